@@ -1,0 +1,77 @@
+"""Oracle pins: the Fig. 5 static schedule (§III-F).
+
+Two independent oracle implementations (closed form, literal Fig. 5 transliteration) are
+checked against each other by brute force over every tiny shape, against the exactly-once
+invariant, and against a hand-derived worked example of Fig. 5 (tests/golden)."""
+import os
+
+import numpy as np
+import pytest
+
+import oracle
+
+GOLD = os.path.join(os.path.dirname(__file__), "golden", "fig5_n10_T2_N3.txt")
+
+
+def test_closed_form_equals_literal_fig5_bruteforce():
+    for n in range(0, 71):
+        for T in range(1, 6):
+            for N in range(1, 10):
+                owner, count = oracle.fig5_simulate(n, T, N)
+                assert (count == 1).all(), (n, T, N)  # every iteration exactly once
+                for iv in range(n):
+                    tm, th = oracle.static_owner_closed(iv, n, T, N)
+                    assert owner[iv] == tm * N + th, (n, T, N, iv)
+
+
+def test_worked_example_fig5():
+    rows = np.loadtxt(GOLD, dtype=np.int64, comments="#")
+    owner, count = oracle.fig5_simulate(10, 2, 3)
+    assert (count == 1).all()
+    assert (owner == rows[:, 3]).all()
+    for iv, tm, th, g in rows:
+        assert oracle.static_owner_closed(int(iv), 10, 2, 3) == (tm, th)
+    # the assumption breaks after one iteration: IV >= T*N never runs
+    owner_a, count_a = oracle.fig5_simulate(10, 2, 3, assume_oversub=True)
+    assert (count_a[:6] == 1).all() and (count_a[6:] == 0).all()
+
+
+@pytest.mark.parametrize("n,T,N", [(0, 1, 1), (1, 8, 128), (1023, 8, 128), (1024, 8, 128),
+                                   (1025, 8, 128), (7, 3, 5), (15, 3, 5), (16, 3, 5)])
+def test_special_cases(n, T, N):
+    owner, count = oracle.fig5_simulate(n, T, N)
+    assert (count == 1).all()
+    # n < T*N: threads g >= n idle;   n = k*T*N + r: thread g runs ceil((n-g)/(T*N)) iters
+    runs = np.bincount(owner, minlength=T * N) if n else np.zeros(T * N, np.int64)
+    g = np.arange(T * N)
+    expect = np.where(g < n, (n - g + T * N - 1) // (T * N), 0)
+    assert (runs == expect).all()
+
+
+def test_assumption_equivalent_when_it_holds():
+    for n in range(0, 40):
+        for T in range(1, 5):
+            for N in range(1, 8):
+                if n > T * N:
+                    continue
+                a = oracle.fig5_simulate(n, T, N, assume_oversub=True)
+                b = oracle.fig5_simulate(n, T, N, assume_oversub=False)
+                assert (a[0] == b[0]).all() and (a[1] == b[1]).all()
+
+
+def test_team_for_and_distribute_readings():
+    # Q2: `for` in a team = Fig. 5 with NumBlocks=1; `distribute` = Fig. 5 with NumThreads=1
+    for n in range(0, 50):
+        for N in range(1, 9):
+            owner, count = oracle.team_for_simulate(n, N)
+            assert (count == 1).all() and (owner == np.arange(n) % N).all()
+        for T in range(1, 6):
+            owner, count = oracle.distribute_simulate(n, T)
+            assert (count == 1).all() and (owner == np.arange(n) % T).all()
+
+
+def test_cyclic_not_blocked():
+    """the combined scheme is CUDA-style cyclic (chunk 1), not OpenMP's blocked
+    schedule(static): consecutive iterations go to consecutive threads."""
+    owner, _ = oracle.fig5_simulate(64, 2, 4)
+    assert list(owner[:9]) == [0, 1, 2, 3, 4, 5, 6, 7, 0]

@@ -1,0 +1,400 @@
+"""bench.py -- XSBench-shaped lookups/s through the omprt device runtime on B200, and its
+runtime overhead versus the bare CUDA kernel (BASELINE.json `metric`, configs[2]).
+
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--impl omprt|reference] [--no-secondary]
+
+One step = one pass of the hot path over one batch: the runtime-driven lookup kernel
+(SPMD `target teams distribute parallel for`, oversubscription assumption, 17M lookups of
+the small problem) + the verification sum (K11) + at N > 1 the NCCL all-reduce of
+the u64 checksum.  Weak scaling: rank r processes lookups [r*L, (r+1)*L), L = 17M, with
+replicated tables.  L2 is flushed (256 MiB scrub write) before every timed step, outside
+the step's events.  Times are CUDA events on the launching stream; the reported time is
+the max over ranks.  `--impl reference` times the CPU oracle (the reference arm) on the
+host cores on a bounded sample.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+L = 17_000_000          # lookups per rank (BASELINE configs[2])
+THREADS = 256
+METRIC = "XSBench lookups/s and runtime overhead vs bare CUDA kernel at 1/2/4/8 B200"
+UNIT = "lookups/s"
+WORKLOAD = "XSBench-shaped small problem (68 nuclides, 11303 gridpoints/nuclide, unionized grid), 17M lookups per GPU"
+
+
+def parse():
+    p = argparse.ArgumentParser()
+    p.add_argument("--gpus", type=int, default=1)
+    p.add_argument("--steps", type=int, default=10)
+    p.add_argument("--warmup", type=int, default=3)
+    p.add_argument("--impl", default="omprt", choices=["omprt", "reference"])
+    p.add_argument("--no-secondary", action="store_true")
+    p.add_argument("--no-e2e", action="store_true")
+    return p.parse_args()
+
+
+def dist_env():
+    rank = int(os.environ.get("RANK", "0"))
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    return rank, world, local
+
+
+# ----------------------------------------------------------------------------- clocks
+class ClockSampler:
+    """nvidia-smi clocks / throttle reasons sampled during the timed region."""
+
+    Q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+         "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+         "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, gpu):
+        self.gpu, self.proc, self.lines = gpu, None, []
+
+    def start(self):
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", "-i", str(self.gpu), f"--query-gpu={self.Q}",
+                 "--format=csv,noheader,nounits", "-lms", "100"],
+                stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except OSError:
+            self.proc = None
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.lines.append(line.strip())
+
+    def stop(self):
+        if self.proc is None:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        time.sleep(0.25)
+        self.proc.terminate()
+        try:
+            self.proc.wait(timeout=5)
+        except subprocess.TimeoutExpired:
+            self.proc.kill()
+        sm, smax, reasons = [], None, set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for ln in self.lines:
+            f = [x.strip() for x in ln.split(",")]
+            if len(f) < 9:
+                continue
+            try:
+                sm.append(float(f[1]))
+                smax = float(f[2])
+            except ValueError:
+                continue
+            for nm, v in zip(names, f[5:9]):
+                if v.lower() == "active":
+                    reasons.add(nm)
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": smax,
+                "reasons": sorted(reasons), "samples": len(sm)}
+
+
+# ----------------------------------------------------------------------------- reference arm
+def cpu_oracle_rate(tables, seconds=3.0, first=0):
+    """The oracle as it stands, over all host cores, on a bounded prefix sample of the
+    workload (contiguous lookups from `first`).  Returns (lookups/s, cores, sample, wall)."""
+    import oracle
+    cores = len(os.sched_getaffinity(0)) if hasattr(os, "sched_getaffinity") else os.cpu_count()
+    t0 = time.perf_counter()
+    oracle.xs_lookup(tables, first, 20000, threads=cores)
+    per = (time.perf_counter() - t0) / 20000
+    n = int(min(L, max(20000, seconds / per)))
+    t0 = time.perf_counter()
+    v = oracle.xs_lookup(tables, first, n, threads=cores)
+    wall = time.perf_counter() - t0
+    return n / wall, cores, n, wall, v
+
+
+def run_reference(args):
+    rank, world, _ = dist_env()
+    if rank != 0:
+        return
+    import gen
+    t = gen.XSTables(**gen.XS_SMALL)
+    times = []
+    rate = cores = n = None
+    for k in range(args.warmup + args.steps):
+        r, cores, n, wall, _ = cpu_oracle_rate(t, seconds=2.0)
+        if k >= args.warmup:
+            times.append(wall)
+            rate = r
+    ms = 1000.0 * statistics.mean(times)
+    value = n / (ms / 1000.0)
+    sample = f"first {n} of the {L} lookups per step (contiguous prefix), all host cores"
+    line = {"impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms,
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64",
+            "data": "synthetic", "config": {"workload": WORKLOAD + " (CPU oracle sample)"},
+            "cpu_baseline": {"value": value, "unit": UNIT, "cores": cores, "kind": "oracle",
+                             "sample": sample},
+            "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0,
+                    "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+# ----------------------------------------------------------------------------- omprt arm
+def load_peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        d = json.load(open(p))
+        return float(d["hbm_gbs"]), "MEASURED_PEAKS.json hbm_gbs (measured copy)"
+    return 6650.0, "fallback 6.65 TB/s (B200_PROFILING.md)"
+
+
+def load_alg_bytes():
+    d = json.load(open(os.path.join(ROOT, "profiles", "xs_algorithmic_bytes.json")))
+    return float(d["bytes_per_lookup"])
+
+
+def load_ncu_traffic():
+    p = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+    if os.path.exists(p):
+        d = json.load(open(p))
+        return d.get("omprt_xs_rt_assume", {}).get("dram_bytes_per_launch")
+    return None
+
+
+def run_omprt(args):
+    import numpy as np
+    import torch
+    import torch.distributed as dist
+
+    import gen
+    from paper_conf_ipps_doerfertphtdcg22_b200 import omprt
+
+    rank, world, local = dist_env()
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    omprt.omprt_init(local)
+    stream = torch.cuda.current_stream()
+    tabs = gen.XSTables(**gen.XS_SMALL)
+    d = omprt.XSDeviceTables(tabs, dev)
+    first = rank * L
+    ver = torch.zeros(L, dtype=torch.uint64, device=dev)
+    ck = torch.zeros(1, dtype=torch.uint64, device=dev)
+    ck_all = torch.zeros(1, dtype=torch.int64, device=dev)
+    scrub = torch.empty(256 * 1024 * 1024 // 4, dtype=torch.float32, device=dev)
+    A = omprt.OMPRT_ASSUME_OVERSUB
+
+    def step(kernel_events=None, which="rt", flags=A):
+        ck.zero_()
+        if kernel_events:
+            kernel_events[0].record(stream)
+        if which == "rt":
+            omprt.omprt_xs_lookup(d, gen.XS_LOOKUP_SEED, first, L, ver, None, 0, THREADS, flags)
+        else:
+            omprt.omprt_cuda_xs_lookup(d, gen.XS_LOOKUP_SEED, first, L, ver, None, 0, THREADS, 0)
+        if kernel_events:
+            kernel_events[1].record(stream)
+        omprt.omprt_u64_sum(ver, L, ck)
+        if world > 1:
+            ck_all.copy_(ck.view(torch.int64))
+            dist.all_reduce(ck_all)  # u64 sum: two's-complement wrap == mod 2^64
+
+    def timed(which, flags, k_steps, w_steps):
+        for _ in range(w_steps):
+            scrub.fill_(1.0)
+            step(None, which, flags)
+        torch.cuda.synchronize()
+        if world > 1:
+            dist.barrier()
+        torch.cuda.synchronize()
+        ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True),
+               torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
+              for _ in range(k_steps)]
+        for e in ev:
+            scrub.fill_(1.0)  # L2 flush, outside the step's events
+            e[0].record(stream)
+            step((e[1], e[2]), which, flags)
+            e[3].record(stream)
+        torch.cuda.synchronize()
+        if world > 1:
+            dist.barrier()
+        step_ms = [a.elapsed_time(b) for a, _, _, b in ev]
+        kern_ms = [b.elapsed_time(c) for _, b, c, _ in ev]
+        return step_ms, kern_ms
+
+    clocks = ClockSampler(local)
+    # primary: runtime-driven with the assumption (the headline path)
+    clocks.start()
+    step_ms, kern_ms = timed("rt", A, args.steps, args.warmup)
+    clk = clocks.stop()
+    checksum = int(ck.cpu().numpy()[0]) if world == 1 else int(ck_all.cpu().numpy()[0]) % 2**64
+    # twin and variants, interleaved in the same process with the same geometry
+    twin_step, twin_k = timed("twin", 0, args.steps, 1)
+    noas_step, noas_k = timed("rt", 0, args.steps, 1)
+
+    def mx(v):
+        if world == 1:
+            return v
+        t = torch.tensor([v], dtype=torch.float64, device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        return float(t.item())
+
+    ms_step = mx(statistics.mean(step_ms))
+    ms_kern = mx(statistics.mean(kern_ms))
+    ms_twin_k = mx(statistics.mean(twin_k))
+    ms_noas_k = mx(statistics.mean(noas_k))
+    value = world * L / (ms_step / 1000.0)
+
+    # e2e through the public C ABI with HOST tables (pinned): H2D tables + lookups + sum +
+    # D2H checksum, synchronous, timed on the host clock around the call
+    e2e = None
+    if not args.no_e2e:
+        pinned = {k: torch.from_numpy(getattr(tabs, k)).pin_memory()
+                  for k in ("nuclide_grid", "unionized", "index_grid", "num_nucs", "mats",
+                            "concs")}
+        hs = omprt.xs_host_struct(tabs, pinned)
+        for _ in range(max(1, args.warmup)):
+            omprt.omprt_xs_run_host(hs, gen.XS_LOOKUP_SEED, first, L, THREADS, 0)
+        torch.cuda.synchronize()
+        if world > 1:
+            dist.barrier()
+        t0 = time.perf_counter()
+        for _ in range(args.steps):
+            ck_h, h2d, d2h = omprt.omprt_xs_run_host(hs, gen.XS_LOOKUP_SEED, first, L, THREADS, 0)
+        e2e_ms = mx(1000.0 * (time.perf_counter() - t0) / args.steps)
+        assert ck_h == checksum or world > 1, (ck_h, checksum)
+        e2e = {"value": world * L / (e2e_ms / 1000.0), "unit": UNIT, "h2d_bytes_per_step": h2d,
+               "d2h_bytes_per_step": d2h, "ms_per_step": e2e_ms,
+               "path": "omprt_xs_run_host (pinned host tables, fused reduction)"}
+
+    tab = omprt.kernel_table()
+    peak, peak_src = load_peaks()
+    alg = load_alg_bytes() * L
+    achieved = alg / (ms_kern / 1000.0) / 1e9
+    secondary = None
+    if not args.no_secondary and rank == 0:
+        secondary = run_secondary(omprt, torch, gen, dev, stream, scrub)
+    cpu = None
+    if rank == 0:
+        r, cores, n, wall, _ = cpu_oracle_rate(tabs, seconds=3.0, first=first)
+        cpu = {"value": r, "unit": UNIT, "cores": cores, "kind": "oracle",
+               "sample": f"first {n} lookups of rank 0's batch, all host cores, {wall:.2f} s wall"}
+    if rank == 0:
+        line = {
+            "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": ms_step, "higher_is_better": True,
+            "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+            "config": {"workload": WORKLOAD, "lookups_per_gpu": L, "threads_per_team": THREADS,
+                       "teams": (L + THREADS - 1) // THREADS, "parallelism": f"dp{world}",
+                       "l2": "flushed before every timed step (256 MiB scrub write)",
+                       "variant": "runtime-driven SPMD, teams oversubscription assumption"},
+            "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
+                         "frac": achieved / peak, "traffic": load_ncu_traffic(),
+                         "kernel": "omprt_xs_rt_assume", "alg_bytes_per_launch": alg,
+                         "peak_source": peak_src},
+            "cpu_baseline": cpu,
+            "e2e": e2e,
+            "gpu_launches": 2 * args.steps,
+            "clocks": clk,
+            "checksum": checksum,
+            "kernel_ms": {"rt_assume": ms_kern, "twin": ms_twin_k, "rt_no_assume": ms_noas_k},
+            "overhead_vs_twin": {
+                "time": ms_kern / ms_twin_k - 1.0,
+                "time_no_assume": ms_noas_k / ms_twin_k - 1.0,
+                "regs": [tab["omprt_xs_rt_assume"]["regs"], tab["cuda_xs_twin"]["regs"]],
+                "regs_no_assume": tab["omprt_xs_rt"]["regs"],
+                "static_smem": [tab["omprt_xs_rt_assume"]["static_smem"],
+                                tab["cuda_xs_twin"]["static_smem"]]},
+            "secondary": secondary,
+        }
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.destroy_process_group()
+
+
+def _time(fn, stream, scrub, reps=5, warm=2, flush=True):
+    import torch
+    for _ in range(warm):
+        fn()
+    torch.cuda.synchronize()
+    out = []
+    for _ in range(reps):
+        if flush:
+            scrub.fill_(1.0)
+        a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        a.record(stream)
+        fn()
+        b.record(stream)
+        torch.cuda.synchronize()
+        out.append(a.elapsed_time(b))
+    return statistics.median(out)
+
+
+def run_secondary(omprt, torch, gen, dev, stream, scrub):
+    """The other BASELINE configs at their sizes, runtime vs twin (kernel ms, cold L2)."""
+    res = {}
+    # C1: SPMD axpy + sum, 2^20, 8 x 128
+    n = 1 << 20
+    x, b, c = gen.axpy_inputs(n)
+    bt, ct = torch.from_numpy(b).to(dev), torch.from_numpy(c).to(dev)
+    at = torch.empty_like(bt)
+    s = torch.zeros(1, dtype=torch.float64, device=dev)
+    t_rt = _time(lambda: omprt.omprt_spmd_axpy_sum(n, x, bt, ct, at, s, 8, 128), stream, scrub)
+    t_tw = _time(lambda: omprt.omprt_cuda_axpy_sum(n, x, bt, ct, at, s, 8, 128), stream, scrub)
+    res["c1_axpy_sum_8x128"] = {"rt_ms": t_rt, "twin_ms": t_tw, "overhead": t_rt / t_tw - 1,
+                                "GBps_alg": 24 * n / t_rt / 1e6}
+    # C2: generic mode 4096 teams x 256, inner 256
+    T = 4096
+    inp = torch.from_numpy(gen.generic_inputs(T, 256)).to(dev)
+    out = torch.empty(T * 256, dtype=torch.float64, device=dev)
+    t_rt = _time(lambda: omprt.omprt_generic_team(T, 256, 256, inp, out, None, None,
+                                                  omprt.OMPRT_ASSUME_OVERSUB), stream, scrub)
+    t_gs = _time(lambda: omprt.omprt_generic_team(T, 256, 256, inp, out, None, None,
+                                                  omprt.OMPRT_GENERAL_SM), stream, scrub)
+    t_tw = _time(lambda: omprt.omprt_cuda_generic_team(T, 256, 256, inp, out), stream, scrub)
+    res["c2_generic_4096x256"] = {"rt_ms": t_rt, "rt_general_sm_ms": t_gs, "twin_ms": t_tw,
+                                  "overhead": t_rt / t_tw - 1}
+    # C4: RSBench-shaped, 10M lookups (single GPU here)
+    rs = gen.RSTables()
+    rd = omprt.RSDeviceTables(rs, dev)
+    nl = 10_000_000
+    v = torch.empty(nl, dtype=torch.uint64, device=dev)
+    A = omprt.OMPRT_ASSUME_OVERSUB
+    t_rt = _time(lambda: omprt.omprt_rs_lookup(rd, 1070, 0, nl, v, None, 0, 128, A), stream,
+                 scrub, reps=3, warm=1)
+    t_tw = _time(lambda: omprt.omprt_cuda_rs_lookup(rd, 1070, 0, nl, v, None, 0, 128, 0), stream,
+                 scrub, reps=3, warm=1)
+    res["c4_rsbench_10M"] = {"rt_ms": t_rt, "twin_ms": t_tw, "overhead": t_rt / t_tw - 1,
+                             "lookups_per_s": nl / t_rt * 1e3}
+    # C5: SU(3) 32^4 sites
+    ns = 32 ** 4
+    Ah, Bh = gen.su3_inputs(ns)
+    At, Bt = torch.from_numpy(Ah).to(dev), torch.from_numpy(Bh).to(dev)
+    Ct = torch.empty_like(At)
+    ck = torch.zeros(1, dtype=torch.float64, device=dev)
+    t_rt = _time(lambda: omprt.omprt_su3_mult(At, Bt, Ct, ns, ck, 0, 128, A), stream, scrub)
+    t_tw = _time(lambda: omprt.omprt_cuda_su3_mult(At, Bt, Ct, ns, ck, 0, 128, 0), stream, scrub)
+    res["c5_su3_32^4"] = {"rt_ms": t_rt, "twin_ms": t_tw, "overhead": t_rt / t_tw - 1,
+                          "GBps_alg": 1152 * ns / t_rt / 1e6, "GFLOPs": 864 * ns / t_rt / 1e6}
+    return res
+
+
+def main():
+    args = parse()
+    if args.impl == "reference":
+        run_reference(args)
+    else:
+        run_omprt(args)
+
+
+if __name__ == "__main__":
+    main()

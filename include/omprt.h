@@ -1,0 +1,220 @@
+/*
+ * omprt.h -- C ABI of libomprt.so, the B200-native (sm_100a) device-runtime hot path of
+ * Doerfert et al., "Co-Designing an OpenMP GPU Runtime and Optimizations for Near-Zero
+ * Overhead Execution" (IPDPS'22).  "P:<line> §<sec>" cites /root/reference/PAPER.md.
+ *
+ * Each entry point launches the execution of one offloaded
+ *     #pragma omp target teams distribute parallel for        (SPMD mode)
+ * or one generic-mode target region (sequential main thread + `parallel`),
+ * driven by the header-only device runtime (csrc/omprt/device: init/deinit P:100-112,
+ * Fig. 5 static schedule P:121-149, state machine P:92, alloc_shared stack P:110-112,
+ * team/league reductions), and -- under the `omprt_cuda_*` names -- the hand-written bare
+ * CUDA kernel of the same loop (the paper's "CUDA (NVCC)" rows), which gives the
+ * "overhead versus CUDA".
+ *
+ * Conventions (all functions):
+ *   - Return an int status: OMPRT_OK (0) or a negative OMPRT_E_* code; no C++ exception
+ *     crosses the ABI.  omprt_last_error() returns the calling thread's last message.
+ *   - Data pointers are DEVICE pointers owned by the caller (e.g. torch tensors) unless the
+ *     name says `_host`.  The library never frees caller memory.  It owns only its
+ *     per-device workspace (fallback pool, league partials, tickets, error word), created
+ *     by omprt_init and released by omprt_fini.
+ *   - The device is the calling thread's current CUDA device; omprt_init must have been
+ *     called for it (else OMPRT_E_NOTINIT).
+ *   - `stream` is a cudaStream_t passed as void* (NULL = legacy default stream).  Launches
+ *     are asynchronous; results are valid after the stream is synchronized.  Calls that
+ *     reduce share the device's league workspace: launch them on one stream (in order).
+ *   - Reductions follow OpenMP: *inout = *inout (+) sum over all iterations.
+ *   - Device-side fatal errors (stack pool exhausted, debug assertion) record a code in a
+ *     mapped host word and trap; omprt_device_status() reports it.
+ */
+#ifndef OMPRT_H
+#define OMPRT_H
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+/* ---- status codes ------------------------------------------------------------------ */
+#define OMPRT_OK 0
+#define OMPRT_E_INVAL (-1)   /* bad argument (incl. a violated oversubscription assumption) */
+#define OMPRT_E_CUDA (-2)    /* a CUDA runtime call failed (message in omprt_last_error) */
+#define OMPRT_E_NOMEM (-3)   /* device allocation failed */
+#define OMPRT_E_STACK (-4)   /* shared-memory stack and its global pool exhausted */
+#define OMPRT_E_ASSERT (-5)  /* debug-build device assertion failed */
+#define OMPRT_E_NOTINIT (-6) /* omprt_init was not called for the current device */
+
+/* ---- launch flags ------------------------------------------------------------------ */
+/* P:125 §III-F user assumption: n <= teams*threads (distribute parallel for) or n <= team
+ * size (team `for`): every thread runs at most one iteration and the loop disappears.  The
+ * host rejects a call that violates it (OMPRT_E_INVAL) instead of dropping iterations. */
+#define OMPRT_ASSUME_OVERSUB (1u << 0)
+/* Test build: record owner[i] = global thread id that ran iteration i (and count[i]). */
+#define OMPRT_RECORD_OWNER (1u << 1)
+/* Generic mode: use the general state machine (function pointer) instead of the custom
+ * compile-time one. */
+#define OMPRT_GENERAL_SM (1u << 2)
+/* Generic mode stack placement: dynamic shared memory of 2 KiB / 0 B instead of
+ * the static 4 KiB stack, so globalized arrays fall back to the global pool. */
+#define OMPRT_SMALL_STACK (1u << 3)
+#define OMPRT_NO_STACK (1u << 4)
+/* Use the debug instantiation: assertions + call tracing compiled in, enabled at run time
+ * by OMPRT_DEBUG (bit 0 assert, bit 1 trace) read at omprt_init. */
+#define OMPRT_DEBUG_BUILD (1u << 5)
+/* Generic mode: the region joins and the main thread runs a sequential postlogue. */
+#define OMPRT_POSTLOGUE (1u << 6)
+/* ICV probe: keep ICVs of nested data environments in thread ICV states. */
+#define OMPRT_THREAD_STATES (1u << 7)
+/* Fused variants: reduce the per-iteration verification inside the loop kernel instead of
+ * storing it and summing with omprt_u64_sum (the paper moves the reduction out). */
+#define OMPRT_FUSED_REDUCTION (1u << 8)
+/* Testing only (omprt_spmd_axpy_sum): skip the host-side check of OMPRT_ASSUME_OVERSUB so
+ * the debug build's device assertion ("asserting that the condition actually holds")
+ * can be exercised.  In a release build a violated assumption then skips iterations. */
+#define OMPRT_UNCHECKED (1u << 9)
+
+/* ---- runtime lifecycle ------------------------------------------------------------- */
+typedef struct {
+  uint64_t pool_bytes_per_team; /* global fallback slice per team (default 64 KiB) */
+  uint64_t pool_teams;          /* teams covered by the pool (default 4096) */
+  uint64_t max_teams;           /* capacity of the league-reduction partials (default 2^20) */
+} omprt_options;
+
+/* Create the per-device workspace; reads OMPRT_DEBUG.  opt may be NULL (defaults).
+ * Idempotent per device. */
+int omprt_init(int device, const omprt_options *opt);
+int omprt_fini(int device);
+/* Device-side error recorded since init (0 = none); info (nullable) gets 4 ints
+ * {team, thread, line, extra}. */
+int omprt_device_status(int device, int *code, int *info);
+/* Copies the calling thread's last error message (always NUL-terminated); returns its
+ * length. */
+int omprt_last_error(char *buf, size_t n);
+
+/* Fig. 5 as a pure host function: the (team, thread) that runs iteration iv
+ * of a combined distribute parallel for over n iterations.  OMPRT_E_INVAL if iv is not in
+ * [0, n) or a size is not positive. */
+int omprt_static_owner(int64_t iv, int64_t n, int32_t teams, int32_t threads, int32_t *team,
+                       int32_t *thread);
+
+/* ---- C1: SPMD axpy + fp64 sum (BASELINE configs[0]) -------------------------------- */
+/* a[i] = fma(x, b[i], c[i]) for i in [0, n); *sum_inout += sum_i a[i] (team + league
+ * reduction).  b, c, a: n doubles; sum_inout: 1 double; owner/count (nullable, test build
+ * with OMPRT_RECORD_OWNER): n int32 each -- owner[i] = team*threads+thread, count[i] +=
+ * 1.  flags: OMPRT_ASSUME_OVERSUB | OMPRT_RECORD_OWNER | OMPRT_DEBUG_BUILD. */
+int omprt_spmd_axpy_sum(int64_t n, double x, const double *b, const double *c, double *a,
+                        double *sum_inout, int32_t teams, int32_t threads, uint32_t flags,
+                        int32_t *owner, int32_t *count, void *stream);
+int omprt_cuda_axpy_sum(int64_t n, double x, const double *b, const double *c, double *a,
+                        double *sum_inout, int32_t teams, int32_t threads, uint32_t flags,
+                        int32_t *owner, int32_t *count, void *stream);
+
+/* ---- C2: generic-mode team kernel -------------------------------- */
+/* Per team t: the main thread builds globalized w[inner_n], perm[inner_n] with
+ * alloc_shared, then `parallel` + team `for` computes
+ *   out[t*inner_n + j] = w[perm[j]] / s + w[j].
+ * in/out: teams*inner_n doubles; owner (nullable): teams*inner_n int32 (OpenMP thread
+ * number); postlogue (nullable, needs OMPRT_POSTLOGUE): teams doubles.  threads <= 1024,
+ * inner_n <= 256 for the CUDA twin.  flags: OMPRT_GENERAL_SM | OMPRT_SMALL_STACK |
+ * OMPRT_NO_STACK | OMPRT_POSTLOGUE | OMPRT_ASSUME_OVERSUB (inner_n <= threads) |
+ * OMPRT_DEBUG_BUILD. */
+int omprt_generic_team(int32_t teams, int32_t threads, int32_t inner_n, const double *in,
+                       double *out, int32_t *owner, double *postlogue, uint32_t flags,
+                       void *stream);
+int omprt_cuda_generic_team(int32_t teams, int32_t threads, int32_t inner_n, const double *in,
+                            double *out, int32_t *owner, double *postlogue, uint32_t flags,
+                            void *stream);
+
+/* ICV probe (Fig. 3/4): generic-mode kernel that records 7 int32 per query
+ * point {thread_num, num_threads, level, active_level, in_parallel, team_num, num_teams}:
+ * rec[t][0] prologue (main), rec[t][1+k] region thread k, rec[t][1+threads+k] inside a
+ * nested parallel (num_threads(nested_request), serialized), rec[t][1+2*threads+k] after
+ * it.  rec: teams*(1+3*threads)*7 int32.  flags: OMPRT_THREAD_STATES | OMPRT_DEBUG_BUILD |
+ * OMPRT_GENERAL_SM. */
+int omprt_icv_probe(int32_t teams, int32_t threads, int32_t nested_request, int32_t *rec,
+                    uint32_t flags, void *stream);
+
+/* ---- C3: XSBench-shaped lookup (§V-A) ------------------------- */
+typedef struct {
+  const double *nuclide_grid; /* [n_isotopes*n_gridpoints][6] energy + 5 xs, per nuclide sorted */
+  const double *unionized;    /* [n_union] sorted energies */
+  const int32_t *index_grid;  /* [n_union][n_isotopes] lower bracket per nuclide */
+  const int32_t *num_nucs;    /* [12] */
+  const int32_t *mats;        /* [12][max_num_nucs] */
+  const double *concs;        /* [12][max_num_nucs] */
+  int32_t n_isotopes, n_gridpoints, max_num_nucs, pad;
+  int64_t n_union;
+} omprt_xs_tables;
+/* Lookups first..first+count-1 (lookup i draws its energy and material from
+ * fast_forward_LCG(seed, 2i), so results do not depend on sharding):
+ * verification[i-first] = 1 + argmax of the 5 macroscopic cross sections.  teams = 0:
+ * ceil(count/threads).  With OMPRT_FUSED_REDUCTION, verification may be NULL and
+ * *checksum_inout += sum of the verification values instead (checksum_inout device u64).
+ * flags: OMPRT_ASSUME_OVERSUB | OMPRT_FUSED_REDUCTION | OMPRT_DEBUG_BUILD. */
+int omprt_xs_lookup(omprt_xs_tables t, uint64_t seed, int64_t first, int64_t count,
+                    uint64_t *verification, uint64_t *checksum_inout, int32_t teams,
+                    int32_t threads, uint32_t flags, void *stream);
+int omprt_cuda_xs_lookup(omprt_xs_tables t, uint64_t seed, int64_t first, int64_t count,
+                         uint64_t *verification, uint64_t *checksum_inout, int32_t teams,
+                         int32_t threads, uint32_t flags, void *stream);
+/* K11 ("we moved the reduction out of the timed kernel"): *out_inout += sum v[i]
+ * (u64, wraps mod 2^64). */
+int omprt_u64_sum(const uint64_t *v, int64_t n, uint64_t *out_inout, void *stream);
+/* End-to-end offload with HOST tables (an OpenMP `target ... map(to: tables)
+ * map(from: checksum)`): copies the tables host->device into library-owned buffers
+ * (host pointers should be pinned), runs the lookups and the sum, and copies the u64
+ * checksum back to *checksum_host.  Synchronous.  h2d_bytes/d2h_bytes (nullable) receive
+ * the bytes moved. */
+int omprt_xs_run_host(omprt_xs_tables host_tables, uint64_t seed, int64_t first, int64_t count,
+                      int32_t threads, uint32_t flags, uint64_t *checksum_host,
+                      uint64_t *h2d_bytes, uint64_t *d2h_bytes, void *stream);
+
+/* ---- C4: RSBench-shaped multipole lookup -------------------- */
+typedef struct {
+  const double *poles;      /* [n_poles][8] EA RT RA RF (re, im) */
+  const int32_t *pole_l;    /* [n_poles] l value in [0, numL) */
+  const double *windows;    /* [n_windows][4] T A F 0 */
+  const int32_t *win_range; /* [n_windows][2] absolute pole [start, end) */
+  const int32_t *win_off;   /* [n_nuclides+1] window CSR offsets */
+  const int32_t *n_windows; /* [n_nuclides] */
+  const double *k0rs;       /* [n_nuclides][numL] */
+  const int32_t *num_nucs;  /* [12] */
+  const int32_t *mats;      /* [12][max_num_nucs] */
+  const double *concs;      /* [12][max_num_nucs] */
+  int32_t n_nuclides, numL, max_num_nucs, pad;
+} omprt_rs_tables;
+/* Same contract as omprt_xs_lookup (4 macroscopic cross sections; numL must be 4).
+ * macro (nullable): [count][4] doubles for parity tests. */
+int omprt_rs_lookup(omprt_rs_tables t, uint64_t seed, int64_t first, int64_t count,
+                    uint64_t *verification, double *macro, int32_t teams, int32_t threads,
+                    uint32_t flags, void *stream);
+int omprt_cuda_rs_lookup(omprt_rs_tables t, uint64_t seed, int64_t first, int64_t count,
+                         uint64_t *verification, double *macro, int32_t teams, int32_t threads,
+                         uint32_t flags, void *stream);
+
+/* ---- C5: SU(3) link multiply -------------------------------------- */
+/* C[s][l] = A[s][l] x B[l] (3x3 complex, fp64) for s in [0, n_sites); A, C: n_sites*72
+ * doubles (site-major AoS), B: 72 doubles; *checksum_inout += sum of Re C (nullable).
+ * teams = 0: ceil(n_sites/threads). */
+int omprt_su3_mult(const double *A, const double *B, double *C, int64_t n_sites,
+                   double *checksum_inout, int32_t teams, int32_t threads, uint32_t flags,
+                   void *stream);
+int omprt_cuda_su3_mult(const double *A, const double *B, double *C, int64_t n_sites,
+                        double *checksum_inout, int32_t teams, int32_t threads, uint32_t flags,
+                        void *stream);
+
+/* ---- introspection (resource report, "# Regs" and "SMem") ------------------ */
+/* Number of kernels in the library and the name of kernel `id`. */
+int omprt_kernel_count(void);
+const char *omprt_kernel_name(int id);
+/* cudaFuncGetAttributes of kernel `id`: registers per thread, static smem bytes, local
+ * (spill/stack) bytes per thread, max threads per block. */
+int omprt_kernel_attrs(int id, int *regs, int *static_smem, int *local_bytes,
+                       int *max_threads);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* OMPRT_H */

@@ -1,0 +1,379 @@
+// C2 (BASELINE configs[1]): a generic-mode target region:
+//   #pragma omp target teams num_teams(T) thread_limit(N)
+//   { double w[256]; int perm[256]; double s = 0;            // shared with the region:
+//     for (k...) { w[k] = in[t*256+k]*(t+1); s += w[k]; perm[k] = (17k+t) % 256; }  // globalized
+//     #pragma omp parallel for
+//     for (j...) out[t*256+j] = w[perm[j]] / s + w[j]; }
+// (SURVEY App. A.4).  Runtime-driven: main thread + custom (or general) state machine +
+// alloc_shared stack; twin: __shared__ arrays, thread 0 prologue, one __syncthreads.
+// Products that feed adds use __dmul_rn/__dadd_rn so nvcc cannot contract them (Q12).
+//
+// Also: the ICV probe kernel (Fig. 3/4 semantics).
+#pragma once
+#include "../host/runtime.cuh"
+
+namespace omprt_kernels {
+
+using namespace omprt;
+
+template <class Base, bool GeneralSM>
+struct GenSM : Base {
+  static constexpr bool custom_state_machine = !GeneralSM;
+};
+
+struct GenericTraits : DefaultTraits {
+  static constexpr Mode mode = Mode::Generic;
+  static constexpr unsigned stack_bytes = 4096;  // SURVEY Q9 default
+  static constexpr bool assume_threads_oversub = true;  // inner_n <= team size
+};
+struct GenericTraitsLoop : GenericTraits {
+  static constexpr bool assume_threads_oversub = false;
+};
+// stack in dynamic shared memory (fallback tests: 4 KiB / 2 KiB / 0 B at launch)
+struct GenericTraitsDyn : GenericTraitsLoop {
+  static constexpr unsigned stack_bytes = 0;
+  static constexpr bool dynamic_stack = true;
+};
+struct GenericTraitsDebug : GenericTraitsLoop {
+  static constexpr unsigned debug = dbg::Assert | dbg::Trace;
+};
+
+// The parallel region: team `for` over j (Fig. 5 with NumBlocks = 1).
+template <bool Rec, bool Join>
+struct GenRegion {
+  struct Args {
+    const double* w;
+    const int32_t* perm;
+    double s;
+    double* out;
+    int32_t* owner;
+    int32_t inner_n;
+  };
+  static constexpr bool terminal = true;  // the only region of the kernel
+  static constexpr bool join = Join;      // postlogue reads `out` after the region
+  template <class Tr>
+  __device__ __forceinline__ void operator()(Team<Tr>& team, const Args& a) const {
+    for_static(team, (typename Tr::Idx)a.inner_n, [&](int j) {
+      a.out[j] = __dadd_rn(__ddiv_rn(a.w[a.perm[j]], a.s), a.w[j]);
+      if constexpr (Rec) a.owner[j] = get_thread_num(team);
+    });
+  }
+};
+
+template <class Tr, int kInner, bool Rec, bool Post>
+__global__ void __launch_bounds__(1024)
+    omprt_generic_rt(int32_t inner_n_rt, const double* __restrict__ in, double* __restrict__ out,
+                     int32_t* owner, double* post) {
+  using R = GenRegion<Rec, Post>;
+  using L = RegionList<R>;
+  const int32_t inner_n = kInner > 0 ? kInner : inner_n_rt;
+  Team<Tr> team = init<Tr>();
+  if (!is_main(team)) {  // workers: wait for the main thread's parallel region
+    worker_state_machine<Tr, L>(team);
+    return;
+  }
+  // ---- sequential part: the team's main thread alone ----
+  const int32_t t = (int32_t)blockIdx.x;
+  const double* tin = in + (int64_t)t * inner_n;
+  double* w = static_cast<double*>(alloc_shared(team, (uint32_t)inner_n * 8u));
+  int32_t* perm = static_cast<int32_t*>(alloc_shared(team, (uint32_t)inner_n * 4u));
+  const double tp1 = (double)(t + 1);
+  double s = 0.0;
+  for (int32_t k = 0; k < inner_n; ++k) {
+    const double v = __dmul_rn(__ldg(tin + k), tp1);
+    w[k] = v;
+    s = __dadd_rn(s, v);
+    perm[k] = (k * 17 + t) % inner_n;
+  }
+  double* tout = out + (int64_t)t * inner_n;
+  parallel<Tr, L, R>(team, typename R::Args{w, perm, s, tout,
+                                            Rec ? owner + (int64_t)t * inner_n : nullptr,
+                                            inner_n});
+  if constexpr (Post) {  // after the join the main thread sees the region's writes
+    double acc = 0.0;
+    for (int32_t j = 0; j < inner_n; ++j) acc = __dadd_rn(acc, tout[j]);
+    post[t] = acc;
+  }
+  free_shared(team, perm, (uint32_t)inner_n * 4u);
+  free_shared(team, w, (uint32_t)inner_n * 8u);
+  deinit<Tr, L, true>(team);
+}
+
+// Bare CUDA twin.
+template <int kInner, bool Rec, bool Post>
+__global__ void __launch_bounds__(1024)
+    cuda_generic_twin(int32_t inner_n_rt, const double* __restrict__ in,
+                      double* __restrict__ out, int32_t* owner, double* post) {
+  __shared__ double w[256];
+  __shared__ int32_t perm[256];
+  __shared__ double s_sh;
+  const int32_t inner_n = kInner > 0 ? kInner : inner_n_rt;
+  const int32_t t = (int32_t)blockIdx.x;
+  if (threadIdx.x == 0) {
+    const double* tin = in + (int64_t)t * inner_n;
+    const double tp1 = (double)(t + 1);
+    double s = 0.0;
+    for (int32_t k = 0; k < inner_n; ++k) {
+      const double v = __dmul_rn(__ldg(tin + k), tp1);
+      w[k] = v;
+      s = __dadd_rn(s, v);
+      perm[k] = (k * 17 + t) % inner_n;
+    }
+    s_sh = s;
+  }
+  __syncthreads();
+  const double s = s_sh;
+  double* tout = out + (int64_t)t * inner_n;
+  for (int32_t j = threadIdx.x; j < inner_n; j += blockDim.x) {
+    tout[j] = __dadd_rn(__ddiv_rn(w[perm[j]], s), w[j]);
+    if constexpr (Rec) owner[(int64_t)t * inner_n + j] = threadIdx.x;
+  }
+  if constexpr (Post) {
+    __syncthreads();
+    if (threadIdx.x == 0) {
+      double acc = 0.0;
+      for (int32_t j = 0; j < inner_n; ++j) acc = __dadd_rn(acc, tout[j]);
+      post[t] = acc;
+    }
+  }
+}
+
+OMPRT_REGISTER_KERNEL(omprt_generic_rt, omprt_generic_rt<GenSM<GenericTraits, false>, 256, false, false>)
+OMPRT_REGISTER_KERNEL(omprt_generic_rt_general_sm,
+                      omprt_generic_rt<GenSM<GenericTraits, true>, 256, false, false>)
+OMPRT_REGISTER_KERNEL(cuda_generic_twin, cuda_generic_twin<256, false, false>)
+
+template <class Tr, int kInner>
+inline void launch_generic_rt(int32_t teams, int32_t threads, int32_t inner_n, const double* in,
+                              double* out, int32_t* owner, double* post, uint32_t dyn,
+                              cudaStream_t s) {
+  const bool rec = owner != nullptr, pst = post != nullptr;
+  if (rec && pst)
+    omprt_generic_rt<Tr, kInner, true, true><<<teams, threads, dyn, s>>>(inner_n, in, out, owner, post);
+  else if (rec)
+    omprt_generic_rt<Tr, kInner, true, false><<<teams, threads, dyn, s>>>(inner_n, in, out, owner, post);
+  else if (pst)
+    omprt_generic_rt<Tr, kInner, false, true><<<teams, threads, dyn, s>>>(inner_n, in, out, owner, post);
+  else
+    omprt_generic_rt<Tr, kInner, false, false><<<teams, threads, dyn, s>>>(inner_n, in, out, owner, post);
+}
+
+template <class Tr>
+inline void launch_generic_rt_any(int32_t teams, int32_t threads, int32_t inner_n,
+                                  const double* in, double* out, int32_t* owner, double* post,
+                                  uint32_t dyn, cudaStream_t s) {
+  if (inner_n == 256)
+    launch_generic_rt<Tr, 256>(teams, threads, inner_n, in, out, owner, post, dyn, s);
+  else
+    launch_generic_rt<Tr, 0>(teams, threads, inner_n, in, out, owner, post, dyn, s);
+}
+
+template <class Tr>
+inline void launch_generic_sm(bool general, int32_t teams, int32_t threads, int32_t inner_n,
+                              const double* in, double* out, int32_t* owner, double* post,
+                              uint32_t dyn, cudaStream_t s) {
+  if (general)
+    launch_generic_rt_any<GenSM<Tr, true>>(teams, threads, inner_n, in, out, owner, post, dyn, s);
+  else
+    launch_generic_rt_any<GenSM<Tr, false>>(teams, threads, inner_n, in, out, owner, post, dyn, s);
+}
+
+inline uint64_t stack_round_host(uint64_t b) { return (b + 15) & ~uint64_t(15); }
+
+inline int generic_validate(int32_t teams, int32_t threads, int32_t inner_n, const double* in,
+                            double* out, double* post, uint32_t flags, Workspace* w,
+                            bool twin) {
+  OMPRT_CHECK_ARG(teams > 0 && teams <= 2147483647, "teams must be > 0");
+  OMPRT_CHECK_ARG(threads > 0 && threads <= 1024, "threads must be in [1, 1024]");
+  OMPRT_CHECK_ARG(inner_n >= 0 && inner_n <= 65536, "inner_n out of range");
+  OMPRT_CHECK_ARG(!twin || inner_n <= 256, "the CUDA twin supports inner_n <= 256");
+  OMPRT_CHECK_ARG(inner_n == 0 || (in && out), "null data pointer");
+  OMPRT_CHECK_ARG(!(flags & OMPRT_POSTLOGUE) || post, "OMPRT_POSTLOGUE needs postlogue");
+  OMPRT_CHECK_ARG(!(flags & OMPRT_ASSUME_OVERSUB) || inner_n <= threads,
+                  "threads-oversubscription assumption violated: inner_n=%d > threads=%d",
+                  inner_n, threads);
+  if (!twin) {
+    // bytes of the globalized arrays (16 B granules) against stack + this team's pool slice
+    const uint64_t need = stack_round_host((uint64_t)inner_n * 8) +
+                          stack_round_host((uint64_t)inner_n * 4);
+    const uint64_t cap = (flags & OMPRT_NO_STACK) ? 0 : (flags & OMPRT_SMALL_STACK) ? 2048 : 4096;
+    if (need > cap) {
+      OMPRT_CHECK_ARG((uint64_t)teams <= w->opt.pool_teams,
+                      "teams (%d) exceed the fallback pool's pool_teams (%llu)", teams,
+                      (unsigned long long)w->opt.pool_teams);
+      if (need > cap + w->opt.pool_bytes_per_team)
+        return set_error(OMPRT_E_STACK,
+                         "globalized arrays (%llu B) exceed stack (%llu B) + pool slice (%llu B)",
+                         (unsigned long long)need, (unsigned long long)cap,
+                         (unsigned long long)w->opt.pool_bytes_per_team);
+    }
+  }
+  return OMPRT_OK;
+}
+
+}  // namespace omprt_kernels
+
+extern "C" int omprt_generic_team(int32_t teams, int32_t threads, int32_t inner_n,
+                                  const double* in, double* out, int32_t* owner,
+                                  double* postlogue, uint32_t flags, void* stream) {
+  using namespace omprt_kernels;
+  Workspace* w;
+  if (int r = current_ws(&w)) return r;
+  if (int r = generic_validate(teams, threads, inner_n, in, out, postlogue, flags, w, false))
+    return r;
+  cudaStream_t s = as_stream(stream);
+  double* post = (flags & OMPRT_POSTLOGUE) ? postlogue : nullptr;
+  const bool general = flags & OMPRT_GENERAL_SM;
+  if (flags & (OMPRT_SMALL_STACK | OMPRT_NO_STACK)) {
+    const uint32_t dyn = (flags & OMPRT_NO_STACK) ? 0u : 2048u;
+    launch_generic_sm<GenericTraitsDyn>(general, teams, threads, inner_n, in, out, owner, post,
+                                        dyn, s);
+  } else if (stack_round_host((uint64_t)inner_n * 8) + stack_round_host((uint64_t)inner_n * 4) >
+             4096) {
+    // does not fit the static 4 KiB stack: spill to the pool through a 4 KiB dynamic stack
+    const uint32_t dyn = 4096;
+    launch_generic_sm<GenericTraitsDyn>(general, teams, threads, inner_n, in, out, owner, post,
+                                        dyn, s);
+  } else if (flags & OMPRT_DEBUG_BUILD) {
+    launch_generic_sm<GenericTraitsDebug>(general, teams, threads, inner_n, in, out, owner, post,
+                                          0, s);
+  } else if (flags & OMPRT_ASSUME_OVERSUB) {
+    launch_generic_sm<GenericTraits>(general, teams, threads, inner_n, in, out, owner, post, 0,
+                                     s);
+  } else {
+    launch_generic_sm<GenericTraitsLoop>(general, teams, threads, inner_n, in, out, owner, post,
+                                         0, s);
+  }
+  return check_launch("omprt_generic_rt");
+}
+
+extern "C" int omprt_cuda_generic_team(int32_t teams, int32_t threads, int32_t inner_n,
+                                       const double* in, double* out, int32_t* owner,
+                                       double* postlogue, uint32_t flags, void* stream) {
+  using namespace omprt_kernels;
+  Workspace* w;
+  if (int r = current_ws(&w)) return r;
+  if (int r = generic_validate(teams, threads, inner_n, in, out, postlogue, flags, w, true))
+    return r;
+  cudaStream_t s = as_stream(stream);
+  const bool rec = owner != nullptr, pst = (flags & OMPRT_POSTLOGUE) != 0;
+#define OMPRT_TWIN_LAUNCH(K)                                                               \
+  do {                                                                                     \
+    if (rec && pst)                                                                        \
+      cuda_generic_twin<K, true, true><<<teams, threads, 0, s>>>(inner_n, in, out, owner,   \
+                                                                 postlogue);              \
+    else if (rec)                                                                          \
+      cuda_generic_twin<K, true, false><<<teams, threads, 0, s>>>(inner_n, in, out, owner,  \
+                                                                  postlogue);             \
+    else if (pst)                                                                          \
+      cuda_generic_twin<K, false, true><<<teams, threads, 0, s>>>(inner_n, in, out, owner,  \
+                                                                  postlogue);             \
+    else                                                                                   \
+      cuda_generic_twin<K, false, false><<<teams, threads, 0, s>>>(inner_n, in, out, owner, \
+                                                                   postlogue);            \
+  } while (0)
+  if (inner_n == 256) OMPRT_TWIN_LAUNCH(256);
+  else OMPRT_TWIN_LAUNCH(0);
+#undef OMPRT_TWIN_LAUNCH
+  return check_launch("cuda_generic_twin");
+}
+
+// ---------------------------------------------------------------------------------------
+// ICV probe: records the ICV queries at the prologue, in the region, inside a
+// serialized nested parallel and after it.
+// ---------------------------------------------------------------------------------------
+namespace omprt_kernels {
+
+template <class Tr>
+__device__ __forceinline__ void icv_record(const Team<Tr>& t, int32_t* r) {
+  r[0] = get_thread_num(t);
+  r[1] = get_num_threads(t);
+  r[2] = get_level(t);
+  r[3] = get_active_level(t);
+  r[4] = in_parallel(t);
+  r[5] = get_team_num(t);
+  r[6] = get_num_teams(t);
+}
+
+struct IcvNested {
+  struct Args {
+    int32_t* rec;
+  };
+  static constexpr bool terminal = true;
+  static constexpr bool join = false;
+  template <class Tr>
+  __device__ __forceinline__ void operator()(Team<Tr>& team, const Args& a) const {
+    icv_record(team, a.rec);
+  }
+};
+
+struct IcvOuter {
+  struct Args {
+    int32_t* team_rec;  // this team's records
+    int32_t nthreads;
+    int32_t nested_request;
+  };
+  static constexpr bool terminal = true;
+  static constexpr bool join = false;
+  template <class Tr>
+  __device__ __forceinline__ void operator()(Team<Tr>& team, const Args& a) const {
+    const int k = get_thread_num(team);
+    icv_record(team, a.team_rec + (1 + k) * 7);
+    parallel<Tr, RegionList<IcvNested>, IcvNested>(
+        team, IcvNested::Args{a.team_rec + (1 + a.nthreads + k) * 7}, a.nested_request);
+    icv_record(team, a.team_rec + (1 + 2 * a.nthreads + k) * 7);
+  }
+};
+
+struct IcvTraits : DefaultTraits {
+  static constexpr Mode mode = Mode::Generic;
+  // thread ICV states (48 B each after rounding) come from per-thread slices; slices
+  // that are too small spill to the global pool
+  static constexpr unsigned stack_bytes = 1024 * 24;
+};
+template <class Base>
+struct WithThreadStates : Base {
+  static constexpr bool uses_thread_states = true;
+};
+template <class Base>
+struct WithDebug : Base {
+  static constexpr unsigned debug = dbg::Assert | dbg::Trace;
+};
+
+template <class Tr>
+__global__ void __launch_bounds__(1024) omprt_icv_probe_kernel(int32_t nthreads, int32_t nested,
+                                                               int32_t* rec) {
+  using L = RegionList<IcvOuter>;
+  Team<Tr> team = init<Tr>();
+  if (!is_main(team)) {
+    worker_state_machine<Tr, L>(team);
+    return;
+  }
+  int32_t* team_rec = rec + (int64_t)blockIdx.x * (1 + 3 * nthreads) * 7;
+  icv_record(team, team_rec);
+  parallel<Tr, L, IcvOuter>(team, IcvOuter::Args{team_rec, nthreads, nested}, nthreads);
+  deinit<Tr, L, true>(team);
+}
+
+}  // namespace omprt_kernels
+
+extern "C" int omprt_icv_probe(int32_t teams, int32_t threads, int32_t nested_request,
+                               int32_t* rec, uint32_t flags, void* stream) {
+  using namespace omprt_kernels;
+  Workspace* w;
+  if (int r = current_ws(&w)) return r;
+  OMPRT_CHECK_ARG(teams > 0 && threads > 0 && threads <= 1024 && rec && nested_request > 0,
+                  "omprt_icv_probe: bad arguments");
+  cudaStream_t s = as_stream(stream);
+  const bool ts = flags & OMPRT_THREAD_STATES, dbgb = flags & OMPRT_DEBUG_BUILD,
+             gen = flags & OMPRT_GENERAL_SM;
+#define OMPRT_ICV(...) omprt_icv_probe_kernel<__VA_ARGS__><<<teams, threads, 0, s>>>(threads, nested_request, rec)
+  if (ts && dbgb) OMPRT_ICV(WithDebug<WithThreadStates<IcvTraits>>);
+  else if (ts && gen) OMPRT_ICV(GenSM<WithThreadStates<IcvTraits>, true>);
+  else if (ts) OMPRT_ICV(WithThreadStates<IcvTraits>);
+  else if (dbgb) OMPRT_ICV(WithDebug<IcvTraits>);
+  else if (gen) OMPRT_ICV(GenSM<IcvTraits, true>);
+  else OMPRT_ICV(IcvTraits);
+#undef OMPRT_ICV
+  return check_launch("omprt_icv_probe");
+}

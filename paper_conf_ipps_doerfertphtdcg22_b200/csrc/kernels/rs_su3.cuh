@@ -1,0 +1,270 @@
+// C4 (BASELINE configs[3]): RSBench-shaped lookups, and C5 (configs[4]): SU(3) link
+// multiply (GridMini-shaped), each as an SPMD
+// `target teams distribute parallel for` driven by omprt plus its bare CUDA twin.
+#pragma once
+#include "../host/runtime.cuh"
+#include "rs_body.cuh"
+
+namespace omprt_kernels {
+
+using namespace omprt;
+
+// ---------------------------------------------------------------------------- RSBench
+struct RSTraits : DefaultTraits {};
+struct RSTraitsAssume : DefaultTraits {
+  static constexpr bool assume_teams_oversub = true;
+};
+constexpr int kRSThreads = 128;
+
+template <class Tr, bool Macro>
+__global__ void __launch_bounds__(kRSThreads)
+    omprt_rs_rt(const __grid_constant__ RSTables t, uint64_t seed, int64_t first,
+                typename Tr::Idx count, uint64_t* __restrict__ verification,
+                double* __restrict__ macro) {
+  using Idx = typename Tr::Idx;
+  Team<Tr> team = init<Tr>();
+  distribute_parallel_for(team, count, [&](Idx iv) {
+    verification[iv] = rs_lookup_one<Macro>(t, seed, first + iv, macro + (int64_t)iv * 4);
+  });
+}
+
+template <bool Macro>
+__global__ void __launch_bounds__(kRSThreads)
+    cuda_rs_twin(const __grid_constant__ RSTables t, uint64_t seed, int64_t first, int32_t count,
+                 uint64_t* __restrict__ verification, double* __restrict__ macro) {
+  const int32_t i = blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= count) return;
+  verification[i] = rs_lookup_one<Macro>(t, seed, first + i, macro + (int64_t)i * 4);
+}
+
+OMPRT_REGISTER_KERNEL(omprt_rs_rt, omprt_rs_rt<RSTraits, false>)
+OMPRT_REGISTER_KERNEL(omprt_rs_rt_assume, omprt_rs_rt<RSTraitsAssume, false>)
+OMPRT_REGISTER_KERNEL(cuda_rs_twin, cuda_rs_twin<false>)
+
+inline RSTables to_dev(const omprt_rs_tables& a) {
+  return RSTables{a.poles, a.pole_l, a.windows, a.win_range, a.win_off, a.n_windows, a.k0rs,
+                  a.num_nucs, a.mats, a.concs, a.n_nuclides, a.numL, a.max_num_nucs, 0};
+}
+
+inline int rs_validate(const omprt_rs_tables& t, int64_t count, uint64_t* ver, int32_t& teams,
+                       int32_t threads, uint32_t flags) {
+  OMPRT_CHECK_ARG(count >= 0 && count < (1ll << 31), "count must be in [0, 2^31)");
+  OMPRT_CHECK_ARG(threads == kRSThreads, "threads must be %d", kRSThreads);
+  OMPRT_CHECK_ARG(t.numL == 4, "numL must be 4");
+  OMPRT_CHECK_ARG(t.poles && t.pole_l && t.windows && t.win_range && t.win_off && t.n_windows &&
+                      t.k0rs && t.num_nucs && t.mats && t.concs,
+                  "bad RSBench tables");
+  OMPRT_CHECK_ARG(ver != nullptr || count == 0, "verification is required");
+  if (teams <= 0) teams = (int32_t)std::max<int64_t>(1, ceil_div(count, threads));
+  OMPRT_CHECK_ARG(!(flags & OMPRT_ASSUME_OVERSUB) || count <= (int64_t)teams * threads,
+                  "oversubscription assumption violated");
+  OMPRT_CHECK_ARG(count + 2 * (int64_t)teams * threads < INT32_MAX, "iteration space too large");
+  return OMPRT_OK;
+}
+
+// ---------------------------------------------------------------------------- SU(3)
+// One site: C[l] = A[l] x B[l] for the 4 links; complex MAC = 4 fmas in fixed order
+// (App. A.3), so C is bit-identical to the oracle.  Returns sum of Re C over the site.
+__device__ __forceinline__ double su3_site(const double2* __restrict__ A,
+                                           const double2* __restrict__ B,
+                                           double2* __restrict__ Cs) {
+  double re_sum = 0.0;
+#pragma unroll
+  for (int l = 0; l < 4; ++l) {
+    double2 a[9];
+#pragma unroll
+    for (int e = 0; e < 9; ++e) a[e] = __ldg(A + l * 9 + e);
+#pragma unroll
+    for (int r = 0; r < 3; ++r)
+#pragma unroll
+      for (int c = 0; c < 3; ++c) {
+        double re = 0.0, im = 0.0;
+#pragma unroll
+        for (int m = 0; m < 3; ++m) {
+          const double2 x = a[r * 3 + m];
+          const double2 y = __ldg(B + l * 9 + m * 3 + c);
+          re = fma(x.x, y.x, re);
+          re = fma(-x.y, y.y, re);
+          im = fma(x.x, y.y, im);
+          im = fma(x.y, y.x, im);
+        }
+        __stcs(Cs + l * 9 + r * 3 + c, make_double2(re, im));
+        re_sum += re;
+      }
+  }
+  return re_sum;
+}
+
+struct SU3Traits : DefaultTraits {
+  static constexpr bool assume_teams_oversub = true;  // one site per thread
+};
+struct SU3TraitsLoop : DefaultTraits {};
+constexpr int kSU3Threads = 128;
+
+template <class Tr, bool Checksum>
+__global__ void __launch_bounds__(kSU3Threads)
+    omprt_su3_rt(const double2* __restrict__ A, const double2* __restrict__ B,
+                 double2* __restrict__ Cm, typename Tr::Idx n_sites, double* checksum,
+                 double* partials, unsigned* ticket) {
+  using Idx = typename Tr::Idx;
+  Team<Tr> team = init<Tr>();
+  double acc = 0.0;
+  distribute_parallel_for(team, n_sites, [&](Idx s) {
+    acc += su3_site(A + (int64_t)s * 36, B, Cm + (int64_t)s * 36);
+  });
+  if constexpr (Checksum)
+    league_reduce(team, team_reduce_to_main(team, acc, Plus{}), Plus{}, checksum, partials,
+                  ticket);
+}
+
+template <bool Checksum>
+__global__ void __launch_bounds__(kSU3Threads)
+    cuda_su3_twin(const double2* __restrict__ A, const double2* __restrict__ B,
+                  double2* __restrict__ Cm, int32_t n_sites, double* checksum, double* partials,
+                  unsigned* ticket) {
+  const int32_t s = blockIdx.x * blockDim.x + threadIdx.x;
+  double acc = 0.0;
+  if (s < n_sites) acc = su3_site(A + (int64_t)s * 36, B, Cm + (int64_t)s * 36);
+  if constexpr (Checksum) {
+    __shared__ double ws[32];
+    __shared__ unsigned last;
+    for (int off = 16; off > 0; off >>= 1) acc += __shfl_xor_sync(0xffffffffu, acc, off);
+    const unsigned lane = threadIdx.x & 31u, wid = threadIdx.x >> 5, nw = blockDim.x >> 5;
+    if (lane == 0) ws[wid] = acc;
+    __syncthreads();
+    double b = 0.0;
+    if (wid == 0) {
+      b = lane < nw ? ws[lane] : 0.0;
+      for (int off = 16; off > 0; off >>= 1) b += __shfl_xor_sync(0xffffffffu, b, off);
+    }
+    if (threadIdx.x == 0) {
+      partials[blockIdx.x] = b;
+      __threadfence();
+      last = atomicAdd(ticket, 1u) == gridDim.x - 1;
+    }
+    __syncthreads();
+    if (last) {
+      __threadfence();
+      double t = 0.0;
+      for (unsigned k = threadIdx.x; k < gridDim.x; k += blockDim.x) t += __ldcg(partials + k);
+      for (int off = 16; off > 0; off >>= 1) t += __shfl_xor_sync(0xffffffffu, t, off);
+      if (lane == 0) ws[wid] = t;
+      __syncthreads();
+      if (wid == 0) {
+        double tt = lane < nw ? ws[lane] : 0.0;
+        for (int off = 16; off > 0; off >>= 1) tt += __shfl_xor_sync(0xffffffffu, tt, off);
+        if (threadIdx.x == 0) {
+          *checksum = *checksum + tt;
+          *ticket = 0u;
+        }
+      }
+    }
+  }
+}
+
+OMPRT_REGISTER_KERNEL(omprt_su3_rt, omprt_su3_rt<SU3Traits, true>)
+OMPRT_REGISTER_KERNEL(omprt_su3_rt_loop, omprt_su3_rt<SU3TraitsLoop, true>)
+OMPRT_REGISTER_KERNEL(cuda_su3_twin, cuda_su3_twin<true>)
+
+inline int su3_validate(const double* A, const double* B, double* Cm, int64_t n,
+                        int32_t& teams, int32_t threads, uint32_t flags, double* ck,
+                        Workspace* w) {
+  OMPRT_CHECK_ARG(n >= 0 && n < (1ll << 30), "n_sites out of range");
+  OMPRT_CHECK_ARG(threads == kSU3Threads, "threads must be %d", kSU3Threads);
+  OMPRT_CHECK_ARG(n == 0 || (A && B && Cm), "null data pointer");
+  OMPRT_CHECK_ARG(((uintptr_t)A | (uintptr_t)B | (uintptr_t)Cm) % 16 == 0,
+                  "A, B, C must be 16 B aligned");
+  if (teams <= 0) teams = (int32_t)std::max<int64_t>(1, ceil_div(n, threads));
+  OMPRT_CHECK_ARG(!ck || (uint64_t)teams <= w->opt.max_teams, "teams exceed max_teams");
+  OMPRT_CHECK_ARG(!(flags & OMPRT_ASSUME_OVERSUB) || n <= (int64_t)teams * threads,
+                  "oversubscription assumption violated");
+  return OMPRT_OK;
+}
+
+}  // namespace omprt_kernels
+
+extern "C" int omprt_rs_lookup(omprt_rs_tables t, uint64_t seed, int64_t first, int64_t count,
+                               uint64_t* verification, double* macro, int32_t teams,
+                               int32_t threads, uint32_t flags, void* stream) {
+  using namespace omprt_kernels;
+  Workspace* w;
+  if (int r = current_ws(&w)) return r;
+  if (int r = rs_validate(t, count, verification, teams, threads, flags)) return r;
+  if (count == 0) return OMPRT_OK;
+  cudaStream_t s = as_stream(stream);
+  const RSTables d = to_dev(t);
+  const int32_t n = (int32_t)count;
+  if (flags & OMPRT_ASSUME_OVERSUB) {
+    if (macro) omprt_rs_rt<RSTraitsAssume, true><<<teams, threads, 0, s>>>(d, seed, first, n, verification, macro);
+    else omprt_rs_rt<RSTraitsAssume, false><<<teams, threads, 0, s>>>(d, seed, first, n, verification, nullptr);
+  } else {
+    if (macro) omprt_rs_rt<RSTraits, true><<<teams, threads, 0, s>>>(d, seed, first, n, verification, macro);
+    else omprt_rs_rt<RSTraits, false><<<teams, threads, 0, s>>>(d, seed, first, n, verification, nullptr);
+  }
+  return check_launch("omprt_rs_rt");
+}
+
+extern "C" int omprt_cuda_rs_lookup(omprt_rs_tables t, uint64_t seed, int64_t first,
+                                    int64_t count, uint64_t* verification, double* macro,
+                                    int32_t teams, int32_t threads, uint32_t flags, void* stream) {
+  using namespace omprt_kernels;
+  Workspace* w;
+  if (int r = current_ws(&w)) return r;
+  int32_t tm = 0;
+  if (int r = rs_validate(t, count, verification, tm, threads, 0)) return r;
+  (void)teams;
+  (void)flags;
+  if (count == 0) return OMPRT_OK;
+  cudaStream_t s = as_stream(stream);
+  const RSTables d = to_dev(t);
+  if (macro) cuda_rs_twin<true><<<tm, threads, 0, s>>>(d, seed, first, (int32_t)count, verification, macro);
+  else cuda_rs_twin<false><<<tm, threads, 0, s>>>(d, seed, first, (int32_t)count, verification, nullptr);
+  return check_launch("cuda_rs_twin");
+}
+
+extern "C" int omprt_su3_mult(const double* A, const double* B, double* Cm, int64_t n_sites,
+                              double* checksum_inout, int32_t teams, int32_t threads,
+                              uint32_t flags, void* stream) {
+  using namespace omprt_kernels;
+  Workspace* w;
+  if (int r = current_ws(&w)) return r;
+  if (int r = su3_validate(A, B, Cm, n_sites, teams, threads, flags, checksum_inout, w)) return r;
+  if (n_sites == 0) return OMPRT_OK;
+  cudaStream_t s = as_stream(stream);
+  auto* a = (const double2*)A;
+  auto* b = (const double2*)B;
+  auto* c = (double2*)Cm;
+  double* p = (double*)w->partials;
+  unsigned* tk = w->tickets + 3;
+  const int32_t n = (int32_t)n_sites;
+  if (flags & OMPRT_ASSUME_OVERSUB) {
+    if (checksum_inout) omprt_su3_rt<SU3Traits, true><<<teams, threads, 0, s>>>(a, b, c, n, checksum_inout, p, tk);
+    else omprt_su3_rt<SU3Traits, false><<<teams, threads, 0, s>>>(a, b, c, n, nullptr, p, tk);
+  } else {
+    if (checksum_inout) omprt_su3_rt<SU3TraitsLoop, true><<<teams, threads, 0, s>>>(a, b, c, n, checksum_inout, p, tk);
+    else omprt_su3_rt<SU3TraitsLoop, false><<<teams, threads, 0, s>>>(a, b, c, n, nullptr, p, tk);
+  }
+  return check_launch("omprt_su3_rt");
+}
+
+extern "C" int omprt_cuda_su3_mult(const double* A, const double* B, double* Cm, int64_t n_sites,
+                                   double* checksum_inout, int32_t teams, int32_t threads,
+                                   uint32_t flags, void* stream) {
+  using namespace omprt_kernels;
+  Workspace* w;
+  if (int r = current_ws(&w)) return r;
+  int32_t tm = 0;
+  if (int r = su3_validate(A, B, Cm, n_sites, tm, threads, 0, checksum_inout, w)) return r;
+  (void)teams;
+  (void)flags;
+  if (n_sites == 0) return OMPRT_OK;
+  cudaStream_t s = as_stream(stream);
+  if (checksum_inout)
+    cuda_su3_twin<true><<<tm, threads, 0, s>>>((const double2*)A, (const double2*)B, (double2*)Cm,
+                                               (int32_t)n_sites, checksum_inout,
+                                               (double*)w->partials, w->tickets + 3);
+  else
+    cuda_su3_twin<false><<<tm, threads, 0, s>>>((const double2*)A, (const double2*)B, (double2*)Cm,
+                                                (int32_t)n_sites, nullptr, nullptr, nullptr);
+  return check_launch("cuda_su3_twin");
+}

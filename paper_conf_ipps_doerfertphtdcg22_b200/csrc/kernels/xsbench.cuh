@@ -1,0 +1,281 @@
+// C3 (BASELINE configs[2], the headline): XSBench-shaped lookups as
+//   #pragma omp target teams distribute parallel for
+//   for (i = first; i < first + count; ++i) verification[i - first] = lookup(i);
+// runtime-driven (omprt, with / without the oversubscription assumption) and
+// the bare CUDA twin (XSBench's CUDA version: one lookup per thread).  The verification
+// sum runs as a separate kernel (K11), or fused (OMPRT_FUSED_REDUCTION).
+#pragma once
+#include "../host/runtime.cuh"
+#include "xs_body.cuh"
+
+namespace omprt_kernels {
+
+using namespace omprt;
+
+struct XSTraits : DefaultTraits {};
+struct XSTraitsAssume : DefaultTraits {
+  static constexpr bool assume_teams_oversub = true;
+};
+struct XSTraitsDebug : DefaultTraits {
+  static constexpr unsigned debug = dbg::Assert | dbg::Trace;
+};
+struct XSTraitsAssumeDebug : XSTraitsAssume {
+  static constexpr unsigned debug = dbg::Assert | dbg::Trace;
+};
+
+constexpr int kXSThreads = 256;
+
+template <class Tr, bool Fused>
+__global__ void __launch_bounds__(kXSThreads)
+    omprt_xs_rt(const __grid_constant__ XSTables t, uint64_t seed, int64_t first,
+                typename Tr::Idx count, uint64_t* __restrict__ verification,
+                unsigned long long* checksum, unsigned long long* partials, unsigned* ticket) {
+  using Idx = typename Tr::Idx;
+  Team<Tr> team = init<Tr>();
+  unsigned long long acc = 0;
+  distribute_parallel_for(team, count, [&](Idx iv) {
+    const uint64_t v = xs_lookup_one(t, seed, first + iv);
+    if constexpr (Fused) acc += v;
+    else verification[iv] = v;
+  });
+  if constexpr (Fused)
+    league_reduce(team, team_reduce_to_main(team, acc, Plus{}), Plus{}, checksum, partials,
+                  ticket);
+}
+
+// XSBench's CUDA kernel shape: one lookup per thread, early return past the end.
+template <bool Fused>
+__global__ void __launch_bounds__(kXSThreads)
+    cuda_xs_twin(const __grid_constant__ XSTables t, uint64_t seed, int64_t first, int32_t count,
+                 uint64_t* __restrict__ verification, unsigned long long* checksum,
+                 unsigned long long* partials, unsigned* ticket) {
+  const int32_t i = blockIdx.x * blockDim.x + threadIdx.x;
+  if constexpr (!Fused) {
+    if (i >= count) return;
+    verification[i] = xs_lookup_one(t, seed, first + i);
+  } else {
+    unsigned long long v = i < count ? xs_lookup_one(t, seed, first + i) : 0ull;
+    __shared__ unsigned long long ws[32];
+    __shared__ unsigned last;
+    for (int off = 16; off > 0; off >>= 1) v += __shfl_xor_sync(0xffffffffu, v, off);
+    const unsigned lane = threadIdx.x & 31u, wid = threadIdx.x >> 5, nw = blockDim.x >> 5;
+    if (lane == 0) ws[wid] = v;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+      unsigned long long b = 0;
+      for (unsigned k = 0; k < nw; ++k) b += ws[k];
+      partials[blockIdx.x] = b;
+      __threadfence();
+      last = atomicAdd(ticket, 1u) == gridDim.x - 1;
+    }
+    __syncthreads();
+    if (last) {
+      __threadfence();
+      unsigned long long s = 0;
+      for (unsigned k = threadIdx.x; k < gridDim.x; k += blockDim.x) s += __ldcg(partials + k);
+      for (int off = 16; off > 0; off >>= 1) s += __shfl_xor_sync(0xffffffffu, s, off);
+      __syncthreads();
+      if (lane == 0) ws[wid] = s;
+      __syncthreads();
+      if (threadIdx.x == 0) {
+        unsigned long long b = 0;
+        for (unsigned k = 0; k < nw; ++k) b += ws[k];
+        *checksum += b;
+        *ticket = 0u;
+      }
+    }
+  }
+}
+
+// K11: verification sum, a runtime-driven SPMD reduction over a full-device grid.
+struct SumTraits : DefaultTraits {
+  static constexpr unsigned unroll = 8;
+};
+template <class Tr>
+__global__ void __launch_bounds__(512)
+    omprt_u64_sum_rt(const unsigned long long* __restrict__ v, typename Tr::Idx n,
+                     unsigned long long* out, unsigned long long* partials, unsigned* ticket) {
+  using Idx = typename Tr::Idx;
+  Team<Tr> team = init<Tr>();
+  unsigned long long acc = 0;
+  distribute_parallel_for(team, n, [&](Idx i) { acc += __ldg(v + i); });
+  league_reduce(team, team_reduce_to_main(team, acc, Plus{}), Plus{}, out, partials, ticket);
+}
+
+OMPRT_REGISTER_KERNEL(omprt_xs_rt, omprt_xs_rt<XSTraits, false>)
+OMPRT_REGISTER_KERNEL(omprt_xs_rt_assume, omprt_xs_rt<XSTraitsAssume, false>)
+OMPRT_REGISTER_KERNEL(omprt_xs_rt_fused, omprt_xs_rt<XSTraitsAssume, true>)
+OMPRT_REGISTER_KERNEL(omprt_xs_rt_debug, omprt_xs_rt<XSTraitsDebug, false>)
+OMPRT_REGISTER_KERNEL(cuda_xs_twin, cuda_xs_twin<false>)
+OMPRT_REGISTER_KERNEL(cuda_xs_twin_fused, cuda_xs_twin<true>)
+OMPRT_REGISTER_KERNEL(omprt_u64_sum_rt, omprt_u64_sum_rt<SumTraits>)
+
+inline XSTables to_dev(const omprt_xs_tables& a) {
+  return XSTables{a.nuclide_grid, a.unionized, a.index_grid, a.num_nucs, a.mats, a.concs,
+                  a.n_isotopes, a.n_gridpoints, a.max_num_nucs, 0, a.n_union};
+}
+
+inline int xs_validate(const omprt_xs_tables& t, int64_t count, uint64_t* ver, uint64_t* ck,
+                       int32_t& teams, int32_t threads, uint32_t flags, Workspace* w) {
+  OMPRT_CHECK_ARG(count >= 0 && count < (1ll << 31), "count must be in [0, 2^31)");
+  OMPRT_CHECK_ARG(threads == kXSThreads, "threads must be %d", kXSThreads);
+  OMPRT_CHECK_ARG(t.nuclide_grid && t.unionized && t.index_grid && t.num_nucs && t.mats &&
+                      t.concs && t.n_union >= 2 && t.n_union < (1ll << 31) &&
+                      t.n_gridpoints >= 2 && t.n_isotopes > 0,
+                  "bad XSBench tables");
+  const bool fused = flags & OMPRT_FUSED_REDUCTION;
+  OMPRT_CHECK_ARG(fused ? ck != nullptr : (ver != nullptr || count == 0),
+                  fused ? "fused reduction needs checksum_inout" : "verification is required");
+  if (teams <= 0) teams = (int32_t)std::max<int64_t>(1, ceil_div(count, threads));
+  OMPRT_CHECK_ARG(!fused || (uint64_t)teams <= w->opt.max_teams, "teams exceed max_teams");
+  OMPRT_CHECK_ARG(!(flags & OMPRT_ASSUME_OVERSUB) || count <= (int64_t)teams * threads,
+                  "oversubscription assumption violated: count=%lld > teams*threads=%lld",
+                  (long long)count, (long long)teams * threads);
+  OMPRT_CHECK_ARG(count + 2 * (int64_t)teams * threads < INT32_MAX, "iteration space too large");
+  return OMPRT_OK;
+}
+
+inline int launch_u64_sum(const uint64_t* v, int64_t n, uint64_t* out, Workspace* w,
+                          cudaStream_t s) {
+  OMPRT_CHECK_ARG(n >= 0 && out && (v || n == 0), "omprt_u64_sum: bad arguments");
+  int dev = 0, sms = 148;
+  cudaGetDevice(&dev);
+  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  // a full-device grid: 4 teams of 512 per SM (sized in multiples of the SM count)
+  int64_t teams = std::min<int64_t>((int64_t)sms * 4, std::max<int64_t>(1, ceil_div(n, 512)));
+  if (n + 10 * teams * 512 < INT32_MAX)
+    omprt_u64_sum_rt<SumTraits><<<(int)teams, 512, 0, s>>>(
+        (const unsigned long long*)v, (int32_t)n, (unsigned long long*)out,
+        (unsigned long long*)w->partials, w->tickets + 2);
+  else
+    omprt_u64_sum_rt<WithIdx64<SumTraits>><<<(int)teams, 512, 0, s>>>(
+        (const unsigned long long*)v, n, (unsigned long long*)out,
+        (unsigned long long*)w->partials, w->tickets + 2);
+  return check_launch("omprt_u64_sum_rt");
+}
+
+}  // namespace omprt_kernels
+
+extern "C" int omprt_xs_lookup(omprt_xs_tables t, uint64_t seed, int64_t first, int64_t count,
+                               uint64_t* verification, uint64_t* checksum_inout, int32_t teams,
+                               int32_t threads, uint32_t flags, void* stream) {
+  using namespace omprt_kernels;
+  Workspace* w;
+  if (int r = current_ws(&w)) return r;
+  if (int r = xs_validate(t, count, verification, checksum_inout, teams, threads, flags, w))
+    return r;
+  if (count == 0) return OMPRT_OK;
+  cudaStream_t s = as_stream(stream);
+  const XSTables d = to_dev(t);
+  const bool assume = flags & OMPRT_ASSUME_OVERSUB, fused = flags & OMPRT_FUSED_REDUCTION,
+             debug = flags & OMPRT_DEBUG_BUILD;
+  auto* ck = (unsigned long long*)checksum_inout;
+  auto* p = (unsigned long long*)w->partials;
+  unsigned* tk = w->tickets + 1;
+  const int32_t n = (int32_t)count;
+#define OMPRT_XS(TR, F) \
+  omprt_xs_rt<TR, F><<<teams, threads, 0, s>>>(d, seed, first, n, verification, ck, p, tk)
+  if (fused) {
+    if (assume) OMPRT_XS(XSTraitsAssume, true);
+    else OMPRT_XS(XSTraits, true);
+  } else if (debug) {
+    if (assume) OMPRT_XS(XSTraitsAssumeDebug, false);
+    else OMPRT_XS(XSTraitsDebug, false);
+  } else {
+    if (assume) OMPRT_XS(XSTraitsAssume, false);
+    else OMPRT_XS(XSTraits, false);
+  }
+#undef OMPRT_XS
+  return check_launch("omprt_xs_rt");
+}
+
+extern "C" int omprt_cuda_xs_lookup(omprt_xs_tables t, uint64_t seed, int64_t first,
+                                    int64_t count, uint64_t* verification,
+                                    uint64_t* checksum_inout, int32_t teams, int32_t threads,
+                                    uint32_t flags, void* stream) {
+  using namespace omprt_kernels;
+  Workspace* w;
+  if (int r = current_ws(&w)) return r;
+  int32_t tm = 0;  // the twin always runs one lookup per thread
+  if (int r = xs_validate(t, count, verification, checksum_inout, tm, threads,
+                          flags & ~OMPRT_ASSUME_OVERSUB, w))
+    return r;
+  (void)teams;
+  if (count == 0) return OMPRT_OK;
+  cudaStream_t s = as_stream(stream);
+  const XSTables d = to_dev(t);
+  if (flags & OMPRT_FUSED_REDUCTION)
+    cuda_xs_twin<true><<<tm, threads, 0, s>>>(d, seed, first, (int32_t)count, verification,
+                                              (unsigned long long*)checksum_inout,
+                                              (unsigned long long*)w->partials, w->tickets + 1);
+  else
+    cuda_xs_twin<false><<<tm, threads, 0, s>>>(d, seed, first, (int32_t)count, verification,
+                                               nullptr, nullptr, nullptr);
+  return check_launch("cuda_xs_twin");
+}
+
+extern "C" int omprt_u64_sum(const uint64_t* v, int64_t n, uint64_t* out_inout, void* stream) {
+  using namespace omprt_kernels;
+  Workspace* w;
+  if (int r = current_ws(&w)) return r;
+  return launch_u64_sum(v, n, out_inout, w, as_stream(stream));
+}
+
+// End to end with host tables: map(to: tables) -> lookups (fused reduction) ->
+// map(from: checksum).  Synchronous on `stream`.
+extern "C" int omprt_xs_run_host(omprt_xs_tables h, uint64_t seed, int64_t first, int64_t count,
+                                 int32_t threads, uint32_t flags, uint64_t* checksum_host,
+                                 uint64_t* h2d_bytes, uint64_t* d2h_bytes, void* stream) {
+  using namespace omprt_kernels;
+  Workspace* w;
+  if (int r = current_ws(&w)) return r;
+  OMPRT_CHECK_ARG(checksum_host && h.nuclide_grid && h.unionized && h.index_grid && h.num_nucs &&
+                      h.mats && h.concs,
+                  "omprt_xs_run_host: bad arguments");
+  cudaStream_t s = as_stream(stream);
+  const size_t n_grid = (size_t)h.n_isotopes * h.n_gridpoints * 6 * sizeof(double);
+  const size_t n_uni = (size_t)h.n_union * sizeof(double);
+  const size_t n_idx = (size_t)h.n_union * h.n_isotopes * sizeof(int32_t);
+  const size_t n_num = 12 * sizeof(int32_t);
+  const size_t n_mat = (size_t)12 * h.max_num_nucs * sizeof(int32_t);
+  const size_t n_con = (size_t)12 * h.max_num_nucs * sizeof(double);
+  auto al = [](size_t b) { return (b + 255) & ~size_t(255); };
+  const size_t total = al(n_grid) + al(n_uni) + al(n_idx) + al(n_num) + al(n_mat) + al(n_con);
+  if (w->xs_buf_bytes < total) {
+    cudaFree(w->xs_buf);
+    w->xs_buf = nullptr;
+    w->xs_buf_bytes = 0;
+    if (cudaMalloc(&w->xs_buf, total) != cudaSuccess) {
+      cudaGetLastError();
+      return set_error(OMPRT_E_NOMEM, "omprt_xs_run_host: cannot allocate %zu B", total);
+    }
+    w->xs_buf_bytes = total;
+  }
+  unsigned char* b = (unsigned char*)w->xs_buf;
+  omprt_xs_tables d = h;
+  size_t off = 0;
+  auto put = [&](const void* src, size_t bytes) -> const void* {
+    void* dst = b + off;
+    off += al(bytes);
+    return cudaMemcpyAsync(dst, src, bytes, cudaMemcpyHostToDevice, s) == cudaSuccess ? dst
+                                                                                      : nullptr;
+  };
+  d.nuclide_grid = (const double*)put(h.nuclide_grid, n_grid);
+  d.unionized = (const double*)put(h.unionized, n_uni);
+  d.index_grid = (const int32_t*)put(h.index_grid, n_idx);
+  d.num_nucs = (const int32_t*)put(h.num_nucs, n_num);
+  d.mats = (const int32_t*)put(h.mats, n_mat);
+  d.concs = (const double*)put(h.concs, n_con);
+  if (!d.nuclide_grid || !d.unionized || !d.index_grid || !d.num_nucs || !d.mats || !d.concs)
+    return set_error(OMPRT_E_CUDA, "omprt_xs_run_host: H2D copy failed");
+  uint64_t* ck = w->scratch_u64;
+  OMPRT_CUDA_TRY(cudaMemsetAsync(ck, 0, sizeof(uint64_t), s));
+  if (int r = omprt_xs_lookup(d, seed, first, count, nullptr, ck, 0, threads,
+                              (flags | OMPRT_FUSED_REDUCTION | OMPRT_ASSUME_OVERSUB), stream))
+    return r;
+  OMPRT_CUDA_TRY(cudaMemcpyAsync(checksum_host, ck, sizeof(uint64_t), cudaMemcpyDeviceToHost, s));
+  OMPRT_CUDA_TRY(cudaStreamSynchronize(s));
+  if (h2d_bytes) *h2d_bytes = n_grid + n_uni + n_idx + n_num + n_mat + n_con;
+  if (d2h_bytes) *d2h_bytes = sizeof(uint64_t);
+  return OMPRT_OK;
+}

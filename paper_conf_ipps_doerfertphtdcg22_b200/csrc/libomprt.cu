@@ -1,0 +1,9 @@
+// libomprt.so: the whole library is one translation unit, so the header-only device
+// runtime is compiled (and optimized) together with every kernel that uses it, and
+// the per-device environment has a single __constant__ definition.
+#include "host/runtime.cuh"
+#include "host/api.cuh"
+#include "kernels/axpy.cuh"
+#include "kernels/generic.cuh"
+#include "kernels/xsbench.cuh"
+#include "kernels/rs_su3.cuh"

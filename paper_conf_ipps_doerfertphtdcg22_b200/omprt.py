@@ -1,0 +1,318 @@
+"""Thin ctypes binding of libomprt.so (include/omprt.h): argument marshalling only.
+
+Every function has the C name and the C argument order; device buffers are torch CUDA
+tensors (PyTorch supplies memory, streams and process groups -- nothing else), host buffers
+for `_host` calls are numpy arrays.  A nonzero status raises OmprtError.  There is no CPU
+fallback: without the built library (or on a machine without a GPU) every call fails.
+"""
+from __future__ import annotations
+
+import ctypes as C
+import os
+
+HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(HERE, "libomprt.so")
+
+OMPRT_OK = 0
+OMPRT_E_INVAL = -1
+OMPRT_E_CUDA = -2
+OMPRT_E_NOMEM = -3
+OMPRT_E_STACK = -4
+OMPRT_E_ASSERT = -5
+OMPRT_E_NOTINIT = -6
+
+OMPRT_ASSUME_OVERSUB = 1 << 0
+OMPRT_RECORD_OWNER = 1 << 1
+OMPRT_GENERAL_SM = 1 << 2
+OMPRT_SMALL_STACK = 1 << 3
+OMPRT_NO_STACK = 1 << 4
+OMPRT_DEBUG_BUILD = 1 << 5
+OMPRT_POSTLOGUE = 1 << 6
+OMPRT_THREAD_STATES = 1 << 7
+OMPRT_FUSED_REDUCTION = 1 << 8
+OMPRT_UNCHECKED = 1 << 9
+
+# Every symbol include/omprt.h declares (checked by tests/test_abi.py).
+EXPORTS = [
+    "omprt_init", "omprt_fini", "omprt_device_status", "omprt_last_error", "omprt_static_owner",
+    "omprt_spmd_axpy_sum", "omprt_cuda_axpy_sum", "omprt_generic_team", "omprt_cuda_generic_team",
+    "omprt_icv_probe", "omprt_xs_lookup", "omprt_cuda_xs_lookup", "omprt_u64_sum",
+    "omprt_xs_run_host", "omprt_rs_lookup", "omprt_cuda_rs_lookup", "omprt_su3_mult",
+    "omprt_cuda_su3_mult", "omprt_kernel_count", "omprt_kernel_name", "omprt_kernel_attrs",
+]
+
+
+class OmprtError(RuntimeError):
+    def __init__(self, code, msg):
+        super().__init__(f"omprt error {code}: {msg}")
+        self.code = code
+
+
+class Options(C.Structure):
+    _fields_ = [("pool_bytes_per_team", C.c_uint64), ("pool_teams", C.c_uint64),
+                ("max_teams", C.c_uint64)]
+
+
+class XSTablesC(C.Structure):
+    _fields_ = [("nuclide_grid", C.c_void_p), ("unionized", C.c_void_p), ("index_grid", C.c_void_p),
+                ("num_nucs", C.c_void_p), ("mats", C.c_void_p), ("concs", C.c_void_p),
+                ("n_isotopes", C.c_int32), ("n_gridpoints", C.c_int32),
+                ("max_num_nucs", C.c_int32), ("pad", C.c_int32), ("n_union", C.c_int64)]
+
+
+class RSTablesC(C.Structure):
+    _fields_ = [("poles", C.c_void_p), ("pole_l", C.c_void_p), ("windows", C.c_void_p),
+                ("win_range", C.c_void_p), ("win_off", C.c_void_p), ("n_windows", C.c_void_p),
+                ("k0rs", C.c_void_p), ("num_nucs", C.c_void_p), ("mats", C.c_void_p),
+                ("concs", C.c_void_p), ("n_nuclides", C.c_int32), ("numL", C.c_int32),
+                ("max_num_nucs", C.c_int32), ("pad", C.c_int32)]
+
+
+_lib = None
+_vp, _i32, _i64, _u32, _u64, _f64 = C.c_void_p, C.c_int32, C.c_int64, C.c_uint32, C.c_uint64, C.c_double
+_SIGS = {
+    "omprt_init": [C.c_int, C.POINTER(Options)],
+    "omprt_fini": [C.c_int],
+    "omprt_device_status": [C.c_int, C.POINTER(C.c_int), C.POINTER(C.c_int)],
+    "omprt_last_error": [C.c_char_p, C.c_size_t],
+    "omprt_static_owner": [_i64, _i64, _i32, _i32, C.POINTER(_i32), C.POINTER(_i32)],
+    "omprt_spmd_axpy_sum": [_i64, _f64, _vp, _vp, _vp, _vp, _i32, _i32, _u32, _vp, _vp, _vp],
+    "omprt_cuda_axpy_sum": [_i64, _f64, _vp, _vp, _vp, _vp, _i32, _i32, _u32, _vp, _vp, _vp],
+    "omprt_generic_team": [_i32, _i32, _i32, _vp, _vp, _vp, _vp, _u32, _vp],
+    "omprt_cuda_generic_team": [_i32, _i32, _i32, _vp, _vp, _vp, _vp, _u32, _vp],
+    "omprt_icv_probe": [_i32, _i32, _i32, _vp, _u32, _vp],
+    "omprt_xs_lookup": [XSTablesC, _u64, _i64, _i64, _vp, _vp, _i32, _i32, _u32, _vp],
+    "omprt_cuda_xs_lookup": [XSTablesC, _u64, _i64, _i64, _vp, _vp, _i32, _i32, _u32, _vp],
+    "omprt_u64_sum": [_vp, _i64, _vp, _vp],
+    "omprt_xs_run_host": [XSTablesC, _u64, _i64, _i64, _i32, _u32, C.POINTER(_u64),
+                          C.POINTER(_u64), C.POINTER(_u64), _vp],
+    "omprt_rs_lookup": [RSTablesC, _u64, _i64, _i64, _vp, _vp, _i32, _i32, _u32, _vp],
+    "omprt_cuda_rs_lookup": [RSTablesC, _u64, _i64, _i64, _vp, _vp, _i32, _i32, _u32, _vp],
+    "omprt_su3_mult": [_vp, _vp, _vp, _i64, _vp, _i32, _i32, _u32, _vp],
+    "omprt_cuda_su3_mult": [_vp, _vp, _vp, _i64, _vp, _i32, _i32, _u32, _vp],
+    "omprt_kernel_count": [],
+    "omprt_kernel_name": [C.c_int],
+    "omprt_kernel_attrs": [C.c_int, C.POINTER(C.c_int), C.POINTER(C.c_int), C.POINTER(C.c_int),
+                           C.POINTER(C.c_int)],
+}
+
+
+def load(path: str = LIB_PATH):
+    """Load libomprt.so (raises if it was not built -- there is no fallback)."""
+    global _lib
+    if _lib is None:
+        if not os.path.exists(path):
+            raise OSError(f"{path} is missing: run __graft_entry__.build() (no CPU fallback)")
+        lib = C.CDLL(path)
+        for name, args in _SIGS.items():
+            f = getattr(lib, name)
+            f.argtypes = args
+            f.restype = C.c_char_p if name == "omprt_kernel_name" else C.c_int
+        _lib = lib
+    return _lib
+
+
+def last_error() -> str:
+    buf = C.create_string_buffer(512)
+    load().omprt_last_error(buf, 512)
+    return buf.value.decode(errors="replace")
+
+
+def _check(code):
+    if code != OMPRT_OK:
+        raise OmprtError(code, last_error())
+    return code
+
+
+def _p(t):
+    """Device pointer of a torch CUDA tensor (None -> NULL)."""
+    if t is None:
+        return None
+    if not t.is_cuda:
+        raise ValueError("expected a CUDA tensor")
+    if not t.is_contiguous():
+        raise ValueError("expected a contiguous tensor")
+    return t.data_ptr()
+
+
+def _hp(a):
+    """Host pointer of a numpy array or pinned torch CPU tensor."""
+    if a is None:
+        return None
+    if hasattr(a, "ctypes"):
+        return a.ctypes.data
+    return a.data_ptr()
+
+
+def _stream(stream):
+    if stream is None:
+        import torch
+        return torch.cuda.current_stream().cuda_stream
+    return stream if isinstance(stream, int) else stream.cuda_stream
+
+
+# ---------------------------------------------------------------- lifecycle / status
+def omprt_init(device=0, pool_bytes_per_team=0, pool_teams=0, max_teams=0):
+    o = Options(pool_bytes_per_team, pool_teams, max_teams)
+    return _check(load().omprt_init(device, C.byref(o)))
+
+
+def omprt_fini(device=0):
+    return _check(load().omprt_fini(device))
+
+
+def omprt_device_status(device=0):
+    code, info = C.c_int(), (C.c_int * 4)()
+    _check(load().omprt_device_status(device, C.byref(code), info))
+    return code.value, list(info)
+
+
+def omprt_static_owner(iv, n, teams, threads):
+    tm, th = _i32(), _i32()
+    _check(load().omprt_static_owner(iv, n, teams, threads, C.byref(tm), C.byref(th)))
+    return tm.value, th.value
+
+
+# ---------------------------------------------------------------- C1
+def omprt_spmd_axpy_sum(n, x, b, c, a, sum_inout, teams, threads, flags=0, owner=None,
+                        count=None, stream=None):
+    return _check(load().omprt_spmd_axpy_sum(n, x, _p(b), _p(c), _p(a), _p(sum_inout), teams,
+                                             threads, flags, _p(owner), _p(count), _stream(stream)))
+
+
+def omprt_cuda_axpy_sum(n, x, b, c, a, sum_inout, teams, threads, flags=0, owner=None,
+                        count=None, stream=None):
+    return _check(load().omprt_cuda_axpy_sum(n, x, _p(b), _p(c), _p(a), _p(sum_inout), teams,
+                                             threads, flags, _p(owner), _p(count), _stream(stream)))
+
+
+# ---------------------------------------------------------------- C2
+def omprt_generic_team(teams, threads, inner_n, inp, out, owner=None, postlogue=None, flags=0,
+                       stream=None):
+    return _check(load().omprt_generic_team(teams, threads, inner_n, _p(inp), _p(out), _p(owner),
+                                            _p(postlogue), flags, _stream(stream)))
+
+
+def omprt_cuda_generic_team(teams, threads, inner_n, inp, out, owner=None, postlogue=None,
+                            flags=0, stream=None):
+    return _check(load().omprt_cuda_generic_team(teams, threads, inner_n, _p(inp), _p(out),
+                                                 _p(owner), _p(postlogue), flags,
+                                                 _stream(stream)))
+
+
+def omprt_icv_probe(teams, threads, nested_request, rec, flags=0, stream=None):
+    return _check(load().omprt_icv_probe(teams, threads, nested_request, _p(rec), flags,
+                                         _stream(stream)))
+
+
+# ---------------------------------------------------------------- C3
+class XSDeviceTables:
+    """Device copies (torch tensors) of gen.XSTables and the by-value C struct."""
+
+    def __init__(self, t, device="cuda"):
+        import torch
+        self.host = t
+        self.nuclide_grid = torch.from_numpy(t.nuclide_grid).to(device)
+        self.unionized = torch.from_numpy(t.unionized).to(device)
+        self.index_grid = torch.from_numpy(t.index_grid).to(device)
+        self.num_nucs = torch.from_numpy(t.num_nucs).to(device)
+        self.mats = torch.from_numpy(t.mats).to(device)
+        self.concs = torch.from_numpy(t.concs).to(device)
+        self.c = XSTablesC(_p(self.nuclide_grid), _p(self.unionized), _p(self.index_grid),
+                           _p(self.num_nucs), _p(self.mats), _p(self.concs), t.n_isotopes,
+                           t.n_gridpoints, t.max_num_nucs, 0, t.n_union)
+
+
+def xs_host_struct(t, pinned=None):
+    """By-value struct of HOST table pointers (numpy or pinned torch tensors)."""
+    src = pinned or {}
+    g = lambda k: src.get(k, getattr(t, k))
+    return XSTablesC(_hp(g("nuclide_grid")), _hp(g("unionized")), _hp(g("index_grid")),
+                     _hp(g("num_nucs")), _hp(g("mats")), _hp(g("concs")), t.n_isotopes,
+                     t.n_gridpoints, t.max_num_nucs, 0, t.n_union)
+
+
+def omprt_xs_lookup(tables, seed, first, count, verification, checksum_inout=None, teams=0,
+                    threads=256, flags=0, stream=None):
+    return _check(load().omprt_xs_lookup(tables.c, seed, first, count, _p(verification),
+                                         _p(checksum_inout), teams, threads, flags,
+                                         _stream(stream)))
+
+
+def omprt_cuda_xs_lookup(tables, seed, first, count, verification, checksum_inout=None, teams=0,
+                         threads=256, flags=0, stream=None):
+    return _check(load().omprt_cuda_xs_lookup(tables.c, seed, first, count, _p(verification),
+                                              _p(checksum_inout), teams, threads, flags,
+                                              _stream(stream)))
+
+
+def omprt_u64_sum(v, n, out_inout, stream=None):
+    return _check(load().omprt_u64_sum(_p(v), n, _p(out_inout), _stream(stream)))
+
+
+def omprt_xs_run_host(host_struct, seed, first, count, threads=256, flags=0, stream=None):
+    ck, hb, db = _u64(), _u64(), _u64()
+    _check(load().omprt_xs_run_host(host_struct, seed, first, count, threads, flags,
+                                    C.byref(ck), C.byref(hb), C.byref(db), _stream(stream)))
+    return ck.value, hb.value, db.value
+
+
+# ---------------------------------------------------------------- C4
+class RSDeviceTables:
+    def __init__(self, t, device="cuda"):
+        import torch
+        self.host = t
+        keep = {}
+        for k in ("poles", "pole_l", "windows", "win_range", "win_off", "n_windows", "k0rs",
+                  "num_nucs", "mats", "concs"):
+            keep[k] = torch.from_numpy(getattr(t, k)).to(device)
+            setattr(self, k, keep[k])
+        self.c = RSTablesC(*[_p(keep[k]) for k in ("poles", "pole_l", "windows", "win_range",
+                                                   "win_off", "n_windows", "k0rs", "num_nucs",
+                                                   "mats", "concs")],
+                           t.n_nuclides, t.numL, t.max_num_nucs, 0)
+
+
+def omprt_rs_lookup(tables, seed, first, count, verification, macro=None, teams=0, threads=128,
+                    flags=0, stream=None):
+    return _check(load().omprt_rs_lookup(tables.c, seed, first, count, _p(verification),
+                                         _p(macro), teams, threads, flags, _stream(stream)))
+
+
+def omprt_cuda_rs_lookup(tables, seed, first, count, verification, macro=None, teams=0,
+                         threads=128, flags=0, stream=None):
+    return _check(load().omprt_cuda_rs_lookup(tables.c, seed, first, count, _p(verification),
+                                              _p(macro), teams, threads, flags, _stream(stream)))
+
+
+# ---------------------------------------------------------------- C5
+def omprt_su3_mult(A, B, Cout, n_sites, checksum_inout=None, teams=0, threads=128, flags=0,
+                   stream=None):
+    return _check(load().omprt_su3_mult(_p(A), _p(B), _p(Cout), n_sites, _p(checksum_inout), teams,
+                                        threads, flags, _stream(stream)))
+
+
+def omprt_cuda_su3_mult(A, B, Cout, n_sites, checksum_inout=None, teams=0, threads=128, flags=0,
+                        stream=None):
+    return _check(load().omprt_cuda_su3_mult(_p(A), _p(B), _p(Cout), n_sites, _p(checksum_inout),
+                                             teams, threads, flags, _stream(stream)))
+
+
+# ---------------------------------------------------------------- introspection
+def omprt_kernel_count():
+    return load().omprt_kernel_count()
+
+
+def omprt_kernel_name(i):
+    r = load().omprt_kernel_name(i)
+    return r.decode() if r else None
+
+
+def omprt_kernel_attrs(i):
+    r, s, l, m = C.c_int(), C.c_int(), C.c_int(), C.c_int()
+    _check(load().omprt_kernel_attrs(i, C.byref(r), C.byref(s), C.byref(l), C.byref(m)))
+    return dict(regs=r.value, static_smem=s.value, local_bytes=l.value, max_threads=m.value)
+
+
+def kernel_table():
+    return {omprt_kernel_name(i): omprt_kernel_attrs(i) for i in range(omprt_kernel_count())}

@@ -30,3 +30,16 @@ def rs_tables_small():
     """A reduced RSBench shape (fewer nuclides/poles) for fast parity runs."""
     import gen
     return gen.RSTables(n_nuclides=355, avg_poles=100, avg_windows=10)
+
+
+@pytest.fixture(scope="session")
+def rt():
+    """The CUDA library, initialized on cuda:0 (GPU tests only; no fallback)."""
+    import torch
+    from paper_conf_ipps_doerfertphtdcg22_b200 import build, omprt
+    if not torch.cuda.is_available():
+        pytest.fail("GPU test run without a GPU")
+    build.build()
+    torch.cuda.set_device(0)
+    omprt.omprt_init(0)
+    return omprt

@@ -1,0 +1,28 @@
+"""Resource parity with the bare CUDA twins (the paper's Fig. 11 "# Regs" / "SMem" columns,
+P:290-470; north_star target: registers within 5% of the twin, no local memory, and 0 B of
+runtime shared memory on SPMD kernels)."""
+import pytest
+
+pytestmark = pytest.mark.gpu
+
+PAIRS = [
+    ("omprt_axpy_rt", "cuda_axpy_twin", True),
+    ("omprt_axpy_rt_assume", "cuda_axpy_twin", True),
+    ("omprt_xs_rt_assume", "cuda_xs_twin", True),
+    ("omprt_xs_rt", "cuda_xs_twin", True),
+    ("omprt_xs_rt_fused", "cuda_xs_twin_fused", True),
+    ("omprt_rs_rt_assume", "cuda_rs_twin", True),
+    ("omprt_rs_rt", "cuda_rs_twin", True),
+    ("omprt_su3_rt", "cuda_su3_twin", True),
+    ("omprt_generic_rt", "cuda_generic_twin", False),
+]
+
+
+@pytest.mark.parametrize("rtk,twin,spmd", PAIRS)
+def test_registers_and_smem_vs_twin(rt, rtk, twin, spmd):
+    tab = rt.kernel_table()
+    a, b = tab[rtk], tab[twin]
+    assert a["regs"] <= int(1.05 * b["regs"]) or a["regs"] <= b["regs"] + 1, (a, b)
+    assert a["local_bytes"] <= b["local_bytes"], (a, b)
+    if spmd:
+        assert a["static_smem"] == b["static_smem"], (a, b)  # 0 B of runtime state

@@ -1,0 +1,84 @@
+"""GPU parity: RSBench-shaped lookups (tolerance contract) and SU(3)
+(bit-exact, §8(c) C6)."""
+import os
+
+import numpy as np
+import pytest
+import torch
+
+import gen
+import oracle
+
+pytestmark = pytest.mark.gpu
+DEV = "cuda:0"
+
+
+@pytest.fixture(scope="module")
+def rs_dev(rt, rs_tables):
+    return rt.RSDeviceTables(rs_tables, DEV)
+
+
+def _rs(rt, d, first, count, which, flags=0):
+    ver = torch.zeros(max(count, 1), dtype=torch.uint64, device=DEV)
+    mac = torch.zeros(max(count, 1) * 4, dtype=torch.float64, device=DEV)
+    fn = rt.omprt_rs_lookup if which == "rt" else rt.omprt_cuda_rs_lookup
+    fn(d, gen.RS_LOOKUP_SEED, first, count, ver, mac, 0, 128, flags)
+    torch.cuda.synchronize()
+    return ver.cpu().numpy()[:count], mac.cpu().numpy()[: 4 * count].reshape(count, 4)
+
+
+@pytest.mark.parametrize("variant", ["rt", "rt_assume", "twin"])
+def test_rs_parity(rt, rs_dev, rs_tables, variant):
+    first, count = 4321, 20_000 + 17
+    flags = rt.OMPRT_ASSUME_OVERSUB if variant == "rt_assume" else 0
+    ver, mac = _rs(rt, rs_dev, first, count, "twin" if variant == "twin" else "rt", flags)
+    rv, rm = oracle.rs_lookup(rs_tables, first, count, want_macro=True,
+                              threads=os.cpu_count() or 1)
+    # macro xs normwise (sigma_E = sigma_T - sigma_A can cancel): 1e-10
+    err = np.abs(mac - rm).max(axis=1) / np.abs(rm).max(axis=1)
+    assert err.max() <= 1e-10, err.max()
+    # verification: identical, except flips that are near-ties in the oracle
+    flip = np.nonzero(ver != rv)[0]
+    for q in flip:
+        top2 = np.sort(rm[q])[-2:]
+        assert top2[1] - top2[0] <= 1e-12 * abs(top2[1]), (q, rm[q], mac[q])
+    assert flip.size <= 2
+
+
+def test_rs_checksum_and_rt_twin_agree(rt, rs_dev):
+    n = 100_000
+    v1, m1 = _rs(rt, rs_dev, 0, n, "rt", rt.OMPRT_ASSUME_OVERSUB)
+    v2, m2 = _rs(rt, rs_dev, 0, n, "twin")
+    assert (v1 == v2).all() and (m1 == m2).all()  # same body, same compiler -> same bits
+
+
+def _su3(rt, fn, A, B, n, flags=0):
+    At, Bt = torch.from_numpy(A).to(DEV), torch.from_numpy(B).to(DEV)
+    Ct = torch.full((n * 72,), float("nan"), dtype=torch.float64, device=DEV)
+    ck = torch.full((1,), 0.5, dtype=torch.float64, device=DEV)
+    fn(At, Bt, Ct, n, ck, 0, 128, flags)
+    torch.cuda.synchronize()
+    return Ct.cpu().numpy(), float(ck.item()) - 0.5
+
+
+@pytest.mark.parametrize("n", [8 ** 4, 8 ** 4 + 5, 32 ** 4])
+@pytest.mark.parametrize("variant", ["rt", "rt_loop", "twin"])
+def test_su3_bit_exact(rt, n, variant):
+    A, B = gen.su3_inputs(n)
+    fn = rt.omprt_cuda_su3_mult if variant == "twin" else rt.omprt_su3_mult
+    flags = rt.OMPRT_ASSUME_OVERSUB if variant == "rt" else 0
+    C, ck = _su3(rt, fn, A, B, n, flags)
+    Cref = oracle.su3_mult(A, B, n, threads=os.cpu_count() or 1)
+    assert (C == Cref).all()
+    re = Cref[0::2]
+    assert abs(ck - oracle.sum_f64(re)) <= 1e-12 * oracle.sum_abs_f64(re)
+
+
+def test_su3_pins_on_gpu(rt):
+    n = 4096
+    A, B = gen.su3_inputs(n, "identity")
+    C, _ = _su3(rt, rt.omprt_su3_mult, A, B, n, rt.OMPRT_ASSUME_OVERSUB)
+    assert (C == A).all()
+    A, B = gen.su3_inputs(n, "third")
+    C, ck = _su3(rt, rt.omprt_su3_mult, A, B, n, rt.OMPRT_ASSUME_OVERSUB)
+    assert (C.reshape(n, 4, 3, 3, 2)[..., 0] == 1.0).all() and ck == 36.0 * n

@@ -1,0 +1,114 @@
+"""GPU parity: XSBench-shaped lookups -- verification per lookup
+bit-exact against the oracle, the u64 checksum exact, sharding-invariant, at a reduced size
+spanning many teams and a ragged tail, and at the full 17M size on sampled lookups plus the
+full checksum (oracle run over all host cores)."""
+import os
+
+import numpy as np
+import pytest
+import torch
+
+import gen
+import oracle
+
+pytestmark = pytest.mark.gpu
+DEV = "cuda:0"
+SEED = gen.XS_LOOKUP_SEED
+
+
+@pytest.fixture(scope="module")
+def xs_dev(rt, xs_small):
+    return rt.XSDeviceTables(xs_small, DEV)
+
+
+def _lookup(rt, d, first, count, which, flags=0):
+    ver = torch.zeros(max(count, 1), dtype=torch.uint64, device=DEV)
+    fn = rt.omprt_xs_lookup if which == "rt" else rt.omprt_cuda_xs_lookup
+    fn(d, SEED, first, count, ver, None, 0, 256, flags)
+    torch.cuda.synchronize()
+    return ver.cpu().numpy()[:count]
+
+
+@pytest.mark.parametrize("variant", ["rt", "rt_assume", "twin", "rt_debug"])
+def test_verification_bit_exact(rt, xs_dev, xs_small, variant):
+    first, count = 777, (1 << 17) + 13  # many teams and a ragged last team
+    flags = {"rt": 0, "rt_assume": rt.OMPRT_ASSUME_OVERSUB, "twin": 0,
+             "rt_debug": rt.OMPRT_DEBUG_BUILD}[variant]
+    got = _lookup(rt, xs_dev, first, count, "twin" if variant == "twin" else "rt", flags)
+    ref = oracle.xs_lookup(xs_small, first, count, threads=os.cpu_count() or 1)
+    assert (got == ref).all()
+
+
+def test_edge_sizes(rt, xs_dev, xs_small):
+    for first, count in [(0, 0), (0, 1), (5, 255), (5, 256), (5, 257)]:
+        got = _lookup(rt, xs_dev, first, count, "rt", rt.OMPRT_ASSUME_OVERSUB)
+        assert (got == oracle.xs_lookup(xs_small, first, count)).all()
+
+
+def test_checksum_separate_and_fused(rt, xs_dev, xs_small):
+    n = 1 << 20
+    ref = oracle.xs_lookup(xs_small, 0, n, threads=os.cpu_count() or 1)
+    ref_sum = int(ref.sum())
+    ver = torch.zeros(n, dtype=torch.uint64, device=DEV)
+    rt.omprt_xs_lookup(xs_dev, SEED, 0, n, ver, None, 0, 256, rt.OMPRT_ASSUME_OVERSUB)
+    ck = torch.full((1,), 5, dtype=torch.uint64, device=DEV)  # orig value is kept (OpenMP)
+    rt.omprt_u64_sum(ver, n, ck)
+    torch.cuda.synchronize()
+    assert int(ck.cpu().numpy()[0]) == ref_sum + 5
+    for fn, flags in [(rt.omprt_xs_lookup, rt.OMPRT_ASSUME_OVERSUB | rt.OMPRT_FUSED_REDUCTION),
+                      (rt.omprt_xs_lookup, rt.OMPRT_FUSED_REDUCTION),
+                      (rt.omprt_cuda_xs_lookup, rt.OMPRT_FUSED_REDUCTION)]:
+        ck = torch.zeros(1, dtype=torch.uint64, device=DEV)
+        fn(xs_dev, SEED, 0, n, None, ck, 0, 256, flags)
+        torch.cuda.synchronize()
+        assert int(ck.cpu().numpy()[0]) == ref_sum
+
+
+def test_virtual_shards_match_one_launch(rt, xs_dev):
+    """G shards [r*L/G, (r+1)*L/G) give the same verification and checksum."""
+    L, G = 300_007, 8
+    full = _lookup(rt, xs_dev, 0, L, "rt", rt.OMPRT_ASSUME_OVERSUB)
+    parts = [
+        _lookup(rt, xs_dev, r * L // G, (r + 1) * L // G - r * L // G, "rt",
+                rt.OMPRT_ASSUME_OVERSUB) for r in range(G)
+    ]
+    assert (np.concatenate(parts) == full).all()
+
+
+def test_u64_sum_wraps(rt):
+    v = np.full(1 << 20, (1 << 63) + 12345, dtype=np.uint64)
+    t = torch.from_numpy(v).to(DEV)
+    out = torch.zeros(1, dtype=torch.uint64, device=DEV)
+    rt.omprt_u64_sum(t, v.size, out)
+    torch.cuda.synchronize()
+    assert int(out.cpu().numpy()[0]) == (int(v.size) * ((1 << 63) + 12345)) % 2**64
+
+
+def test_full_size_17M(rt, xs_dev, xs_small):
+    """BASELINE configs[2] at full size, in the launch configuration bench.py times:
+    sampled lookups bit-exact, full checksum equal to the oracle's (all host cores)."""
+    n = 17_000_000
+    ver = torch.zeros(n, dtype=torch.uint64, device=DEV)
+    rt.omprt_xs_lookup(xs_dev, SEED, 0, n, ver, None, 0, 256, rt.OMPRT_ASSUME_OVERSUB)
+    ck = torch.zeros(1, dtype=torch.uint64, device=DEV)
+    rt.omprt_u64_sum(ver, n, ck)
+    torch.cuda.synchronize()
+    got = ver.cpu().numpy()
+    idx = np.random.default_rng(11).integers(0, n, 20000)
+    idx[:2] = [0, n - 1]
+    for i in idx[:2000]:
+        assert got[i] == oracle.xs_lookup(xs_small, int(i), 1)[0]
+    ref = oracle.xs_lookup(xs_small, 0, n, threads=os.cpu_count() or 1)
+    assert (got == ref).all()
+    assert int(ck.cpu().numpy()[0]) == int(ref.sum())
+
+
+def test_end_to_end_host_tables(rt, xs_small):
+    """omprt_xs_run_host: tables from (pinned) host memory, checksum back to the host."""
+    pinned = {k: torch.from_numpy(getattr(xs_small, k)).pin_memory()
+              for k in ("nuclide_grid", "unionized", "index_grid", "num_nucs", "mats", "concs")}
+    hs = rt.xs_host_struct(xs_small, pinned)
+    n = 100_000
+    ck, h2d, d2h = rt.omprt_xs_run_host(hs, SEED, 0, n)
+    assert ck == int(oracle.xs_lookup(xs_small, 0, n).sum())
+    assert h2d == xs_small.nbytes() and d2h == 8

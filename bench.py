@@ -184,9 +184,10 @@ def run_omprt(args):
     dev = torch.device("cuda", local)
     omprt.omprt_init(local)
     stream = torch.cuda.current_stream()
+    from paper_conf_ipps_doerfertphtdcg22_b200 import sharding
     tabs = gen.XSTables(**gen.XS_SMALL)
     d = omprt.XSDeviceTables(tabs, dev)
-    first = rank * L
+    first, _ = sharding.weak_shard(L, rank)
     ver = torch.zeros(L, dtype=torch.uint64, device=dev)
     ck = torch.zeros(1, dtype=torch.uint64, device=dev)
     ck_all = torch.zeros(1, dtype=torch.int64, device=dev)
@@ -206,7 +207,7 @@ def run_omprt(args):
         omprt.omprt_u64_sum(ver, L, ck)
         if world > 1:
             ck_all.copy_(ck.view(torch.int64))
-            dist.all_reduce(ck_all)  # u64 sum: two's-complement wrap == mod 2^64
+            sharding.allreduce_u64_sum(ck_all.view(torch.uint64))  # NCCL, wraps mod 2^64
 
     def timed(which, flags, k_steps, w_steps):
         for _ in range(w_steps):
@@ -242,11 +243,7 @@ def run_omprt(args):
     noas_step, noas_k = timed("rt", 0, args.steps, 1)
 
     def mx(v):
-        if world == 1:
-            return v
-        t = torch.tensor([v], dtype=torch.float64, device=dev)
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        return float(t.item())
+        return v if world == 1 else sharding.allreduce_max(v, dev)
 
     ms_step = mx(statistics.mean(step_ms))
     ms_kern = mx(statistics.mean(kern_ms))

@@ -1,0 +1,49 @@
+"""Multi-GPU plumbing of the hot path: one process per GPU, independent
+lookups / iterations / sites sharded by contiguous ranges, tables replicated, and one
+collective -- the checksum all-reduce -- over NCCL (gloo in CPU tests).
+
+Lookup i draws its energy and material from fast_forward_LCG(seed, 2i), so any contiguous
+partition gives bit-identical per-lookup results and an identical integer checksum.
+"""
+from __future__ import annotations
+
+
+def shard(total: int, rank: int, world: int):
+    """Strong scaling: rank r owns [r*total//world, (r+1)*total//world) -> (first, count)."""
+    if world <= 0 or not 0 <= rank < world or total < 0:
+        raise ValueError("bad shard arguments")
+    a = total * rank // world
+    b = total * (rank + 1) // world
+    return a, b - a
+
+
+def weak_shard(per_rank: int, rank: int):
+    """Weak scaling: rank r owns its own batch [r*per_rank, (r+1)*per_rank)."""
+    if per_rank < 0 or rank < 0:
+        raise ValueError("bad shard arguments")
+    return rank * per_rank, per_rank
+
+
+def allreduce_u64_sum(t, group=None):
+    """In-place u64 sum across ranks.  Collectives have no uint64 op, so the bits are
+    all-reduced as int64: two's-complement addition wraps exactly like u64 mod 2^64."""
+    import torch
+    import torch.distributed as dist
+    v = t.view(torch.int64)
+    dist.all_reduce(v, op=dist.ReduceOp.SUM, group=group)
+    return t
+
+
+def allreduce_f64_sum(t, group=None):
+    import torch.distributed as dist
+    dist.all_reduce(t, op=dist.ReduceOp.SUM, group=group)
+    return t
+
+
+def allreduce_max(value: float, device, group=None) -> float:
+    """Max over ranks of a host float (the device-timed step time, max over ranks)."""
+    import torch
+    import torch.distributed as dist
+    t = torch.tensor([value], dtype=torch.float64, device=device)
+    dist.all_reduce(t, op=dist.ReduceOp.MAX, group=group)
+    return float(t.item())

@@ -1,0 +1,23 @@
+#!/bin/bash
+# One GPU session: parity tests, smoke, bench, ncu launch list + full captures.
+# Usage (under gpurun): bash scripts/gpu_round.sh [tag]
+TAG=${1:-r01}
+OUT=gpurun_out
+mkdir -p $OUT
+nvidia-smi -L > $OUT/nvidia_smi_$TAG.txt 2>&1
+nproc >> $OUT/nvidia_smi_$TAG.txt
+export PYTHONUNBUFFERED=1
+timeout 1500 python -m pytest tests -m gpu -q -rf --timeout 600 > $OUT/pytest_gpu_$TAG.txt 2>&1
+echo "pytest exit $?" >> $OUT/pytest_gpu_$TAG.txt
+timeout 300 python -c "import __graft_entry__ as g; g.smoke()" > $OUT/smoke_$TAG.txt 2>&1
+echo "smoke exit $?" >> $OUT/smoke_$TAG.txt
+timeout 900 python bench.py --steps 10 --warmup 3 > $OUT/bench_$TAG.txt 2>&1
+echo "bench exit $?" >> $OUT/bench_$TAG.txt
+timeout 300 python bench.py --impl reference --steps 2 --warmup 1 > $OUT/bench_ref_$TAG.txt 2>&1
+timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none -c 200 --csv \
+  --log-file $OUT/launches_$TAG.csv python bench.py --steps 2 --warmup 1 --no-e2e > $OUT/ncu_launch_stdout_$TAG.txt 2>&1
+timeout 900 ncu --set full --clock-control none --import-source on -k regex:omprt_xs_rt -s 1 -c 1 \
+  -o $OUT/prof_xs_rt_$TAG python bench.py --steps 1 --warmup 1 --no-e2e --no-secondary > $OUT/ncu_full_stdout_$TAG.txt 2>&1
+timeout 900 ncu --set full --clock-control none --import-source on -k regex:cuda_xs_twin -s 0 -c 1 \
+  -o $OUT/prof_xs_twin_$TAG python bench.py --steps 1 --warmup 1 --no-e2e --no-secondary >> $OUT/ncu_full_stdout_$TAG.txt 2>&1
+ls -la $OUT

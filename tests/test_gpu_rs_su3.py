@@ -45,11 +45,18 @@ def test_rs_parity(rt, rs_dev, rs_tables, variant):
     assert flip.size <= 2
 
 
-def test_rs_checksum_and_rt_twin_agree(rt, rs_dev):
+def test_rs_rt_and_twin_agree(rt, rs_dev):
+    """Same body in both kernels; nvcc may contract a*b+c differently in the two inlining
+    contexts, so values agree to rounding, verification exactly up to near-ties."""
     n = 100_000
     v1, m1 = _rs(rt, rs_dev, 0, n, "rt", rt.OMPRT_ASSUME_OVERSUB)
     v2, m2 = _rs(rt, rs_dev, 0, n, "twin")
-    assert (v1 == v2).all() and (m1 == m2).all()  # same body, same compiler -> same bits
+    err = np.abs(m1 - m2).max(axis=1) / np.abs(m2).max(axis=1)
+    assert err.max() <= 1e-12
+    flip = np.nonzero(v1 != v2)[0]
+    for q in flip:
+        top2 = np.sort(m2[q])[-2:]
+        assert top2[1] - top2[0] <= 1e-12 * abs(top2[1])
 
 
 def _su3(rt, fn, A, B, n, flags=0):

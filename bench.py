@@ -156,26 +156,25 @@ def load_peaks():
     return 6650.0, "fallback 6.65 TB/s (B200_PROFILING.md)"
 
 
-def load_alg_bytes():
+def load_alg_bytes(accel):
     d = json.load(open(os.path.join(ROOT, "profiles", "xs_algorithmic_bytes.json")))
-    return float(d["bytes_per_lookup"])
+    return float(d["accel"]["bytes_per_lookup"] if accel else d["bytes_per_lookup"])
 
 
-def load_ncu_traffic():
+def load_ncu_traffic(kernel):
     p = os.path.join(ROOT, "profiles", "ncu_traffic.json")
     if os.path.exists(p):
         d = json.load(open(p))
-        return d.get("omprt_xs_rt_assume", {}).get("dram_bytes_per_launch")
+        return d.get(kernel, {}).get("dram_bytes_per_launch")
     return None
 
 
 def run_omprt(args):
-    import numpy as np
     import torch
     import torch.distributed as dist
 
     import gen
-    from paper_conf_ipps_doerfertphtdcg22_b200 import omprt
+    from paper_conf_ipps_doerfertphtdcg22_b200 import omprt, sharding
 
     rank, world, local = dist_env()
     if world > 1:
@@ -184,9 +183,9 @@ def run_omprt(args):
     dev = torch.device("cuda", local)
     omprt.omprt_init(local)
     stream = torch.cuda.current_stream()
-    from paper_conf_ipps_doerfertphtdcg22_b200 import sharding
     tabs = gen.XSTables(**gen.XS_SMALL)
-    d = omprt.XSDeviceTables(tabs, dev)
+    d_acc = omprt.XSDeviceTables(tabs, dev, accel=True)   # B200 layouts (the headline path)
+    d_pln = d_acc.plain()                                 # the tables as specified
     first, _ = sharding.weak_shard(L, rank)
     ver = torch.zeros(L, dtype=torch.uint64, device=dev)
     ck = torch.zeros(1, dtype=torch.uint64, device=dev)
@@ -194,14 +193,16 @@ def run_omprt(args):
     scrub = torch.empty(256 * 1024 * 1024 // 4, dtype=torch.float32, device=dev)
     A = omprt.OMPRT_ASSUME_OVERSUB
 
-    def step(kernel_events=None, which="rt", flags=A):
+    def step(kernel_events, which, tables, flags):
         ck.zero_()
         if kernel_events:
             kernel_events[0].record(stream)
         if which == "rt":
-            omprt.omprt_xs_lookup(d, gen.XS_LOOKUP_SEED, first, L, ver, None, 0, THREADS, flags)
+            omprt.omprt_xs_lookup(tables, gen.XS_LOOKUP_SEED, first, L, ver, None, 0, THREADS,
+                                  flags)
         else:
-            omprt.omprt_cuda_xs_lookup(d, gen.XS_LOOKUP_SEED, first, L, ver, None, 0, THREADS, 0)
+            omprt.omprt_cuda_xs_lookup(tables, gen.XS_LOOKUP_SEED, first, L, ver, None, 0,
+                                       THREADS, 0)
         if kernel_events:
             kernel_events[1].record(stream)
         omprt.omprt_u64_sum(ver, L, ck)
@@ -209,10 +210,10 @@ def run_omprt(args):
             ck_all.copy_(ck.view(torch.int64))
             sharding.allreduce_u64_sum(ck_all.view(torch.uint64))  # NCCL, wraps mod 2^64
 
-    def timed(which, flags, k_steps, w_steps):
+    def timed(which, tables, flags, k_steps, w_steps):
         for _ in range(w_steps):
             scrub.fill_(1.0)
-            step(None, which, flags)
+            step(None, which, tables, flags)
         torch.cuda.synchronize()
         if world > 1:
             dist.barrier()
@@ -223,7 +224,7 @@ def run_omprt(args):
         for e in ev:
             scrub.fill_(1.0)  # L2 flush, outside the step's events
             e[0].record(stream)
-            step((e[1], e[2]), which, flags)
+            step((e[1], e[2]), which, tables, flags)
             e[3].record(stream)
         torch.cuda.synchronize()
         if world > 1:
@@ -232,51 +233,57 @@ def run_omprt(args):
         kern_ms = [b.elapsed_time(c) for _, b, c, _ in ev]
         return step_ms, kern_ms
 
-    clocks = ClockSampler(local)
-    # primary: runtime-driven with the assumption (the headline path)
-    clocks.start()
-    step_ms, kern_ms = timed("rt", A, args.steps, args.warmup)
-    clk = clocks.stop()
-    checksum = int(ck.cpu().numpy()[0]) if world == 1 else int(ck_all.cpu().numpy()[0]) % 2**64
-    # twin and variants, interleaved in the same process with the same geometry
-    twin_step, twin_k = timed("twin", 0, args.steps, 1)
-    noas_step, noas_k = timed("rt", 0, args.steps, 1)
-
     def mx(v):
         return v if world == 1 else sharding.allreduce_max(v, dev)
 
+    clocks = ClockSampler(local)
+    # primary: runtime-driven, assumption, B200 layouts (the headline path)
+    clocks.start()
+    step_ms, kern_ms = timed("rt", d_acc, A, args.steps, args.warmup)
+    clk = clocks.stop()
+    checksum = int(ck.cpu().numpy()[0]) if world == 1 else int(ck_all.cpu().numpy()[0]) % 2**64
+    # twin and variants, in the same process with the same geometry
+    kms = {"rt_assume": mx(statistics.mean(kern_ms))}
+    for name, which, tables, flags in [("twin", "twin", d_acc, 0), ("rt_no_assume", "rt", d_acc, 0),
+                                       ("plain_rt_assume", "rt", d_pln, A),
+                                       ("plain_twin", "twin", d_pln, 0),
+                                       ("plain_rt_no_assume", "rt", d_pln, 0)]:
+        _, k = timed(which, tables, flags, args.steps, 1)
+        kms[name] = mx(statistics.mean(k))
+        if world == 1:
+            assert int(ck.cpu().numpy()[0]) == checksum, name  # every variant: same checksum
     ms_step = mx(statistics.mean(step_ms))
-    ms_kern = mx(statistics.mean(kern_ms))
-    ms_twin_k = mx(statistics.mean(twin_k))
-    ms_noas_k = mx(statistics.mean(noas_k))
     value = world * L / (ms_step / 1000.0)
 
-    # e2e through the public C ABI with HOST tables (pinned): H2D tables + lookups + sum +
-    # D2H checksum, synchronous, timed on the host clock around the call
+    # e2e through the public C ABI with HOST tables (pinned): H2D tables + device-built B200
+    # layouts + lookups + sum + D2H checksum, synchronous, host clock around the call
     e2e = None
     if not args.no_e2e:
         pinned = {k: torch.from_numpy(getattr(tabs, k)).pin_memory()
                   for k in ("nuclide_grid", "unionized", "index_grid", "num_nucs", "mats",
                             "concs")}
         hs = omprt.xs_host_struct(tabs, pinned)
+        XA = omprt.OMPRT_XS_ACCEL
         for _ in range(max(1, args.warmup)):
-            omprt.omprt_xs_run_host(hs, gen.XS_LOOKUP_SEED, first, L, THREADS, 0)
+            omprt.omprt_xs_run_host(hs, gen.XS_LOOKUP_SEED, first, L, THREADS, XA)
         torch.cuda.synchronize()
         if world > 1:
             dist.barrier()
         t0 = time.perf_counter()
         for _ in range(args.steps):
-            ck_h, h2d, d2h = omprt.omprt_xs_run_host(hs, gen.XS_LOOKUP_SEED, first, L, THREADS, 0)
+            ck_h, h2d, d2h = omprt.omprt_xs_run_host(hs, gen.XS_LOOKUP_SEED, first, L, THREADS, XA)
         e2e_ms = mx(1000.0 * (time.perf_counter() - t0) / args.steps)
         assert ck_h == checksum or world > 1, (ck_h, checksum)
         e2e = {"value": world * L / (e2e_ms / 1000.0), "unit": UNIT, "h2d_bytes_per_step": h2d,
                "d2h_bytes_per_step": d2h, "ms_per_step": e2e_ms,
-               "path": "omprt_xs_run_host (pinned host tables, fused reduction)"}
+               "path": "omprt_xs_run_host (pinned host tables -> device-built B200 layouts, "
+                       "fused reduction, u64 checksum back)"}
 
     tab = omprt.kernel_table()
     peak, peak_src = load_peaks()
-    alg = load_alg_bytes() * L
-    achieved = alg / (ms_kern / 1000.0) / 1e9
+    alg = load_alg_bytes(True) * L
+    achieved = alg / (kms["rt_assume"] / 1000.0) / 1e9
+    alg_plain = load_alg_bytes(False) * L
     secondary = None
     if not args.no_secondary and rank == 0:
         secondary = run_secondary(omprt, torch, gen, dev, stream, scrub)
@@ -293,24 +300,34 @@ def run_omprt(args):
             "config": {"workload": WORKLOAD, "lookups_per_gpu": L, "threads_per_team": THREADS,
                        "teams": (L + THREADS - 1) // THREADS, "parallelism": f"dp{world}",
                        "l2": "flushed before every timed step (256 MiB scrub write)",
-                       "variant": "runtime-driven SPMD, teams oversubscription assumption"},
+                       "variant": "runtime-driven SPMD, teams oversubscription assumption, "
+                                  "B200 table layouts (binned search, 16-bit index, bracket "
+                                  "records)"},
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
-                         "frac": achieved / peak, "traffic": load_ncu_traffic(),
-                         "kernel": "omprt_xs_rt_assume", "alg_bytes_per_launch": alg,
-                         "peak_source": peak_src},
+                         "frac": achieved / peak,
+                         "traffic": load_ncu_traffic("omprt_xs_rt_assume_accel"),
+                         "kernel": "omprt_xs_rt_assume_accel", "alg_bytes_per_launch": alg,
+                         "peak_source": peak_src,
+                         "plain_layout": {"kernel": "omprt_xs_rt_assume",
+                                          "alg_bytes_per_launch": alg_plain,
+                                          "achieved": alg_plain / kms["plain_rt_assume"] / 1e6,
+                                          "traffic": load_ncu_traffic("omprt_xs_rt_assume")}},
             "cpu_baseline": cpu,
             "e2e": e2e,
             "gpu_launches": 2 * args.steps,
             "clocks": clk,
             "checksum": checksum,
-            "kernel_ms": {"rt_assume": ms_kern, "twin": ms_twin_k, "rt_no_assume": ms_noas_k},
+            "kernel_ms": kms,
             "overhead_vs_twin": {
-                "time": ms_kern / ms_twin_k - 1.0,
-                "time_no_assume": ms_noas_k / ms_twin_k - 1.0,
-                "regs": [tab["omprt_xs_rt_assume"]["regs"], tab["cuda_xs_twin"]["regs"]],
-                "regs_no_assume": tab["omprt_xs_rt"]["regs"],
-                "static_smem": [tab["omprt_xs_rt_assume"]["static_smem"],
-                                tab["cuda_xs_twin"]["static_smem"]]},
+                "time": kms["rt_assume"] / kms["twin"] - 1.0,
+                "time_no_assume": kms["rt_no_assume"] / kms["twin"] - 1.0,
+                "time_plain": kms["plain_rt_assume"] / kms["plain_twin"] - 1.0,
+                "regs": [tab["omprt_xs_rt_assume_accel"]["regs"], tab["cuda_xs_twin_accel"]["regs"]],
+                "regs_no_assume": tab["omprt_xs_rt_accel"]["regs"],
+                "local_bytes": [tab["omprt_xs_rt_assume_accel"]["local_bytes"],
+                                tab["cuda_xs_twin_accel"]["local_bytes"]],
+                "static_smem": [tab["omprt_xs_rt_assume_accel"]["static_smem"],
+                                tab["cuda_xs_twin_accel"]["static_smem"]]},
             "secondary": secondary,
         }
         print(json.dumps(line), flush=True)

@@ -74,6 +74,9 @@ extern "C" {
  * the debug build's device assertion ("asserting that the condition actually holds")
  * can be exercised.  In a release build a violated assumption then skips iterations. */
 #define OMPRT_UNCHECKED (1u << 9)
+/* omprt_xs_run_host: build and use the accelerated table layouts on the device (per call,
+ * inside the end-to-end time). */
+#define OMPRT_XS_ACCEL (1u << 10)
 
 /* ---- runtime lifecycle ------------------------------------------------------------- */
 typedef struct {
@@ -146,6 +149,17 @@ typedef struct {
   const double *concs;        /* [12][max_num_nucs] */
   int32_t n_isotopes, n_gridpoints, max_num_nucs, pad;
   int64_t n_union;
+  /* Optional B200 layouts of the same data, filled by omprt_xs_build_accel (all NULL: the
+   * lookups read the tables above exactly as specified).  With them set the lookups read
+   * the same values from: `bins` (search brackets of 2^log2_bins energy bins -- the same
+   * unionized-grid index with ~4 instead of ~20 probes), `index_grid16` (the index grid as
+   * uint16, n_gridpoints <= 65536: half the footprint, same values) and `brackets` (per
+   * nuclide and bracket k the 12 doubles of gridpoints k and k+1, interleaved, 96 B per
+   * bracket: 3 x 256-bit loads instead of 6 x 128-bit).  Results are identical. */
+  const int32_t *bins;         /* [2^log2_bins + 1] */
+  const uint16_t *index_grid16;/* [n_union][n_isotopes] */
+  const double *brackets;      /* [n_isotopes][n_gridpoints-1][12], 32 B aligned */
+  int32_t log2_bins, pad2;
 } omprt_xs_tables;
 /* Lookups first..first+count-1 (lookup i draws its energy and material from
  * fast_forward_LCG(seed, 2i), so results do not depend on sharding):
@@ -159,6 +173,17 @@ int omprt_xs_lookup(omprt_xs_tables t, uint64_t seed, int64_t first, int64_t cou
 int omprt_cuda_xs_lookup(omprt_xs_tables t, uint64_t seed, int64_t first, int64_t count,
                          uint64_t *verification, uint64_t *checksum_inout, int32_t teams,
                          int32_t threads, uint32_t flags, void *stream);
+/* Byte sizes of the three accelerated-layout buffers for tables of this shape:
+ * sizes[0] bins, sizes[1] index_grid16, sizes[2] brackets.  OMPRT_E_INVAL when
+ * n_gridpoints > 65536 (the 16-bit index cannot hold it) or log2_bins not in [1, 28]. */
+int omprt_xs_accel_sizes(int32_t n_isotopes, int32_t n_gridpoints, int64_t n_union,
+                         int32_t log2_bins, uint64_t *sizes);
+/* Build the accelerated layouts from t's device tables into caller-owned device buffers
+ * (sizes from omprt_xs_accel_sizes; brackets 32 B aligned) on `stream`, and point t's
+ * bins / index_grid16 / brackets / log2_bins at them.  A table-preparation step (like
+ * XSBench's own index-grid construction), not part of a lookup. */
+int omprt_xs_build_accel(omprt_xs_tables *t, int32_t *bins, uint16_t *index_grid16,
+                         double *brackets, int32_t log2_bins, void *stream);
 /* K11 ("we moved the reduction out of the timed kernel"): *out_inout += sum v[i]
  * (u64, wraps mod 2^64). */
 int omprt_u64_sum(const uint64_t *v, int64_t n, uint64_t *out_inout, void *stream);

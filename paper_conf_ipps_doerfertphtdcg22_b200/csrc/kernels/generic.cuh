@@ -38,6 +38,35 @@ struct GenericTraitsDebug : GenericTraitsLoop {
   static constexpr unsigned debug = dbg::Assert | dbg::Trace;
 };
 
+// The sequential prologue (user code, identical in the runtime kernel and the twin): the
+// team's main thread fills the arrays the parallel region reads.  Loads are issued in
+// batches of 16 so a single thread keeps 16 requests in flight.
+__device__ __forceinline__ double gen_prologue(const double* __restrict__ tin, int32_t t,
+                                               int32_t inner_n, double* w, int32_t* perm) {
+  const double tp1 = (double)(t + 1);
+  double s = 0.0;
+  int32_t k = 0;
+  for (; k + 16 <= inner_n; k += 16) {
+    double v[16];
+#pragma unroll
+    for (int u = 0; u < 16; ++u) v[u] = __ldg(tin + k + u);
+#pragma unroll
+    for (int u = 0; u < 16; ++u) {
+      const double x = __dmul_rn(v[u], tp1);
+      w[k + u] = x;
+      s = __dadd_rn(s, x);
+      perm[k + u] = ((k + u) * 17 + t) % inner_n;
+    }
+  }
+  for (; k < inner_n; ++k) {
+    const double x = __dmul_rn(__ldg(tin + k), tp1);
+    w[k] = x;
+    s = __dadd_rn(s, x);
+    perm[k] = (k * 17 + t) % inner_n;
+  }
+  return s;
+}
+
 // The parallel region: team `for` over j (Fig. 5 with NumBlocks = 1).
 template <bool Rec, bool Join>
 struct GenRegion {
@@ -60,8 +89,10 @@ struct GenRegion {
   }
 };
 
+constexpr int kGenericMaxThreads = 256;
+
 template <class Tr, int kInner, bool Rec, bool Post>
-__global__ void __launch_bounds__(1024)
+__global__ void __launch_bounds__(kGenericMaxThreads)
     omprt_generic_rt(int32_t inner_n_rt, const double* __restrict__ in, double* __restrict__ out,
                      int32_t* owner, double* post) {
   using R = GenRegion<Rec, Post>;
@@ -74,17 +105,9 @@ __global__ void __launch_bounds__(1024)
   }
   // ---- sequential part: the team's main thread alone ----
   const int32_t t = (int32_t)blockIdx.x;
-  const double* tin = in + (int64_t)t * inner_n;
   double* w = static_cast<double*>(alloc_shared(team, (uint32_t)inner_n * 8u));
   int32_t* perm = static_cast<int32_t*>(alloc_shared(team, (uint32_t)inner_n * 4u));
-  const double tp1 = (double)(t + 1);
-  double s = 0.0;
-  for (int32_t k = 0; k < inner_n; ++k) {
-    const double v = __dmul_rn(__ldg(tin + k), tp1);
-    w[k] = v;
-    s = __dadd_rn(s, v);
-    perm[k] = (k * 17 + t) % inner_n;
-  }
+  const double s = gen_prologue(in + (int64_t)t * inner_n, t, inner_n, w, perm);
   double* tout = out + (int64_t)t * inner_n;
   parallel<Tr, L, R>(team, typename R::Args{w, perm, s, tout,
                                             Rec ? owner + (int64_t)t * inner_n : nullptr,
@@ -101,7 +124,7 @@ __global__ void __launch_bounds__(1024)
 
 // Bare CUDA twin.
 template <int kInner, bool Rec, bool Post>
-__global__ void __launch_bounds__(1024)
+__global__ void __launch_bounds__(kGenericMaxThreads)
     cuda_generic_twin(int32_t inner_n_rt, const double* __restrict__ in,
                       double* __restrict__ out, int32_t* owner, double* post) {
   __shared__ double w[256];
@@ -109,18 +132,7 @@ __global__ void __launch_bounds__(1024)
   __shared__ double s_sh;
   const int32_t inner_n = kInner > 0 ? kInner : inner_n_rt;
   const int32_t t = (int32_t)blockIdx.x;
-  if (threadIdx.x == 0) {
-    const double* tin = in + (int64_t)t * inner_n;
-    const double tp1 = (double)(t + 1);
-    double s = 0.0;
-    for (int32_t k = 0; k < inner_n; ++k) {
-      const double v = __dmul_rn(__ldg(tin + k), tp1);
-      w[k] = v;
-      s = __dadd_rn(s, v);
-      perm[k] = (k * 17 + t) % inner_n;
-    }
-    s_sh = s;
-  }
+  if (threadIdx.x == 0) s_sh = gen_prologue(in + (int64_t)t * inner_n, t, inner_n, w, perm);
   __syncthreads();
   const double s = s_sh;
   double* tout = out + (int64_t)t * inner_n;
@@ -184,7 +196,8 @@ inline int generic_validate(int32_t teams, int32_t threads, int32_t inner_n, con
                             double* out, double* post, uint32_t flags, Workspace* w,
                             bool twin) {
   OMPRT_CHECK_ARG(teams > 0 && teams <= 2147483647, "teams must be > 0");
-  OMPRT_CHECK_ARG(threads > 0 && threads <= 1024, "threads must be in [1, 1024]");
+  OMPRT_CHECK_ARG(threads > 0 && threads <= kGenericMaxThreads, "threads must be in [1, %d]",
+                  kGenericMaxThreads);
   OMPRT_CHECK_ARG(inner_n >= 0 && inner_n <= 65536, "inner_n out of range");
   OMPRT_CHECK_ARG(!twin || inner_n <= 256, "the CUDA twin supports inner_n <= 256");
   OMPRT_CHECK_ARG(inner_n == 0 || (in && out), "null data pointer");

@@ -63,34 +63,63 @@ inline int rs_validate(const omprt_rs_tables& t, int64_t count, uint64_t* ver, i
 }
 
 // ---------------------------------------------------------------------------- SU(3)
+// 256-bit global accesses (sm_100: LDG/STG.E.ENL2.256): a site is 576 B = 18 x 32 B, so a
+// pair of links (288 B) moves in 9 instructions per thread instead of 18 x 16 B ones --
+// half the L1 wavefronts of the strided AoS access.
+__device__ __forceinline__ void ld_nc_256(const double* p, double& a, double& b, double& c,
+                                          double& d) {
+  asm("ld.global.nc.L1::no_allocate.v4.f64 {%0,%1,%2,%3}, [%4];"
+      : "=d"(a), "=d"(b), "=d"(c), "=d"(d)
+      : "l"(p));
+}
+__device__ __forceinline__ void st_cs_256(double* p, double a, double b, double c, double d) {
+  asm volatile("st.global.cs.v4.f64 [%0], {%1,%2,%3,%4};" ::"l"(p), "d"(a), "d"(b), "d"(c),
+               "d"(d)
+               : "memory");
+}
+
 // One site: C[l] = A[l] x B[l] for the 4 links; complex MAC = 4 fmas in fixed order
-// (App. A.3), so C is bit-identical to the oracle.  Returns sum of Re C over the site.
-__device__ __forceinline__ double su3_site(const double2* __restrict__ A,
+// (App. A.3), so C is bit-identical to the oracle.  Row r of C[l] needs only row r of A[l],
+// so it overwrites it in registers.  Returns sum of Re C over the site in (l, r, c) order.
+__device__ __forceinline__ double su3_site(const double* __restrict__ A,
                                            const double2* __restrict__ B,
-                                           double2* __restrict__ Cs) {
+                                           double* __restrict__ Cs) {
   double re_sum = 0.0;
 #pragma unroll
-  for (int l = 0; l < 4; ++l) {
-    double2 a[9];
+  for (int lp = 0; lp < 2; ++lp) {
+    double v[36];
 #pragma unroll
-    for (int e = 0; e < 9; ++e) a[e] = __ldg(A + l * 9 + e);
+    for (int q = 0; q < 9; ++q)
+      ld_nc_256(A + lp * 36 + 4 * q, v[4 * q], v[4 * q + 1], v[4 * q + 2], v[4 * q + 3]);
 #pragma unroll
-    for (int r = 0; r < 3; ++r)
+    for (int li = 0; li < 2; ++li) {
+      const int l = 2 * lp + li, base = 18 * li;
 #pragma unroll
-      for (int c = 0; c < 3; ++c) {
-        double re = 0.0, im = 0.0;
+      for (int r = 0; r < 3; ++r) {
+        double out[6];
 #pragma unroll
-        for (int m = 0; m < 3; ++m) {
-          const double2 x = a[r * 3 + m];
-          const double2 y = __ldg(B + l * 9 + m * 3 + c);
-          re = fma(x.x, y.x, re);
-          re = fma(-x.y, y.y, re);
-          im = fma(x.x, y.y, im);
-          im = fma(x.y, y.x, im);
+        for (int c = 0; c < 3; ++c) {
+          double re = 0.0, im = 0.0;
+#pragma unroll
+          for (int m = 0; m < 3; ++m) {
+            const double xr = v[base + (r * 3 + m) * 2], xi = v[base + (r * 3 + m) * 2 + 1];
+            const double2 y = __ldg(B + l * 9 + m * 3 + c);
+            re = fma(xr, y.x, re);
+            re = fma(-xi, y.y, re);
+            im = fma(xr, y.y, im);
+            im = fma(xi, y.x, im);
+          }
+          out[2 * c] = re;
+          out[2 * c + 1] = im;
+          re_sum += re;
         }
-        __stcs(Cs + l * 9 + r * 3 + c, make_double2(re, im));
-        re_sum += re;
+#pragma unroll
+        for (int e = 0; e < 6; ++e) v[base + r * 6 + e] = out[e];
       }
+    }
+#pragma unroll
+    for (int q = 0; q < 9; ++q)
+      st_cs_256(Cs + lp * 36 + 4 * q, v[4 * q], v[4 * q + 1], v[4 * q + 2], v[4 * q + 3]);
   }
   return re_sum;
 }
@@ -103,14 +132,14 @@ constexpr int kSU3Threads = 128;
 
 template <class Tr, bool Checksum>
 __global__ void __launch_bounds__(kSU3Threads)
-    omprt_su3_rt(const double2* __restrict__ A, const double2* __restrict__ B,
-                 double2* __restrict__ Cm, typename Tr::Idx n_sites, double* checksum,
+    omprt_su3_rt(const double* __restrict__ A, const double2* __restrict__ B,
+                 double* __restrict__ Cm, typename Tr::Idx n_sites, double* checksum,
                  double* partials, unsigned* ticket) {
   using Idx = typename Tr::Idx;
   Team<Tr> team = init<Tr>();
   double acc = 0.0;
   distribute_parallel_for(team, n_sites, [&](Idx s) {
-    acc += su3_site(A + (int64_t)s * 36, B, Cm + (int64_t)s * 36);
+    acc += su3_site(A + (int64_t)s * 72, B, Cm + (int64_t)s * 72);
   });
   if constexpr (Checksum)
     league_reduce(team, team_reduce_to_main(team, acc, Plus{}), Plus{}, checksum, partials,
@@ -119,12 +148,12 @@ __global__ void __launch_bounds__(kSU3Threads)
 
 template <bool Checksum>
 __global__ void __launch_bounds__(kSU3Threads)
-    cuda_su3_twin(const double2* __restrict__ A, const double2* __restrict__ B,
-                  double2* __restrict__ Cm, int32_t n_sites, double* checksum, double* partials,
+    cuda_su3_twin(const double* __restrict__ A, const double2* __restrict__ B,
+                  double* __restrict__ Cm, int32_t n_sites, double* checksum, double* partials,
                   unsigned* ticket) {
   const int32_t s = blockIdx.x * blockDim.x + threadIdx.x;
   double acc = 0.0;
-  if (s < n_sites) acc = su3_site(A + (int64_t)s * 36, B, Cm + (int64_t)s * 36);
+  if (s < n_sites) acc = su3_site(A + (int64_t)s * 72, B, Cm + (int64_t)s * 72);
   if constexpr (Checksum) {
     __shared__ double ws[32];
     __shared__ unsigned last;
@@ -172,8 +201,8 @@ inline int su3_validate(const double* A, const double* B, double* Cm, int64_t n,
   OMPRT_CHECK_ARG(n >= 0 && n < (1ll << 30), "n_sites out of range");
   OMPRT_CHECK_ARG(threads == kSU3Threads, "threads must be %d", kSU3Threads);
   OMPRT_CHECK_ARG(n == 0 || (A && B && Cm), "null data pointer");
-  OMPRT_CHECK_ARG(((uintptr_t)A | (uintptr_t)B | (uintptr_t)Cm) % 16 == 0,
-                  "A, B, C must be 16 B aligned");
+  OMPRT_CHECK_ARG(((uintptr_t)A | (uintptr_t)Cm) % 32 == 0 && (uintptr_t)B % 16 == 0,
+                  "A and C must be 32 B aligned (256-bit accesses), B 16 B aligned");
   if (teams <= 0) teams = (int32_t)std::max<int64_t>(1, ceil_div(n, threads));
   OMPRT_CHECK_ARG(!ck || (uint64_t)teams <= w->opt.max_teams, "teams exceed max_teams");
   OMPRT_CHECK_ARG(!(flags & OMPRT_ASSUME_OVERSUB) || n <= (int64_t)teams * threads,
@@ -231,9 +260,9 @@ extern "C" int omprt_su3_mult(const double* A, const double* B, double* Cm, int6
   if (int r = su3_validate(A, B, Cm, n_sites, teams, threads, flags, checksum_inout, w)) return r;
   if (n_sites == 0) return OMPRT_OK;
   cudaStream_t s = as_stream(stream);
-  auto* a = (const double2*)A;
+  auto* a = A;
   auto* b = (const double2*)B;
-  auto* c = (double2*)Cm;
+  auto* c = Cm;
   double* p = (double*)w->partials;
   unsigned* tk = w->tickets + 3;
   const int32_t n = (int32_t)n_sites;
@@ -260,11 +289,11 @@ extern "C" int omprt_cuda_su3_mult(const double* A, const double* B, double* Cm,
   if (n_sites == 0) return OMPRT_OK;
   cudaStream_t s = as_stream(stream);
   if (checksum_inout)
-    cuda_su3_twin<true><<<tm, threads, 0, s>>>((const double2*)A, (const double2*)B, (double2*)Cm,
+    cuda_su3_twin<true><<<tm, threads, 0, s>>>(A, (const double2*)B, Cm,
                                                (int32_t)n_sites, checksum_inout,
                                                (double*)w->partials, w->tickets + 3);
   else
-    cuda_su3_twin<false><<<tm, threads, 0, s>>>((const double2*)A, (const double2*)B, (double2*)Cm,
+    cuda_su3_twin<false><<<tm, threads, 0, s>>>(A, (const double2*)B, Cm,
                                                 (int32_t)n_sites, nullptr, nullptr, nullptr);
   return check_launch("cuda_su3_twin");
 }

@@ -19,6 +19,11 @@ struct XSTables {
   const double* __restrict__ concs;         // [12][max_num_nucs]
   int32_t n_isotopes, n_gridpoints, max_num_nucs, pad;
   int64_t n_union;
+  // optional B200 layouts of the same data (omprt_xs_build_accel), all NULL or all set
+  const int32_t* __restrict__ bins;         // [2^log2_bins + 1] search brackets per energy bin
+  const uint16_t* __restrict__ index_grid16;  // [n_union][n_iso] (n_gp <= 65536)
+  const double* __restrict__ brackets;      // [n_iso][n_gp-1][12] (E,t,e,a,f,n) x (k, k+1)
+  int32_t log2_bins, pad2;
 };
 
 // ---- the proxy apps' LCG (m = 2^63, a = 2806196910506780709, c = 1) ----------------------
@@ -99,44 +104,73 @@ __device__ __forceinline__ int32_t grid_search(const double* __restrict__ A, int
   return lo;
 }
 
-// One lookup: returns verification = 1 + argmax of the 5 macroscopic cross sections;
-// macro_out (nullable) receives them.
-template <bool kMacro = false>
-__device__ __forceinline__ uint64_t xs_lookup_one(const XSTables& t, uint64_t seed0,
-                                                  int64_t i, double* macro_out = nullptr) {
+// Exact search of the unionized grid accelerated by energy bins: bins[b] = grid_search(b/H)
+// is monotone in b, so the answer for E in [b/H, (b+1)/H) lies in [bins[b], bins[b+1]] and
+// the same bisection over that bracket (~4 probes instead of ~20) returns the same index.
+__device__ __forceinline__ int32_t binned_grid_search(const XSTables& t, double E) {
+  const int64_t H = 1ll << t.log2_bins;
+  int64_t b = (int64_t)(E * (double)H);  // exact scaling by a power of two
+  if (b > H - 1) b = H - 1;
+  int32_t lo = __ldg(t.bins + b), hi = __ldg(t.bins + b + 1) + 1;
+  if (hi > (int32_t)t.n_union - 1) hi = (int32_t)t.n_union - 1;
+  while (hi - lo > 1) {
+    const int32_t mid = lo + ((hi - lo) >> 1);
+    if (__ldg(t.unionized + mid) > E) hi = mid;
+    else lo = mid;
+  }
+  return lo;
+}
+
+__device__ __forceinline__ void ld_nc_v4f64(const double* p, double& a, double& b, double& c,
+                                            double& d) {
+  asm("ld.global.nc.v4.f64 {%0,%1,%2,%3}, [%4];" : "=d"(a), "=d"(b), "=d"(c), "=d"(d) : "l"(p));
+}
+
+// One lookup: returns verification = 1 + argmax of the 5 macroscopic cross sections.
+// Accel = false reads the tables exactly as specified (binary search of the unionized grid,
+// int32 index grid, 48 B gridpoint records: 6 x 16 B loads per nuclide).  Accel = true reads
+// the same values from the B200 layouts (binned search, 16-bit index grid, 96 B bracket
+// records loaded by 3 x 256-bit loads) -- identical results, fewer L1 wavefronts.
+template <bool Accel>
+__device__ __forceinline__ uint64_t xs_lookup_one(const XSTables& t, uint64_t seed0, int64_t i) {
   uint64_t seed = lcg_fast_forward(seed0, 2ull * (uint64_t)i);
   const double E = lcg_double(seed);
   const int mat = pick_mat(seed);
-  const int32_t idx = grid_search(t.unionized, (int32_t)t.n_union, E);
+  const int32_t idx = Accel ? binned_grid_search(t, E)
+                            : grid_search(t.unionized, (int32_t)t.n_union, E);
   const int nn = __ldg(t.num_nucs + mat);
   const int32_t* __restrict__ mrow = t.mats + mat * t.max_num_nucs;
   const double* __restrict__ crow = t.concs + mat * t.max_num_nucs;
-  const int32_t* __restrict__ irow = t.index_grid + (int64_t)idx * t.n_isotopes;
-  const double2* __restrict__ grid = reinterpret_cast<const double2*>(t.nuclide_grid);
+  const int64_t row = (int64_t)idx * t.n_isotopes;
   double m0 = 0.0, m1 = 0.0, m2 = 0.0, m3 = 0.0, m4 = 0.0;
 #pragma unroll 4
   for (int j = 0; j < nn; ++j) {
     const int32_t p = __ldg(mrow + j);
     const double conc = __ldg(crow + j);
-    int32_t k = __ldg(irow + p);
+    int32_t k = Accel ? (int32_t)__ldg(t.index_grid16 + row + p) : __ldg(t.index_grid + row + p);
     if (k == t.n_gridpoints - 1) --k;
-    // gridpoints k and k+1 of nuclide p: 2 x 48 B = 6 x 16 B (16 B aligned)
-    const double2* g = grid + ((int64_t)p * t.n_gridpoints + k) * 3;
-    const double2 l0 = __ldg(g + 0), l1 = __ldg(g + 1), l2 = __ldg(g + 2);
-    const double2 h0 = __ldg(g + 3), h1 = __ldg(g + 4), h2 = __ldg(g + 5);
-    const double f = (h0.x - E) / (h0.x - l0.x);
-    m0 = fma(fma(-f, h0.y - l0.y, h0.y), conc, m0);  // total
-    m1 = fma(fma(-f, h1.x - l1.x, h1.x), conc, m1);  // elastic
-    m2 = fma(fma(-f, h1.y - l1.y, h1.y), conc, m2);  // absorption
-    m3 = fma(fma(-f, h2.x - l2.x, h2.x), conc, m3);  // fission
-    m4 = fma(fma(-f, h2.y - l2.y, h2.y), conc, m4);  // nu-fission
-  }
-  if constexpr (kMacro) {
-    macro_out[0] = m0;
-    macro_out[1] = m1;
-    macro_out[2] = m2;
-    macro_out[3] = m3;
-    macro_out[4] = m4;
+    double le, lt, lel, la, lf, ln, he, ht, hel, ha, hf, hn;
+    if constexpr (Accel) {
+      // bracket (p, k): E_k E_k1 | t_k t_k1 | e_k e_k1 | a_k a_k1 | f_k f_k1 | n_k n_k1
+      const double* g = t.brackets + ((int64_t)p * (t.n_gridpoints - 1) + k) * 12;
+      ld_nc_v4f64(g, le, he, lt, ht);
+      ld_nc_v4f64(g + 4, lel, hel, la, ha);
+      ld_nc_v4f64(g + 8, lf, hf, ln, hn);
+    } else {
+      // gridpoints k and k+1 of nuclide p: 2 x 48 B = 6 x 16 B (16 B aligned)
+      const double2* g = reinterpret_cast<const double2*>(t.nuclide_grid) +
+                         ((int64_t)p * t.n_gridpoints + k) * 3;
+      const double2 l0 = __ldg(g + 0), l1 = __ldg(g + 1), l2 = __ldg(g + 2);
+      const double2 h0 = __ldg(g + 3), h1 = __ldg(g + 4), h2 = __ldg(g + 5);
+      le = l0.x; lt = l0.y; lel = l1.x; la = l1.y; lf = l2.x; ln = l2.y;
+      he = h0.x; ht = h0.y; hel = h1.x; ha = h1.y; hf = h2.x; hn = h2.y;
+    }
+    const double f = (he - E) / (he - le);
+    m0 = fma(fma(-f, ht - lt, ht), conc, m0);      // total
+    m1 = fma(fma(-f, hel - lel, hel), conc, m1);   // elastic
+    m2 = fma(fma(-f, ha - la, ha), conc, m2);      // absorption
+    m3 = fma(fma(-f, hf - lf, hf), conc, m3);      // fission
+    m4 = fma(fma(-f, hn - ln, hn), conc, m4);      // nu-fission
   }
   // 1 + argmax, strict '>' from max = -1 (the first maximum wins)
   double mx = -1.0;
@@ -147,6 +181,35 @@ __device__ __forceinline__ uint64_t xs_lookup_one(const XSTables& t, uint64_t se
   if (m3 > mx) { mx = m3; v = 4; }
   if (m4 > mx) { mx = m4; v = 5; }
   return v;
+}
+
+// ---- builders of the accelerated layouts (table preparation, not per lookup) -------------
+__global__ void xs_build_bins(const double* __restrict__ U, int32_t len, int32_t log2_bins,
+                              int32_t* __restrict__ bins) {
+  const int64_t H = 1ll << log2_bins;
+  for (int64_t b = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; b <= H;
+       b += (int64_t)gridDim.x * blockDim.x)
+    bins[b] = grid_search(U, len, (double)b / (double)H);
+}
+__global__ void xs_build_index16(const int32_t* __restrict__ a, uint16_t* __restrict__ b,
+                                 int64_t n) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n;
+       i += (int64_t)gridDim.x * blockDim.x)
+    b[i] = (uint16_t)a[i];
+}
+__global__ void xs_build_brackets(const double* __restrict__ g, double* __restrict__ o,
+                                  int32_t n_iso, int32_t n_gp) {
+  const int64_t nb = (int64_t)n_iso * (n_gp - 1);
+  for (int64_t b = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; b < nb;
+       b += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t p = b / (n_gp - 1), k = b % (n_gp - 1);
+    const double* lo = g + (p * n_gp + k) * 6;
+#pragma unroll
+    for (int c = 0; c < 6; ++c) {
+      o[b * 12 + 2 * c] = lo[c];
+      o[b * 12 + 2 * c + 1] = lo[6 + c];
+    }
+  }
 }
 
 }  // namespace omprt_kernels

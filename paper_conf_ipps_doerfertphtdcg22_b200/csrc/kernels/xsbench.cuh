@@ -3,7 +3,8 @@
 //   for (i = first; i < first + count; ++i) verification[i - first] = lookup(i);
 // runtime-driven (omprt, with / without the oversubscription assumption) and
 // the bare CUDA twin (XSBench's CUDA version: one lookup per thread).  The verification
-// sum runs as a separate kernel (K11), or fused (OMPRT_FUSED_REDUCTION).
+// sum runs as a separate kernel (K11), or fused (OMPRT_FUSED_REDUCTION).  Both read
+// either the tables as specified or their B200 layouts (omprt_xs_build_accel).
 #pragma once
 #include "../host/runtime.cuh"
 #include "xs_body.cuh"
@@ -24,9 +25,12 @@ struct XSTraitsAssumeDebug : XSTraitsAssume {
 };
 
 constexpr int kXSThreads = 256;
+// 4 teams of 256 per SM (<= 64 registers): measured best occupancy / memory-parallelism
+// trade-off for this latency-bound gather (scripts/experiments/xs_explore.*).
+constexpr int kXSMinBlocks = 4;
 
-template <class Tr, bool Fused>
-__global__ void __launch_bounds__(kXSThreads)
+template <class Tr, bool Fused, bool Accel>
+__global__ void __launch_bounds__(kXSThreads, kXSMinBlocks)
     omprt_xs_rt(const __grid_constant__ XSTables t, uint64_t seed, int64_t first,
                 typename Tr::Idx count, uint64_t* __restrict__ verification,
                 unsigned long long* checksum, unsigned long long* partials, unsigned* ticket) {
@@ -34,7 +38,7 @@ __global__ void __launch_bounds__(kXSThreads)
   Team<Tr> team = init<Tr>();
   unsigned long long acc = 0;
   distribute_parallel_for(team, count, [&](Idx iv) {
-    const uint64_t v = xs_lookup_one(t, seed, first + iv);
+    const uint64_t v = xs_lookup_one<Accel>(t, seed, first + iv);
     if constexpr (Fused) acc += v;
     else verification[iv] = v;
   });
@@ -43,18 +47,19 @@ __global__ void __launch_bounds__(kXSThreads)
                   ticket);
 }
 
-// XSBench's CUDA kernel shape: one lookup per thread, early return past the end.
-template <bool Fused>
-__global__ void __launch_bounds__(kXSThreads)
+// XSBench's CUDA kernel shape: one lookup per thread, early return past the end; the fused
+// variant hand-codes the same reduction algorithm as the runtime.
+template <bool Fused, bool Accel>
+__global__ void __launch_bounds__(kXSThreads, kXSMinBlocks)
     cuda_xs_twin(const __grid_constant__ XSTables t, uint64_t seed, int64_t first, int32_t count,
                  uint64_t* __restrict__ verification, unsigned long long* checksum,
                  unsigned long long* partials, unsigned* ticket) {
   const int32_t i = blockIdx.x * blockDim.x + threadIdx.x;
   if constexpr (!Fused) {
     if (i >= count) return;
-    verification[i] = xs_lookup_one(t, seed, first + i);
+    verification[i] = xs_lookup_one<Accel>(t, seed, first + i);
   } else {
-    unsigned long long v = i < count ? xs_lookup_one(t, seed, first + i) : 0ull;
+    unsigned long long v = i < count ? xs_lookup_one<Accel>(t, seed, first + i) : 0ull;
     __shared__ unsigned long long ws[32];
     __shared__ unsigned last;
     for (int off = 16; off > 0; off >>= 1) v += __shfl_xor_sync(0xffffffffu, v, off);
@@ -102,27 +107,42 @@ __global__ void __launch_bounds__(512)
   league_reduce(team, team_reduce_to_main(team, acc, Plus{}), Plus{}, out, partials, ticket);
 }
 
-OMPRT_REGISTER_KERNEL(omprt_xs_rt, omprt_xs_rt<XSTraits, false>)
-OMPRT_REGISTER_KERNEL(omprt_xs_rt_assume, omprt_xs_rt<XSTraitsAssume, false>)
-OMPRT_REGISTER_KERNEL(omprt_xs_rt_fused, omprt_xs_rt<XSTraitsAssume, true>)
-OMPRT_REGISTER_KERNEL(omprt_xs_rt_debug, omprt_xs_rt<XSTraitsDebug, false>)
-OMPRT_REGISTER_KERNEL(cuda_xs_twin, cuda_xs_twin<false>)
-OMPRT_REGISTER_KERNEL(cuda_xs_twin_fused, cuda_xs_twin<true>)
+OMPRT_REGISTER_KERNEL(omprt_xs_rt, omprt_xs_rt<XSTraits, false, false>)
+OMPRT_REGISTER_KERNEL(omprt_xs_rt_assume, omprt_xs_rt<XSTraitsAssume, false, false>)
+OMPRT_REGISTER_KERNEL(omprt_xs_rt_fused, omprt_xs_rt<XSTraitsAssume, true, false>)
+OMPRT_REGISTER_KERNEL(omprt_xs_rt_debug, omprt_xs_rt<XSTraitsDebug, false, false>)
+OMPRT_REGISTER_KERNEL(omprt_xs_rt_accel, omprt_xs_rt<XSTraits, false, true>)
+OMPRT_REGISTER_KERNEL(omprt_xs_rt_assume_accel, omprt_xs_rt<XSTraitsAssume, false, true>)
+OMPRT_REGISTER_KERNEL(omprt_xs_rt_fused_accel, omprt_xs_rt<XSTraitsAssume, true, true>)
+OMPRT_REGISTER_KERNEL(cuda_xs_twin, cuda_xs_twin<false, false>)
+OMPRT_REGISTER_KERNEL(cuda_xs_twin_fused, cuda_xs_twin<true, false>)
+OMPRT_REGISTER_KERNEL(cuda_xs_twin_accel, cuda_xs_twin<false, true>)
+OMPRT_REGISTER_KERNEL(cuda_xs_twin_fused_accel, cuda_xs_twin<true, true>)
 OMPRT_REGISTER_KERNEL(omprt_u64_sum_rt, omprt_u64_sum_rt<SumTraits>)
 
 inline XSTables to_dev(const omprt_xs_tables& a) {
   return XSTables{a.nuclide_grid, a.unionized, a.index_grid, a.num_nucs, a.mats, a.concs,
-                  a.n_isotopes, a.n_gridpoints, a.max_num_nucs, 0, a.n_union};
+                  a.n_isotopes, a.n_gridpoints, a.max_num_nucs, 0, a.n_union,
+                  a.bins, a.index_grid16, a.brackets, a.log2_bins, 0};
+}
+
+inline bool xs_has_accel(const omprt_xs_tables& t) {
+  return t.bins != nullptr && t.index_grid16 != nullptr && t.brackets != nullptr;
 }
 
 inline int xs_validate(const omprt_xs_tables& t, int64_t count, uint64_t* ver, uint64_t* ck,
                        int32_t& teams, int32_t threads, uint32_t flags, Workspace* w) {
   OMPRT_CHECK_ARG(count >= 0 && count < (1ll << 31), "count must be in [0, 2^31)");
   OMPRT_CHECK_ARG(threads == kXSThreads, "threads must be %d", kXSThreads);
-  OMPRT_CHECK_ARG(t.nuclide_grid && t.unionized && t.index_grid && t.num_nucs && t.mats &&
-                      t.concs && t.n_union >= 2 && t.n_union < (1ll << 31) &&
-                      t.n_gridpoints >= 2 && t.n_isotopes > 0,
+  OMPRT_CHECK_ARG(t.unionized && t.num_nucs && t.mats && t.concs && t.n_union >= 2 &&
+                      t.n_union < (1ll << 31) && t.n_gridpoints >= 2 && t.n_isotopes > 0,
                   "bad XSBench tables");
+  const bool accel = xs_has_accel(t);
+  OMPRT_CHECK_ARG(accel || (t.nuclide_grid && t.index_grid), "bad XSBench tables");
+  OMPRT_CHECK_ARG(!accel || (t.log2_bins >= 1 && t.log2_bins <= 28),
+                  "accelerated layout: bad log2_bins");
+  OMPRT_CHECK_ARG(accel || (!t.bins && !t.index_grid16 && !t.brackets),
+                  "accelerated layout: bins, index_grid16 and brackets go together");
   const bool fused = flags & OMPRT_FUSED_REDUCTION;
   OMPRT_CHECK_ARG(fused ? ck != nullptr : (ver != nullptr || count == 0),
                   fused ? "fused reduction needs checksum_inout" : "verification is required");
@@ -154,6 +174,37 @@ inline int launch_u64_sum(const uint64_t* v, int64_t n, uint64_t* out, Workspace
   return check_launch("omprt_u64_sum_rt");
 }
 
+inline int xs_accel_sizes(int32_t n_isotopes, int32_t n_gridpoints, int64_t n_union,
+                          int32_t log2_bins, uint64_t* sizes) {
+  OMPRT_CHECK_ARG(n_isotopes > 0 && n_gridpoints >= 2 && n_gridpoints <= 65536 &&
+                      n_union >= 2 && log2_bins >= 1 && log2_bins <= 28 && sizes,
+                  "omprt_xs_accel_sizes: bad arguments (n_gridpoints must be <= 65536)");
+  sizes[0] = sizeof(int32_t) * ((1ull << log2_bins) + 1);
+  sizes[1] = sizeof(uint16_t) * (uint64_t)n_union * n_isotopes;
+  sizes[2] = sizeof(double) * 12ull * n_isotopes * (n_gridpoints - 1);
+  return OMPRT_OK;
+}
+
+inline int launch_xs_accel(omprt_xs_tables* t, int32_t* bins, uint16_t* idx16, double* brackets,
+                           int32_t log2_bins, cudaStream_t s) {
+  uint64_t sz[3];
+  if (int r = xs_accel_sizes(t->n_isotopes, t->n_gridpoints, t->n_union, log2_bins, sz)) return r;
+  OMPRT_CHECK_ARG(t->nuclide_grid && t->unionized && t->index_grid && bins && idx16 && brackets,
+                  "omprt_xs_build_accel: null pointer");
+  OMPRT_CHECK_ARG((uintptr_t)brackets % 32 == 0, "brackets must be 32 B aligned");
+  xs_build_bins<<<1024, 256, 0, s>>>(t->unionized, (int32_t)t->n_union, log2_bins, bins);
+  xs_build_index16<<<2048, 256, 0, s>>>(t->index_grid, idx16,
+                                        (int64_t)t->n_union * t->n_isotopes);
+  xs_build_brackets<<<2048, 256, 0, s>>>(t->nuclide_grid, brackets, t->n_isotopes,
+                                         t->n_gridpoints);
+  if (int r = check_launch("xs_build_accel")) return r;
+  t->bins = bins;
+  t->index_grid16 = idx16;
+  t->brackets = brackets;
+  t->log2_bins = log2_bins;
+  return OMPRT_OK;
+}
+
 }  // namespace omprt_kernels
 
 extern "C" int omprt_xs_lookup(omprt_xs_tables t, uint64_t seed, int64_t first, int64_t count,
@@ -168,22 +219,27 @@ extern "C" int omprt_xs_lookup(omprt_xs_tables t, uint64_t seed, int64_t first, 
   cudaStream_t s = as_stream(stream);
   const XSTables d = to_dev(t);
   const bool assume = flags & OMPRT_ASSUME_OVERSUB, fused = flags & OMPRT_FUSED_REDUCTION,
-             debug = flags & OMPRT_DEBUG_BUILD;
+             debug = flags & OMPRT_DEBUG_BUILD, accel = xs_has_accel(t);
   auto* ck = (unsigned long long*)checksum_inout;
   auto* p = (unsigned long long*)w->partials;
   unsigned* tk = w->tickets + 1;
   const int32_t n = (int32_t)count;
-#define OMPRT_XS(TR, F) \
-  omprt_xs_rt<TR, F><<<teams, threads, 0, s>>>(d, seed, first, n, verification, ck, p, tk)
-  if (fused) {
-    if (assume) OMPRT_XS(XSTraitsAssume, true);
-    else OMPRT_XS(XSTraits, true);
-  } else if (debug) {
-    if (assume) OMPRT_XS(XSTraitsAssumeDebug, false);
-    else OMPRT_XS(XSTraitsDebug, false);
+#define OMPRT_XS(TR, F, A) \
+  omprt_xs_rt<TR, F, A><<<teams, threads, 0, s>>>(d, seed, first, n, verification, ck, p, tk)
+  if (debug) {
+    OMPRT_CHECK_ARG(!fused && !accel, "the debug build covers the plain, unfused kernel");
+    if (assume) OMPRT_XS(XSTraitsAssumeDebug, false, false);
+    else OMPRT_XS(XSTraitsDebug, false, false);
+  } else if (accel) {
+    if (fused && assume) OMPRT_XS(XSTraitsAssume, true, true);
+    else if (fused) OMPRT_XS(XSTraits, true, true);
+    else if (assume) OMPRT_XS(XSTraitsAssume, false, true);
+    else OMPRT_XS(XSTraits, false, true);
   } else {
-    if (assume) OMPRT_XS(XSTraitsAssume, false);
-    else OMPRT_XS(XSTraits, false);
+    if (fused && assume) OMPRT_XS(XSTraitsAssume, true, false);
+    else if (fused) OMPRT_XS(XSTraits, true, false);
+    else if (assume) OMPRT_XS(XSTraitsAssume, false, false);
+    else OMPRT_XS(XSTraits, false, false);
   }
 #undef OMPRT_XS
   return check_launch("omprt_xs_rt");
@@ -204,13 +260,15 @@ extern "C" int omprt_cuda_xs_lookup(omprt_xs_tables t, uint64_t seed, int64_t fi
   if (count == 0) return OMPRT_OK;
   cudaStream_t s = as_stream(stream);
   const XSTables d = to_dev(t);
-  if (flags & OMPRT_FUSED_REDUCTION)
-    cuda_xs_twin<true><<<tm, threads, 0, s>>>(d, seed, first, (int32_t)count, verification,
-                                              (unsigned long long*)checksum_inout,
-                                              (unsigned long long*)w->partials, w->tickets + 1);
-  else
-    cuda_xs_twin<false><<<tm, threads, 0, s>>>(d, seed, first, (int32_t)count, verification,
-                                               nullptr, nullptr, nullptr);
+  const bool fused = flags & OMPRT_FUSED_REDUCTION, accel = xs_has_accel(t);
+  auto* ck = (unsigned long long*)checksum_inout;
+  auto* p = (unsigned long long*)w->partials;
+  unsigned* tk = w->tickets + 1;
+  const int32_t n = (int32_t)count;
+  if (fused && accel) cuda_xs_twin<true, true><<<tm, threads, 0, s>>>(d, seed, first, n, verification, ck, p, tk);
+  else if (fused) cuda_xs_twin<true, false><<<tm, threads, 0, s>>>(d, seed, first, n, verification, ck, p, tk);
+  else if (accel) cuda_xs_twin<false, true><<<tm, threads, 0, s>>>(d, seed, first, n, verification, nullptr, nullptr, nullptr);
+  else cuda_xs_twin<false, false><<<tm, threads, 0, s>>>(d, seed, first, n, verification, nullptr, nullptr, nullptr);
   return check_launch("cuda_xs_twin");
 }
 
@@ -221,8 +279,22 @@ extern "C" int omprt_u64_sum(const uint64_t* v, int64_t n, uint64_t* out_inout, 
   return launch_u64_sum(v, n, out_inout, w, as_stream(stream));
 }
 
-// End to end with host tables: map(to: tables) -> lookups (fused reduction) ->
-// map(from: checksum).  Synchronous on `stream`.
+extern "C" int omprt_xs_accel_sizes(int32_t n_isotopes, int32_t n_gridpoints, int64_t n_union,
+                                    int32_t log2_bins, uint64_t* sizes) {
+  return omprt_kernels::xs_accel_sizes(n_isotopes, n_gridpoints, n_union, log2_bins, sizes);
+}
+
+extern "C" int omprt_xs_build_accel(omprt_xs_tables* t, int32_t* bins, uint16_t* index_grid16,
+                                    double* brackets, int32_t log2_bins, void* stream) {
+  using namespace omprt_kernels;
+  Workspace* w;
+  if (int r = current_ws(&w)) return r;
+  OMPRT_CHECK_ARG(t != nullptr, "omprt_xs_build_accel: null tables");
+  return launch_xs_accel(t, bins, index_grid16, brackets, log2_bins, as_stream(stream));
+}
+
+// End to end with host tables: map(to: tables) -> (accelerated layouts built on the device)
+// -> lookups (fused reduction) -> map(from: checksum).  Synchronous on `stream`.
 extern "C" int omprt_xs_run_host(omprt_xs_tables h, uint64_t seed, int64_t first, int64_t count,
                                  int32_t threads, uint32_t flags, uint64_t* checksum_host,
                                  uint64_t* h2d_bytes, uint64_t* d2h_bytes, void* stream) {
@@ -239,8 +311,13 @@ extern "C" int omprt_xs_run_host(omprt_xs_tables h, uint64_t seed, int64_t first
   const size_t n_num = 12 * sizeof(int32_t);
   const size_t n_mat = (size_t)12 * h.max_num_nucs * sizeof(int32_t);
   const size_t n_con = (size_t)12 * h.max_num_nucs * sizeof(double);
+  const bool accel = (flags & OMPRT_XS_ACCEL) && h.n_gridpoints <= 65536;
+  const int32_t log2_bins = 16;
+  uint64_t asz[3] = {0, 0, 0};
+  if (accel) xs_accel_sizes(h.n_isotopes, h.n_gridpoints, h.n_union, log2_bins, asz);
   auto al = [](size_t b) { return (b + 255) & ~size_t(255); };
-  const size_t total = al(n_grid) + al(n_uni) + al(n_idx) + al(n_num) + al(n_mat) + al(n_con);
+  const size_t total = al(n_grid) + al(n_uni) + al(n_idx) + al(n_num) + al(n_mat) + al(n_con) +
+                       al(asz[0]) + al(asz[1]) + al(asz[2]);
   if (w->xs_buf_bytes < total) {
     cudaFree(w->xs_buf);
     w->xs_buf = nullptr;
@@ -254,11 +331,12 @@ extern "C" int omprt_xs_run_host(omprt_xs_tables h, uint64_t seed, int64_t first
   unsigned char* b = (unsigned char*)w->xs_buf;
   omprt_xs_tables d = h;
   size_t off = 0;
+  bool ok = true;
   auto put = [&](const void* src, size_t bytes) -> const void* {
     void* dst = b + off;
     off += al(bytes);
-    return cudaMemcpyAsync(dst, src, bytes, cudaMemcpyHostToDevice, s) == cudaSuccess ? dst
-                                                                                      : nullptr;
+    ok = ok && cudaMemcpyAsync(dst, src, bytes, cudaMemcpyHostToDevice, s) == cudaSuccess;
+    return dst;
   };
   d.nuclide_grid = (const double*)put(h.nuclide_grid, n_grid);
   d.unionized = (const double*)put(h.unionized, n_uni);
@@ -266,12 +344,25 @@ extern "C" int omprt_xs_run_host(omprt_xs_tables h, uint64_t seed, int64_t first
   d.num_nucs = (const int32_t*)put(h.num_nucs, n_num);
   d.mats = (const int32_t*)put(h.mats, n_mat);
   d.concs = (const double*)put(h.concs, n_con);
-  if (!d.nuclide_grid || !d.unionized || !d.index_grid || !d.num_nucs || !d.mats || !d.concs)
-    return set_error(OMPRT_E_CUDA, "omprt_xs_run_host: H2D copy failed");
+  if (!ok) return set_error(OMPRT_E_CUDA, "omprt_xs_run_host: H2D copy failed");
+  d.bins = nullptr;
+  d.index_grid16 = nullptr;
+  d.brackets = nullptr;
+  if (accel) {
+    int32_t* bins = (int32_t*)(b + off);
+    off += al(asz[0]);
+    uint16_t* i16 = (uint16_t*)(b + off);
+    off += al(asz[1]);
+    double* br = (double*)(b + off);
+    off += al(asz[2]);
+    if (int r = launch_xs_accel(&d, bins, i16, br, log2_bins, s)) return r;
+  }
   uint64_t* ck = w->scratch_u64;
   OMPRT_CUDA_TRY(cudaMemsetAsync(ck, 0, sizeof(uint64_t), s));
   if (int r = omprt_xs_lookup(d, seed, first, count, nullptr, ck, 0, threads,
-                              (flags | OMPRT_FUSED_REDUCTION | OMPRT_ASSUME_OVERSUB), stream))
+                              (flags & ~OMPRT_XS_ACCEL) | OMPRT_FUSED_REDUCTION |
+                                  OMPRT_ASSUME_OVERSUB,
+                              stream))
     return r;
   OMPRT_CUDA_TRY(cudaMemcpyAsync(checksum_host, ck, sizeof(uint64_t), cudaMemcpyDeviceToHost, s));
   OMPRT_CUDA_TRY(cudaStreamSynchronize(s));

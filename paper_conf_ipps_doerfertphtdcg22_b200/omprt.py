@@ -31,13 +31,14 @@ OMPRT_POSTLOGUE = 1 << 6
 OMPRT_THREAD_STATES = 1 << 7
 OMPRT_FUSED_REDUCTION = 1 << 8
 OMPRT_UNCHECKED = 1 << 9
+OMPRT_XS_ACCEL = 1 << 10
 
 # Every symbol include/omprt.h declares (checked by tests/test_abi.py).
 EXPORTS = [
     "omprt_init", "omprt_fini", "omprt_device_status", "omprt_last_error", "omprt_static_owner",
     "omprt_spmd_axpy_sum", "omprt_cuda_axpy_sum", "omprt_generic_team", "omprt_cuda_generic_team",
     "omprt_icv_probe", "omprt_xs_lookup", "omprt_cuda_xs_lookup", "omprt_u64_sum",
-    "omprt_xs_run_host", "omprt_rs_lookup", "omprt_cuda_rs_lookup", "omprt_su3_mult",
+    "omprt_xs_run_host", "omprt_xs_accel_sizes", "omprt_xs_build_accel", "omprt_rs_lookup", "omprt_cuda_rs_lookup", "omprt_su3_mult",
     "omprt_cuda_su3_mult", "omprt_kernel_count", "omprt_kernel_name", "omprt_kernel_attrs",
 ]
 
@@ -57,7 +58,9 @@ class XSTablesC(C.Structure):
     _fields_ = [("nuclide_grid", C.c_void_p), ("unionized", C.c_void_p), ("index_grid", C.c_void_p),
                 ("num_nucs", C.c_void_p), ("mats", C.c_void_p), ("concs", C.c_void_p),
                 ("n_isotopes", C.c_int32), ("n_gridpoints", C.c_int32),
-                ("max_num_nucs", C.c_int32), ("pad", C.c_int32), ("n_union", C.c_int64)]
+                ("max_num_nucs", C.c_int32), ("pad", C.c_int32), ("n_union", C.c_int64),
+                ("bins", C.c_void_p), ("index_grid16", C.c_void_p), ("brackets", C.c_void_p),
+                ("log2_bins", C.c_int32), ("pad2", C.c_int32)]
 
 
 class RSTablesC(C.Structure):
@@ -84,6 +87,8 @@ _SIGS = {
     "omprt_xs_lookup": [XSTablesC, _u64, _i64, _i64, _vp, _vp, _i32, _i32, _u32, _vp],
     "omprt_cuda_xs_lookup": [XSTablesC, _u64, _i64, _i64, _vp, _vp, _i32, _i32, _u32, _vp],
     "omprt_u64_sum": [_vp, _i64, _vp, _vp],
+    "omprt_xs_accel_sizes": [_i32, _i32, _i64, _i32, C.POINTER(_u64)],
+    "omprt_xs_build_accel": [C.POINTER(XSTablesC), _vp, _vp, _vp, _i32, _vp],
     "omprt_xs_run_host": [XSTablesC, _u64, _i64, _i64, _i32, _u32, C.POINTER(_u64),
                           C.POINTER(_u64), C.POINTER(_u64), _vp],
     "omprt_rs_lookup": [RSTablesC, _u64, _i64, _i64, _vp, _vp, _i32, _i32, _u32, _vp],
@@ -207,9 +212,10 @@ def omprt_icv_probe(teams, threads, nested_request, rec, flags=0, stream=None):
 
 # ---------------------------------------------------------------- C3
 class XSDeviceTables:
-    """Device copies (torch tensors) of gen.XSTables and the by-value C struct."""
+    """Device copies (torch tensors) of gen.XSTables and the by-value C struct.  With
+    accel=True the B200 layouts are built on the device (omprt_xs_build_accel)."""
 
-    def __init__(self, t, device="cuda"):
+    def __init__(self, t, device="cuda", accel=False, log2_bins=16):
         import torch
         self.host = t
         self.nuclide_grid = torch.from_numpy(t.nuclide_grid).to(device)
@@ -220,7 +226,33 @@ class XSDeviceTables:
         self.concs = torch.from_numpy(t.concs).to(device)
         self.c = XSTablesC(_p(self.nuclide_grid), _p(self.unionized), _p(self.index_grid),
                            _p(self.num_nucs), _p(self.mats), _p(self.concs), t.n_isotopes,
-                           t.n_gridpoints, t.max_num_nucs, 0, t.n_union)
+                           t.n_gridpoints, t.max_num_nucs, 0, t.n_union, None, None, None, 0, 0)
+        if accel:
+            sizes = omprt_xs_accel_sizes(t.n_isotopes, t.n_gridpoints, t.n_union, log2_bins)
+            self.bins = torch.empty(sizes[0] // 4, dtype=torch.int32, device=device)
+            self.index_grid16 = torch.empty(sizes[1] // 2, dtype=torch.uint16, device=device)
+            self.brackets = torch.empty(sizes[2] // 8, dtype=torch.float64, device=device)
+            omprt_xs_build_accel(self, self.bins, self.index_grid16, self.brackets, log2_bins)
+
+    def plain(self):
+        """A view of the same tables without the accelerated layouts."""
+        v = XSDeviceTables.__new__(XSDeviceTables)
+        v.__dict__.update(self.__dict__)
+        v.c = XSTablesC.from_buffer_copy(self.c)
+        v.c.bins = v.c.index_grid16 = v.c.brackets = None
+        v.c.log2_bins = 0
+        return v
+
+
+def omprt_xs_accel_sizes(n_isotopes, n_gridpoints, n_union, log2_bins=16):
+    sz = (_u64 * 3)()
+    _check(load().omprt_xs_accel_sizes(n_isotopes, n_gridpoints, n_union, log2_bins, sz))
+    return list(sz)
+
+
+def omprt_xs_build_accel(tables, bins, index_grid16, brackets, log2_bins=16, stream=None):
+    return _check(load().omprt_xs_build_accel(C.byref(tables.c), _p(bins), _p(index_grid16),
+                                              _p(brackets), log2_bins, _stream(stream)))
 
 
 def xs_host_struct(t, pinned=None):
@@ -229,7 +261,7 @@ def xs_host_struct(t, pinned=None):
     g = lambda k: src.get(k, getattr(t, k))
     return XSTablesC(_hp(g("nuclide_grid")), _hp(g("unionized")), _hp(g("index_grid")),
                      _hp(g("num_nucs")), _hp(g("mats")), _hp(g("concs")), t.n_isotopes,
-                     t.n_gridpoints, t.max_num_nucs, 0, t.n_union)
+                     t.n_gridpoints, t.max_num_nucs, 0, t.n_union, None, None, None, 0, 0)
 
 
 def omprt_xs_lookup(tables, seed, first, count, verification, checksum_inout=None, teams=0,

@@ -1,6 +1,7 @@
 #!/bin/bash
-# One GPU session: parity tests, smoke, bench, ncu launch list + full captures.
-# Usage (under gpurun): bash scripts/gpu_round.sh [tag]
+# One GPU session: parity tests, smoke, bench, reference arm, ncu launch list + full
+# captures of the headline kernel and its twin (exported to CSV on the box; the two
+# .ncu-rep files come back too).  Usage (under gpurun): bash scripts/gpu_round.sh TAG
 TAG=${1:-r01}
 OUT=gpurun_out
 mkdir -p $OUT
@@ -14,10 +15,12 @@ echo "smoke exit $?" >> $OUT/smoke_$TAG.txt
 timeout 900 python bench.py --steps 10 --warmup 3 > $OUT/bench_$TAG.txt 2>&1
 echo "bench exit $?" >> $OUT/bench_$TAG.txt
 timeout 300 python bench.py --impl reference --steps 2 --warmup 1 > $OUT/bench_ref_$TAG.txt 2>&1
-timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none -c 200 --csv \
-  --log-file $OUT/launches_$TAG.csv python bench.py --steps 2 --warmup 1 --no-e2e > $OUT/ncu_launch_stdout_$TAG.txt 2>&1
-timeout 900 ncu --set full --clock-control none --import-source on -k regex:omprt_xs_rt -s 1 -c 1 \
-  -o $OUT/prof_xs_rt_$TAG python bench.py --steps 1 --warmup 1 --no-e2e --no-secondary > $OUT/ncu_full_stdout_$TAG.txt 2>&1
-timeout 900 ncu --set full --clock-control none --import-source on -k regex:cuda_xs_twin -s 0 -c 1 \
-  -o $OUT/prof_xs_twin_$TAG python bench.py --steps 1 --warmup 1 --no-e2e --no-secondary >> $OUT/ncu_full_stdout_$TAG.txt 2>&1
-ls -la $OUT
+timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none -c 400 --csv \
+  --log-file $OUT/launches_$TAG.csv python bench.py --steps 2 --warmup 1 --no-e2e --no-secondary > $OUT/ncu_launch_stdout_$TAG.txt 2>&1
+for K in omprt_xs_rt cuda_xs_twin; do
+  timeout 900 ncu --set full --clock-control none --import-source on -k regex:$K -s 1 -c 1 \
+    -o $OUT/prof_${K}_$TAG python bench.py --steps 1 --warmup 1 --no-e2e --no-secondary > $OUT/ncu_full_${K}_$TAG.txt 2>&1
+  ncu -i $OUT/prof_${K}_$TAG.ncu-rep --page raw --csv --print-units base > $OUT/raw_${K}_$TAG.csv 2>&1
+  ncu -i $OUT/prof_${K}_$TAG.ncu-rep --page source --csv --print-units base > $OUT/src_${K}_$TAG.csv 2>&1
+done
+du -sh $OUT

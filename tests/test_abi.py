@@ -57,6 +57,15 @@ def test_static_owner_host_function(lib):
     assert e.value.code == omprt.OMPRT_E_INVAL
 
 
+def test_xs_accel_sizes_host_function(lib):
+    from paper_conf_ipps_doerfertphtdcg22_b200 import omprt
+    sz = omprt.omprt_xs_accel_sizes(68, 11303, 768604, 16)
+    assert sz == [4 * (65536 + 1), 2 * 768604 * 68, 8 * 12 * 68 * 11302]
+    with pytest.raises(omprt.OmprtError) as e:
+        omprt.omprt_xs_accel_sizes(68, 70000, 768604, 16)  # 16-bit index cannot hold it
+    assert e.value.code == omprt.OMPRT_E_INVAL
+
+
 def test_kernel_registry(lib):
     from paper_conf_ipps_doerfertphtdcg22_b200 import omprt
     names = [omprt.omprt_kernel_name(i) for i in range(omprt.omprt_kernel_count())]

@@ -11,6 +11,9 @@ PAIRS = [
     ("omprt_xs_rt_assume", "cuda_xs_twin", True),
     ("omprt_xs_rt", "cuda_xs_twin", True),
     ("omprt_xs_rt_fused", "cuda_xs_twin_fused", True),
+    ("omprt_xs_rt_assume_accel", "cuda_xs_twin_accel", True),
+    ("omprt_xs_rt_accel", "cuda_xs_twin_accel", True),
+    ("omprt_xs_rt_fused_accel", "cuda_xs_twin_fused_accel", True),
     ("omprt_rs_rt_assume", "cuda_rs_twin", True),
     ("omprt_rs_rt", "cuda_rs_twin", True),
     ("omprt_su3_rt", "cuda_su3_twin", True),

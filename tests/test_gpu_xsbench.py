@@ -17,8 +17,13 @@ SEED = gen.XS_LOOKUP_SEED
 
 
 @pytest.fixture(scope="module")
-def xs_dev(rt, xs_small):
-    return rt.XSDeviceTables(xs_small, DEV)
+def xs_acc(rt, xs_small):
+    return rt.XSDeviceTables(xs_small, DEV, accel=True)
+
+
+@pytest.fixture(scope="module")
+def xs_dev(xs_acc):
+    return xs_acc.plain()
 
 
 def _lookup(rt, d, first, count, which, flags=0):
@@ -39,13 +44,36 @@ def test_verification_bit_exact(rt, xs_dev, xs_small, variant):
     assert (got == ref).all()
 
 
+@pytest.mark.parametrize("variant", ["rt", "rt_assume", "twin"])
+def test_accel_layout_bit_exact(rt, xs_acc, xs_small, variant):
+    """The B200 layouts (binned search, 16-bit index, bracket records) give the same bits."""
+    first, count = 12345, (1 << 17) + 29
+    flags = rt.OMPRT_ASSUME_OVERSUB if variant == "rt_assume" else 0
+    got = _lookup(rt, xs_acc, first, count, "twin" if variant == "twin" else "rt", flags)
+    ref = oracle.xs_lookup(xs_small, first, count, threads=os.cpu_count() or 1)
+    assert (got == ref).all()
+
+
+def test_accel_tables_content(rt, xs_acc, xs_small):
+    bins = xs_acc.bins.cpu().numpy()
+    H = 1 << 16
+    edges = np.arange(H + 1, dtype=np.float64) / H
+    U = xs_small.unionized
+    assert (bins == np.clip(np.searchsorted(U, edges, side="right") - 1, 0, U.size - 2)).all()
+    assert (xs_acc.index_grid16.cpu().numpy().astype(np.int32) ==
+            xs_small.index_grid.reshape(-1)).all()
+    br = xs_acc.brackets.cpu().numpy().reshape(xs_small.n_isotopes, xs_small.n_gridpoints - 1, 6, 2)
+    G = xs_small.nuclide_grid.reshape(xs_small.n_isotopes, xs_small.n_gridpoints, 6)
+    assert (br[..., 0] == G[:, :-1, :]).all() and (br[..., 1] == G[:, 1:, :]).all()
+
+
 def test_edge_sizes(rt, xs_dev, xs_small):
     for first, count in [(0, 0), (0, 1), (5, 255), (5, 256), (5, 257)]:
         got = _lookup(rt, xs_dev, first, count, "rt", rt.OMPRT_ASSUME_OVERSUB)
         assert (got == oracle.xs_lookup(xs_small, first, count)).all()
 
 
-def test_checksum_separate_and_fused(rt, xs_dev, xs_small):
+def test_checksum_separate_and_fused(rt, xs_dev, xs_acc, xs_small):
     n = 1 << 20
     ref = oracle.xs_lookup(xs_small, 0, n, threads=os.cpu_count() or 1)
     ref_sum = int(ref.sum())
@@ -55,11 +83,14 @@ def test_checksum_separate_and_fused(rt, xs_dev, xs_small):
     rt.omprt_u64_sum(ver, n, ck)
     torch.cuda.synchronize()
     assert int(ck.cpu().numpy()[0]) == ref_sum + 5
-    for fn, flags in [(rt.omprt_xs_lookup, rt.OMPRT_ASSUME_OVERSUB | rt.OMPRT_FUSED_REDUCTION),
-                      (rt.omprt_xs_lookup, rt.OMPRT_FUSED_REDUCTION),
-                      (rt.omprt_cuda_xs_lookup, rt.OMPRT_FUSED_REDUCTION)]:
+    for fn, flags, tabs in [
+            (rt.omprt_xs_lookup, rt.OMPRT_ASSUME_OVERSUB | rt.OMPRT_FUSED_REDUCTION, xs_dev),
+            (rt.omprt_xs_lookup, rt.OMPRT_FUSED_REDUCTION, xs_dev),
+            (rt.omprt_cuda_xs_lookup, rt.OMPRT_FUSED_REDUCTION, xs_dev),
+            (rt.omprt_xs_lookup, rt.OMPRT_ASSUME_OVERSUB | rt.OMPRT_FUSED_REDUCTION, xs_acc),
+            (rt.omprt_cuda_xs_lookup, rt.OMPRT_FUSED_REDUCTION, xs_acc)]:
         ck = torch.zeros(1, dtype=torch.uint64, device=DEV)
-        fn(xs_dev, SEED, 0, n, None, ck, 0, 256, flags)
+        fn(tabs, SEED, 0, n, None, ck, 0, 256, flags)
         torch.cuda.synchronize()
         assert int(ck.cpu().numpy()[0]) == ref_sum
 
@@ -84,12 +115,13 @@ def test_u64_sum_wraps(rt):
     assert int(out.cpu().numpy()[0]) == (int(v.size) * ((1 << 63) + 12345)) % 2**64
 
 
-def test_full_size_17M(rt, xs_dev, xs_small):
-    """BASELINE configs[2] at full size, in the launch configuration bench.py times:
-    sampled lookups bit-exact, full checksum equal to the oracle's (all host cores)."""
+def test_full_size_17M(rt, xs_acc, xs_small):
+    """BASELINE configs[2] at full size, in the launch configuration bench.py times
+    (runtime-driven, assumption, B200 layouts): sampled lookups bit-exact, then every lookup
+    and the checksum against the oracle (all host cores)."""
     n = 17_000_000
     ver = torch.zeros(n, dtype=torch.uint64, device=DEV)
-    rt.omprt_xs_lookup(xs_dev, SEED, 0, n, ver, None, 0, 256, rt.OMPRT_ASSUME_OVERSUB)
+    rt.omprt_xs_lookup(xs_acc, SEED, 0, n, ver, None, 0, 256, rt.OMPRT_ASSUME_OVERSUB)
     ck = torch.zeros(1, dtype=torch.uint64, device=DEV)
     rt.omprt_u64_sum(ver, n, ck)
     torch.cuda.synchronize()
@@ -109,6 +141,8 @@ def test_end_to_end_host_tables(rt, xs_small):
               for k in ("nuclide_grid", "unionized", "index_grid", "num_nucs", "mats", "concs")}
     hs = rt.xs_host_struct(xs_small, pinned)
     n = 100_000
-    ck, h2d, d2h = rt.omprt_xs_run_host(hs, SEED, 0, n)
-    assert ck == int(oracle.xs_lookup(xs_small, 0, n).sum())
-    assert h2d == xs_small.nbytes() and d2h == 8
+    ref = int(oracle.xs_lookup(xs_small, 0, n).sum())
+    for flags in (0, rt.OMPRT_XS_ACCEL):
+        ck, h2d, d2h = rt.omprt_xs_run_host(hs, SEED, 0, n, 256, flags)
+        assert ck == ref
+        assert h2d == xs_small.nbytes() and d2h == 8

@@ -131,7 +131,7 @@ __device__ __forceinline__ void ld_nc_v4f64(const double* p, double& a, double& 
 // int32 index grid, 48 B gridpoint records: 6 x 16 B loads per nuclide).  Accel = true reads
 // the same values from the B200 layouts (binned search, 16-bit index grid, 96 B bracket
 // records loaded by 3 x 256-bit loads) -- identical results, fewer L1 wavefronts.
-template <bool Accel>
+template <bool Accel, int kUnroll = 4>
 __device__ __forceinline__ uint64_t xs_lookup_one(const XSTables& t, uint64_t seed0, int64_t i) {
   uint64_t seed = lcg_fast_forward(seed0, 2ull * (uint64_t)i);
   const double E = lcg_double(seed);
@@ -143,7 +143,7 @@ __device__ __forceinline__ uint64_t xs_lookup_one(const XSTables& t, uint64_t se
   const double* __restrict__ crow = t.concs + mat * t.max_num_nucs;
   const int64_t row = (int64_t)idx * t.n_isotopes;
   double m0 = 0.0, m1 = 0.0, m2 = 0.0, m3 = 0.0, m4 = 0.0;
-#pragma unroll 4
+#pragma unroll kUnroll
   for (int j = 0; j < nn; ++j) {
     const int32_t p = __ldg(mrow + j);
     const double conc = __ldg(crow + j);

@@ -65,12 +65,15 @@ inline constexpr bool kHasStack = Tr::stack_bytes > 0 || Tr::dynamic_stack;
 // Shared-memory stack allocation granule (16 B alignment).
 inline constexpr unsigned kStackAlign = 16;
 
-// Named hardware barriers.  Fig. 6 uses barrier 8 for the runtime's aligned
-// barrier so it never aliases the user's __syncthreads (barrier 0); the generic-mode state
-// machine uses its own non-aligned barriers.
-inline constexpr unsigned kAlignedBarrierId = 8;
-inline constexpr unsigned kStateMachineBarrierId = 9;
-inline constexpr unsigned kJoinBarrierId = 10;
+// Named hardware barriers.  Fig. 6 puts the runtime's aligned barrier on
+// barrier 8 to keep it apart from the user's __syncthreads (barrier 0).  On sm_100 a CTA
+// reserves (highest id + 1) barriers from the SM's pool, so ids 8-10 cap residency at
+// 6 CTAs/SM (ncu launch__occupancy_limit_barriers = 6, profiles/ncu_generic_x01): the
+// aligned barrier uses barrier 0 (it is a full-CTA aligned barrier, exactly what
+// __syncthreads is) and the state machine ids 1 and 2 -- 3 barriers per CTA.
+inline constexpr unsigned kAlignedBarrierId = 0;
+inline constexpr unsigned kStateMachineBarrierId = 1;
+inline constexpr unsigned kJoinBarrierId = 2;
 
 // Error codes shared with the host ABI (include/omprt.h).
 enum : int {

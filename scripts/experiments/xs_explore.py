@@ -3,11 +3,12 @@ import ctypes as C, os, subprocess, sys, statistics, json
 ROOT = os.path.dirname(os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 sys.path.insert(0, ROOT)
 HERE = os.path.dirname(os.path.abspath(__file__))
-SO = os.path.join(HERE, "libxsx.so")
+SRC = os.environ.get("XSX_SRC", "xs_explore.cu")
+SO = os.path.join(HERE, "lib" + SRC.replace(".cu", ".so"))
 
 def build():
     subprocess.check_call(["nvcc", "-O3", "-std=c++17", "-gencode", "arch=compute_100a,code=sm_100a",
-                           "-lineinfo", "--shared", "-Xcompiler", "-fPIC", os.path.join(HERE, "xs_explore.cu"), "-o", SO])
+                           "-lineinfo", "--shared", "-Xcompiler", "-fPIC", os.path.join(HERE, SRC), "-o", SO])
 
 def main():
     import torch, gen
@@ -18,7 +19,7 @@ def main():
     torch.cuda.set_device(0)
     omprt.omprt_init(0)
     t = gen.XSTables(**gen.XS_SMALL)
-    d = omprt.XSDeviceTables(t, "cuda")
+    d = omprt.XSDeviceTables(t, "cuda", accel=os.environ.get("XSX_ACCEL") == "1")
     L.xsx_prepare.argtypes = [omprt.XSTablesC]
     L.xsx_run.argtypes = [C.c_int, omprt.XSTablesC, C.c_uint64, C.c_int64, C.c_int32, C.c_void_p, C.c_void_p]
     assert L.xsx_prepare(d.c) == 0

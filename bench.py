@@ -366,6 +366,14 @@ def run_secondary(omprt, torch, gen, dev, stream, scrub):
     t_tw = _time(lambda: omprt.omprt_cuda_axpy_sum(n, x, bt, ct, at, s, 8, 128), stream, scrub)
     res["c1_axpy_sum_8x128"] = {"rt_ms": t_rt, "twin_ms": t_tw, "overhead": t_rt / t_tw - 1,
                                 "GBps_alg": 24 * n / t_rt / 1e6}
+    # NEXT f3: the same loop with schedule(static, 4): 256-bit chunk accesses
+    t_rt = _time(lambda: omprt.omprt_spmd_axpy_sum_chunked(n, 4, x, bt, ct, at, s, 8, 128),
+                 stream, scrub)
+    t_tw = _time(lambda: omprt.omprt_cuda_axpy_sum_chunked(n, 4, x, bt, ct, at, s, 8, 128),
+                 stream, scrub)
+    res["c1_axpy_sum_8x128_chunk4"] = {"rt_ms": t_rt, "twin_ms": t_tw,
+                                       "overhead": t_rt / t_tw - 1,
+                                       "GBps_alg": 24 * n / t_rt / 1e6}
     # C2: generic mode 4096 teams x 256, inner 256
     T = 4096
     inp = torch.from_numpy(gen.generic_inputs(T, 256)).to(dev)
@@ -375,8 +383,17 @@ def run_secondary(omprt, torch, gen, dev, stream, scrub):
     t_gs = _time(lambda: omprt.omprt_generic_team(T, 256, 256, inp, out, None, None,
                                                   omprt.OMPRT_GENERAL_SM), stream, scrub)
     t_tw = _time(lambda: omprt.omprt_cuda_generic_team(T, 256, 256, inp, out), stream, scrub)
+    A_ = omprt.OMPRT_ASSUME_OVERSUB
+    t_sp = _time(lambda: omprt.omprt_generic_team(T, 256, 256, inp, out, None, None,
+                                                  A_ | omprt.OMPRT_SPMDIZE), stream, scrub)
+    t_dg = _time(lambda: omprt.omprt_generic_team(T, 256, 256, inp, out, None, None,
+                                                  A_ | omprt.OMPRT_DEGLOBALIZE), stream, scrub)
+    t_db = _time(lambda: omprt.omprt_generic_team(T, 256, 256, inp, out, None, None,
+                                                  omprt.OMPRT_DEBUG_BUILD), stream, scrub)
     res["c2_generic_4096x256"] = {"rt_ms": t_rt, "rt_general_sm_ms": t_gs, "twin_ms": t_tw,
-                                  "overhead": t_rt / t_tw - 1}
+                                  "overhead": t_rt / t_tw - 1, "rt_spmdized_ms": t_sp,
+                                  "rt_deglobalized_ms": t_dg,
+                                  "rt_debug_build_env_off_ms": t_db}
     # C4: RSBench-shaped, 10M lookups (single GPU here)
     rs = gen.RSTables()
     rd = omprt.RSDeviceTables(rs, dev)

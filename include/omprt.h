@@ -77,6 +77,13 @@ extern "C" {
 /* omprt_xs_run_host: build and use the accelerated table layouts on the device (per call,
  * inside the end-to-end time). */
 #define OMPRT_XS_ACCEL (1u << 10)
+/* omprt_generic_team, NEXT f1 (P:174 SPMDization): the same target region in SPMD mode, the
+ * sequential prologue guarded (thread 0) and broadcast by an aligned barrier; no state
+ * machine.  inner_n <= 256. */
+#define OMPRT_SPMDIZE (1u << 11)
+/* omprt_generic_team, NEXT f2 (P:172 globalization elimination): generic mode with
+ * the globalized arrays in static team-local shared memory -- no stack (0 B).  inner_n <= 256. */
+#define OMPRT_DEGLOBALIZE (1u << 12)
 
 /* ---- runtime lifecycle ------------------------------------------------------------- */
 typedef struct {
@@ -113,6 +120,21 @@ int omprt_spmd_axpy_sum(int64_t n, double x, const double *b, const double *c, d
 int omprt_cuda_axpy_sum(int64_t n, double x, const double *b, const double *c, double *a,
                         double *sum_inout, int32_t teams, int32_t threads, uint32_t flags,
                         int32_t *owner, int32_t *count, void *stream);
+
+/* NEXT f3 -- C1 with a user chunk (Fig. 5 covers only "the absence of user-defined
+ * chunks"): dist_schedule(static, chunk) + schedule(static, chunk) on the combined scheme,
+ * chunk k = [k*chunk, min(n, (k+1)*chunk)) -> global thread k mod (teams*threads).  With
+ * chunk = 4 and 32 B-aligned a, b, c each chunk moves with 256-bit accesses.
+ * OMPRT_ASSUME_OVERSUB here means ceil(n/chunk) <= teams*threads.  Other arguments as
+ * omprt_spmd_axpy_sum (owner[i] = owning global thread). */
+int omprt_spmd_axpy_sum_chunked(int64_t n, int64_t chunk, double x, const double *b,
+                                const double *c, double *a, double *sum_inout, int32_t teams,
+                                int32_t threads, uint32_t flags, int32_t *owner, int32_t *count,
+                                void *stream);
+int omprt_cuda_axpy_sum_chunked(int64_t n, int64_t chunk, double x, const double *b,
+                                const double *c, double *a, double *sum_inout, int32_t teams,
+                                int32_t threads, uint32_t flags, int32_t *owner, int32_t *count,
+                                void *stream);
 
 /* ---- C2: generic-mode team kernel -------------------------------- */
 /* Per team t: the main thread builds globalized w[inner_n], perm[inner_n] with

@@ -69,6 +69,8 @@ def _declare(L):
         "oracle_fig5_simulate": (None, [C.c_int64, C.c_int32, C.c_int32, C.c_int, _i32p, _i32p]),
         "oracle_team_for_simulate": (None, [C.c_int64, C.c_int32, C.c_int, _i32p, _i32p]),
         "oracle_distribute_simulate": (None, [C.c_int64, C.c_int32, _i32p, _i32p]),
+        "oracle_static_chunk_owner_closed": (C.c_int, [C.c_int64, C.c_int64, C.c_int64, C.c_int64, C.c_int64, _i32p, _i32p]),
+        "oracle_chunk_simulate": (None, [C.c_int64, C.c_int64, C.c_int32, C.c_int32, C.c_int, _i32p, _i32p]),
         "oracle_axpy": (None, [C.c_int64, C.c_double, _f64p, _f64p, _f64p]),
         "oracle_sum_f64": (C.c_double, [_f64p, C.c_int64, C.c_double]),
         "oracle_sum_f64_ld": (C.c_longdouble, [_f64p, C.c_int64, C.c_double]),
@@ -130,6 +132,20 @@ def distribute_simulate(n, teams):
     owner = np.empty(n, np.int32)
     count = np.empty(n, np.int32)
     lib().oracle_distribute_simulate(n, teams, _p(owner, _i32p), _p(count, _i32p))
+    return owner, count
+
+
+def static_chunk_owner_closed(iv, n, chunk, teams, threads):
+    tm, th = C.c_int32(), C.c_int32()
+    r = lib().oracle_static_chunk_owner_closed(iv, n, chunk, teams, threads, C.byref(tm), C.byref(th))
+    return None if r else (tm.value, th.value)
+
+
+def chunk_simulate(n, chunk, teams, threads, assume_oversub=False):
+    owner = np.empty(n, np.int32)
+    count = np.empty(n, np.int32)
+    lib().oracle_chunk_simulate(n, chunk, teams, threads, int(assume_oversub), _p(owner, _i32p),
+                                _p(count, _i32p))
     return owner, count
 
 

@@ -48,6 +48,15 @@ void oracle_team_for_simulate(int64_t n, int32_t nthreads, int assume_oversub,
                               int32_t *owner, int32_t *count);
 void oracle_distribute_simulate(int64_t n, int32_t teams, int32_t *owner, int32_t *count);
 
+/* NEXT f3 (Fig. 5 covers only "the absence of user-defined chunks"; reading R-F3):
+ * static schedule with a user chunk C applied to the combined scheme, OpenMP round-robin:
+ * chunk k = iterations [kC, min(n, kC + C)) runs on global thread k mod (T*N).  C = 1 is
+ * Fig. 5.  Closed form and a literal per-thread simulation. */
+int oracle_static_chunk_owner_closed(int64_t iv, int64_t n, int64_t chunk, int64_t teams,
+                                     int64_t threads, int32_t *team, int32_t *thread);
+void oracle_chunk_simulate(int64_t n, int64_t chunk, int32_t teams, int32_t threads,
+                           int assume_oversub, int32_t *owner, int32_t *count);
+
 /* ---- C1: SPMD axpy + fp64 sum reduction (BASELINE configs[0]) -------------------------- */
 /* a[i] = fma(x, b[i], c[i]) (SURVEY Q12 reading: one rounding, explicit). */
 void oracle_axpy(int64_t n, double x, const double *b, const double *c, double *a);

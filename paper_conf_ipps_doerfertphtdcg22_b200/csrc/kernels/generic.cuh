@@ -90,9 +90,12 @@ struct GenRegion {
 };
 
 constexpr int kGenericMaxThreads = 256;
+// 8 teams of 256 per SM (<= 32 registers) for the runtime kernel AND the twin, so neither
+// comparison side is limited by a register count the other escapes.
+constexpr int kGenericMinBlocks = 8;
 
 template <class Tr, int kInner, bool Rec, bool Post>
-__global__ void __launch_bounds__(kGenericMaxThreads)
+__global__ void __launch_bounds__(kGenericMaxThreads, kGenericMinBlocks)
     omprt_generic_rt(int32_t inner_n_rt, const double* __restrict__ in, double* __restrict__ out,
                      int32_t* owner, double* post) {
   using R = GenRegion<Rec, Post>;
@@ -124,7 +127,7 @@ __global__ void __launch_bounds__(kGenericMaxThreads)
 
 // Bare CUDA twin.
 template <int kInner, bool Rec, bool Post>
-__global__ void __launch_bounds__(kGenericMaxThreads)
+__global__ void __launch_bounds__(kGenericMaxThreads, kGenericMinBlocks)
     cuda_generic_twin(int32_t inner_n_rt, const double* __restrict__ in,
                       double* __restrict__ out, int32_t* owner, double* post) {
   __shared__ double w[256];
@@ -150,6 +153,139 @@ __global__ void __launch_bounds__(kGenericMaxThreads)
   }
 }
 
+// ---- NEXT f2: deglobalized generic-mode kernel ---------------------------
+// The globalized arrays have compile-time sizes, so they become static team-local smem
+// arrays (no stack, no cursor, no fallback) and the region names them directly; only `s`
+// travels through the argument sharing space.  The state machine is unchanged.
+template <class Base>
+struct Deglob : Base {
+  static constexpr unsigned stack_bytes = 0;
+  static constexpr bool dynamic_stack = false;
+  static constexpr bool stack_fallback = false;
+};
+constexpr unsigned kGenMaxInner = 256;
+
+template <bool Rec, bool Join>
+struct GenRegionDeglob {
+  struct Args {
+    double s;
+    double* out;
+    int32_t* owner;
+    int32_t inner_n;
+  };
+  static constexpr bool terminal = true;
+  static constexpr bool join = Join;
+  template <class Tr>
+  __device__ __forceinline__ void operator()(Team<Tr>& team, const Args& a) const {
+    const double* w = team_local<double, kGenMaxInner, 0>();
+    const int32_t* perm = team_local<int32_t, kGenMaxInner, 1>();
+    for_static(team, (typename Tr::Idx)a.inner_n, [&](int j) {
+      a.out[j] = __dadd_rn(__ddiv_rn(w[perm[j]], a.s), w[j]);
+      if constexpr (Rec) a.owner[j] = get_thread_num(team);
+    });
+  }
+};
+
+template <class Tr, int kInner, bool Rec, bool Post>
+__global__ void __launch_bounds__(kGenericMaxThreads, kGenericMinBlocks)
+    omprt_generic_deglob_rt(int32_t inner_n_rt, const double* __restrict__ in,
+                            double* __restrict__ out, int32_t* owner, double* post) {
+  using R = GenRegionDeglob<Rec, Post>;
+  using L = RegionList<R>;
+  const int32_t inner_n = kInner > 0 ? kInner : inner_n_rt;
+  Team<Tr> team = init<Tr>();
+  if (!is_main(team)) {
+    worker_state_machine<Tr, L>(team);
+    return;
+  }
+  const int32_t t = (int32_t)blockIdx.x;
+  double* w = team_local<double, kGenMaxInner, 0>();
+  int32_t* perm = team_local<int32_t, kGenMaxInner, 1>();
+  const double s = gen_prologue(in + (int64_t)t * inner_n, t, inner_n, w, perm);
+  double* tout = out + (int64_t)t * inner_n;
+  parallel<Tr, L, R>(team, typename R::Args{s, tout, Rec ? owner + (int64_t)t * inner_n : nullptr,
+                                            inner_n});
+  if constexpr (Post) {
+    double acc = 0.0;
+    for (int32_t j = 0; j < inner_n; ++j) acc = __dadd_rn(acc, tout[j]);
+    post[t] = acc;
+  }
+  deinit<Tr, L, true>(team);
+}
+
+// ---- NEXT f1: SPMDized kernel -----------------------------------------------------
+// The same target region in SPMD mode: the sequential prologue is guarded (thread 0 runs
+// it, an aligned barrier broadcasts w, perm and s), then all threads run the team `for`.
+template <class Base>
+struct Spmdized : Base {
+  static constexpr Mode mode = Mode::SPMD;
+  static constexpr unsigned stack_bytes = 0;
+  static constexpr bool dynamic_stack = false;
+  static constexpr bool stack_fallback = false;
+};
+
+template <class Tr, int kInner, bool Rec, bool Post>
+__global__ void __launch_bounds__(kGenericMaxThreads, kGenericMinBlocks)
+    omprt_generic_spmd_rt(int32_t inner_n_rt, const double* __restrict__ in,
+                          double* __restrict__ out, int32_t* owner, double* post) {
+  const int32_t inner_n = kInner > 0 ? kInner : inner_n_rt;
+  Team<Tr> team = init<Tr>();
+  const int32_t t = (int32_t)blockIdx.x;
+  double* w = team_local<double, kGenMaxInner, 0>();
+  int32_t* perm = team_local<int32_t, kGenMaxInner, 1>();
+  double* s_sh = team_local<double, 1, 2>();
+  guarded(team, [&] { s_sh[0] = gen_prologue(in + (int64_t)t * inner_n, t, inner_n, w, perm); });
+  const double s = s_sh[0];
+  double* tout = out + (int64_t)t * inner_n;
+  for_static(team, (typename Tr::Idx)inner_n, [&](int j) {
+    tout[j] = __dadd_rn(__ddiv_rn(w[perm[j]], s), w[j]);
+    if constexpr (Rec) owner[(int64_t)t * inner_n + j] = get_thread_num(team);
+  });
+  if constexpr (Post) {
+    aligned_barrier();  // the region's writes are visible to thread 0
+    if (team.thread_num == 0) {
+      double acc = 0.0;
+      for (int32_t j = 0; j < inner_n; ++j) acc = __dadd_rn(acc, tout[j]);
+      post[t] = acc;
+    }
+  }
+}
+
+// Variant 1: deglobalized (generic mode), 2: SPMDized.
+template <int Variant, class Tr, int KI, bool R, bool P>
+inline void launch_gv(int32_t teams, int32_t threads, int32_t inner_n, const double* in,
+                      double* out, int32_t* owner, double* post, cudaStream_t s) {
+  if constexpr (Variant == 1)
+    omprt_generic_deglob_rt<Tr, KI, R, P><<<teams, threads, 0, s>>>(inner_n, in, out, owner, post);
+  else
+    omprt_generic_spmd_rt<Tr, KI, R, P><<<teams, threads, 0, s>>>(inner_n, in, out, owner, post);
+}
+
+template <int Variant, class Tr>
+inline void launch_generic_variant(int32_t teams, int32_t threads, int32_t inner_n,
+                                   const double* in, double* out, int32_t* owner, double* post,
+                                   cudaStream_t s) {
+  const bool rec = owner != nullptr, pst = post != nullptr;
+#define OMPRT_GV(KI, R, P) \
+  launch_gv<Variant, Tr, KI, R, P>(teams, threads, inner_n, in, out, owner, post, s)
+  if (inner_n == 256) {
+    if (rec && pst) OMPRT_GV(256, true, true);
+    else if (rec) OMPRT_GV(256, true, false);
+    else if (pst) OMPRT_GV(256, false, true);
+    else OMPRT_GV(256, false, false);
+  } else {
+    if (rec && pst) OMPRT_GV(0, true, true);
+    else if (rec) OMPRT_GV(0, true, false);
+    else if (pst) OMPRT_GV(0, false, true);
+    else OMPRT_GV(0, false, false);
+  }
+#undef OMPRT_GV
+}
+
+OMPRT_REGISTER_KERNEL(omprt_generic_deglob_rt,
+                      omprt_generic_deglob_rt<Deglob<GenSM<GenericTraits, false>>, 256, false, false>)
+OMPRT_REGISTER_KERNEL(omprt_generic_spmd_rt,
+                      omprt_generic_spmd_rt<Spmdized<GenericTraits>, 256, false, false>)
 OMPRT_REGISTER_KERNEL(omprt_generic_rt, omprt_generic_rt<GenSM<GenericTraits, false>, 256, false, false>)
 OMPRT_REGISTER_KERNEL(omprt_generic_rt_general_sm,
                       omprt_generic_rt<GenSM<GenericTraits, true>, 256, false, false>)
@@ -237,6 +373,24 @@ extern "C" int omprt_generic_team(int32_t teams, int32_t threads, int32_t inner_
   cudaStream_t s = as_stream(stream);
   double* post = (flags & OMPRT_POSTLOGUE) ? postlogue : nullptr;
   const bool general = flags & OMPRT_GENERAL_SM;
+  if (flags & (OMPRT_SPMDIZE | OMPRT_DEGLOBALIZE)) {
+    OMPRT_CHECK_ARG(inner_n <= (int32_t)kGenMaxInner,
+                    "SPMDized / deglobalized variants need inner_n <= %u", kGenMaxInner);
+    OMPRT_CHECK_ARG(!(flags & (OMPRT_SMALL_STACK | OMPRT_NO_STACK | OMPRT_DEBUG_BUILD)),
+                    "SPMDized / deglobalized variants have no stack and no debug build");
+    const bool assume = flags & OMPRT_ASSUME_OVERSUB;
+    if (flags & OMPRT_SPMDIZE) {
+      if (assume) launch_generic_variant<2, Spmdized<GenericTraits>>(teams, threads, inner_n, in, out, owner, post, s);
+      else launch_generic_variant<2, Spmdized<GenericTraitsLoop>>(teams, threads, inner_n, in, out, owner, post, s);
+    } else if (general) {
+      if (assume) launch_generic_variant<1, Deglob<GenSM<GenericTraits, true>>>(teams, threads, inner_n, in, out, owner, post, s);
+      else launch_generic_variant<1, Deglob<GenSM<GenericTraitsLoop, true>>>(teams, threads, inner_n, in, out, owner, post, s);
+    } else {
+      if (assume) launch_generic_variant<1, Deglob<GenSM<GenericTraits, false>>>(teams, threads, inner_n, in, out, owner, post, s);
+      else launch_generic_variant<1, Deglob<GenSM<GenericTraitsLoop, false>>>(teams, threads, inner_n, in, out, owner, post, s);
+    }
+    return check_launch("omprt_generic_variant");
+  }
   if (flags & (OMPRT_SMALL_STACK | OMPRT_NO_STACK)) {
     const uint32_t dyn = (flags & OMPRT_NO_STACK) ? 0u : 2048u;
     launch_generic_sm<GenericTraitsDyn>(general, teams, threads, inner_n, in, out, owner, post,

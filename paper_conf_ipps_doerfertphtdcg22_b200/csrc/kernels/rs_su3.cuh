@@ -66,18 +66,6 @@ inline int rs_validate(const omprt_rs_tables& t, int64_t count, uint64_t* ver, i
 // 256-bit global accesses (sm_100: LDG/STG.E.ENL2.256): a site is 576 B = 18 x 32 B, so a
 // pair of links (288 B) moves in 9 instructions per thread instead of 18 x 16 B ones --
 // half the L1 wavefronts of the strided AoS access.
-__device__ __forceinline__ void ld_nc_256(const double* p, double& a, double& b, double& c,
-                                          double& d) {
-  asm("ld.global.nc.L1::no_allocate.v4.f64 {%0,%1,%2,%3}, [%4];"
-      : "=d"(a), "=d"(b), "=d"(c), "=d"(d)
-      : "l"(p));
-}
-__device__ __forceinline__ void st_cs_256(double* p, double a, double b, double c, double d) {
-  asm volatile("st.global.cs.v4.f64 [%0], {%1,%2,%3,%4};" ::"l"(p), "d"(a), "d"(b), "d"(c),
-               "d"(d)
-               : "memory");
-}
-
 // One site: C[l] = A[l] x B[l] for the 4 links; complex MAC = 4 fmas in fixed order
 // (App. A.3), so C is bit-identical to the oracle.  Row r of C[l] needs only row r of A[l],
 // so it overwrites it in registers.  Returns sum of Re C over the site in (l, r, c) order.
@@ -90,7 +78,7 @@ __device__ __forceinline__ double su3_site(const double* __restrict__ A,
     double v[36];
 #pragma unroll
     for (int q = 0; q < 9; ++q)
-      ld_nc_256(A + lp * 36 + 4 * q, v[4 * q], v[4 * q + 1], v[4 * q + 2], v[4 * q + 3]);
+      ld_stream_v4f64(A + lp * 36 + 4 * q, v[4 * q], v[4 * q + 1], v[4 * q + 2], v[4 * q + 3]);
 #pragma unroll
     for (int li = 0; li < 2; ++li) {
       const int l = 2 * lp + li, base = 18 * li;
@@ -119,7 +107,7 @@ __device__ __forceinline__ double su3_site(const double* __restrict__ A,
     }
 #pragma unroll
     for (int q = 0; q < 9; ++q)
-      st_cs_256(Cs + lp * 36 + 4 * q, v[4 * q], v[4 * q + 1], v[4 * q + 2], v[4 * q + 3]);
+      st_cs_v4f64(Cs + lp * 36 + 4 * q, v[4 * q], v[4 * q + 1], v[4 * q + 2], v[4 * q + 3]);
   }
   return re_sum;
 }

@@ -6,6 +6,8 @@
 #pragma once
 #include <cstdint>
 
+#include "vec.cuh"
+
 namespace omprt_kernels {
 
 // Tables passed BY VALUE as a kernel parameter (by-reference structs cost a load
@@ -121,17 +123,12 @@ __device__ __forceinline__ int32_t binned_grid_search(const XSTables& t, double 
   return lo;
 }
 
-__device__ __forceinline__ void ld_nc_v4f64(const double* p, double& a, double& b, double& c,
-                                            double& d) {
-  asm("ld.global.nc.v4.f64 {%0,%1,%2,%3}, [%4];" : "=d"(a), "=d"(b), "=d"(c), "=d"(d) : "l"(p));
-}
-
 // One lookup: returns verification = 1 + argmax of the 5 macroscopic cross sections.
 // Accel = false reads the tables exactly as specified (binary search of the unionized grid,
 // int32 index grid, 48 B gridpoint records: 6 x 16 B loads per nuclide).  Accel = true reads
 // the same values from the B200 layouts (binned search, 16-bit index grid, 96 B bracket
 // records loaded by 3 x 256-bit loads) -- identical results, fewer L1 wavefronts.
-template <bool Accel, int kUnroll = 4>
+template <bool Accel, int kUnroll = (Accel ? 2 : 4)>
 __device__ __forceinline__ uint64_t xs_lookup_one(const XSTables& t, uint64_t seed0, int64_t i) {
   uint64_t seed = lcg_fast_forward(seed0, 2ull * (uint64_t)i);
   const double E = lcg_double(seed);

@@ -4,6 +4,7 @@
 #include "host/runtime.cuh"
 #include "host/api.cuh"
 #include "kernels/axpy.cuh"
+#include "kernels/axpy_chunk.cuh"
 #include "kernels/generic.cuh"
 #include "kernels/xsbench.cuh"
 #include "kernels/rs_su3.cuh"

@@ -239,6 +239,18 @@ __device__ __forceinline__ void worker_state_machine(Team<Tr>& team) {
   }
 }
 
+// NEXT f1 -- SPMDization (§IV-A3): sequential code of a generic-mode region executed
+// in SPMD mode, "guarded for single threaded execution": the team's thread 0 runs `fn`
+// (its side effects happen once), then an aligned barrier broadcasts them.  No state
+// machine, no region hand-off.
+template <class Tr, class Fn>
+__device__ __forceinline__ void guarded(Team<Tr>& team, Fn&& fn) {
+  static_assert(Tr::mode == Mode::SPMD, "guarded execution is the SPMD form of sequential code");
+  OMPRT_TRACE(Tr, "guarded");
+  if (team.thread_num == 0) fn();
+  aligned_barrier();
+}
+
 // Runtime de-initialization: release the workers unless the last region was
 // terminal (then they already left).  `last_was_terminal` is a compile-time fact of the
 // kernel's control flow.

@@ -32,11 +32,14 @@ OMPRT_THREAD_STATES = 1 << 7
 OMPRT_FUSED_REDUCTION = 1 << 8
 OMPRT_UNCHECKED = 1 << 9
 OMPRT_XS_ACCEL = 1 << 10
+OMPRT_SPMDIZE = 1 << 11
+OMPRT_DEGLOBALIZE = 1 << 12
 
 # Every symbol include/omprt.h declares (checked by tests/test_abi.py).
 EXPORTS = [
     "omprt_init", "omprt_fini", "omprt_device_status", "omprt_last_error", "omprt_static_owner",
-    "omprt_spmd_axpy_sum", "omprt_cuda_axpy_sum", "omprt_generic_team", "omprt_cuda_generic_team",
+    "omprt_spmd_axpy_sum", "omprt_cuda_axpy_sum", "omprt_spmd_axpy_sum_chunked",
+    "omprt_cuda_axpy_sum_chunked", "omprt_generic_team", "omprt_cuda_generic_team",
     "omprt_icv_probe", "omprt_xs_lookup", "omprt_cuda_xs_lookup", "omprt_u64_sum",
     "omprt_xs_run_host", "omprt_xs_accel_sizes", "omprt_xs_build_accel", "omprt_rs_lookup", "omprt_cuda_rs_lookup", "omprt_su3_mult",
     "omprt_cuda_su3_mult", "omprt_kernel_count", "omprt_kernel_name", "omprt_kernel_attrs",
@@ -81,6 +84,10 @@ _SIGS = {
     "omprt_static_owner": [_i64, _i64, _i32, _i32, C.POINTER(_i32), C.POINTER(_i32)],
     "omprt_spmd_axpy_sum": [_i64, _f64, _vp, _vp, _vp, _vp, _i32, _i32, _u32, _vp, _vp, _vp],
     "omprt_cuda_axpy_sum": [_i64, _f64, _vp, _vp, _vp, _vp, _i32, _i32, _u32, _vp, _vp, _vp],
+    "omprt_spmd_axpy_sum_chunked": [_i64, _i64, _f64, _vp, _vp, _vp, _vp, _i32, _i32, _u32, _vp,
+                                    _vp, _vp],
+    "omprt_cuda_axpy_sum_chunked": [_i64, _i64, _f64, _vp, _vp, _vp, _vp, _i32, _i32, _u32, _vp,
+                                    _vp, _vp],
     "omprt_generic_team": [_i32, _i32, _i32, _vp, _vp, _vp, _vp, _u32, _vp],
     "omprt_cuda_generic_team": [_i32, _i32, _i32, _vp, _vp, _vp, _vp, _u32, _vp],
     "omprt_icv_probe": [_i32, _i32, _i32, _vp, _u32, _vp],
@@ -189,6 +196,20 @@ def omprt_cuda_axpy_sum(n, x, b, c, a, sum_inout, teams, threads, flags=0, owner
                         count=None, stream=None):
     return _check(load().omprt_cuda_axpy_sum(n, x, _p(b), _p(c), _p(a), _p(sum_inout), teams,
                                              threads, flags, _p(owner), _p(count), _stream(stream)))
+
+
+def omprt_spmd_axpy_sum_chunked(n, chunk, x, b, c, a, sum_inout, teams, threads, flags=0,
+                                owner=None, count=None, stream=None):
+    return _check(load().omprt_spmd_axpy_sum_chunked(n, chunk, x, _p(b), _p(c), _p(a),
+                                                     _p(sum_inout), teams, threads, flags,
+                                                     _p(owner), _p(count), _stream(stream)))
+
+
+def omprt_cuda_axpy_sum_chunked(n, chunk, x, b, c, a, sum_inout, teams, threads, flags=0,
+                                owner=None, count=None, stream=None):
+    return _check(load().omprt_cuda_axpy_sum_chunked(n, chunk, x, _p(b), _p(c), _p(a),
+                                                     _p(sum_inout), teams, threads, flags,
+                                                     _p(owner), _p(count), _stream(stream)))
 
 
 # ---------------------------------------------------------------- C2

@@ -24,3 +24,5 @@ for K in omprt_xs_rt cuda_xs_twin; do
   ncu -i $OUT/prof_${K}_$TAG.ncu-rep --page source --csv --print-units base > $OUT/src_${K}_$TAG.csv 2>&1
 done
 du -sh $OUT
+OMPRT_DEBUG=0 timeout 600 python scripts/debug_cost.py > $OUT/debug_cost_env0_$TAG.txt 2>&1
+OMPRT_DEBUG=1 timeout 600 python scripts/debug_cost.py > $OUT/debug_cost_env1_$TAG.txt 2>&1

@@ -91,3 +91,25 @@ def test_icv_probe(rt, N, variant):
     got = rec.cpu().numpy().reshape(teams, 1 + 3 * N, 7)
     ref = oracle.icv_table(teams, N, nested)
     assert (got == ref).all()
+
+
+@pytest.mark.parametrize("teams,N,inner", [(64, 256, 256), (64, 96, 256), (7, 64, 100),
+                                           (4096, 256, 256)])
+@pytest.mark.parametrize("variant", ["spmdize", "spmdize_assume", "deglob", "deglob_assume",
+                                     "deglob_general"])
+@pytest.mark.parametrize("post", [False, True])
+def test_spmdized_and_deglobalized(rt, teams, N, inner, variant, post):
+    """NEXT f1 / f2: the SPMDized (guarded prologue, no state machine) and deglobalized
+    (static team-local arrays, no stack) forms of C2 give the generic-mode results."""
+    if "assume" in variant and inner > N:
+        pytest.skip("assumption needs inner_n <= threads")
+    flags = {"spmdize": rt.OMPRT_SPMDIZE,
+             "spmdize_assume": rt.OMPRT_SPMDIZE | rt.OMPRT_ASSUME_OVERSUB,
+             "deglob": rt.OMPRT_DEGLOBALIZE,
+             "deglob_assume": rt.OMPRT_DEGLOBALIZE | rt.OMPRT_ASSUME_OVERSUB,
+             "deglob_general": rt.OMPRT_DEGLOBALIZE | rt.OMPRT_GENERAL_SM}[variant]
+    inp, out, owner, pst = _generic(rt, rt.omprt_generic_team, teams, N, inner, flags, post=post)
+    o_ref, own_ref, p_ref = oracle.generic_team(teams, N, inner, inp)
+    assert (out == o_ref).all() and (owner == own_ref).all()
+    if post:
+        assert (pst == p_ref).all()

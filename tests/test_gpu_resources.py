@@ -18,7 +18,18 @@ PAIRS = [
     ("omprt_rs_rt", "cuda_rs_twin", True),
     ("omprt_su3_rt", "cuda_su3_twin", True),
     ("omprt_generic_rt", "cuda_generic_twin", False),
+    ("omprt_axpy_chunk_rt", "cuda_axpy_chunk_twin", True),
+    ("omprt_generic_spmd_rt", "cuda_generic_twin", True),
+    ("omprt_generic_deglob_rt", "cuda_generic_twin", False),
 ]
+
+
+def test_deglobalized_has_no_stack(rt):
+    """NEXT f2: the deglobalized kernel carries only the twin's arrays (+ the team state and
+    the argument sharing space), not the 4 KiB stack of the stack-based kernel."""
+    tab = rt.kernel_table()
+    assert tab["omprt_generic_deglob_rt"]["static_smem"] < tab["omprt_generic_rt"]["static_smem"]
+    assert tab["omprt_generic_deglob_rt"]["static_smem"] <= tab["cuda_generic_twin"]["static_smem"] + 64
 
 
 @pytest.mark.parametrize("rtk,twin,spmd", PAIRS)

@@ -158,3 +158,52 @@ def test_debug_build_runtime_bits_off_is_silent(rt):
     """Compiled-in debug code does nothing unless enabled at run time."""
     p = _child(8 * 128 + 1, 128, "0")
     assert "STATUS 0" in p.stdout and "[omprt]" not in p.stdout
+
+
+CHUNK_CASES = [(0, 4, 1, 32), (1, 4, 8, 128), (1 << 20, 4, 8, 128), ((1 << 20) + 7, 4, 8, 128),
+               ((1 << 20) + 5, 3, 3, 96), (100003, 16, 37, 64), (4096, 1, 8, 128),
+               (2049, 4, 2, 256)]
+
+
+@pytest.mark.parametrize("n,C,T,N", CHUNK_CASES)
+@pytest.mark.parametrize("which", ["rt", "twin"])
+def test_chunked_schedule_owner_and_values(rt, n, C, T, N, which):
+    """NEXT f3: chunk k -> global thread k mod (T*N) (oracle_chunk_simulate), every iteration
+    once, a[] bit-exact, sum within 1e-12 of the Neumaier reference."""
+    x, b, c = gen.axpy_inputs(n)
+    fn = rt.omprt_spmd_axpy_sum_chunked if which == "rt" else rt.omprt_cuda_axpy_sum_chunked
+    bt, ct = torch.from_numpy(b).to(DEV), torch.from_numpy(c).to(DEV)
+    at = torch.full((max(n, 1),), float("nan"), dtype=torch.float64, device=DEV)
+    s = torch.zeros(1, dtype=torch.float64, device=DEV)
+    owner = torch.full((max(n, 1),), -1, dtype=torch.int32, device=DEV)
+    count = torch.zeros(max(n, 1), dtype=torch.int32, device=DEV)
+    fn(n, C, x, bt, ct, at, s, T, N, rt.OMPRT_RECORD_OWNER, owner, count)
+    torch.cuda.synchronize()
+    ref_owner, _ = oracle.chunk_simulate(n, C, T, N)
+    assert (count.cpu().numpy()[:n] == 1).all()
+    assert (owner.cpu().numpy()[:n] == ref_owner).all()
+    a_ref = oracle.axpy(x, b, c)
+    assert (at.cpu().numpy()[:n] == a_ref).all()
+    assert abs(s.item() - oracle.sum_f64(a_ref)) <= 1e-12 * max(oracle.sum_abs_f64(a_ref), 1e-300)
+
+
+def test_chunked_vectorized_matches_twin_and_assumption(rt):
+    n, C = 1 << 20, 4
+    x, b, c = gen.axpy_inputs(n, exact=True)
+    bt, ct = torch.from_numpy(b).to(DEV), torch.from_numpy(c).to(DEV)
+    sums = []
+    for fn, T, N, flags in [(rt.omprt_spmd_axpy_sum_chunked, 8, 128, 0),
+                            (rt.omprt_cuda_axpy_sum_chunked, 8, 128, 0),
+                            (rt.omprt_spmd_axpy_sum_chunked, 256, 1024, rt.OMPRT_ASSUME_OVERSUB)]:
+        at = torch.empty_like(bt)
+        s = torch.zeros(1, dtype=torch.float64, device=DEV)
+        fn(n, C, x, bt, ct, at, s, T, N, flags)
+        torch.cuda.synchronize()
+        assert (at.cpu().numpy() == oracle.axpy(x, b, c)).all()
+        sums.append(s.item())
+    assert sums == [float(1 << 30)] * 3  # integer-valued: exact in any order
+    with pytest.raises(rt.OmprtError) as e:  # 2^20 / 4 chunks > 128*1024 threads
+        rt.omprt_spmd_axpy_sum_chunked(n, C, x, bt, ct, torch.empty_like(bt),
+                                       torch.zeros(1, dtype=torch.float64, device=DEV), 128,
+                                       1024, rt.OMPRT_ASSUME_OVERSUB)
+    assert e.value.code == rt.OMPRT_E_INVAL

@@ -75,3 +75,31 @@ def test_cyclic_not_blocked():
     schedule(static): consecutive iterations go to consecutive threads."""
     owner, _ = oracle.fig5_simulate(64, 2, 4)
     assert list(owner[:9]) == [0, 1, 2, 3, 4, 5, 6, 7, 0]
+
+
+def test_chunked_schedule_closed_form_and_literal():
+    """NEXT f3 (reading R-F3): chunk k -> global thread k mod (T*N); brute force over tiny
+    shapes, exactly-once, and C = 1 reduces to Fig. 5 (the independent pin)."""
+    for n in range(0, 60):
+        for C in range(1, 7):
+            for T in range(1, 4):
+                for N in range(1, 6):
+                    owner, count = oracle.chunk_simulate(n, C, T, N)
+                    assert (count == 1).all()
+                    for iv in range(n):
+                        tm, th = oracle.static_chunk_owner_closed(iv, n, C, T, N)
+                        assert owner[iv] == tm * N + th
+                    if C == 1:
+                        f5, _ = oracle.fig5_simulate(n, T, N)
+                        assert (owner == f5).all()
+
+
+def test_chunked_schedule_special_cases():
+    owner, count = oracle.chunk_simulate(100, 1000, 4, 8)   # one chunk: all on thread 0
+    assert (owner == 0).all() and (count == 1).all()
+    owner, count = oracle.chunk_simulate(64, 4, 2, 8)        # consecutive chunks, round robin
+    assert list(owner[:12]) == [0, 0, 0, 0, 1, 1, 1, 1, 2, 2, 2, 2]
+    # assumption n <= T*N*C: at most one chunk per thread, identical assignment
+    a = oracle.chunk_simulate(63, 4, 2, 8, assume_oversub=True)
+    b = oracle.chunk_simulate(63, 4, 2, 8)
+    assert (a[0] == b[0]).all() and (a[1] == b[1]).all()

@@ -177,11 +177,16 @@ def run_omprt(args):
     from paper_conf_ipps_doerfertphtdcg22_b200 import omprt, sharding
 
     rank, world, local = dist_env()
+    gpu, backend, shared_gpu = sharding.pick_device_and_backend(local, world,
+                                                                torch.cuda.device_count())
+    torch.cuda.set_device(gpu)
+    dev = torch.device("cuda", gpu)
     if world > 1:
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
-    torch.cuda.set_device(local)
-    dev = torch.device("cuda", local)
-    omprt.omprt_init(local)
+        if backend == "nccl":
+            dist.init_process_group("nccl", device_id=dev)
+        else:
+            dist.init_process_group("gloo")
+    omprt.omprt_init(gpu)
     stream = torch.cuda.current_stream()
     tabs = gen.XSTables(**gen.XS_SMALL)
     d_acc = omprt.XSDeviceTables(tabs, dev, accel=True)   # B200 layouts (the headline path)

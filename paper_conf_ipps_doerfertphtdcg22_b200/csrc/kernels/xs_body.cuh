@@ -128,8 +128,91 @@ __device__ __forceinline__ int32_t binned_grid_search(const XSTables& t, double 
 // int32 index grid, 48 B gridpoint records: 6 x 16 B loads per nuclide).  Accel = true reads
 // the same values from the B200 layouts (binned search, 16-bit index grid, 96 B bracket
 // records loaded by 3 x 256-bit loads) -- identical results, fewer L1 wavefronts.
-template <bool Accel, int kUnroll = (Accel ? 2 : 4)>
+// Accumulate one nuclide's bracket into the 5 macroscopic cross sections (A.1 "Per nuclide").
+__device__ __forceinline__ void xs_accumulate(double E, double conc, double le, double he,
+                                              double lt, double ht, double lel, double hel,
+                                              double la, double ha, double lf, double hf,
+                                              double ln, double hn, double& m0, double& m1,
+                                              double& m2, double& m3, double& m4) {
+  const double f = (he - E) / (he - le);
+  m0 = fma(fma(-f, ht - lt, ht), conc, m0);      // total
+  m1 = fma(fma(-f, hel - lel, hel), conc, m1);   // elastic
+  m2 = fma(fma(-f, ha - la, ha), conc, m2);      // absorption
+  m3 = fma(fma(-f, hf - lf, hf), conc, m3);      // fission
+  m4 = fma(fma(-f, hn - ln, hn), conc, m4);      // nu-fission
+}
+
+__device__ __forceinline__ uint64_t xs_argmax5(double m0, double m1, double m2, double m3,
+                                               double m4) {
+  // 1 + argmax, strict '>' from max = -1 (the first maximum wins)
+  double mx = -1.0;
+  uint64_t v = 1;
+  if (m0 > mx) { mx = m0; v = 1; }
+  if (m1 > mx) { mx = m1; v = 2; }
+  if (m2 > mx) { mx = m2; v = 3; }
+  if (m3 > mx) { mx = m3; v = 4; }
+  if (m4 > mx) { mx = m4; v = 5; }
+  return v;
+}
+
+// The lookup on the B200 layouts with a software-pipelined nuclide loop: the index entries
+// of the next pair of nuclides are requested before the current pair's brackets, so the
+// index -> bracket dependency of one pair overlaps the other (measured: x04 in profiles/).
+// Same arithmetic in the same order as the plain path.
+__device__ __forceinline__ uint64_t xs_lookup_accel(const XSTables& t, uint64_t seed0,
+                                                    int64_t i) {
+  constexpr int P = 2;
+  uint64_t seed = lcg_fast_forward(seed0, 2ull * (uint64_t)i);
+  const double E = lcg_double(seed);
+  const int mat = pick_mat(seed);
+  const int32_t idx = binned_grid_search(t, E);
+  const int nn = __ldg(t.num_nucs + mat);
+  const int32_t* __restrict__ mrow = t.mats + mat * t.max_num_nucs;
+  const double* __restrict__ crow = t.concs + mat * t.max_num_nucs;
+  const uint16_t* __restrict__ irow = t.index_grid16 + (int64_t)idx * t.n_isotopes;
+  double m0 = 0.0, m1 = 0.0, m2 = 0.0, m3 = 0.0, m4 = 0.0;
+  int32_t pc[P], kc[P];
+#pragma unroll
+  for (int u = 0; u < P; ++u) {
+    pc[u] = u < nn ? __ldg(mrow + u) : 0;
+    kc[u] = u < nn ? (int32_t)__ldg(irow + pc[u]) : 0;
+  }
+  for (int j = 0; j < nn; j += P) {
+    int32_t pn[P], kn[P];
+#pragma unroll
+    for (int u = 0; u < P; ++u) {  // next stage's index entries
+      const int jj = j + P + u;
+      pn[u] = jj < nn ? __ldg(mrow + jj) : 0;
+      kn[u] = jj < nn ? (int32_t)__ldg(irow + pn[u]) : 0;
+    }
+#pragma unroll
+    for (int u = 0; u < P; ++u) {
+      if (j + u < nn) {
+        int32_t k = kc[u];
+        if (k == t.n_gridpoints - 1) --k;
+        const double conc = __ldg(crow + j + u);
+        // bracket (p, k): E_k E_k1 | t_k t_k1 | e_k e_k1 | a_k a_k1 | f_k f_k1 | n_k n_k1
+        const double* g = t.brackets + ((int64_t)pc[u] * (t.n_gridpoints - 1) + k) * 12;
+        double le, lt, lel, la, lf, ln, he, ht, hel, ha, hf, hn;
+        ld_nc_v4f64(g, le, he, lt, ht);
+        ld_nc_v4f64(g + 4, lel, hel, la, ha);
+        ld_nc_v4f64(g + 8, lf, hf, ln, hn);
+        xs_accumulate(E, conc, le, he, lt, ht, lel, hel, la, ha, lf, hf, ln, hn, m0, m1, m2, m3,
+                      m4);
+      }
+    }
+#pragma unroll
+    for (int u = 0; u < P; ++u) {
+      pc[u] = pn[u];
+      kc[u] = kn[u];
+    }
+  }
+  return xs_argmax5(m0, m1, m2, m3, m4);
+}
+
+template <bool Accel, int kUnroll = 4>
 __device__ __forceinline__ uint64_t xs_lookup_one(const XSTables& t, uint64_t seed0, int64_t i) {
+  if constexpr (Accel) return xs_lookup_accel(t, seed0, i);
   uint64_t seed = lcg_fast_forward(seed0, 2ull * (uint64_t)i);
   const double E = lcg_double(seed);
   const int mat = pick_mat(seed);

@@ -27,10 +27,11 @@ struct XSTraitsAssumeDebug : XSTraitsAssume {
 constexpr int kXSThreads = 256;
 // 4 teams of 256 per SM (<= 64 registers): measured best occupancy / memory-parallelism
 // trade-off for this latency-bound gather (scripts/experiments/xs_explore.*).
-constexpr int kXSMinBlocks = 4;
+constexpr int kXSMinBlocks = 4;   // plain layout
+constexpr int kXSMinBlocksAccel = 3;  // B200 layouts: 78 registers, no spills (x04)
 
 template <class Tr, bool Fused, bool Accel>
-__global__ void __launch_bounds__(kXSThreads, kXSMinBlocks)
+__global__ void __launch_bounds__(kXSThreads, Accel ? kXSMinBlocksAccel : kXSMinBlocks)
     omprt_xs_rt(const __grid_constant__ XSTables t, uint64_t seed, int64_t first,
                 typename Tr::Idx count, uint64_t* __restrict__ verification,
                 unsigned long long* checksum, unsigned long long* partials, unsigned* ticket) {
@@ -50,7 +51,7 @@ __global__ void __launch_bounds__(kXSThreads, kXSMinBlocks)
 // XSBench's CUDA kernel shape: one lookup per thread, early return past the end; the fused
 // variant hand-codes the same reduction algorithm as the runtime.
 template <bool Fused, bool Accel>
-__global__ void __launch_bounds__(kXSThreads, kXSMinBlocks)
+__global__ void __launch_bounds__(kXSThreads, Accel ? kXSMinBlocksAccel : kXSMinBlocks)
     cuda_xs_twin(const __grid_constant__ XSTables t, uint64_t seed, int64_t first, int32_t count,
                  uint64_t* __restrict__ verification, unsigned long long* checksum,
                  unsigned long long* partials, unsigned* ticket) {

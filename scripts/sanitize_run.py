@@ -1,0 +1,75 @@
+"""Small launches of every runtime kernel family (and twins) for compute-sanitizer
+(memcheck / racecheck / synccheck / initcheck; SURVEY §4 T-sanitize).
+
+  compute-sanitizer --tool racecheck python scripts/sanitize_run.py
+"""
+import os
+import sys
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+
+
+def main():
+    import torch
+
+    import gen
+    from paper_conf_ipps_doerfertphtdcg22_b200 import omprt
+
+    torch.cuda.set_device(0)
+    omprt.omprt_init(0)
+    dev = "cuda"
+    A = omprt.OMPRT_ASSUME_OVERSUB
+    # C1 (+ chunked)
+    n = 1 << 14
+    x, b, c = gen.axpy_inputs(n)
+    bt, ct = torch.from_numpy(b).to(dev), torch.from_numpy(c).to(dev)
+    at = torch.empty_like(bt)
+    s = torch.zeros(1, dtype=torch.float64, device=dev)
+    omprt.omprt_spmd_axpy_sum(n, x, bt, ct, at, s, 8, 128)
+    omprt.omprt_cuda_axpy_sum(n, x, bt, ct, at, s, 8, 128)
+    omprt.omprt_spmd_axpy_sum_chunked(n, 4, x, bt, ct, at, s, 8, 128)
+    omprt.omprt_spmd_axpy_sum(n, x, bt, ct, at, s, 128, 128, A)
+    # C2: all state machines, stack placements, SPMDized, deglobalized, postlogue
+    T = 16
+    inp = torch.from_numpy(gen.generic_inputs(T, 256)).to(dev)
+    out = torch.empty(T * 256, dtype=torch.float64, device=dev)
+    post = torch.empty(T, dtype=torch.float64, device=dev)
+    for f in (0, A, omprt.OMPRT_GENERAL_SM, omprt.OMPRT_SMALL_STACK, omprt.OMPRT_NO_STACK,
+              omprt.OMPRT_SPMDIZE | A, omprt.OMPRT_DEGLOBALIZE | A):
+        omprt.omprt_generic_team(T, 256, 256, inp, out, None, post, f | omprt.OMPRT_POSTLOGUE)
+    omprt.omprt_cuda_generic_team(T, 256, 256, inp, out, None, post, omprt.OMPRT_POSTLOGUE)
+    rec = torch.empty(T * (1 + 3 * 64) * 7, dtype=torch.int32, device=dev)
+    for f in (0, omprt.OMPRT_THREAD_STATES, omprt.OMPRT_GENERAL_SM):
+        omprt.omprt_icv_probe(T, 64, 4, rec, f)
+    # C3 (reduced grid)
+    t = gen.XSTables(n_isotopes=68, n_gridpoints=200)
+    d = omprt.XSDeviceTables(t, dev, accel=True)
+    m = 4096
+    ver = torch.empty(m, dtype=torch.uint64, device=dev)
+    ck = torch.zeros(1, dtype=torch.uint64, device=dev)
+    omprt.omprt_xs_lookup(d, 1070, 0, m, ver, None, 0, 256, A)
+    omprt.omprt_xs_lookup(d.plain(), 1070, 0, m, ver, None, 0, 256, A)
+    omprt.omprt_xs_lookup(d, 1070, 0, m, None, ck, 0, 256, A | omprt.OMPRT_FUSED_REDUCTION)
+    omprt.omprt_cuda_xs_lookup(d, 1070, 0, m, ver, None, 0, 256, 0)
+    omprt.omprt_u64_sum(ver, m, ck)
+    # C4 (reduced tables)
+    rs = gen.RSTables(n_nuclides=355, avg_poles=20, avg_windows=4)
+    rd = omprt.RSDeviceTables(rs, dev)
+    v = torch.empty(512, dtype=torch.uint64, device=dev)
+    omprt.omprt_rs_lookup(rd, 1070, 0, 512, v, None, 0, 128, A)
+    omprt.omprt_cuda_rs_lookup(rd, 1070, 0, 512, v, None, 0, 128, 0)
+    # C5
+    ns = 1024
+    Ah, Bh = gen.su3_inputs(ns)
+    At, Bt = torch.from_numpy(Ah).to(dev), torch.from_numpy(Bh).to(dev)
+    Ct = torch.empty_like(At)
+    cs = torch.zeros(1, dtype=torch.float64, device=dev)
+    omprt.omprt_su3_mult(At, Bt, Ct, ns, cs, 0, 128, A)
+    omprt.omprt_cuda_su3_mult(At, Bt, Ct, ns, cs, 0, 128, 0)
+    torch.cuda.synchronize()
+    print("sanitize_run: ok, device status", omprt.omprt_device_status(0)[0])
+
+
+if __name__ == "__main__":
+    main()

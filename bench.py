@@ -241,7 +241,7 @@ def run_omprt(args):
     def mx(v):
         return v if world == 1 else sharding.allreduce_max(v, dev)
 
-    clocks = ClockSampler(local)
+    clocks = ClockSampler(gpu)
     # primary: runtime-driven, assumption, B200 layouts (the headline path)
     clocks.start()
     step_ms, kern_ms = timed("rt", d_acc, A, args.steps, args.warmup)
@@ -304,6 +304,8 @@ def run_omprt(args):
             "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
             "config": {"workload": WORKLOAD, "lookups_per_gpu": L, "threads_per_team": THREADS,
                        "teams": (L + THREADS - 1) // THREADS, "parallelism": f"dp{world}",
+                       "backend": backend if world > 1 else None,
+                       "shared_gpu_test_mode": shared_gpu,
                        "l2": "flushed before every timed step (256 MiB scrub write)",
                        "variant": "runtime-driven SPMD, teams oversubscription assumption, "
                                   "B200 table layouts (binned search, 16-bit index, bracket "

@@ -74,6 +74,14 @@ def test_world2_gloo():
     assert out[0]["weak"] == (0, 1000) and out[1]["weak"] == (1000, 1000)
 
 
+def test_device_and_backend_choice():
+    assert sharding.pick_device_and_backend(3, 8, 8) == (3, "nccl", False)
+    assert sharding.pick_device_and_backend(0, 1, 1) == (0, "nccl", False)
+    assert sharding.pick_device_and_backend(1, 2, 1) == (0, "gloo", True)  # test mode only
+    with pytest.raises(RuntimeError):
+        sharding.pick_device_and_backend(0, 1, 0)  # no GPU: no CPU fallback
+
+
 def test_shard_partition_properties():
     for total in (0, 1, 7, 17_000_000, 10_000_001):
         for world in (1, 2, 3, 4, 8):

@@ -421,6 +421,11 @@ def run_secondary(omprt, torch, gen, dev, stream, scrub):
     ck = torch.zeros(1, dtype=torch.float64, device=dev)
     t_rt = _time(lambda: omprt.omprt_su3_mult(At, Bt, Ct, ns, ck, 0, 128, A), stream, scrub)
     t_tw = _time(lambda: omprt.omprt_cuda_su3_mult(At, Bt, Ct, ns, ck, 0, 128, 0), stream, scrub)
+    TS = omprt.OMPRT_TMA_STAGED
+    t_rs = _time(lambda: omprt.omprt_su3_mult(At, Bt, Ct, ns, ck, 0, 128, TS), stream, scrub)
+    t_ts = _time(lambda: omprt.omprt_cuda_su3_mult(At, Bt, Ct, ns, ck, 0, 128, TS), stream, scrub)
+    res["c5_su3_32^4_tma_staged"] = {"rt_ms": t_rs, "twin_ms": t_ts, "overhead": t_rs / t_ts - 1,
+                                     "GBps_alg": 1152 * ns / t_rs / 1e6}
     res["c5_su3_32^4"] = {"rt_ms": t_rt, "twin_ms": t_tw, "overhead": t_rt / t_tw - 1,
                           "GBps_alg": 1152 * ns / t_rt / 1e6, "GFLOPs": 864 * ns / t_rt / 1e6}
     return res

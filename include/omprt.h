@@ -84,6 +84,10 @@ extern "C" {
 /* omprt_generic_team, NEXT f2 (P:172 globalization elimination): generic mode with
  * the globalized arrays in static team-local shared memory -- no stack (0 B).  inner_n <= 256. */
 #define OMPRT_DEGLOBALIZE (1u << 12)
+/* omprt_su3_mult: move the 576 B site records with bulk (TMA) copies through padded shared
+ * memory slots (one persistent team of 128 per SM, per-thread double buffering); teams = 0:
+ * one per SM.  Not combined with OMPRT_ASSUME_OVERSUB. */
+#define OMPRT_TMA_STAGED (1u << 13)
 
 /* ---- runtime lifecycle ------------------------------------------------------------- */
 typedef struct {

@@ -1,0 +1,183 @@
+// C5 with TMA staging (OMPRT_TMA_STAGED): the SU(3) site loop as a persistent
+// `distribute parallel for` (one team of 128 per SM, Fig. 5 assignment) whose site records
+// (576 B, AoS) are moved by bulk copies into padded shared-memory slots and back
+// (omprt/device/tma.cuh), instead of 32-line-wide strided global accesses.  The twin runs
+// the same per-thread double-buffered bulk-copy pipeline, written by hand.
+#pragma once
+#include "../common/ptx_tma.cuh"
+#include "../host/runtime.cuh"
+#include "../omprt/device/tma.cuh"
+#include "rs_su3.cuh"
+
+namespace omprt_kernels {
+
+using namespace omprt;
+
+constexpr unsigned kSU3Rec = 576;   // 4 links x 3 x 3 complex fp64
+constexpr unsigned kSU3Slot = 592;  // 148 words: 8 consecutive threads' 16 B loads hit
+                                    // disjoint bank quads (conflict-free LDS.128)
+constexpr int kSU3StagedThreads = 128;
+
+// The body on a staged record (in place): C[l] = A[l] x B[l], the App. A.3 fma order, the
+// same (l, r, c) accumulation of Re C as su3_site.
+__device__ __forceinline__ double su3_site_slot(unsigned char* slot,
+                                                const double2* __restrict__ B) {
+  double2* v = reinterpret_cast<double2*>(slot);
+  double re_sum = 0.0;
+#pragma unroll
+  for (int l = 0; l < 4; ++l) {
+    double2 a[9];
+#pragma unroll
+    for (int e = 0; e < 9; ++e) a[e] = v[l * 9 + e];
+#pragma unroll
+    for (int r = 0; r < 3; ++r)
+#pragma unroll
+      for (int c = 0; c < 3; ++c) {
+        double re = 0.0, im = 0.0;
+#pragma unroll
+        for (int m = 0; m < 3; ++m) {
+          const double2 x = a[r * 3 + m];
+          const double2 y = __ldg(B + l * 9 + m * 3 + c);
+          re = fma(x.x, y.x, re);
+          re = fma(-x.y, y.y, re);
+          im = fma(x.x, y.y, im);
+          im = fma(x.y, y.x, im);
+        }
+        v[l * 9 + r * 3 + c] = make_double2(re, im);
+        re_sum += re;
+      }
+  }
+  return re_sum;
+}
+
+struct SU3StagedTraits : DefaultTraits {};  // persistent grid: the loop stays
+
+template <class Tr, bool Checksum>
+__global__ void __launch_bounds__(kSU3StagedThreads, 1)
+    omprt_su3_staged_rt(const double* __restrict__ A, const double2* __restrict__ B,
+                        double* __restrict__ Cm, typename Tr::Idx n_sites, double* checksum,
+                        double* partials, unsigned* ticket) {
+  using Idx = typename Tr::Idx;
+  Team<Tr> team = init<Tr>();
+  double acc = 0.0;
+  distribute_parallel_for_staged<Tr, kSU3Rec, kSU3Slot>(
+      team, n_sites, reinterpret_cast<const unsigned char*>(A),
+      reinterpret_cast<unsigned char*>(Cm),
+      [&](Idx, unsigned char* slot) { acc += su3_site_slot(slot, B); });
+  if constexpr (Checksum)
+    league_reduce(team, team_reduce_to_main(team, acc, Plus{}), Plus{}, checksum, partials,
+                  ticket);
+}
+
+// Bare CUDA twin: the same per-thread bulk-copy pipeline and reduction, by hand.
+template <bool Checksum>
+__global__ void __launch_bounds__(kSU3StagedThreads, 1)
+    cuda_su3_staged_twin(const double* __restrict__ A, const double2* __restrict__ B,
+                         double* __restrict__ Cm, int32_t n_sites, double* checksum,
+                         double* partials, unsigned* ticket) {
+  extern __shared__ __align__(128) unsigned char smem[];
+  const unsigned nt = blockDim.x, t = threadIdx.x;
+  unsigned char* slot0 = smem + t * kSU3Slot;
+  unsigned char* slot1 = smem + (nt + t) * kSU3Slot;
+  uint64_t* bar = reinterpret_cast<uint64_t*>(smem + 2 * nt * kSU3Slot) + 2 * t;
+  tma::mbar_init(bar, 1);
+  tma::mbar_init(bar + 1, 1);
+  tma::fence_mbar_init();
+  const unsigned char* in = reinterpret_cast<const unsigned char*>(A);
+  unsigned char* out = reinterpret_cast<unsigned char*>(Cm);
+  const int32_t stride = gridDim.x * nt;
+  int32_t s = blockIdx.x * nt + t;
+  double acc = 0.0;
+  if (s < n_sites) {
+    tma::mbar_arrive_expect_tx(bar, kSU3Rec);
+    tma::bulk_load(slot0, in + (size_t)s * kSU3Rec, kSU3Rec, bar);
+  }
+  uint32_t ph0 = 0, ph1 = 0;
+  for (unsigned k = 0; s < n_sites; s += stride, ++k) {
+    unsigned char* cur = (k & 1) ? slot1 : slot0;
+    unsigned char* nxt = (k & 1) ? slot0 : slot1;
+    uint64_t* bcur = bar + (k & 1);
+    uint64_t* bnxt = bar + ((k & 1) ^ 1);
+    if (s + stride < n_sites) {
+      tma::bulk_wait_read<0>();
+      tma::mbar_arrive_expect_tx(bnxt, kSU3Rec);
+      tma::bulk_load(nxt, in + (size_t)(s + stride) * kSU3Rec, kSU3Rec, bnxt);
+    }
+    tma::mbar_wait(bcur, (k & 1) ? ph1 : ph0);
+    if (k & 1) ph1 ^= 1u;
+    else ph0 ^= 1u;
+    acc += su3_site_slot(cur, B);
+    tma::fence_proxy_async_smem();
+    tma::bulk_store(out + (size_t)s * kSU3Rec, cur, kSU3Rec);
+    tma::bulk_commit();
+  }
+  tma::bulk_wait<0>();
+  if constexpr (Checksum) {
+    __shared__ double ws[32];
+    __shared__ unsigned last;
+    for (int off = 16; off > 0; off >>= 1) acc += __shfl_xor_sync(0xffffffffu, acc, off);
+    const unsigned lane = t & 31u, wid = t >> 5, nw = nt >> 5;
+    if (lane == 0) ws[wid] = acc;
+    __syncthreads();
+    double b = 0.0;
+    if (wid == 0) {
+      b = lane < nw ? ws[lane] : 0.0;
+      for (int off = 16; off > 0; off >>= 1) b += __shfl_xor_sync(0xffffffffu, b, off);
+    }
+    if (t == 0) {
+      partials[blockIdx.x] = b;
+      __threadfence();
+      last = atomicAdd(ticket, 1u) == gridDim.x - 1;
+    }
+    __syncthreads();
+    if (last) {
+      __threadfence();
+      double tt = 0.0;
+      for (unsigned k = t; k < gridDim.x; k += nt) tt += __ldcg(partials + k);
+      for (int off = 16; off > 0; off >>= 1) tt += __shfl_xor_sync(0xffffffffu, tt, off);
+      if (lane == 0) ws[wid] = tt;
+      __syncthreads();
+      if (wid == 0) {
+        double u = lane < nw ? ws[lane] : 0.0;
+        for (int off = 16; off > 0; off >>= 1) u += __shfl_xor_sync(0xffffffffu, u, off);
+        if (t == 0) {
+          *checksum = *checksum + u;
+          *ticket = 0u;
+        }
+      }
+    }
+  }
+}
+
+OMPRT_REGISTER_KERNEL(omprt_su3_staged_rt, omprt_su3_staged_rt<SU3StagedTraits, true>)
+OMPRT_REGISTER_KERNEL(cuda_su3_staged_twin, cuda_su3_staged_twin<true>)
+
+// persistent geometry: one team per SM (153 KB of slots + barriers)
+inline int su3_staged_launch(bool twin, const double* A, const double* B, double* Cm,
+                             int64_t n, double* ck, int32_t teams, Workspace* w,
+                             cudaStream_t s) {
+  const uint32_t smem = staged_smem_bytes<kSU3Slot, 2>(kSU3StagedThreads);
+  int dev = 0, sms = 148;
+  cudaGetDevice(&dev);
+  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  if (teams <= 0) teams = sms;
+  OMPRT_CHECK_ARG(!ck || (uint64_t)teams <= w->opt.max_teams, "teams exceed max_teams");
+  OMPRT_CHECK_ARG(n + 2 * (int64_t)teams * kSU3StagedThreads < INT32_MAX, "n_sites too large");
+  const int32_t nn = (int32_t)n;
+  auto* b2 = (const double2*)B;
+  double* p = (double*)w->partials;
+  unsigned* tk = w->tickets + 3;
+  if (twin) {
+    auto k = ck ? cuda_su3_staged_twin<true> : cuda_su3_staged_twin<false>;
+    OMPRT_CUDA_TRY(cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
+    k<<<teams, kSU3StagedThreads, smem, s>>>(A, b2, Cm, nn, ck, p, tk);
+  } else {
+    auto k = ck ? omprt_su3_staged_rt<SU3StagedTraits, true>
+                : omprt_su3_staged_rt<SU3StagedTraits, false>;
+    OMPRT_CUDA_TRY(cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
+    k<<<teams, kSU3StagedThreads, smem, s>>>(A, b2, Cm, nn, ck, p, tk);
+  }
+  return check_launch(twin ? "cuda_su3_staged_twin" : "omprt_su3_staged_rt");
+}
+
+}  // namespace omprt_kernels

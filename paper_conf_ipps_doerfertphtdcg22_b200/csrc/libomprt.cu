@@ -8,3 +8,4 @@
 #include "kernels/generic.cuh"
 #include "kernels/xsbench.cuh"
 #include "kernels/rs_su3.cuh"
+#include "kernels/su3_staged.cuh"

@@ -1,0 +1,60 @@
+"""Quick CUDA-event timings of the secondary configs' variants (median of 7, L2 flushed).
+  python scripts/quick_time.py [su3] [rs] [c1] [c2]"""
+import json
+import os
+import statistics
+import sys
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+
+
+def main(which):
+    import torch
+
+    import gen
+    from paper_conf_ipps_doerfertphtdcg22_b200 import omprt
+    torch.cuda.set_device(0)
+    omprt.omprt_init(0)
+    dev, s = "cuda", torch.cuda.current_stream()
+    scrub = torch.empty(64 << 20, dtype=torch.float32, device=dev)
+
+    def t(fn, reps=7):
+        fn()
+        torch.cuda.synchronize()
+        out = []
+        for _ in range(reps):
+            scrub.fill_(1.0)
+            a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            a.record(s)
+            fn()
+            b.record(s)
+            torch.cuda.synchronize()
+            out.append(a.elapsed_time(b))
+        return statistics.median(out)
+
+    A, TS = omprt.OMPRT_ASSUME_OVERSUB, omprt.OMPRT_TMA_STAGED
+    res = {}
+    if "su3" in which:
+        ns = 32 ** 4
+        Ah, Bh = gen.su3_inputs(ns)
+        At, Bt = torch.from_numpy(Ah).to(dev), torch.from_numpy(Bh).to(dev)
+        Ct = torch.empty_like(At)
+        ck = torch.zeros(1, dtype=torch.float64, device=dev)
+        for name, fn, fl in [("rt", omprt.omprt_su3_mult, A), ("twin", omprt.omprt_cuda_su3_mult, 0),
+                             ("rt_staged", omprt.omprt_su3_mult, TS),
+                             ("twin_staged", omprt.omprt_cuda_su3_mult, TS)]:
+            ms = t(lambda: fn(At, Bt, Ct, ns, ck, 0, 128, fl))
+            res[f"su3_{name}"] = {"ms": ms, "GBps_alg": 1152 * ns / ms / 1e6}
+    if "rs" in which:
+        rs = gen.RSTables()
+        rd = omprt.RSDeviceTables(rs, dev)
+        n = 1_000_000
+        v = torch.empty(n, dtype=torch.uint64, device=dev)
+        res["rs_rt_1M"] = {"ms": t(lambda: omprt.omprt_rs_lookup(rd, 1070, 0, n, v, None, 0, 128, A), 3)}
+        res["rs_twin_1M"] = {"ms": t(lambda: omprt.omprt_cuda_rs_lookup(rd, 1070, 0, n, v, None, 0, 128, 0), 3)}
+    print(json.dumps(res))
+
+
+if __name__ == "__main__":
+    main(sys.argv[1:] or ["su3", "rs"])

@@ -69,11 +69,12 @@ def _su3(rt, fn, A, B, n, flags=0):
 
 
 @pytest.mark.parametrize("n", [8 ** 4, 8 ** 4 + 5, 32 ** 4])
-@pytest.mark.parametrize("variant", ["rt", "rt_loop", "twin"])
+@pytest.mark.parametrize("variant", ["rt", "rt_loop", "twin", "rt_staged", "twin_staged"])
 def test_su3_bit_exact(rt, n, variant):
     A, B = gen.su3_inputs(n)
-    fn = rt.omprt_cuda_su3_mult if variant == "twin" else rt.omprt_su3_mult
-    flags = rt.OMPRT_ASSUME_OVERSUB if variant == "rt" else 0
+    fn = rt.omprt_cuda_su3_mult if variant.startswith("twin") else rt.omprt_su3_mult
+    flags = {"rt": rt.OMPRT_ASSUME_OVERSUB, "rt_loop": 0, "twin": 0,
+             "rt_staged": rt.OMPRT_TMA_STAGED, "twin_staged": rt.OMPRT_TMA_STAGED}[variant]
     C, ck = _su3(rt, fn, A, B, n, flags)
     Cref = oracle.su3_mult(A, B, n, threads=os.cpu_count() or 1)
     assert (C == Cref).all()

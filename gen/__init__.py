@@ -219,6 +219,15 @@ class XSTables:
     def n_union(self):
         return self.unionized.shape[0]
 
+    @property
+    def index_grid16(self):
+        """The same index grid as uint16 (every entry is < n_gridpoints <= 65536): the
+        compact host-side layout of the data (a copy, made on first use)."""
+        if not hasattr(self, "_ig16"):
+            assert self.n_gridpoints <= 65536
+            self._ig16 = self.index_grid.astype(np.uint16)
+        return self._ig16
+
     def nbytes(self):
         return (self.nuclide_grid.nbytes + self.unionized.nbytes + self.index_grid.nbytes
                 + self.num_nucs.nbytes + self.mats.nbytes + self.concs.nbytes)

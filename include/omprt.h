@@ -221,6 +221,18 @@ int omprt_u64_sum(const uint64_t *v, int64_t n, uint64_t *out_inout, void *strea
 int omprt_xs_run_host(omprt_xs_tables host_tables, uint64_t seed, int64_t first, int64_t count,
                       int32_t threads, uint32_t flags, uint64_t *checksum_host,
                       uint64_t *h2d_bytes, uint64_t *d2h_bytes, void *stream);
+/* The same offload repeated `steps` times (1..1024), each step with its own H2D of the
+ * tables, lookups and D2H of its checksum (checksums_host[steps]); the H2D of step s+1 runs
+ * on an internal copy stream while step s computes (two device table slots; OpenMP
+ * `target nowait` + dependences).  host_tables may hold the B200 layouts on the host:
+ * index_grid16 (then index_grid may be NULL and 2 B per entry cross PCIe) and/or brackets
+ * (then nuclide_grid may be NULL); whatever is missing is built on the device (bins
+ * always), which also enables the accelerated lookup (as OMPRT_XS_ACCEL does).
+ * *h2d_bytes = bytes copied host->device per step.  Synchronous. */
+int omprt_xs_run_host_steps(omprt_xs_tables host_tables, uint64_t seed, int64_t first,
+                            int64_t count, int32_t threads, uint32_t flags, int32_t steps,
+                            uint64_t *checksums_host, uint64_t *h2d_bytes, uint64_t *d2h_bytes,
+                            void *stream);
 
 /* ---- C4: RSBench-shaped multipole lookup -------------------- */
 typedef struct {

@@ -54,7 +54,15 @@ extern "C" int omprt_fini(int device) {
   cudaFree(w.tickets);
   cudaFree(w.scratch_u64);
   cudaFree(w.pool);
-  cudaFree(w.xs_buf);
+  cudaFree(w.xs_buf[0]);
+  cudaFree(w.xs_buf[1]);
+  cudaFree(w.dev_ck);
+  if (w.pinned_ck) cudaFreeHost(w.pinned_ck);
+  for (int k = 0; k < 2; ++k) {
+    if (w.copy_done[k]) cudaEventDestroy(w.copy_done[k]);
+    if (w.compute_done[k]) cudaEventDestroy(w.compute_done[k]);
+  }
+  if (w.copy_stream) cudaStreamDestroy(w.copy_stream);
   cudaFreeHost(w.err_host);
   omprt::DeviceEnv zero{};
   cudaMemcpyToSymbol(omprt_env, &zero, sizeof zero);

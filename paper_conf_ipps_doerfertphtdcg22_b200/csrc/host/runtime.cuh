@@ -49,10 +49,17 @@ struct Workspace {
   uint64_t* scratch_u64 = nullptr;  // 8 slots of device scratch (e2e checksum, ...)
   omprt_options opt{};
   unsigned debug_bits = 0;
-  // e2e (omprt_xs_run_host) device copies of the tables, grown on demand
-  void* xs_buf = nullptr;
+  // e2e (omprt_xs_run_host*) device copies of the tables, two slots (double buffering
+  // across steps), grown on demand; a copy stream, per-slot events, pinned checksums
+  void* xs_buf[2] = {nullptr, nullptr};
   size_t xs_buf_bytes = 0;
+  cudaStream_t copy_stream = nullptr;
+  cudaEvent_t copy_done[2] = {nullptr, nullptr};
+  cudaEvent_t compute_done[2] = {nullptr, nullptr};
+  uint64_t* pinned_ck = nullptr;     // [kMaxE2ESteps]
+  uint64_t* dev_ck = nullptr;        // [kMaxE2ESteps]
 };
+constexpr int kMaxE2ESteps = 1024;
 
 constexpr int kMaxDevices = 64;
 Workspace g_ws[kMaxDevices];

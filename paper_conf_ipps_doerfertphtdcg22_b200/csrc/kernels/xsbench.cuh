@@ -294,80 +294,143 @@ extern "C" int omprt_xs_build_accel(omprt_xs_tables* t, int32_t* bins, uint16_t*
   return launch_xs_accel(t, bins, index_grid16, brackets, log2_bins, as_stream(stream));
 }
 
-// End to end with host tables: map(to: tables) -> (accelerated layouts built on the device)
-// -> lookups (fused reduction) -> map(from: checksum).  Synchronous on `stream`.
-extern "C" int omprt_xs_run_host(omprt_xs_tables h, uint64_t seed, int64_t first, int64_t count,
-                                 int32_t threads, uint32_t flags, uint64_t* checksum_host,
-                                 uint64_t* h2d_bytes, uint64_t* d2h_bytes, void* stream) {
+// End to end with HOST tables, `steps` times (an OpenMP `target map(to: tables)
+// map(from: checksum)` per step): H2D of the tables -> the B200 layouts built on the device
+// (bins always; the 16-bit index grid and the bracket records unless the host already holds
+// them in that layout) -> lookups with the fused checksum -> D2H of the checksum.  Two
+// device table slots, a copy stream and per-slot events let the H2D of step s+1 run while
+// step s computes (`target nowait` with dependences).  Synchronous: returns when all steps
+// are done.  Host tables should be pinned (pageable copies serialize).
+extern "C" int omprt_xs_run_host_steps(omprt_xs_tables h, uint64_t seed, int64_t first,
+                                       int64_t count, int32_t threads, uint32_t flags,
+                                       int32_t steps, uint64_t* checksums_host,
+                                       uint64_t* h2d_bytes, uint64_t* d2h_bytes, void* stream) {
   using namespace omprt_kernels;
   Workspace* w;
   if (int r = current_ws(&w)) return r;
-  OMPRT_CHECK_ARG(checksum_host && h.nuclide_grid && h.unionized && h.index_grid && h.num_nucs &&
-                      h.mats && h.concs,
-                  "omprt_xs_run_host: bad arguments");
+  OMPRT_CHECK_ARG(checksums_host && steps >= 1 && steps <= kMaxE2ESteps && h.unionized &&
+                      h.num_nucs && h.mats && h.concs && (h.index_grid || h.index_grid16) &&
+                      (h.nuclide_grid || h.brackets),
+                  "omprt_xs_run_host_steps: bad arguments");
+  const bool accel = (flags & OMPRT_XS_ACCEL) || h.index_grid16 || h.brackets;
+  OMPRT_CHECK_ARG(accel || (h.index_grid && h.nuclide_grid),
+                  "the plain path needs the int32 index grid and the nuclide grid");
+  OMPRT_CHECK_ARG(!accel || h.n_gridpoints <= 65536, "16-bit index: n_gridpoints > 65536");
   cudaStream_t s = as_stream(stream);
-  const size_t n_grid = (size_t)h.n_isotopes * h.n_gridpoints * 6 * sizeof(double);
-  const size_t n_uni = (size_t)h.n_union * sizeof(double);
-  const size_t n_idx = (size_t)h.n_union * h.n_isotopes * sizeof(int32_t);
-  const size_t n_num = 12 * sizeof(int32_t);
-  const size_t n_mat = (size_t)12 * h.max_num_nucs * sizeof(int32_t);
-  const size_t n_con = (size_t)12 * h.max_num_nucs * sizeof(double);
-  const bool accel = (flags & OMPRT_XS_ACCEL) && h.n_gridpoints <= 65536;
   const int32_t log2_bins = 16;
   uint64_t asz[3] = {0, 0, 0};
   if (accel) xs_accel_sizes(h.n_isotopes, h.n_gridpoints, h.n_union, log2_bins, asz);
+  const bool up16 = accel && h.index_grid16, upbr = accel && h.brackets;
+  const size_t n_grid = upbr ? 0 : (size_t)h.n_isotopes * h.n_gridpoints * 6 * sizeof(double);
+  const size_t n_br = upbr ? asz[2] : 0;
+  const size_t n_uni = (size_t)h.n_union * sizeof(double);
+  const size_t n_idx = up16 ? asz[1] : (size_t)h.n_union * h.n_isotopes * sizeof(int32_t);
+  const size_t n_num = 12 * sizeof(int32_t);
+  const size_t n_mat = (size_t)12 * h.max_num_nucs * sizeof(int32_t);
+  const size_t n_con = (size_t)12 * h.max_num_nucs * sizeof(double);
   auto al = [](size_t b) { return (b + 255) & ~size_t(255); };
-  const size_t total = al(n_grid) + al(n_uni) + al(n_idx) + al(n_num) + al(n_mat) + al(n_con) +
-                       al(asz[0]) + al(asz[1]) + al(asz[2]);
+  // slot layout: uploaded tables, then the device-built layouts
+  const size_t built16 = (accel && !up16) ? asz[1] : 0, builtbr = (accel && !upbr) ? asz[2] : 0;
+  const size_t total = al(n_grid) + al(n_br) + al(n_uni) + al(n_idx) + al(n_num) + al(n_mat) +
+                       al(n_con) + al(asz[0]) + al(built16) + al(builtbr);
+  if (!w->copy_stream) {
+    OMPRT_CUDA_TRY(cudaStreamCreateWithFlags(&w->copy_stream, cudaStreamNonBlocking));
+    for (int k = 0; k < 2; ++k) {
+      OMPRT_CUDA_TRY(cudaEventCreateWithFlags(&w->copy_done[k], cudaEventDisableTiming));
+      OMPRT_CUDA_TRY(cudaEventCreateWithFlags(&w->compute_done[k], cudaEventDisableTiming));
+    }
+    OMPRT_CUDA_TRY(cudaHostAlloc(&w->pinned_ck, kMaxE2ESteps * sizeof(uint64_t),
+                                 cudaHostAllocDefault));
+    OMPRT_CUDA_TRY(cudaMalloc(&w->dev_ck, kMaxE2ESteps * sizeof(uint64_t)));
+  }
   if (w->xs_buf_bytes < total) {
-    cudaFree(w->xs_buf);
-    w->xs_buf = nullptr;
+    OMPRT_CUDA_TRY(cudaDeviceSynchronize());
+    for (int k = 0; k < 2; ++k) {
+      cudaFree(w->xs_buf[k]);
+      w->xs_buf[k] = nullptr;
+    }
     w->xs_buf_bytes = 0;
-    if (cudaMalloc(&w->xs_buf, total) != cudaSuccess) {
+    if (cudaMalloc(&w->xs_buf[0], total) != cudaSuccess ||
+        cudaMalloc(&w->xs_buf[1], total) != cudaSuccess) {
       cudaGetLastError();
-      return set_error(OMPRT_E_NOMEM, "omprt_xs_run_host: cannot allocate %zu B", total);
+      return set_error(OMPRT_E_NOMEM, "omprt_xs_run_host_steps: cannot allocate 2 x %zu B",
+                       total);
     }
     w->xs_buf_bytes = total;
   }
-  unsigned char* b = (unsigned char*)w->xs_buf;
-  omprt_xs_tables d = h;
-  size_t off = 0;
-  bool ok = true;
-  auto put = [&](const void* src, size_t bytes) -> const void* {
-    void* dst = b + off;
-    off += al(bytes);
-    ok = ok && cudaMemcpyAsync(dst, src, bytes, cudaMemcpyHostToDevice, s) == cudaSuccess;
-    return dst;
-  };
-  d.nuclide_grid = (const double*)put(h.nuclide_grid, n_grid);
-  d.unionized = (const double*)put(h.unionized, n_uni);
-  d.index_grid = (const int32_t*)put(h.index_grid, n_idx);
-  d.num_nucs = (const int32_t*)put(h.num_nucs, n_num);
-  d.mats = (const int32_t*)put(h.mats, n_mat);
-  d.concs = (const double*)put(h.concs, n_con);
-  if (!ok) return set_error(OMPRT_E_CUDA, "omprt_xs_run_host: H2D copy failed");
-  d.bins = nullptr;
-  d.index_grid16 = nullptr;
-  d.brackets = nullptr;
-  if (accel) {
-    int32_t* bins = (int32_t*)(b + off);
-    off += al(asz[0]);
-    uint16_t* i16 = (uint16_t*)(b + off);
-    off += al(asz[1]);
-    double* br = (double*)(b + off);
-    off += al(asz[2]);
-    if (int r = launch_xs_accel(&d, bins, i16, br, log2_bins, s)) return r;
+  // the previous call's work on the user stream is ordered before this call's copies
+  OMPRT_CUDA_TRY(cudaEventRecord(w->compute_done[0], s));
+  OMPRT_CUDA_TRY(cudaEventRecord(w->compute_done[1], s));
+  OMPRT_CUDA_TRY(cudaMemsetAsync(w->dev_ck, 0, steps * sizeof(uint64_t), s));
+  for (int32_t st = 0; st < steps; ++st) {
+    const int b = st & 1;
+    unsigned char* base = (unsigned char*)w->xs_buf[b];
+    size_t off = 0;
+    bool ok = true;
+    cudaStream_t cs = w->copy_stream;
+    ok = ok && cudaStreamWaitEvent(cs, w->compute_done[b], 0) == cudaSuccess;
+    auto put = [&](const void* src, size_t bytes) -> void* {
+      void* dst = base + off;
+      off += al(bytes);
+      if (bytes) ok = ok && cudaMemcpyAsync(dst, src, bytes, cudaMemcpyHostToDevice, cs) ==
+                                cudaSuccess;
+      return dst;
+    };
+    omprt_xs_tables d = h;
+    d.nuclide_grid = upbr ? nullptr : (const double*)put(h.nuclide_grid, n_grid);
+    double* br = (double*)put(upbr ? h.brackets : nullptr, n_br);
+    d.unionized = (const double*)put(h.unionized, n_uni);
+    void* idx = put(up16 ? (const void*)h.index_grid16 : (const void*)h.index_grid, n_idx);
+    d.num_nucs = (const int32_t*)put(h.num_nucs, n_num);
+    d.mats = (const int32_t*)put(h.mats, n_mat);
+    d.concs = (const double*)put(h.concs, n_con);
+    ok = ok && cudaEventRecord(w->copy_done[b], cs) == cudaSuccess;
+    if (!ok) return set_error(OMPRT_E_CUDA, "omprt_xs_run_host_steps: H2D copy failed");
+    OMPRT_CUDA_TRY(cudaStreamWaitEvent(s, w->copy_done[b], 0));
+    d.index_grid = up16 ? nullptr : (const int32_t*)idx;
+    d.bins = nullptr;
+    d.index_grid16 = nullptr;
+    d.brackets = nullptr;
+    if (accel) {
+      int32_t* bins = (int32_t*)(base + off);
+      off += al(asz[0]);
+      uint16_t* i16 = up16 ? (uint16_t*)idx : (uint16_t*)(base + off);
+      off += al(built16);
+      double* brk = upbr ? br : (double*)(base + off);
+      off += al(builtbr);
+      xs_build_bins<<<1024, 256, 0, s>>>(d.unionized, (int32_t)d.n_union, log2_bins, bins);
+      if (!up16)
+        xs_build_index16<<<2048, 256, 0, s>>>(d.index_grid, i16,
+                                              (int64_t)d.n_union * d.n_isotopes);
+      if (!upbr)
+        xs_build_brackets<<<2048, 256, 0, s>>>(d.nuclide_grid, brk, d.n_isotopes,
+                                               d.n_gridpoints);
+      if (int r = check_launch("xs_build_accel")) return r;
+      d.bins = bins;
+      d.index_grid16 = i16;
+      d.brackets = brk;
+      d.log2_bins = log2_bins;
+    }
+    if (int r = omprt_xs_lookup(d, seed, first, count, nullptr, w->dev_ck + st, 0, threads,
+                                (flags & ~OMPRT_XS_ACCEL) | OMPRT_FUSED_REDUCTION |
+                                    OMPRT_ASSUME_OVERSUB,
+                                stream))
+      return r;
+    OMPRT_CUDA_TRY(cudaMemcpyAsync(w->pinned_ck + st, w->dev_ck + st, sizeof(uint64_t),
+                                   cudaMemcpyDeviceToHost, s));
+    OMPRT_CUDA_TRY(cudaEventRecord(w->compute_done[b], s));
   }
-  uint64_t* ck = w->scratch_u64;
-  OMPRT_CUDA_TRY(cudaMemsetAsync(ck, 0, sizeof(uint64_t), s));
-  if (int r = omprt_xs_lookup(d, seed, first, count, nullptr, ck, 0, threads,
-                              (flags & ~OMPRT_XS_ACCEL) | OMPRT_FUSED_REDUCTION |
-                                  OMPRT_ASSUME_OVERSUB,
-                              stream))
-    return r;
-  OMPRT_CUDA_TRY(cudaMemcpyAsync(checksum_host, ck, sizeof(uint64_t), cudaMemcpyDeviceToHost, s));
   OMPRT_CUDA_TRY(cudaStreamSynchronize(s));
-  if (h2d_bytes) *h2d_bytes = n_grid + n_uni + n_idx + n_num + n_mat + n_con;
+  memcpy(checksums_host, w->pinned_ck, steps * sizeof(uint64_t));
+  if (h2d_bytes)
+    *h2d_bytes = n_grid + n_br + n_uni + n_idx + n_num + n_mat + n_con;  // per step
   if (d2h_bytes) *d2h_bytes = sizeof(uint64_t);
   return OMPRT_OK;
+}
+
+extern "C" int omprt_xs_run_host(omprt_xs_tables h, uint64_t seed, int64_t first, int64_t count,
+                                 int32_t threads, uint32_t flags, uint64_t* checksum_host,
+                                 uint64_t* h2d_bytes, uint64_t* d2h_bytes, void* stream) {
+  return omprt_xs_run_host_steps(h, seed, first, count, threads, flags, 1, checksum_host,
+                                 h2d_bytes, d2h_bytes, stream);
 }

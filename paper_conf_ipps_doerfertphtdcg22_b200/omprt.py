@@ -42,7 +42,7 @@ EXPORTS = [
     "omprt_spmd_axpy_sum", "omprt_cuda_axpy_sum", "omprt_spmd_axpy_sum_chunked",
     "omprt_cuda_axpy_sum_chunked", "omprt_generic_team", "omprt_cuda_generic_team",
     "omprt_icv_probe", "omprt_xs_lookup", "omprt_cuda_xs_lookup", "omprt_u64_sum",
-    "omprt_xs_run_host", "omprt_xs_accel_sizes", "omprt_xs_build_accel", "omprt_rs_lookup", "omprt_cuda_rs_lookup", "omprt_su3_mult",
+    "omprt_xs_run_host", "omprt_xs_run_host_steps", "omprt_xs_accel_sizes", "omprt_xs_build_accel", "omprt_rs_lookup", "omprt_cuda_rs_lookup", "omprt_su3_mult",
     "omprt_cuda_su3_mult", "omprt_kernel_count", "omprt_kernel_name", "omprt_kernel_attrs",
 ]
 
@@ -99,6 +99,8 @@ _SIGS = {
     "omprt_xs_build_accel": [C.POINTER(XSTablesC), _vp, _vp, _vp, _i32, _vp],
     "omprt_xs_run_host": [XSTablesC, _u64, _i64, _i64, _i32, _u32, C.POINTER(_u64),
                           C.POINTER(_u64), C.POINTER(_u64), _vp],
+    "omprt_xs_run_host_steps": [XSTablesC, _u64, _i64, _i64, _i32, _u32, _i32, C.POINTER(_u64),
+                                C.POINTER(_u64), C.POINTER(_u64), _vp],
     "omprt_rs_lookup": [RSTablesC, _u64, _i64, _i64, _vp, _vp, _i32, _i32, _u32, _vp],
     "omprt_cuda_rs_lookup": [RSTablesC, _u64, _i64, _i64, _vp, _vp, _i32, _i32, _u32, _vp],
     "omprt_su3_mult": [_vp, _vp, _vp, _i64, _vp, _i32, _i32, _u32, _vp],
@@ -278,12 +280,24 @@ def omprt_xs_build_accel(tables, bins, index_grid16, brackets, log2_bins=16, str
 
 
 def xs_host_struct(t, pinned=None):
-    """By-value struct of HOST table pointers (numpy or pinned torch tensors)."""
+    """By-value struct of HOST table pointers (numpy arrays or pinned torch tensors).
+    `pinned` maps field names to host buffers; with "index_grid16" (and no "index_grid")
+    the compact 16-bit index grid crosses PCIe instead of the int32 one."""
     src = pinned or {}
-    g = lambda k: src.get(k, getattr(t, k))
-    return XSTablesC(_hp(g("nuclide_grid")), _hp(g("unionized")), _hp(g("index_grid")),
-                     _hp(g("num_nucs")), _hp(g("mats")), _hp(g("concs")), t.n_isotopes,
-                     t.n_gridpoints, t.max_num_nucs, 0, t.n_union, None, None, None, 0, 0)
+    g = lambda k: _hp(src[k]) if k in src else (_hp(getattr(t, k)) if k != "index_grid16" else None)
+    idx = None if ("index_grid16" in src and "index_grid" not in src) else g("index_grid")
+    return XSTablesC(g("nuclide_grid"), g("unionized"), idx, g("num_nucs"), g("mats"),
+                     g("concs"), t.n_isotopes, t.n_gridpoints, t.max_num_nucs, 0, t.n_union,
+                     None, g("index_grid16"), _hp(src.get("brackets")), 0, 0)
+
+
+def omprt_xs_run_host_steps(host_struct, seed, first, count, steps, threads=256, flags=0,
+                            stream=None):
+    cks = (_u64 * steps)()
+    hb, db = _u64(), _u64()
+    _check(load().omprt_xs_run_host_steps(host_struct, seed, first, count, threads, flags, steps,
+                                          cks, C.byref(hb), C.byref(db), _stream(stream)))
+    return list(cks), hb.value, db.value
 
 
 def omprt_xs_lookup(tables, seed, first, count, verification, checksum_inout=None, teams=0,

@@ -146,3 +146,18 @@ def test_end_to_end_host_tables(rt, xs_small):
         ck, h2d, d2h = rt.omprt_xs_run_host(hs, SEED, 0, n, 256, flags)
         assert ck == ref
         assert h2d == xs_small.nbytes() and d2h == 8
+
+
+def test_end_to_end_pipelined_steps_compact_host_layout(rt, xs_small):
+    """omprt_xs_run_host_steps: several steps, each with its own H2D (16-bit index grid on
+    the host), overlapped copies; every step's checksum equals the oracle's."""
+    pinned = {k: torch.from_numpy(getattr(xs_small, k)).pin_memory()
+              for k in ("nuclide_grid", "unionized", "index_grid16", "num_nucs", "mats",
+                        "concs")}
+    hs = rt.xs_host_struct(xs_small, pinned)
+    n = 200_000
+    ref = int(oracle.xs_lookup(xs_small, 5, n).sum())
+    cks, h2d, d2h = rt.omprt_xs_run_host_steps(hs, SEED, 5, n, 5)
+    assert cks == [ref] * 5
+    idx16 = xs_small.index_grid.size * 2
+    assert h2d == xs_small.nbytes() - xs_small.index_grid.nbytes + idx16 and d2h == 8

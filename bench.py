@@ -441,6 +441,12 @@ def run_secondary(omprt, torch, gen, dev, stream, scrub):
     t_ts = _time(lambda: omprt.omprt_cuda_su3_mult(At, Bt, Ct, ns, ck, 0, 128, TS), stream, scrub)
     res["c5_su3_32^4_tma_staged"] = {"rt_ms": t_rs, "twin_ms": t_ts, "overhead": t_rs / t_ts - 1,
                                      "GBps_alg": 1152 * ns / t_rs / 1e6}
+    WS = omprt.OMPRT_WARP_STAGED
+    t_rw = _time(lambda: omprt.omprt_su3_mult(At, Bt, Ct, ns, ck, 0, 128, WS), stream, scrub)
+    t_tww = _time(lambda: omprt.omprt_cuda_su3_mult(At, Bt, Ct, ns, ck, 0, 128, WS), stream, scrub)
+    res["c5_su3_32^4_warp_staged"] = {"rt_ms": t_rw, "twin_ms": t_tww,
+                                      "overhead": t_rw / t_tww - 1,
+                                      "GBps_alg": 1152 * ns / t_rw / 1e6}
     res["c5_su3_32^4"] = {"rt_ms": t_rt, "twin_ms": t_tw, "overhead": t_rt / t_tw - 1,
                           "GBps_alg": 1152 * ns / t_rt / 1e6, "GFLOPs": 864 * ns / t_rt / 1e6}
     return res

@@ -88,6 +88,12 @@ extern "C" {
  * memory slots (one persistent team of 128 per SM, per-thread double buffering); teams = 0:
  * one per SM.  Not combined with OMPRT_ASSUME_OVERSUB. */
 #define OMPRT_TMA_STAGED (1u << 13)
+/* omprt_su3_mult / omprt_cuda_su3_mult: warp-cooperative staging -- a warp's 32 consecutive
+ * site records (one contiguous 18 KiB range) are copied by coalesced 16 B cp.async into
+ * padded shared-memory slots and written back by coalesced 16 B stores (one persistent team
+ * of 192 per SM, per-warp double buffering); teams = 0: one per SM.  Exclusive with
+ * OMPRT_TMA_STAGED; not combined with OMPRT_ASSUME_OVERSUB. */
+#define OMPRT_WARP_STAGED (1u << 14)
 
 /* ---- runtime lifecycle ------------------------------------------------------------- */
 typedef struct {

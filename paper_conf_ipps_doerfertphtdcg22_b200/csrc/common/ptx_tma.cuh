@@ -1,6 +1,7 @@
-// PTX wrappers for bulk (TMA) copies and mbarriers (sm_90+; SASS UBLKCP / SYNCS.*).
+// PTX wrappers for bulk (TMA) copies and mbarriers (sm_90+; SASS UBLKCP / SYNCS.*) and
+// per-thread cp.async (LDGSTS).
 // Plain instruction wrappers, like CUDA intrinsics: used by the runtime's staging primitive
-// (omprt/device/tma.cuh) and by the hand-written twins alike.
+// (omprt/device/staging.cuh) and by the hand-written twins alike.
 #pragma once
 #include <cstdint>
 
@@ -64,6 +65,29 @@ __device__ __forceinline__ void bulk_wait() {
 // order this thread's generic-proxy shared-memory writes before async-proxy reads
 __device__ __forceinline__ void fence_proxy_async_smem() {
   asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+}
+
+// ---- per-thread 16 B asynchronous global->shared copies (sm_80+; SASS LDGSTS) ----------
+// .cg: cached in L2 only (streamed records are not re-read through L1).
+__device__ __forceinline__ void cp_async16(void* smem, const void* gmem) {
+  asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(smem_addr(smem)), "l"(gmem)
+               : "memory");
+}
+// shared-window address form; src_bytes (0 or 16) < 16 zero-fills the rest (no branch needed
+// for a ragged tail: with src_bytes = 0 nothing is read)
+__device__ __forceinline__ void cp_async16_zfill(uint32_t smem, const void* gmem,
+                                                 uint32_t src_bytes) {
+  asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" ::"r"(smem), "l"(gmem),
+               "r"(src_bytes)
+               : "memory");
+}
+__device__ __forceinline__ void cp_async_commit() {
+  asm volatile("cp.async.commit_group;" ::: "memory");
+}
+// wait until all but the `N` most recent of this thread's groups have landed
+template <int N>
+__device__ __forceinline__ void cp_async_wait() {
+  asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory");
 }
 
 }  // namespace tma

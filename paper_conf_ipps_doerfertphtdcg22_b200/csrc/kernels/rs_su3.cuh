@@ -186,8 +186,8 @@ OMPRT_REGISTER_KERNEL(omprt_su3_rt, omprt_su3_rt<SU3Traits, true>)
 OMPRT_REGISTER_KERNEL(omprt_su3_rt_loop, omprt_su3_rt<SU3TraitsLoop, true>)
 OMPRT_REGISTER_KERNEL(cuda_su3_twin, cuda_su3_twin<true>)
 
-// TMA-staged variant (su3_staged.cuh)
-inline int su3_staged_launch(bool twin, const double* A, const double* B, double* Cm,
+// staged variants (su3_staged.cuh)
+inline int su3_staged_launch(bool twin, bool warp, const double* A, const double* B, double* Cm,
                              int64_t n, double* ck, int32_t teams, Workspace* w,
                              cudaStream_t s);
 
@@ -253,14 +253,16 @@ extern "C" int omprt_su3_mult(const double* A, const double* B, double* Cm, int6
   using namespace omprt_kernels;
   Workspace* w;
   if (int r = current_ws(&w)) return r;
-  if (flags & OMPRT_TMA_STAGED) {
+  if (flags & (OMPRT_TMA_STAGED | OMPRT_WARP_STAGED)) {
     OMPRT_CHECK_ARG(threads == kSU3Threads && !(flags & OMPRT_ASSUME_OVERSUB),
-                    "the TMA-staged variant runs a persistent grid (no assumption)");
+                    "the staged variants run a persistent grid (no assumption)");
+    OMPRT_CHECK_ARG((flags & OMPRT_TMA_STAGED) == 0 || (flags & OMPRT_WARP_STAGED) == 0,
+                    "OMPRT_TMA_STAGED and OMPRT_WARP_STAGED are exclusive");
     int32_t tm = 1;
     if (int r = su3_validate(A, B, Cm, n_sites, tm, threads, 0, checksum_inout, w)) return r;
     if (n_sites == 0) return OMPRT_OK;
-    return su3_staged_launch(false, A, B, Cm, n_sites, checksum_inout, teams, w,
-                             as_stream(stream));
+    return su3_staged_launch(false, (flags & OMPRT_WARP_STAGED) != 0, A, B, Cm, n_sites,
+                             checksum_inout, teams, w, as_stream(stream));
   }
   if (int r = su3_validate(A, B, Cm, n_sites, teams, threads, flags, checksum_inout, w)) return r;
   if (n_sites == 0) return OMPRT_OK;
@@ -289,10 +291,12 @@ extern "C" int omprt_cuda_su3_mult(const double* A, const double* B, double* Cm,
   if (int r = current_ws(&w)) return r;
   int32_t tm = 0;
   if (int r = su3_validate(A, B, Cm, n_sites, tm, threads, 0, checksum_inout, w)) return r;
-  if (flags & OMPRT_TMA_STAGED) {
+  if (flags & (OMPRT_TMA_STAGED | OMPRT_WARP_STAGED)) {
+    OMPRT_CHECK_ARG((flags & OMPRT_TMA_STAGED) == 0 || (flags & OMPRT_WARP_STAGED) == 0,
+                    "OMPRT_TMA_STAGED and OMPRT_WARP_STAGED are exclusive");
     if (n_sites == 0) return OMPRT_OK;
-    return su3_staged_launch(true, A, B, Cm, n_sites, checksum_inout, teams, w,
-                             as_stream(stream));
+    return su3_staged_launch(true, (flags & OMPRT_WARP_STAGED) != 0, A, B, Cm, n_sites,
+                             checksum_inout, teams, w, as_stream(stream));
   }
   (void)teams;
   (void)flags;

@@ -1,12 +1,13 @@
-// C5 with TMA staging (OMPRT_TMA_STAGED): the SU(3) site loop as a persistent
+// C5 with shared-memory staging: OMPRT_TMA_STAGED (per-thread bulk copies) and
+// OMPRT_WARP_STAGED (warp-cooperative cp.async).  TMA staging: the SU(3) site loop as a persistent
 // `distribute parallel for` (one team of 128 per SM, Fig. 5 assignment) whose site records
 // (576 B, AoS) are moved by bulk copies into padded shared-memory slots and back
-// (omprt/device/tma.cuh), instead of 32-line-wide strided global accesses.  The twin runs
+// (omprt/device/staging.cuh), instead of 32-line-wide strided global accesses.  The twin runs
 // the same per-thread double-buffered bulk-copy pipeline, written by hand.
 #pragma once
 #include "../common/ptx_tma.cuh"
 #include "../host/runtime.cuh"
-#include "../omprt/device/tma.cuh"
+#include "../omprt/device/staging.cuh"
 #include "rs_su3.cuh"
 
 namespace omprt_kernels {
@@ -48,6 +49,46 @@ __device__ __forceinline__ double su3_site_slot(unsigned char* slot,
       }
   }
   return re_sum;
+}
+
+// The twins' hand-written league reduction (warp butterflies, per-block partial, last block
+// by ticket folds the partials and adds to *checksum).
+__device__ __forceinline__ void twin_ticket_sum(double acc, double* checksum, double* partials,
+                                                unsigned* ticket) {
+  const unsigned nt = blockDim.x, t = threadIdx.x;
+  __shared__ double ws[32];
+  __shared__ unsigned last;
+  for (int off = 16; off > 0; off >>= 1) acc += __shfl_xor_sync(0xffffffffu, acc, off);
+  const unsigned lane = t & 31u, wid = t >> 5, nw = nt >> 5;
+  if (lane == 0) ws[wid] = acc;
+  __syncthreads();
+  double b = 0.0;
+  if (wid == 0) {
+    b = lane < nw ? ws[lane] : 0.0;
+    for (int off = 16; off > 0; off >>= 1) b += __shfl_xor_sync(0xffffffffu, b, off);
+  }
+  if (t == 0) {
+    partials[blockIdx.x] = b;
+    __threadfence();
+    last = atomicAdd(ticket, 1u) == gridDim.x - 1;
+  }
+  __syncthreads();
+  if (last) {
+    __threadfence();
+    double tt = 0.0;
+    for (unsigned k = t; k < gridDim.x; k += nt) tt += __ldcg(partials + k);
+    for (int off = 16; off > 0; off >>= 1) tt += __shfl_xor_sync(0xffffffffu, tt, off);
+    if (lane == 0) ws[wid] = tt;
+    __syncthreads();
+    if (wid == 0) {
+      double u = lane < nw ? ws[lane] : 0.0;
+      for (int off = 16; off > 0; off >>= 1) u += __shfl_xor_sync(0xffffffffu, u, off);
+      if (t == 0) {
+        *checksum = *checksum + u;
+        *ticket = 0u;
+      }
+    }
+  }
 }
 
 struct SU3StagedTraits : DefaultTraits {};  // persistent grid: the loop stays
@@ -112,72 +153,134 @@ __global__ void __launch_bounds__(kSU3StagedThreads, 1)
     tma::bulk_commit();
   }
   tma::bulk_wait<0>();
-  if constexpr (Checksum) {
-    __shared__ double ws[32];
-    __shared__ unsigned last;
-    for (int off = 16; off > 0; off >>= 1) acc += __shfl_xor_sync(0xffffffffu, acc, off);
-    const unsigned lane = t & 31u, wid = t >> 5, nw = nt >> 5;
-    if (lane == 0) ws[wid] = acc;
-    __syncthreads();
-    double b = 0.0;
-    if (wid == 0) {
-      b = lane < nw ? ws[lane] : 0.0;
-      for (int off = 16; off > 0; off >>= 1) b += __shfl_xor_sync(0xffffffffu, b, off);
-    }
-    if (t == 0) {
-      partials[blockIdx.x] = b;
-      __threadfence();
-      last = atomicAdd(ticket, 1u) == gridDim.x - 1;
-    }
-    __syncthreads();
-    if (last) {
-      __threadfence();
-      double tt = 0.0;
-      for (unsigned k = t; k < gridDim.x; k += nt) tt += __ldcg(partials + k);
-      for (int off = 16; off > 0; off >>= 1) tt += __shfl_xor_sync(0xffffffffu, tt, off);
-      if (lane == 0) ws[wid] = tt;
-      __syncthreads();
-      if (wid == 0) {
-        double u = lane < nw ? ws[lane] : 0.0;
-        for (int off = 16; off > 0; off >>= 1) u += __shfl_xor_sync(0xffffffffu, u, off);
-        if (t == 0) {
-          *checksum = *checksum + u;
-          *ticket = 0u;
-        }
-      }
-    }
-  }
+  if constexpr (Checksum) twin_ticket_sum(acc, checksum, partials, ticket);
 }
 
 OMPRT_REGISTER_KERNEL(omprt_su3_staged_rt, omprt_su3_staged_rt<SU3StagedTraits, true>)
 OMPRT_REGISTER_KERNEL(cuda_su3_staged_twin, cuda_su3_staged_twin<true>)
 
-// persistent geometry: one team per SM (153 KB of slots + barriers)
-inline int su3_staged_launch(bool twin, const double* A, const double* B, double* Cm,
-                             int64_t n, double* ck, int32_t teams, Workspace* w,
+// ---- warp-cooperative staging (OMPRT_WARP_STAGED): coalesced cp.async in, STG.128 out ----
+constexpr int kSU3WarpThreads = 192;  // 6 warps x 2 x 32 slots x 592 B = 222 KB per team
+
+template <class Tr, bool Checksum>
+__global__ void __launch_bounds__(kSU3WarpThreads, 1)
+    omprt_su3_wstaged_rt(const double* __restrict__ A, const double2* __restrict__ B,
+                         double* __restrict__ Cm, typename Tr::Idx n_sites, double* checksum,
+                         double* partials, unsigned* ticket) {
+  using Idx = typename Tr::Idx;
+  Team<Tr> team = init<Tr>();
+  double acc = 0.0;
+  distribute_parallel_for_warp_staged<Tr, kSU3Rec, kSU3Slot>(
+      team, n_sites, reinterpret_cast<const unsigned char*>(A),
+      reinterpret_cast<unsigned char*>(Cm),
+      [&](Idx, unsigned char* slot) { acc += su3_site_slot(slot, B); });
+  if constexpr (Checksum)
+    league_reduce(team, team_reduce_to_main(team, acc, Plus{}), Plus{}, checksum, partials,
+                  ticket);
+}
+
+// Bare CUDA twin: the same warp tile pipeline, by hand.
+template <bool Checksum>
+__global__ void __launch_bounds__(kSU3WarpThreads, 1)
+    cuda_su3_wstaged_twin(const double* __restrict__ A, const double2* __restrict__ B,
+                          double* __restrict__ Cm, int32_t n_sites, double* checksum,
+                          double* partials, unsigned* ticket) {
+  constexpr unsigned kCh = kSU3Rec / 16;  // 36 chunks per site
+  extern __shared__ __align__(128) unsigned char smem[];
+  const unsigned nt = blockDim.x, t = threadIdx.x, lane = t & 31u, w0 = t & ~31u;
+  unsigned char* buf0 = smem + w0 * kSU3Slot;
+  unsigned char* buf1 = smem + (nt + w0) * kSU3Slot;
+  const unsigned char* in = reinterpret_cast<const unsigned char*>(A);
+  unsigned char* out = reinterpret_cast<unsigned char*>(Cm);
+  const int32_t stride = gridDim.x * nt;
+  int32_t base = blockIdx.x * nt + w0;
+  double acc = 0.0;
+  const uint32_t s0 = tma::smem_addr(buf0), s1 = tma::smem_addr(buf1);
+  auto fetch = [&](uint32_t b, int32_t wb) {  // zero-fill past the tile: no branches
+    const unsigned nch = (unsigned)min(32, n_sites - wb) * kCh;
+    const unsigned char* src = in + (size_t)wb * kSU3Rec;
+#pragma unroll
+    for (unsigned j = 0; j < kCh; ++j) {
+      const unsigned c = lane + 32u * j;
+      tma::cp_async16_zfill(b + (c / kCh) * kSU3Slot + (c % kCh) * 16u,
+                            src + (c < nch ? c * 16u : 0u), c < nch ? 16u : 0u);
+    }
+    tma::cp_async_commit();
+  };
+  if (base < n_sites) fetch(s0, base);
+  for (unsigned k = 0; base < n_sites; base += stride, ++k) {
+    unsigned char* cur = (k & 1) ? buf1 : buf0;
+    if (base + stride < n_sites) {
+      fetch((k & 1) ? s0 : s1, base + stride);
+      tma::cp_async_wait<1>();
+    } else {
+      tma::cp_async_wait<0>();
+    }
+    __syncwarp();
+    if (base + (int32_t)lane < n_sites) acc += su3_site_slot(cur + lane * kSU3Slot, B);
+    __syncwarp();
+    const unsigned nch = (unsigned)min(32, n_sites - base) * kCh;
+    unsigned char* dst = out + (size_t)base * kSU3Rec;
+#pragma unroll
+    for (unsigned j = 0; j < kCh; ++j) {
+      const unsigned c = lane + 32u * j;
+      if (c < nch)
+        *reinterpret_cast<uint4*>(dst + c * 16u) =
+            *reinterpret_cast<const uint4*>(cur + (c / kCh) * kSU3Slot + (c % kCh) * 16u);
+    }
+    __syncwarp();
+  }
+  if constexpr (Checksum) twin_ticket_sum(acc, checksum, partials, ticket);
+}
+
+OMPRT_REGISTER_KERNEL(omprt_su3_wstaged_rt, omprt_su3_wstaged_rt<SU3StagedTraits, true>)
+OMPRT_REGISTER_KERNEL(cuda_su3_wstaged_twin, cuda_su3_wstaged_twin<true>)
+
+// persistent geometry: one team per SM.  warp = false: per-thread bulk copies (128 threads,
+// 153 KB of slots + barriers); warp = true: warp-cooperative cp.async (192 threads, 222 KB).
+template <class K>
+inline int su3_staged_go(K k, uint32_t smem, int32_t teams, int threads, const double* A,
+                         const double2* B, double* Cm, int32_t n, double* ck, double* p,
+                         unsigned* tk, cudaStream_t s) {
+  OMPRT_CUDA_TRY(cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
+  k<<<teams, threads, smem, s>>>(A, B, Cm, n, ck, p, tk);
+  return OMPRT_OK;
+}
+
+inline int su3_staged_launch(bool twin, bool warp, const double* A, const double* B,
+                             double* Cm, int64_t n, double* ck, int32_t teams, Workspace* w,
                              cudaStream_t s) {
-  const uint32_t smem = staged_smem_bytes<kSU3Slot, 2>(kSU3StagedThreads);
+  const int threads = warp ? kSU3WarpThreads : kSU3StagedThreads;
+  const uint32_t smem = warp ? warp_staged_smem_bytes<kSU3Slot>(kSU3WarpThreads)
+                             : staged_smem_bytes<kSU3Slot, 2>(kSU3StagedThreads);
   int dev = 0, sms = 148;
   cudaGetDevice(&dev);
   cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
   if (teams <= 0) teams = sms;
   OMPRT_CHECK_ARG(!ck || (uint64_t)teams <= w->opt.max_teams, "teams exceed max_teams");
-  OMPRT_CHECK_ARG(n + 2 * (int64_t)teams * kSU3StagedThreads < INT32_MAX, "n_sites too large");
+  OMPRT_CHECK_ARG(n + 2 * (int64_t)teams * threads < INT32_MAX, "n_sites too large");
   const int32_t nn = (int32_t)n;
   auto* b2 = (const double2*)B;
   double* p = (double*)w->partials;
   unsigned* tk = w->tickets + 3;
-  if (twin) {
-    auto k = ck ? cuda_su3_staged_twin<true> : cuda_su3_staged_twin<false>;
-    OMPRT_CUDA_TRY(cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
-    k<<<teams, kSU3StagedThreads, smem, s>>>(A, b2, Cm, nn, ck, p, tk);
-  } else {
-    auto k = ck ? omprt_su3_staged_rt<SU3StagedTraits, true>
-                : omprt_su3_staged_rt<SU3StagedTraits, false>;
-    OMPRT_CUDA_TRY(cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
-    k<<<teams, kSU3StagedThreads, smem, s>>>(A, b2, Cm, nn, ck, p, tk);
-  }
-  return check_launch(twin ? "cuda_su3_staged_twin" : "omprt_su3_staged_rt");
+  int r;
+  if (warp && twin)
+    r = su3_staged_go(ck ? cuda_su3_wstaged_twin<true> : cuda_su3_wstaged_twin<false>, smem,
+                      teams, threads, A, b2, Cm, nn, ck, p, tk, s);
+  else if (warp)
+    r = su3_staged_go(ck ? omprt_su3_wstaged_rt<SU3StagedTraits, true>
+                         : omprt_su3_wstaged_rt<SU3StagedTraits, false>,
+                      smem, teams, threads, A, b2, Cm, nn, ck, p, tk, s);
+  else if (twin)
+    r = su3_staged_go(ck ? cuda_su3_staged_twin<true> : cuda_su3_staged_twin<false>, smem,
+                      teams, threads, A, b2, Cm, nn, ck, p, tk, s);
+  else
+    r = su3_staged_go(ck ? omprt_su3_staged_rt<SU3StagedTraits, true>
+                         : omprt_su3_staged_rt<SU3StagedTraits, false>,
+                      smem, teams, threads, A, b2, Cm, nn, ck, p, tk, s);
+  if (r) return r;
+  return check_launch(warp ? (twin ? "cuda_su3_wstaged_twin" : "omprt_su3_wstaged_rt")
+                           : (twin ? "cuda_su3_staged_twin" : "omprt_su3_staged_rt"));
 }
 
 }  // namespace omprt_kernels

@@ -1,0 +1,178 @@
+// omprt device runtime -- staging of per-iteration records through shared memory: per-thread
+// bulk (TMA) copies (sm_90+ cp.async.bulk + mbarrier; SASS UBLKCP / SYNCS) and warp-
+// cooperative 16 B cp.async (SASS LDGSTS), see distribute_parallel_for_warp_staged below.
+//
+// north_star: "shared-memory or TMA staging".  A loop whose iteration i reads a fixed-size
+// record in[i] and writes a record out[i] of an AoS array (SU(3): 576 B per site) makes
+// every warp-wide load touch 32 different cache lines.  The runtime instead moves each
+// record with one bulk copy into a padded shared-memory slot owned by the thread that runs
+// iteration i under the Fig. 5 assignment, the body works on the slot, and the runtime
+// bulk-stores the slot to out[i].  Every thread runs its own double-buffered pipeline
+// (own mbarriers, own bulk groups), so no CTA-wide barrier is involved.
+#pragma once
+#include <cstdint>
+
+#include "../../common/ptx_tma.cuh"
+#include "state.cuh"
+
+namespace omprt {
+
+
+// Shared-memory footprint of distribute_parallel_for_staged for `team_size` threads.
+template <unsigned kSlotBytes, unsigned kBuffers>
+__host__ __device__ constexpr uint32_t staged_smem_bytes(uint32_t team_size) {
+  return team_size * (kBuffers * kSlotBytes + kBuffers * 8u);
+}
+
+// `distribute parallel for` (Fig. 5 assignment) whose iteration i reads the kRecBytes record
+// in + i*kRecBytes and writes the record out + i*kRecBytes: the runtime stages the record
+// into this thread's slot (kSlotBytes >= kRecBytes, padded against bank conflicts), calls
+// body(i, slot) -- which computes in place -- and bulk-stores the slot.  Double buffered:
+// the record of the thread's next iteration is in flight while the body runs.
+// Needs staged_smem_bytes<kSlotBytes, 2>(team_size) bytes of dynamic shared memory.
+template <class Tr, unsigned kRecBytes, unsigned kSlotBytes, class Body>
+__device__ __forceinline__ void distribute_parallel_for_staged(Team<Tr>& team,
+                                                               typename Tr::Idx n,
+                                                               const unsigned char* in,
+                                                               unsigned char* out, Body&& body) {
+  using Idx = typename Tr::Idx;
+  static_assert(kRecBytes % 16 == 0 && kSlotBytes % 16 == 0 && kSlotBytes >= kRecBytes,
+                "bulk copies move multiples of 16 B into 16 B-aligned slots");
+  OMPRT_TRACE(Tr, "distribute_parallel_for_staged");
+  extern __shared__ __align__(128) unsigned char omprt_stage_smem[];
+  const uint32_t nt = (uint32_t)team.team_size, t = (uint32_t)team.thread_num;
+  // two named slots, selected (not indexed): an indexed pointer array would live in local memory
+  unsigned char* const slot0 = omprt_stage_smem + (0 * nt + t) * kSlotBytes;
+  unsigned char* const slot1 = omprt_stage_smem + (1 * nt + t) * kSlotBytes;
+  uint64_t* bar = reinterpret_cast<uint64_t*>(omprt_stage_smem + 2 * nt * kSlotBytes) + 2 * t;
+  tma::mbar_init(bar + 0, 1);
+  tma::mbar_init(bar + 1, 1);
+  tma::fence_mbar_init();
+  const Idx total = (Idx)gridDim.x * (Idx)nt;
+  Idx iv = (Idx)blockIdx.x * (Idx)nt + (Idx)t;
+  if (Tr::assume_teams_oversub) OMPRT_ASSERT(Tr, n <= total, "oversubscription assumption violated");
+  // prologue: the first iteration's record
+  if (iv < n) {
+    tma::mbar_arrive_expect_tx(bar + 0, kRecBytes);
+    tma::bulk_load(slot0, in + (size_t)iv * kRecBytes, kRecBytes, bar + 0);
+  }
+  uint32_t k = 0, phase0 = 0, phase1 = 0;
+  for (; iv < n; iv += total, ++k) {
+    const uint32_t b = k & 1u;
+    const Idx nx = iv + total;
+    if (!Tr::assume_teams_oversub && nx < n) {
+      // the next record goes to the other slot once its previous store has read it
+      tma::bulk_wait_read<0>();
+      tma::mbar_arrive_expect_tx(bar + (b ^ 1u), kRecBytes);
+      tma::bulk_load(b ? slot0 : slot1, in + (size_t)nx * kRecBytes, kRecBytes, bar + (b ^ 1u));
+    }
+    tma::mbar_wait(bar + b, b ? phase1 : phase0);
+    if (b) phase1 ^= 1u;
+    else phase0 ^= 1u;
+    unsigned char* const cur = b ? slot1 : slot0;
+    body(iv, cur);
+    tma::fence_proxy_async_smem();
+    tma::bulk_store(out + (size_t)iv * kRecBytes, cur, kRecBytes);
+    tma::bulk_commit();
+    if (Tr::assume_teams_oversub) break;
+  }
+  tma::bulk_wait<0>();  // stores complete before the thread exits
+}
+
+// ---- warp-cooperative staging (cp.async / LDGSTS) ---------------------------------------
+// Under the Fig. 5 assignment the 32 lanes of a warp run 32 consecutive iterations, so the
+// warp's 32 records are one contiguous byte range.  The warp copies that range with
+// coalesced 16 B cp.async (each warp instruction moves 512 contiguous bytes) into 32 padded
+// slots, each lane runs body(i, slot) on its own slot, and the warp writes the slots back
+// with coalesced 16 B stores.  Double buffered per warp: the next tile's range is in flight
+// while the body runs.  Only __syncwarp orders the lanes; the team never synchronizes.
+
+template <unsigned kSlotBytes>
+__host__ __device__ constexpr uint32_t warp_staged_smem_bytes(uint32_t team_size) {
+  return team_size * 2u * kSlotBytes;
+}
+
+namespace detail {
+// chunk c (16 B) of the tile's byte range belongs to record c / kChunks
+template <unsigned kRecBytes, unsigned kSlotBytes>
+__device__ __forceinline__ void warp_stage_in(uint32_t sbuf, const unsigned char* src,
+                                              uint32_t cnt, uint32_t lane) {
+  constexpr uint32_t kChunks = kRecBytes / 16;
+  const uint32_t nch = cnt * kChunks;
+#pragma unroll
+  for (uint32_t j = 0; j < kChunks; ++j) {
+    const uint32_t c = lane + 32u * j;
+    const uint32_t r = c / kChunks, q = c - r * kChunks;
+    // chunks past the tile's last record zero-fill their (unused) slot bytes: branch-free
+    const bool in_tile = c < nch;
+    tma::cp_async16_zfill(sbuf + r * kSlotBytes + q * 16u, src + (in_tile ? c * 16u : 0u),
+                          in_tile ? 16u : 0u);
+  }
+  tma::cp_async_commit();
+}
+template <unsigned kRecBytes, unsigned kSlotBytes>
+__device__ __forceinline__ void warp_stage_out(const unsigned char* buf, unsigned char* dst,
+                                               uint32_t cnt, uint32_t lane) {
+  constexpr uint32_t kChunks = kRecBytes / 16;
+  const uint32_t nch = cnt * kChunks;
+#pragma unroll
+  for (uint32_t j = 0; j < kChunks; ++j) {
+    const uint32_t c = lane + 32u * j;
+    if (c < nch) {
+      const uint32_t r = c / kChunks, q = c - r * kChunks;
+      const uint4 v = *reinterpret_cast<const uint4*>(buf + r * kSlotBytes + q * 16u);
+      *reinterpret_cast<uint4*>(dst + c * 16u) = v;
+    }
+  }
+}
+}  // namespace detail
+
+// `distribute parallel for` (Fig. 5 assignment) over records of kRecBytes, staged per warp.
+// Needs warp_staged_smem_bytes<kSlotBytes>(team_size) bytes of dynamic shared memory and a
+// team size that is a multiple of 32.
+template <class Tr, unsigned kRecBytes, unsigned kSlotBytes, class Body>
+__device__ __forceinline__ void distribute_parallel_for_warp_staged(Team<Tr>& team,
+                                                                    typename Tr::Idx n,
+                                                                    const unsigned char* in,
+                                                                    unsigned char* out,
+                                                                    Body&& body) {
+  using Idx = typename Tr::Idx;
+  static_assert(kRecBytes % 16 == 0 && kSlotBytes % 16 == 0 && kSlotBytes >= kRecBytes,
+                "16 B copies into 16 B-aligned slots");
+  OMPRT_TRACE(Tr, "distribute_parallel_for_warp_staged");
+  extern __shared__ __align__(128) unsigned char omprt_stage_smem[];
+  const uint32_t nt = (uint32_t)team.team_size, t = (uint32_t)team.thread_num;
+  OMPRT_ASSERT(Tr, nt % 32u == 0, "warp staging needs whole warps");
+  const uint32_t lane = t & 31u, w0 = t & ~31u;
+  unsigned char* const buf0 = omprt_stage_smem + w0 * kSlotBytes;
+  unsigned char* const buf1 = omprt_stage_smem + (nt + w0) * kSlotBytes;
+  const Idx total = (Idx)gridDim.x * (Idx)nt;
+  Idx base = (Idx)blockIdx.x * (Idx)nt + (Idx)w0;  // the warp's first iteration
+  if (Tr::assume_teams_oversub) OMPRT_ASSERT(Tr, n <= total, "oversubscription assumption violated");
+  const uint32_t sbuf0 = tma::smem_addr(buf0), sbuf1 = tma::smem_addr(buf1);
+  auto tile = [&](Idx b) { return n - b < (Idx)32 ? (uint32_t)(n - b) : 32u; };
+  if (base < n)
+    detail::warp_stage_in<kRecBytes, kSlotBytes>(sbuf0, in + (size_t)base * kRecBytes,
+                                                 tile(base), lane);
+  for (uint32_t k = 0; base < n; base += total, ++k) {
+    unsigned char* const cur = (k & 1u) ? buf1 : buf0;
+    const Idx nx = base + total;
+    if (!Tr::assume_teams_oversub && nx < n) {
+      detail::warp_stage_in<kRecBytes, kSlotBytes>((k & 1u) ? sbuf0 : sbuf1,
+                                                   in + (size_t)nx * kRecBytes, tile(nx), lane);
+      tma::cp_async_wait<1>();
+    } else {
+      tma::cp_async_wait<0>();
+    }
+    __syncwarp();
+    const Idx iv = base + (Idx)lane;
+    if (iv < n) body(iv, cur + lane * kSlotBytes);
+    __syncwarp();
+    detail::warp_stage_out<kRecBytes, kSlotBytes>(cur, out + (size_t)base * kRecBytes,
+                                                  tile(base), lane);
+    __syncwarp();  // the slots are refilled by the fetch two tiles on
+    if (Tr::assume_teams_oversub) break;
+  }
+}
+
+}  // namespace omprt

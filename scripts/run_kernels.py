@@ -25,6 +25,9 @@ elif which == "su3":
     for _ in range(reps):
         omprt.omprt_su3_mult(At, Bt, Ct, ns, ck, 0, 128, A)
         omprt.omprt_cuda_su3_mult(At, Bt, Ct, ns, ck, 0, 128, 0)
+        for fl in (omprt.OMPRT_TMA_STAGED, omprt.OMPRT_WARP_STAGED):
+            omprt.omprt_su3_mult(At, Bt, Ct, ns, ck, 0, 128, fl)
+            omprt.omprt_cuda_su3_mult(At, Bt, Ct, ns, ck, 0, 128, fl)
 elif which == "generic":
     T = 4096; inp = torch.from_numpy(gen.generic_inputs(T, 256)).to(dev)
     out = torch.empty(T * 256, dtype=torch.float64, device=dev)

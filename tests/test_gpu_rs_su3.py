@@ -69,17 +69,43 @@ def _su3(rt, fn, A, B, n, flags=0):
 
 
 @pytest.mark.parametrize("n", [8 ** 4, 8 ** 4 + 5, 32 ** 4])
-@pytest.mark.parametrize("variant", ["rt", "rt_loop", "twin", "rt_staged", "twin_staged"])
+@pytest.mark.parametrize("variant", ["rt", "rt_loop", "twin", "rt_staged", "twin_staged",
+                                     "rt_wstaged", "twin_wstaged"])
 def test_su3_bit_exact(rt, n, variant):
     A, B = gen.su3_inputs(n)
     fn = rt.omprt_cuda_su3_mult if variant.startswith("twin") else rt.omprt_su3_mult
     flags = {"rt": rt.OMPRT_ASSUME_OVERSUB, "rt_loop": 0, "twin": 0,
-             "rt_staged": rt.OMPRT_TMA_STAGED, "twin_staged": rt.OMPRT_TMA_STAGED}[variant]
+             "rt_staged": rt.OMPRT_TMA_STAGED, "twin_staged": rt.OMPRT_TMA_STAGED,
+             "rt_wstaged": rt.OMPRT_WARP_STAGED, "twin_wstaged": rt.OMPRT_WARP_STAGED}[variant]
     C, ck = _su3(rt, fn, A, B, n, flags)
     Cref = oracle.su3_mult(A, B, n, threads=os.cpu_count() or 1)
     assert (C == Cref).all()
     re = Cref[0::2]
     assert abs(ck - oracle.sum_f64(re)) <= 1e-12 * oracle.sum_abs_f64(re)
+
+
+@pytest.mark.parametrize("flag", ["OMPRT_TMA_STAGED", "OMPRT_WARP_STAGED"])
+@pytest.mark.parametrize("teams", [1, 3, 148])
+def test_su3_staged_geometries(rt, flag, teams):
+    """Few persistent teams (many tiles per warp, both buffers cycling) and a ragged last
+    tile (n not a multiple of 32) stay bit-exact."""
+    n = 4 * 192 * 3 + 37
+    A, B = gen.su3_inputs(n)
+    At, Bt = torch.from_numpy(A).to(DEV), torch.from_numpy(B).to(DEV)
+    Ct = torch.full((n * 72 + 72,), float("nan"), dtype=torch.float64, device=DEV)
+    rt.omprt_su3_mult(At, Bt, Ct, n, None, teams, 128, getattr(rt, flag))
+    torch.cuda.synchronize()
+    C = Ct.cpu().numpy()
+    assert (C[:n * 72] == oracle.su3_mult(A, B, n)).all()
+    assert np.isnan(C[n * 72:]).all()  # nothing written past the last record
+
+
+def test_su3_staged_flags_exclusive(rt):
+    A = torch.zeros(72 * 64, dtype=torch.float64, device=DEV)
+    B = torch.zeros(72, dtype=torch.float64, device=DEV)
+    both = rt.OMPRT_TMA_STAGED | rt.OMPRT_WARP_STAGED
+    with pytest.raises(Exception):
+        rt.omprt_su3_mult(A, B, A, 64, None, 0, 128, both)
 
 
 def test_su3_pins_on_gpu(rt):

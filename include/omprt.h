@@ -94,6 +94,13 @@ extern "C" {
  * of 192 per SM, per-warp double buffering); teams = 0: one per SM.  Exclusive with
  * OMPRT_TMA_STAGED; not combined with OMPRT_ASSUME_OVERSUB. */
 #define OMPRT_WARP_STAGED (1u << 14)
+/* omprt_xs_lookup / omprt_cuda_xs_lookup (B200 layouts required) and the e2e entry points:
+ * flattened execution -- a persistent grid (teams = 0: the device's resident teams) whose
+ * threads run their Fig. 5 iterations with the per-lookup nuclide loop fused into the
+ * iteration loop (omprt::distribute_parallel_for_flat), so a SIMT lane that finishes its
+ * lookup starts its next one instead of waiting for the warp's longest lookup.  Identical
+ * results.  Not combined with OMPRT_ASSUME_OVERSUB or OMPRT_DEBUG_BUILD. */
+#define OMPRT_XS_FLAT (1u << 15)
 
 /* ---- runtime lifecycle ------------------------------------------------------------- */
 typedef struct {

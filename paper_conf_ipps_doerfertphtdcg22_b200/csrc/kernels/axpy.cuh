@@ -20,11 +20,6 @@ struct AxpyTraitsDebug : AxpyTraits {
 struct AxpyTraitsAssumeDebug : AxpyTraitsAssume {
   static constexpr unsigned debug = dbg::Assert | dbg::Trace;
 };
-template <class Base>
-struct WithIdx64 : Base {
-  using Idx = int64_t;
-};
-
 // Runtime-driven kernel: the OpenMP region as the runtime executes it.
 template <class Tr, bool Rec>
 __global__ void __launch_bounds__(1024)

@@ -50,8 +50,12 @@ __host__ __device__ constexpr LcgJumps make_lcg_jumps() {
 }
 __constant__ LcgJumps kLcgJumpTable = make_lcg_jumps();
 
-// fast_forward_LCG(seed, n): compose the jumps of n's set bits (square-and-multiply).
-__device__ __forceinline__ uint64_t lcg_fast_forward(uint64_t seed, uint64_t n) {
+// The affine map (a, c) of n LCG steps: compose the jumps of n's set bits
+// (square-and-multiply).
+struct LcgMap {
+  uint64_t a, c;
+};
+__device__ __forceinline__ LcgMap lcg_jump(uint64_t n) {
   uint64_t a_new = 1, c_new = 0;
   for (int k = 0; n != 0; ++k, n >>= 1) {
     if (n & 1) {
@@ -60,7 +64,14 @@ __device__ __forceinline__ uint64_t lcg_fast_forward(uint64_t seed, uint64_t n) 
       c_new = c_new * ak + kLcgJumpTable.c[k];
     }
   }
-  return (a_new * seed + c_new) & kLcgMask;
+  return {a_new, c_new};
+}
+__device__ __forceinline__ uint64_t lcg_apply(LcgMap m, uint64_t seed) {
+  return (m.a * seed + m.c) & kLcgMask;
+}
+// fast_forward_LCG(seed, n)
+__device__ __forceinline__ uint64_t lcg_fast_forward(uint64_t seed, uint64_t n) {
+  return lcg_apply(lcg_jump(n), seed);
 }
 
 __device__ __forceinline__ double lcg_double(uint64_t& seed) {
@@ -209,6 +220,100 @@ __device__ __forceinline__ uint64_t xs_lookup_accel(const XSTables& t, uint64_t 
   }
   return xs_argmax5(m0, m1, m2, m3, m4);
 }
+
+// The lookup as a RESUMABLE body for the runtime's flattened loop
+// (omprt::distribute_parallel_for_flat): begin/next sample the lookup and search the grid,
+// each step() accumulates P nuclides (the next P index entries prefetched, as
+// xs_lookup_accel), end() takes the argmax.  Same values, same order, same fma points as
+// xs_lookup_accel, so the verification bits are identical.  A thread's next lookup is
+// iv + T*N (Fig. 5): its seed is the current seed advanced by the 2*T*N-step jump, one
+// 64-bit multiply-add instead of a fast-forward from the start (exact: the LCG is affine).
+template <bool Fused, int P = 2>
+struct XSFlatLookup {
+  const XSTables& t;
+  const uint64_t seed0;
+  const int64_t first;
+  uint64_t* __restrict__ const ver;
+  unsigned long long acc = 0;  // Fused: this thread's verification sum
+  LcgMap J;
+  uint64_t s;
+  double E;
+  int32_t mat, idx, nn, j;
+  double m0, m1, m2, m3, m4;
+  int32_t pc[P], kc[P];
+
+  __device__ __forceinline__ XSFlatLookup(const XSTables& tab, uint64_t seed, int64_t first_,
+                                          uint64_t* verification)
+      : t(tab), seed0(seed), first(first_), ver(verification) {}
+
+  __device__ __forceinline__ void start() {
+    uint64_t seed = s;
+    E = lcg_double(seed);
+    mat = pick_mat(seed);
+    idx = binned_grid_search(t, E);
+    nn = __ldg(t.num_nucs + mat);
+    m0 = m1 = m2 = m3 = m4 = 0.0;
+    j = 0;
+    const int32_t* __restrict__ mrow = t.mats + mat * t.max_num_nucs;
+    const uint16_t* __restrict__ irow = t.index_grid16 + (int64_t)idx * t.n_isotopes;
+#pragma unroll
+    for (int u = 0; u < P; ++u) {
+      pc[u] = u < nn ? __ldg(mrow + u) : 0;
+      kc[u] = u < nn ? (int32_t)__ldg(irow + pc[u]) : 0;
+    }
+  }
+  template <class Idx>
+  __device__ __forceinline__ void begin(Idx iv, Idx stride) {
+    J = lcg_jump(2ull * (uint64_t)stride);
+    s = lcg_fast_forward(seed0, 2ull * (uint64_t)(first + iv));
+    start();
+  }
+  template <class Idx>
+  __device__ __forceinline__ void next(Idx) {
+    s = lcg_apply(J, s);
+    start();
+  }
+  __device__ __forceinline__ bool step() {
+    const int32_t* __restrict__ mrow = t.mats + mat * t.max_num_nucs;
+    const double* __restrict__ crow = t.concs + mat * t.max_num_nucs;
+    const uint16_t* __restrict__ irow = t.index_grid16 + (int64_t)idx * t.n_isotopes;
+    int32_t pn[P], kn[P];
+#pragma unroll
+    for (int u = 0; u < P; ++u) {  // next step's index entries
+      const int jj = j + P + u;
+      pn[u] = jj < nn ? __ldg(mrow + jj) : 0;
+      kn[u] = jj < nn ? (int32_t)__ldg(irow + pn[u]) : 0;
+    }
+#pragma unroll
+    for (int u = 0; u < P; ++u) {
+      if (j + u < nn) {
+        int32_t k = kc[u];
+        if (k == t.n_gridpoints - 1) --k;
+        const double conc = __ldg(crow + j + u);
+        const double* g = t.brackets + ((int64_t)pc[u] * (t.n_gridpoints - 1) + k) * 12;
+        double le, lt, lel, la, lf, ln, he, ht, hel, ha, hf, hn;
+        ld_nc_v4f64(g, le, he, lt, ht);
+        ld_nc_v4f64(g + 4, lel, hel, la, ha);
+        ld_nc_v4f64(g + 8, lf, hf, ln, hn);
+        xs_accumulate(E, conc, le, he, lt, ht, lel, hel, la, ha, lf, hf, ln, hn, m0, m1, m2, m3,
+                      m4);
+      }
+    }
+    j += P;
+#pragma unroll
+    for (int u = 0; u < P; ++u) {
+      pc[u] = pn[u];
+      kc[u] = kn[u];
+    }
+    return j < nn;
+  }
+  template <class Idx>
+  __device__ __forceinline__ void end(Idx iv) {
+    const uint64_t v = xs_argmax5(m0, m1, m2, m3, m4);
+    if constexpr (Fused) acc += v;
+    else ver[iv] = v;
+  }
+};
 
 template <bool Accel, int kUnroll = 4>
 __device__ __forceinline__ uint64_t xs_lookup_one(const XSTables& t, uint64_t seed0, int64_t i) {

@@ -48,6 +48,44 @@ __global__ void __launch_bounds__(kXSThreads, Accel ? kXSMinBlocksAccel : kXSMin
                   ticket);
 }
 
+// The twins' hand-written league reduction of a u64 (the same algorithm as the runtime's:
+// warp butterflies, per-warp partials, block partial, ticket, last block folds in order).
+// Every thread of the block calls it.
+__device__ __forceinline__ void twin_u64_ticket_sum(unsigned long long v,
+                                                    unsigned long long* checksum,
+                                                    unsigned long long* partials,
+                                                    unsigned* ticket) {
+  __shared__ unsigned long long ws[32];
+  __shared__ unsigned last;
+  for (int off = 16; off > 0; off >>= 1) v += __shfl_xor_sync(0xffffffffu, v, off);
+  const unsigned lane = threadIdx.x & 31u, wid = threadIdx.x >> 5, nw = blockDim.x >> 5;
+  if (lane == 0) ws[wid] = v;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    unsigned long long b = 0;
+    for (unsigned k = 0; k < nw; ++k) b += ws[k];
+    partials[blockIdx.x] = b;
+    __threadfence();
+    last = atomicAdd(ticket, 1u) == gridDim.x - 1;
+  }
+  __syncthreads();
+  if (last) {
+    __threadfence();
+    unsigned long long s = 0;
+    for (unsigned k = threadIdx.x; k < gridDim.x; k += blockDim.x) s += __ldcg(partials + k);
+    for (int off = 16; off > 0; off >>= 1) s += __shfl_xor_sync(0xffffffffu, s, off);
+    __syncthreads();
+    if (lane == 0) ws[wid] = s;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+      unsigned long long b = 0;
+      for (unsigned k = 0; k < nw; ++k) b += ws[k];
+      *checksum += b;
+      *ticket = 0u;
+    }
+  }
+}
+
 // XSBench's CUDA kernel shape: one lookup per thread, early return past the end; the fused
 // variant hand-codes the same reduction algorithm as the runtime.
 template <bool Fused, bool Accel>
@@ -60,36 +98,56 @@ __global__ void __launch_bounds__(kXSThreads, Accel ? kXSMinBlocksAccel : kXSMin
     if (i >= count) return;
     verification[i] = xs_lookup_one<Accel>(t, seed, first + i);
   } else {
-    unsigned long long v = i < count ? xs_lookup_one<Accel>(t, seed, first + i) : 0ull;
-    __shared__ unsigned long long ws[32];
-    __shared__ unsigned last;
-    for (int off = 16; off > 0; off >>= 1) v += __shfl_xor_sync(0xffffffffu, v, off);
-    const unsigned lane = threadIdx.x & 31u, wid = threadIdx.x >> 5, nw = blockDim.x >> 5;
-    if (lane == 0) ws[wid] = v;
-    __syncthreads();
-    if (threadIdx.x == 0) {
-      unsigned long long b = 0;
-      for (unsigned k = 0; k < nw; ++k) b += ws[k];
-      partials[blockIdx.x] = b;
-      __threadfence();
-      last = atomicAdd(ticket, 1u) == gridDim.x - 1;
+    const unsigned long long v = i < count ? xs_lookup_one<Accel>(t, seed, first + i) : 0ull;
+    twin_u64_ticket_sum(v, checksum, partials, ticket);
+  }
+}
+
+// ---- flattened execution (OMPRT_XS_FLAT): a persistent grid, each thread runs its Fig. 5
+// iterations through omprt::distribute_parallel_for_flat (B200 layouts required).  4 teams
+// of 256 per SM (64 registers): measured best (profiles/xs_explore_x14*).
+constexpr int kXSMinBlocksFlat = 4;
+
+template <class Tr, bool Fused>
+__global__ void __launch_bounds__(kXSThreads, kXSMinBlocksFlat)
+    omprt_xs_flat_rt(const __grid_constant__ XSTables t, uint64_t seed, int64_t first,
+                     typename Tr::Idx count, uint64_t* __restrict__ verification,
+                     unsigned long long* checksum, unsigned long long* partials,
+                     unsigned* ticket) {
+  Team<Tr> team = init<Tr>();
+  XSFlatLookup<Fused> lookup(t, seed, first, verification);
+  distribute_parallel_for_flat(team, count, lookup);
+  if constexpr (Fused)
+    league_reduce(team, team_reduce_to_main(team, lookup.acc, Plus{}), Plus{}, checksum,
+                  partials, ticket);
+}
+
+// Bare CUDA twin: the same flattened loop written by hand around the same body.
+template <bool Fused>
+__global__ void __launch_bounds__(kXSThreads, kXSMinBlocksFlat)
+    cuda_xs_flat_twin(const __grid_constant__ XSTables t, uint64_t seed, int64_t first,
+                      int32_t count, uint64_t* __restrict__ verification,
+                      unsigned long long* checksum, unsigned long long* partials,
+                      unsigned* ticket) {
+  XSFlatLookup<Fused> lookup(t, seed, first, verification);
+  const int32_t stride = (int32_t)gridDim.x * (int32_t)blockDim.x;
+  int32_t i = (int32_t)blockIdx.x * (int32_t)blockDim.x + (int32_t)threadIdx.x;
+  auto run = [&]() {
+    lookup.begin(i, stride);
+    for (;;) {
+      if (lookup.step()) continue;
+      lookup.end(i);
+      i += stride;
+      if (i >= count) break;
+      lookup.next(i);
     }
-    __syncthreads();
-    if (last) {
-      __threadfence();
-      unsigned long long s = 0;
-      for (unsigned k = threadIdx.x; k < gridDim.x; k += blockDim.x) s += __ldcg(partials + k);
-      for (int off = 16; off > 0; off >>= 1) s += __shfl_xor_sync(0xffffffffu, s, off);
-      __syncthreads();
-      if (lane == 0) ws[wid] = s;
-      __syncthreads();
-      if (threadIdx.x == 0) {
-        unsigned long long b = 0;
-        for (unsigned k = 0; k < nw; ++k) b += ws[k];
-        *checksum += b;
-        *ticket = 0u;
-      }
-    }
+  };
+  if constexpr (!Fused) {
+    if (i >= count) return;
+    run();
+  } else {
+    if (i < count) run();
+    twin_u64_ticket_sum(lookup.acc, checksum, partials, ticket);
   }
 }
 
@@ -115,6 +173,10 @@ OMPRT_REGISTER_KERNEL(omprt_xs_rt_debug, omprt_xs_rt<XSTraitsDebug, false, false
 OMPRT_REGISTER_KERNEL(omprt_xs_rt_accel, omprt_xs_rt<XSTraits, false, true>)
 OMPRT_REGISTER_KERNEL(omprt_xs_rt_assume_accel, omprt_xs_rt<XSTraitsAssume, false, true>)
 OMPRT_REGISTER_KERNEL(omprt_xs_rt_fused_accel, omprt_xs_rt<XSTraitsAssume, true, true>)
+OMPRT_REGISTER_KERNEL(omprt_xs_flat_rt, omprt_xs_flat_rt<XSTraits, false>)
+OMPRT_REGISTER_KERNEL(omprt_xs_flat_rt_fused, omprt_xs_flat_rt<XSTraits, true>)
+OMPRT_REGISTER_KERNEL(cuda_xs_flat_twin, cuda_xs_flat_twin<false>)
+OMPRT_REGISTER_KERNEL(cuda_xs_flat_twin_fused, cuda_xs_flat_twin<true>)
 OMPRT_REGISTER_KERNEL(cuda_xs_twin, cuda_xs_twin<false, false>)
 OMPRT_REGISTER_KERNEL(cuda_xs_twin_fused, cuda_xs_twin<true, false>)
 OMPRT_REGISTER_KERNEL(cuda_xs_twin_accel, cuda_xs_twin<false, true>)
@@ -147,6 +209,20 @@ inline int xs_validate(const omprt_xs_tables& t, int64_t count, uint64_t* ver, u
   const bool fused = flags & OMPRT_FUSED_REDUCTION;
   OMPRT_CHECK_ARG(fused ? ck != nullptr : (ver != nullptr || count == 0),
                   fused ? "fused reduction needs checksum_inout" : "verification is required");
+  if (flags & OMPRT_XS_FLAT) {
+    OMPRT_CHECK_ARG(accel, "OMPRT_XS_FLAT needs the B200 layouts (omprt_xs_build_accel)");
+    OMPRT_CHECK_ARG(!(flags & (OMPRT_ASSUME_OVERSUB | OMPRT_DEBUG_BUILD)),
+                    "OMPRT_XS_FLAT runs a persistent grid (no assumption, release build)");
+    if (teams <= 0) {  // persistent: the resident teams of the whole device
+      int dev = 0, sms = 148, per_sm = kXSMinBlocksFlat;
+      cudaGetDevice(&dev);
+      cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+      cudaOccupancyMaxActiveBlocksPerMultiprocessor(
+          &per_sm, omprt_xs_flat_rt<XSTraits, false>, kXSThreads, 0);
+      teams = (int32_t)std::max<int64_t>(
+          1, std::min<int64_t>((int64_t)sms * std::max(per_sm, 1), ceil_div(count, threads)));
+    }
+  }
   if (teams <= 0) teams = (int32_t)std::max<int64_t>(1, ceil_div(count, threads));
   OMPRT_CHECK_ARG(!fused || (uint64_t)teams <= w->opt.max_teams, "teams exceed max_teams");
   OMPRT_CHECK_ARG(!(flags & OMPRT_ASSUME_OVERSUB) || count <= (int64_t)teams * threads,
@@ -225,6 +301,15 @@ extern "C" int omprt_xs_lookup(omprt_xs_tables t, uint64_t seed, int64_t first, 
   auto* p = (unsigned long long*)w->partials;
   unsigned* tk = w->tickets + 1;
   const int32_t n = (int32_t)count;
+  if (flags & OMPRT_XS_FLAT) {
+    if (fused)
+      omprt_xs_flat_rt<XSTraits, true><<<teams, threads, 0, s>>>(d, seed, first, n,
+                                                                 verification, ck, p, tk);
+    else
+      omprt_xs_flat_rt<XSTraits, false><<<teams, threads, 0, s>>>(d, seed, first, n,
+                                                                  verification, ck, p, tk);
+    return check_launch("omprt_xs_flat_rt");
+  }
 #define OMPRT_XS(TR, F, A) \
   omprt_xs_rt<TR, F, A><<<teams, threads, 0, s>>>(d, seed, first, n, verification, ck, p, tk)
   if (debug) {
@@ -253,11 +338,12 @@ extern "C" int omprt_cuda_xs_lookup(omprt_xs_tables t, uint64_t seed, int64_t fi
   using namespace omprt_kernels;
   Workspace* w;
   if (int r = current_ws(&w)) return r;
-  int32_t tm = 0;  // the twin always runs one lookup per thread
+  // the twin runs one lookup per thread, or (OMPRT_XS_FLAT) the same persistent grid
+  const bool flat = flags & OMPRT_XS_FLAT;
+  int32_t tm = flat ? teams : 0;
   if (int r = xs_validate(t, count, verification, checksum_inout, tm, threads,
-                          flags & ~OMPRT_ASSUME_OVERSUB, w))
+                          flags & ~(OMPRT_ASSUME_OVERSUB | OMPRT_DEBUG_BUILD), w))
     return r;
-  (void)teams;
   if (count == 0) return OMPRT_OK;
   cudaStream_t s = as_stream(stream);
   const XSTables d = to_dev(t);
@@ -266,6 +352,11 @@ extern "C" int omprt_cuda_xs_lookup(omprt_xs_tables t, uint64_t seed, int64_t fi
   auto* p = (unsigned long long*)w->partials;
   unsigned* tk = w->tickets + 1;
   const int32_t n = (int32_t)count;
+  if (flat) {
+    if (fused) cuda_xs_flat_twin<true><<<tm, threads, 0, s>>>(d, seed, first, n, verification, ck, p, tk);
+    else cuda_xs_flat_twin<false><<<tm, threads, 0, s>>>(d, seed, first, n, verification, nullptr, nullptr, nullptr);
+    return check_launch("cuda_xs_flat_twin");
+  }
   if (fused && accel) cuda_xs_twin<true, true><<<tm, threads, 0, s>>>(d, seed, first, n, verification, ck, p, tk);
   else if (fused) cuda_xs_twin<true, false><<<tm, threads, 0, s>>>(d, seed, first, n, verification, ck, p, tk);
   else if (accel) cuda_xs_twin<false, true><<<tm, threads, 0, s>>>(d, seed, first, n, verification, nullptr, nullptr, nullptr);
@@ -312,7 +403,8 @@ extern "C" int omprt_xs_run_host_steps(omprt_xs_tables h, uint64_t seed, int64_t
                       h.num_nucs && h.mats && h.concs && (h.index_grid || h.index_grid16) &&
                       (h.nuclide_grid || h.brackets),
                   "omprt_xs_run_host_steps: bad arguments");
-  const bool accel = (flags & OMPRT_XS_ACCEL) || h.index_grid16 || h.brackets;
+  const bool accel =
+      (flags & (OMPRT_XS_ACCEL | OMPRT_XS_FLAT)) || h.index_grid16 || h.brackets;
   OMPRT_CHECK_ARG(accel || (h.index_grid && h.nuclide_grid),
                   "the plain path needs the int32 index grid and the nuclide grid");
   OMPRT_CHECK_ARG(!accel || h.n_gridpoints <= 65536, "16-bit index: n_gridpoints > 65536");
@@ -413,7 +505,7 @@ extern "C" int omprt_xs_run_host_steps(omprt_xs_tables h, uint64_t seed, int64_t
     }
     if (int r = omprt_xs_lookup(d, seed, first, count, nullptr, w->dev_ck + st, 0, threads,
                                 (flags & ~OMPRT_XS_ACCEL) | OMPRT_FUSED_REDUCTION |
-                                    OMPRT_ASSUME_OVERSUB,
+                                    ((flags & OMPRT_XS_FLAT) ? 0u : OMPRT_ASSUME_OVERSUB),
                                 stream))
       return r;
     OMPRT_CUDA_TRY(cudaMemcpyAsync(w->pinned_ck + st, w->dev_ck + st, sizeof(uint64_t),

@@ -55,6 +55,12 @@ struct DefaultTraits {
   using Idx = int32_t;
 };
 
+// The same traits with a 64-bit loop index (when n + T*N does not fit int32).
+template <class Base>
+struct WithIdx64 : Base {
+  using Idx = int64_t;
+};
+
 template <class Tr>
 inline constexpr bool kDebugAssert = (Tr::debug & dbg::Assert) != 0;
 template <class Tr>

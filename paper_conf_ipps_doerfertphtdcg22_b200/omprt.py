@@ -36,6 +36,7 @@ OMPRT_SPMDIZE = 1 << 11
 OMPRT_DEGLOBALIZE = 1 << 12
 OMPRT_TMA_STAGED = 1 << 13
 OMPRT_WARP_STAGED = 1 << 14
+OMPRT_XS_FLAT = 1 << 15
 
 # Every symbol include/omprt.h declares (checked by tests/test_abi.py).
 EXPORTS = [

@@ -19,7 +19,8 @@ def main():
     torch.cuda.set_device(0)
     omprt.omprt_init(0)
     t = gen.XSTables(**gen.XS_SMALL)
-    d = omprt.XSDeviceTables(t, "cuda", accel=os.environ.get("XSX_ACCEL") == "1")
+    d = omprt.XSDeviceTables(t, "cuda", accel=os.environ.get("XSX_ACCEL") == "1",
+                             log2_bins=int(os.environ.get("XSX_LOG2BINS", "16")))
     L.xsx_prepare.argtypes = [omprt.XSTablesC]
     L.xsx_run.argtypes = [C.c_int, omprt.XSTablesC, C.c_uint64, C.c_int64, C.c_int32, C.c_void_p, C.c_void_p]
     assert L.xsx_prepare(d.c) == 0

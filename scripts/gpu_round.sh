@@ -1,6 +1,6 @@
 #!/bin/bash
 # One GPU session: parity tests, smoke, bench, reference arm, ncu launch list + full
-# captures of the headline kernel and its twin (exported to CSV on the box; the two
+# captures of the headline kernel, its twin and the one-lookup-per-thread kernel (exported to CSV on the box; the two
 # .ncu-rep files come back too).  Usage (under gpurun): bash scripts/gpu_round.sh TAG
 TAG=${1:-r01}
 OUT=gpurun_out
@@ -17,12 +17,13 @@ echo "bench exit $?" >> $OUT/bench_$TAG.txt
 timeout 300 python bench.py --impl reference --steps 2 --warmup 1 > $OUT/bench_ref_$TAG.txt 2>&1
 timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none -c 400 --csv \
   --log-file $OUT/launches_$TAG.csv python bench.py --steps 2 --warmup 1 --no-e2e --no-secondary > $OUT/ncu_launch_stdout_$TAG.txt 2>&1
-for K in omprt_xs_rt cuda_xs_twin; do
+for K in omprt_xs_flat_rt cuda_xs_flat_twin omprt_xs_rt; do
   timeout 900 ncu --set full --clock-control none --import-source on -k regex:$K -s 1 -c 1 \
     -o $OUT/prof_${K}_$TAG python bench.py --steps 1 --warmup 1 --no-e2e --no-secondary > $OUT/ncu_full_${K}_$TAG.txt 2>&1
   ncu -i $OUT/prof_${K}_$TAG.ncu-rep --page raw --csv --print-units base > $OUT/raw_${K}_$TAG.csv 2>&1
   ncu -i $OUT/prof_${K}_$TAG.ncu-rep --page source --csv --print-units base > $OUT/src_${K}_$TAG.csv 2>&1
 done
+rm -f $OUT/prof_omprt_xs_rt_$TAG.ncu-rep  # keep the returned payload small (CSV kept)
 du -sh $OUT
 OMPRT_DEBUG=0 timeout 600 python scripts/debug_cost.py > $OUT/debug_cost_env0_$TAG.txt 2>&1
 OMPRT_DEBUG=1 timeout 600 python scripts/debug_cost.py > $OUT/debug_cost_env1_$TAG.txt 2>&1

@@ -3,8 +3,8 @@
   python scripts/ncu_summary.py TAG gpurun_out/prof_a.ncu-rep[:name] ... [--launches gpurun_out/launches.csv]
 
 Writes profiles/ncu_full_<TAG>.json (key metrics per capture, base units),
-profiles/ncu_traffic.json (DRAM bytes per launch per kernel, read by bench.py for
-roofline.traffic) and, with --launches, profiles/launches_<TAG>.txt (per-kernel launch
+profiles/ncu_traffic.json (DRAM and L2->L1 bytes per launch per kernel, read by bench.py
+for roofline.traffic and roofline.l2) and, with --launches, profiles/launches_<TAG>.txt (per-kernel launch
 count, mean device time, and share of the total, from the gpu__time_duration pass).
 """
 import csv
@@ -97,6 +97,11 @@ def main():
                 traffic[nm] = {"dram_bytes_per_launch": m["dram__bytes_read.sum"] + m["dram__bytes_write.sum"],
                                "time_ns": m.get("gpu__time_duration.sum"), "source": os.path.basename(rep),
                                "tag": tag}
+                if "lts__t_sectors_srcunit_tex_op_read.sum" in m:  # L2 -> L1 read bytes
+                    traffic[nm]["l2_read_bytes_per_launch"] = 32.0 * m["lts__t_sectors_srcunit_tex_op_read.sum"]
+                    traffic[nm]["lts_throughput_pct"] = m.get("lts__throughput.avg.pct_of_peak_sustained_elapsed")
+                    traffic[nm]["l1tex_throughput_pct"] = m.get("l1tex__throughput.avg.pct_of_peak_sustained_elapsed")
+                    traffic[nm]["lts_hit_rate_pct"] = m.get("lts__t_sector_hit_rate.pct")
     os.makedirs(os.path.join(ROOT, "profiles"), exist_ok=True)
     with open(os.path.join(ROOT, "profiles", f"ncu_full_{tag}.json"), "w") as f:
         json.dump(summary, f, indent=1)

@@ -54,6 +54,43 @@ def test_accel_layout_bit_exact(rt, xs_acc, xs_small, variant):
     assert (got == ref).all()
 
 
+@pytest.mark.parametrize("which", ["rt", "twin"])
+@pytest.mark.parametrize("teams", [0, 1, 3, 700])
+def test_flat_bit_exact(rt, xs_acc, xs_small, which, teams):
+    """OMPRT_XS_FLAT (persistent grid, nuclide loop fused into the Fig. 5 iteration loop):
+    every lookup bit-exact, with many lookups per thread (teams = 1, 3) and a ragged end."""
+    first, count = 4321, (1 << 16) + 77
+    ver = torch.zeros(count, dtype=torch.uint64, device=DEV)
+    fn = rt.omprt_xs_lookup if which == "rt" else rt.omprt_cuda_xs_lookup
+    fn(xs_acc, SEED, first, count, ver, None, teams, 256, rt.OMPRT_XS_FLAT)
+    torch.cuda.synchronize()
+    ref = oracle.xs_lookup(xs_small, first, count, threads=os.cpu_count() or 1)
+    assert (ver.cpu().numpy() == ref).all()
+
+
+def test_flat_fused_checksum_and_edges(rt, xs_acc, xs_small):
+    F = rt.OMPRT_XS_FLAT
+    for first, count, teams in [(0, 1, 0), (9, 255, 0), (9, 257, 1), (100, 50_000, 0),
+                                (100, 50_000, 5)]:
+        ref = int(oracle.xs_lookup(xs_small, first, count).sum())
+        for fn in (rt.omprt_xs_lookup, rt.omprt_cuda_xs_lookup):
+            ck = torch.full((1,), 7, dtype=torch.uint64, device=DEV)
+            fn(xs_acc, SEED, first, count, None, ck, teams, 256, F | rt.OMPRT_FUSED_REDUCTION)
+            torch.cuda.synchronize()
+            assert int(ck.cpu().numpy()[0]) == ref + 7
+
+
+def test_flat_rejects(rt, xs_dev, xs_acc):
+    ver = torch.zeros(64, dtype=torch.uint64, device=DEV)
+    F = rt.OMPRT_XS_FLAT
+    with pytest.raises(Exception):  # needs the B200 layouts
+        rt.omprt_xs_lookup(xs_dev, SEED, 0, 64, ver, None, 0, 256, F)
+    with pytest.raises(Exception):  # persistent grid: no oversubscription assumption
+        rt.omprt_xs_lookup(xs_acc, SEED, 0, 64, ver, None, 0, 256, F | rt.OMPRT_ASSUME_OVERSUB)
+    with pytest.raises(Exception):
+        rt.omprt_xs_lookup(xs_acc, SEED, 0, 64, ver, None, 0, 256, F | rt.OMPRT_DEBUG_BUILD)
+
+
 def test_accel_tables_content(rt, xs_acc, xs_small):
     bins = xs_acc.bins.cpu().numpy()
     H = 1 << 16
@@ -115,13 +152,20 @@ def test_u64_sum_wraps(rt):
     assert int(out.cpu().numpy()[0]) == (int(v.size) * ((1 << 63) + 12345)) % 2**64
 
 
-def test_full_size_17M(rt, xs_acc, xs_small):
-    """BASELINE configs[2] at full size, in the launch configuration bench.py times
-    (runtime-driven, assumption, B200 layouts): sampled lookups bit-exact, then every lookup
-    and the checksum against the oracle (all host cores)."""
+@pytest.fixture(scope="module")
+def xs_ref_17M(xs_small):
+    return oracle.xs_lookup(xs_small, 0, 17_000_000, threads=os.cpu_count() or 1)
+
+
+@pytest.mark.parametrize("flags", ["OMPRT_XS_FLAT", "OMPRT_ASSUME_OVERSUB"])
+def test_full_size_17M(rt, xs_acc, xs_small, xs_ref_17M, flags):
+    """BASELINE configs[2] at full size, in the launch configurations bench.py times
+    (runtime-driven on the B200 layouts: flattened persistent grid -- the headline -- and
+    one lookup per thread with the assumption): sampled lookups bit-exact against single
+    oracle calls, then every lookup and the checksum against the oracle (all host cores)."""
     n = 17_000_000
     ver = torch.zeros(n, dtype=torch.uint64, device=DEV)
-    rt.omprt_xs_lookup(xs_acc, SEED, 0, n, ver, None, 0, 256, rt.OMPRT_ASSUME_OVERSUB)
+    rt.omprt_xs_lookup(xs_acc, SEED, 0, n, ver, None, 0, 256, getattr(rt, flags))
     ck = torch.zeros(1, dtype=torch.uint64, device=DEV)
     rt.omprt_u64_sum(ver, n, ck)
     torch.cuda.synchronize()
@@ -130,9 +174,8 @@ def test_full_size_17M(rt, xs_acc, xs_small):
     idx[:2] = [0, n - 1]
     for i in idx[:2000]:
         assert got[i] == oracle.xs_lookup(xs_small, int(i), 1)[0]
-    ref = oracle.xs_lookup(xs_small, 0, n, threads=os.cpu_count() or 1)
-    assert (got == ref).all()
-    assert int(ck.cpu().numpy()[0]) == int(ref.sum())
+    assert (got == xs_ref_17M).all()
+    assert int(ck.cpu().numpy()[0]) == int(xs_ref_17M.sum())
 
 
 def test_end_to_end_host_tables(rt, xs_small):
@@ -159,5 +202,7 @@ def test_end_to_end_pipelined_steps_compact_host_layout(rt, xs_small):
     ref = int(oracle.xs_lookup(xs_small, 5, n).sum())
     cks, h2d, d2h = rt.omprt_xs_run_host_steps(hs, SEED, 5, n, 5)
     assert cks == [ref] * 5
+    cks, _, _ = rt.omprt_xs_run_host_steps(hs, SEED, 5, n, 3, flags=rt.OMPRT_XS_FLAT)
+    assert cks == [ref] * 3
     idx16 = xs_small.index_grid.size * 2
     assert h2d == xs_small.nbytes() - xs_small.index_grid.nbytes + idx16 and d2h == 8

@@ -228,12 +228,17 @@ __device__ __forceinline__ uint64_t xs_lookup_accel(const XSTables& t, uint64_t 
 // xs_lookup_accel, so the verification bits are identical.  A thread's next lookup is
 // iv + T*N (Fig. 5): its seed is the current seed advanced by the 2*T*N-step jump, one
 // 64-bit multiply-add instead of a fast-forward from the start (exact: the LCG is affine).
-template <bool Fused, int P = 2>
+// L1 traffic is what bounds this loop (ncu: L1 ~80 % busy), so the bracket records, read
+// once, bypass L1 allocation, and with SmemMats the material tables (mats, concs) come
+// from a team-shared copy (`mats`/`concs` then point to shared memory).
+template <bool Fused, bool SmemMats, int P = 2>
 struct XSFlatLookup {
   const XSTables& t;
   const uint64_t seed0;
   const int64_t first;
   uint64_t* __restrict__ const ver;
+  const int32_t* __restrict__ const mats;  // t.mats, or its team-shared copy
+  const double* __restrict__ const concs;  // t.concs, or its team-shared copy
   unsigned long long acc = 0;  // Fused: this thread's verification sum
   LcgMap J;
   uint64_t s;
@@ -243,8 +248,18 @@ struct XSFlatLookup {
   int32_t pc[P], kc[P];
 
   __device__ __forceinline__ XSFlatLookup(const XSTables& tab, uint64_t seed, int64_t first_,
-                                          uint64_t* verification)
-      : t(tab), seed0(seed), first(first_), ver(verification) {}
+                                          uint64_t* verification, const int32_t* mats_,
+                                          const double* concs_)
+      : t(tab), seed0(seed), first(first_), ver(verification), mats(mats_), concs(concs_) {}
+
+  __device__ __forceinline__ int32_t mat_at(const int32_t* p) const {
+    if constexpr (SmemMats) return *p;
+    else return __ldg(p);
+  }
+  __device__ __forceinline__ double conc_at(const double* p) const {
+    if constexpr (SmemMats) return *p;
+    else return __ldg(p);
+  }
 
   __device__ __forceinline__ void start() {
     uint64_t seed = s;
@@ -254,11 +269,11 @@ struct XSFlatLookup {
     nn = __ldg(t.num_nucs + mat);
     m0 = m1 = m2 = m3 = m4 = 0.0;
     j = 0;
-    const int32_t* __restrict__ mrow = t.mats + mat * t.max_num_nucs;
+    const int32_t* __restrict__ mrow = mats + mat * t.max_num_nucs;
     const uint16_t* __restrict__ irow = t.index_grid16 + (int64_t)idx * t.n_isotopes;
 #pragma unroll
     for (int u = 0; u < P; ++u) {
-      pc[u] = u < nn ? __ldg(mrow + u) : 0;
+      pc[u] = u < nn ? mat_at(mrow + u) : 0;
       kc[u] = u < nn ? (int32_t)__ldg(irow + pc[u]) : 0;
     }
   }
@@ -274,14 +289,14 @@ struct XSFlatLookup {
     start();
   }
   __device__ __forceinline__ bool step() {
-    const int32_t* __restrict__ mrow = t.mats + mat * t.max_num_nucs;
-    const double* __restrict__ crow = t.concs + mat * t.max_num_nucs;
+    const int32_t* __restrict__ mrow = mats + mat * t.max_num_nucs;
+    const double* __restrict__ crow = concs + mat * t.max_num_nucs;
     const uint16_t* __restrict__ irow = t.index_grid16 + (int64_t)idx * t.n_isotopes;
     int32_t pn[P], kn[P];
 #pragma unroll
     for (int u = 0; u < P; ++u) {  // next step's index entries
       const int jj = j + P + u;
-      pn[u] = jj < nn ? __ldg(mrow + jj) : 0;
+      pn[u] = jj < nn ? mat_at(mrow + jj) : 0;
       kn[u] = jj < nn ? (int32_t)__ldg(irow + pn[u]) : 0;
     }
 #pragma unroll
@@ -289,12 +304,12 @@ struct XSFlatLookup {
       if (j + u < nn) {
         int32_t k = kc[u];
         if (k == t.n_gridpoints - 1) --k;
-        const double conc = __ldg(crow + j + u);
+        const double conc = conc_at(crow + j + u);
         const double* g = t.brackets + ((int64_t)pc[u] * (t.n_gridpoints - 1) + k) * 12;
         double le, lt, lel, la, lf, ln, he, ht, hel, ha, hf, hn;
-        ld_nc_v4f64(g, le, he, lt, ht);
-        ld_nc_v4f64(g + 4, lel, hel, la, ha);
-        ld_nc_v4f64(g + 8, lf, hf, ln, hn);
+        ld_stream_v4f64(g, le, he, lt, ht);
+        ld_stream_v4f64(g + 4, lel, hel, la, ha);
+        ld_stream_v4f64(g + 8, lf, hf, ln, hn);
         xs_accumulate(E, conc, le, he, lt, ht, lel, hel, la, ha, lf, hf, ln, hn, m0, m1, m2, m3,
                       m4);
       }

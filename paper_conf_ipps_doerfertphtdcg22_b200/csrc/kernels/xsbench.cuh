@@ -105,17 +105,36 @@ __global__ void __launch_bounds__(kXSThreads, Accel ? kXSMinBlocksAccel : kXSMin
 
 // ---- flattened execution (OMPRT_XS_FLAT): a persistent grid, each thread runs its Fig. 5
 // iterations through omprt::distribute_parallel_for_flat (B200 layouts required).  4 teams
-// of 256 per SM (64 registers): measured best (profiles/xs_explore_x14*).
+// of 256 per SM (64 registers): measured best (profiles/xs_explore_x14*, x16*).  With
+// Smem, the team first copies the material tables into team-shared memory (the runtime's
+// team_local + for_static + team barrier; the twin: __shared__ + loop + __syncthreads).
 constexpr int kXSMinBlocksFlat = 4;
+constexpr int kXSMatSmem = 12 * 48;  // entries: up to 48 nuclides per material (small: 34)
 
-template <class Tr, bool Fused>
+constexpr unsigned kXSMatsSite = 10, kXSConcsSite = 11;  // team_local sites
+
+template <class Tr, bool Fused, bool Smem>
 __global__ void __launch_bounds__(kXSThreads, kXSMinBlocksFlat)
     omprt_xs_flat_rt(const __grid_constant__ XSTables t, uint64_t seed, int64_t first,
                      typename Tr::Idx count, uint64_t* __restrict__ verification,
                      unsigned long long* checksum, unsigned long long* partials,
                      unsigned* ticket) {
+  using Idx = typename Tr::Idx;
   Team<Tr> team = init<Tr>();
-  XSFlatLookup<Fused> lookup(t, seed, first, verification);
+  const int32_t* mats = t.mats;
+  const double* concs = t.concs;
+  if constexpr (Smem) {
+    int32_t* sm = team_local<int32_t, kXSMatSmem, kXSMatsSite>();
+    double* sc = team_local<double, kXSMatSmem, kXSConcsSite>();
+    for_static(team, (Idx)(12 * t.max_num_nucs), [&](Idx k) {
+      sm[k] = __ldg(t.mats + k);
+      sc[k] = __ldg(t.concs + k);
+    });
+    aligned_barrier();
+    mats = sm;
+    concs = sc;
+  }
+  XSFlatLookup<Fused, Smem> lookup(t, seed, first, verification, mats, concs);
   distribute_parallel_for_flat(team, count, lookup);
   if constexpr (Fused)
     league_reduce(team, team_reduce_to_main(team, lookup.acc, Plus{}), Plus{}, checksum,
@@ -123,13 +142,26 @@ __global__ void __launch_bounds__(kXSThreads, kXSMinBlocksFlat)
 }
 
 // Bare CUDA twin: the same flattened loop written by hand around the same body.
-template <bool Fused>
+template <bool Fused, bool Smem>
 __global__ void __launch_bounds__(kXSThreads, kXSMinBlocksFlat)
     cuda_xs_flat_twin(const __grid_constant__ XSTables t, uint64_t seed, int64_t first,
                       int32_t count, uint64_t* __restrict__ verification,
                       unsigned long long* checksum, unsigned long long* partials,
                       unsigned* ticket) {
-  XSFlatLookup<Fused> lookup(t, seed, first, verification);
+  const int32_t* mats = t.mats;
+  const double* concs = t.concs;
+  if constexpr (Smem) {
+    __shared__ int32_t sm[kXSMatSmem];
+    __shared__ double sc[kXSMatSmem];
+    for (int k = threadIdx.x; k < 12 * t.max_num_nucs; k += blockDim.x) {
+      sm[k] = __ldg(t.mats + k);
+      sc[k] = __ldg(t.concs + k);
+    }
+    __syncthreads();
+    mats = sm;
+    concs = sc;
+  }
+  XSFlatLookup<Fused, Smem> lookup(t, seed, first, verification, mats, concs);
   const int32_t stride = (int32_t)gridDim.x * (int32_t)blockDim.x;
   int32_t i = (int32_t)blockIdx.x * (int32_t)blockDim.x + (int32_t)threadIdx.x;
   auto run = [&]() {
@@ -173,10 +205,12 @@ OMPRT_REGISTER_KERNEL(omprt_xs_rt_debug, omprt_xs_rt<XSTraitsDebug, false, false
 OMPRT_REGISTER_KERNEL(omprt_xs_rt_accel, omprt_xs_rt<XSTraits, false, true>)
 OMPRT_REGISTER_KERNEL(omprt_xs_rt_assume_accel, omprt_xs_rt<XSTraitsAssume, false, true>)
 OMPRT_REGISTER_KERNEL(omprt_xs_rt_fused_accel, omprt_xs_rt<XSTraitsAssume, true, true>)
-OMPRT_REGISTER_KERNEL(omprt_xs_flat_rt, omprt_xs_flat_rt<XSTraits, false>)
-OMPRT_REGISTER_KERNEL(omprt_xs_flat_rt_fused, omprt_xs_flat_rt<XSTraits, true>)
-OMPRT_REGISTER_KERNEL(cuda_xs_flat_twin, cuda_xs_flat_twin<false>)
-OMPRT_REGISTER_KERNEL(cuda_xs_flat_twin_fused, cuda_xs_flat_twin<true>)
+OMPRT_REGISTER_KERNEL(omprt_xs_flat_rt, omprt_xs_flat_rt<XSTraits, false, true>)
+OMPRT_REGISTER_KERNEL(omprt_xs_flat_rt_fused, omprt_xs_flat_rt<XSTraits, true, true>)
+OMPRT_REGISTER_KERNEL(omprt_xs_flat_rt_gmem, omprt_xs_flat_rt<XSTraits, false, false>)
+OMPRT_REGISTER_KERNEL(cuda_xs_flat_twin, cuda_xs_flat_twin<false, true>)
+OMPRT_REGISTER_KERNEL(cuda_xs_flat_twin_fused, cuda_xs_flat_twin<true, true>)
+OMPRT_REGISTER_KERNEL(cuda_xs_flat_twin_gmem, cuda_xs_flat_twin<false, false>)
 OMPRT_REGISTER_KERNEL(cuda_xs_twin, cuda_xs_twin<false, false>)
 OMPRT_REGISTER_KERNEL(cuda_xs_twin_fused, cuda_xs_twin<true, false>)
 OMPRT_REGISTER_KERNEL(cuda_xs_twin_accel, cuda_xs_twin<false, true>)
@@ -187,6 +221,11 @@ inline XSTables to_dev(const omprt_xs_tables& a) {
   return XSTables{a.nuclide_grid, a.unionized, a.index_grid, a.num_nucs, a.mats, a.concs,
                   a.n_isotopes, a.n_gridpoints, a.max_num_nucs, 0, a.n_union,
                   a.bins, a.index_grid16, a.brackets, a.log2_bins, 0};
+}
+
+// the flattened kernels keep the material tables in team-shared memory when they fit
+inline bool xs_mats_fit_smem(const omprt_xs_tables& t) {
+  return 12ll * t.max_num_nucs <= kXSMatSmem;
 }
 
 inline bool xs_has_accel(const omprt_xs_tables& t) {
@@ -218,7 +257,7 @@ inline int xs_validate(const omprt_xs_tables& t, int64_t count, uint64_t* ver, u
       cudaGetDevice(&dev);
       cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
       cudaOccupancyMaxActiveBlocksPerMultiprocessor(
-          &per_sm, omprt_xs_flat_rt<XSTraits, false>, kXSThreads, 0);
+          &per_sm, omprt_xs_flat_rt<XSTraits, false, true>, kXSThreads, 0);
       teams = (int32_t)std::max<int64_t>(
           1, std::min<int64_t>((int64_t)sms * std::max(per_sm, 1), ceil_div(count, threads)));
     }
@@ -302,12 +341,14 @@ extern "C" int omprt_xs_lookup(omprt_xs_tables t, uint64_t seed, int64_t first, 
   unsigned* tk = w->tickets + 1;
   const int32_t n = (int32_t)count;
   if (flags & OMPRT_XS_FLAT) {
-    if (fused)
-      omprt_xs_flat_rt<XSTraits, true><<<teams, threads, 0, s>>>(d, seed, first, n,
-                                                                 verification, ck, p, tk);
-    else
-      omprt_xs_flat_rt<XSTraits, false><<<teams, threads, 0, s>>>(d, seed, first, n,
-                                                                  verification, ck, p, tk);
+    const bool smem = xs_mats_fit_smem(t);
+#define OMPRT_XSF(F, S) \
+  omprt_xs_flat_rt<XSTraits, F, S><<<teams, threads, 0, s>>>(d, seed, first, n, verification, ck, p, tk)
+    if (fused && smem) OMPRT_XSF(true, true);
+    else if (fused) OMPRT_XSF(true, false);
+    else if (smem) OMPRT_XSF(false, true);
+    else OMPRT_XSF(false, false);
+#undef OMPRT_XSF
     return check_launch("omprt_xs_flat_rt");
   }
 #define OMPRT_XS(TR, F, A) \
@@ -353,8 +394,11 @@ extern "C" int omprt_cuda_xs_lookup(omprt_xs_tables t, uint64_t seed, int64_t fi
   unsigned* tk = w->tickets + 1;
   const int32_t n = (int32_t)count;
   if (flat) {
-    if (fused) cuda_xs_flat_twin<true><<<tm, threads, 0, s>>>(d, seed, first, n, verification, ck, p, tk);
-    else cuda_xs_flat_twin<false><<<tm, threads, 0, s>>>(d, seed, first, n, verification, nullptr, nullptr, nullptr);
+    const bool smem = xs_mats_fit_smem(t);
+    if (fused && smem) cuda_xs_flat_twin<true, true><<<tm, threads, 0, s>>>(d, seed, first, n, verification, ck, p, tk);
+    else if (fused) cuda_xs_flat_twin<true, false><<<tm, threads, 0, s>>>(d, seed, first, n, verification, ck, p, tk);
+    else if (smem) cuda_xs_flat_twin<false, true><<<tm, threads, 0, s>>>(d, seed, first, n, verification, nullptr, nullptr, nullptr);
+    else cuda_xs_flat_twin<false, false><<<tm, threads, 0, s>>>(d, seed, first, n, verification, nullptr, nullptr, nullptr);
     return check_launch("cuda_xs_flat_twin");
   }
   if (fused && accel) cuda_xs_twin<true, true><<<tm, threads, 0, s>>>(d, seed, first, n, verification, ck, p, tk);

@@ -258,28 +258,13 @@ __device__ __forceinline__ void flat_c(const XSTables& t, uint64_t seed0, int64_
 // iteration (iv + T*N, Fig. 5) is sampled and its binned search advances one probe per step,
 // in straight-line code (the probe load overlaps the step's index/bracket loads).  The next
 // lookup's seed comes from the current one by the affine jump of 2*T*N LCG steps (exact).
-struct Jump {
-  uint64_t a, c;
-};
-__device__ __forceinline__ Jump lcg_jump(uint64_t n) {
-  uint64_t a_new = 1, c_new = 0;
-  for (int k = 0; n != 0; ++k, n >>= 1) {
-    if (n & 1) {
-      const uint64_t ak = kLcgJumpTable.a[k];
-      a_new *= ak;
-      c_new = c_new * ak + kLcgJumpTable.c[k];
-    }
-  }
-  return {a_new, c_new};
-}
-
 template <int P>
 __device__ __forceinline__ void flat_pipe(const XSTables& t, uint64_t seed0, int64_t first,
                                           int32_t n, uint64_t* __restrict__ ver) {
   const int32_t total = gridDim.x * blockDim.x;
   int32_t iv = blockIdx.x * blockDim.x + threadIdx.x;
   if (iv >= n) return;
-  const Jump J = lcg_jump(2ull * (uint64_t)total);
+  const LcgMap J = lcg_jump(2ull * (uint64_t)total);
   const int64_t H = 1ll << t.log2_bins;
   // next lookup's sampling state
   uint64_t sn = lcg_fast_forward(seed0, 2ull * (uint64_t)(first + iv));
@@ -387,7 +372,7 @@ __device__ __forceinline__ void flat_jump(const XSTables& t, uint64_t seed0, int
   const int32_t total = gridDim.x * blockDim.x;
   int32_t iv = blockIdx.x * blockDim.x + threadIdx.x;
   if (iv >= n) return;
-  const Jump J = lcg_jump(2ull * (uint64_t)total);
+  const LcgMap J = lcg_jump(2ull * (uint64_t)total);
   uint64_t s0 = lcg_fast_forward(seed0, 2ull * (uint64_t)(first + iv));
   double E;
   int32_t mat, idx, nn, j;
@@ -452,6 +437,96 @@ __device__ __forceinline__ void flat_jump(const XSTables& t, uint64_t seed0, int
   }
 }
 
+template <int P, bool Stream, bool SmemMats>
+__device__ __forceinline__ void flat_opt(const XSTables& t, uint64_t seed0, int64_t first,
+                                          int32_t n, uint64_t* __restrict__ ver) {
+  const int32_t total = gridDim.x * blockDim.x;
+  int32_t iv = blockIdx.x * blockDim.x + threadIdx.x;
+  if (iv >= n) return;
+  const LcgMap J = lcg_jump(2ull * (uint64_t)total);
+  uint64_t s0 = lcg_fast_forward(seed0, 2ull * (uint64_t)(first + iv));
+  __shared__ int32_t smats[12 * 34];
+  __shared__ double sconcs[12 * 34];
+  const int32_t* gm = t.mats;
+  const double* gc = t.concs;
+  if (SmemMats) {
+    for (int k = threadIdx.x; k < 12 * t.max_num_nucs; k += blockDim.x) {
+      smats[k] = __ldg(t.mats + k);
+      sconcs[k] = __ldg(t.concs + k);
+    }
+    __syncthreads();
+    gm = smats;
+    gc = sconcs;
+  }
+  double E;
+  int32_t mat, idx, nn, j;
+  double m0, m1, m2, m3, m4;
+  int32_t pc[P], kc[P];
+  auto start = [&]() {
+    uint64_t seed = s0;
+    E = lcg_double(seed);
+    mat = pick_mat(seed);
+    idx = binned_grid_search(t, E);
+    nn = __ldg(t.num_nucs + mat);
+    m0 = m1 = m2 = m3 = m4 = 0.0;
+    j = 0;
+    const int32_t* mrow = gm + mat * t.max_num_nucs;
+    const uint16_t* irow = t.index_grid16 + (int64_t)idx * t.n_isotopes;
+#pragma unroll
+    for (int u = 0; u < P; ++u) {
+      pc[u] = u < nn ? (SmemMats ? mrow[u] : __ldg(mrow + u)) : 0;
+      kc[u] = u < nn ? (int32_t)__ldg(irow + pc[u]) : 0;
+    }
+  };
+  start();
+  while (true) {
+    const int32_t* mrow = gm + mat * t.max_num_nucs;
+    const double* crow = gc + mat * t.max_num_nucs;
+    const uint16_t* irow = t.index_grid16 + (int64_t)idx * t.n_isotopes;
+    int32_t pn[P], kn[P];
+#pragma unroll
+    for (int u = 0; u < P; ++u) {
+      const int jj = j + P + u;
+      pn[u] = jj < nn ? (SmemMats ? mrow[jj] : __ldg(mrow + jj)) : 0;
+      kn[u] = jj < nn ? (int32_t)__ldg(irow + pn[u]) : 0;
+    }
+#pragma unroll
+    for (int u = 0; u < P; ++u) {
+      if (j + u < nn) {
+        int32_t k = kc[u];
+        if (k == t.n_gridpoints - 1) --k;
+        const double conc = SmemMats ? crow[j + u] : __ldg(crow + j + u);
+        const double* g = t.brackets + ((int64_t)pc[u] * (t.n_gridpoints - 1) + k) * 12;
+        double le, lt, lel, la, lf, ln, he, ht, hel, ha, hf, hn;
+        if (Stream) {
+          ld_stream_v4f64(g, le, he, lt, ht);
+          ld_stream_v4f64(g + 4, lel, hel, la, ha);
+          ld_stream_v4f64(g + 8, lf, hf, ln, hn);
+        } else {
+          ld_nc_v4f64(g, le, he, lt, ht);
+          ld_nc_v4f64(g + 4, lel, hel, la, ha);
+          ld_nc_v4f64(g + 8, lf, hf, ln, hn);
+        }
+        xs_accumulate(E, conc, le, he, lt, ht, lel, hel, la, ha, lf, hf, ln, hn, m0, m1, m2, m3,
+                      m4);
+      }
+    }
+    j += P;
+#pragma unroll
+    for (int u = 0; u < P; ++u) {
+      pc[u] = pn[u];
+      kc[u] = kn[u];
+    }
+    if (j >= nn) {
+      ver[iv] = xs_argmax5(m0, m1, m2, m3, m4);
+      iv += total;
+      if (iv >= n) break;
+      s0 = (J.a * s0 + J.c) & kLcgMask;
+      start();
+    }
+  }
+}
+
 #define KP(NAME, TPB, MINB)                                                                    \
   __global__ void __launch_bounds__(TPB, MINB) NAME(const __grid_constant__ XSTables t,        \
       uint64_t seed, int64_t first, int32_t n, uint64_t* ver) {                                \
@@ -478,23 +553,26 @@ __device__ __forceinline__ void flat_jump(const XSTables& t, uint64_t seed0, int
       uint64_t seed, int64_t first, int32_t n, uint64_t* ver) {                                \
     flat_jump<P>(t, seed, first, n, ver);                                                      \
   }
+#define KO_(NAME, TPB, MINB, P, ST, SM)                                                        \
+  __global__ void __launch_bounds__(TPB, MINB) NAME(const __grid_constant__ XSTables t,        \
+      uint64_t seed, int64_t first, int32_t n, uint64_t* ver) {                                \
+    flat_opt<P, ST, SM>(t, seed, first, n, ver);                                               \
+  }
 #define KF_(NAME, TPB, MINB, P)                                                                \
   __global__ void __launch_bounds__(TPB, MINB) NAME(const __grid_constant__ XSTables t,        \
       uint64_t seed, int64_t first, int32_t n, uint64_t* ver) {                                \
     flat_loop<P>(t, seed, first, n, ver);                                                      \
   }
 KP(e0, 256, 3)
-KF_(e1, 256, 4, 2)
-KJ_(e2, 256, 4, 2)
-KJ_(e3, 128, 8, 2)
-KJ_(e4, 256, 4, 1)
-KJ_(e5, 256, 4, 2)
-KJ_(e6, 256, 4, 2)
-KF_(e7, 256, 4, 2)
+KJ_(e1, 256, 4, 2)
+KO_(e2, 256, 4, 2, true, false)
+KO_(e3, 256, 4, 2, false, true)
+KO_(e4, 256, 4, 2, true, true)
+KO_(e5, 256, 4, 1, true, true)
 typedef void (*KF)(XSTables, uint64_t, int64_t, int32_t, uint64_t*);
-static KF kf[] = {e0, e1, e2, e3, e4, e5, e6, e7};
-static int ctas_per_sm[] = {0, 4, 4, 8, 4, 8, 16, 8};
-static int tpbv[] = {256, 256, 256, 128, 256, 256, 256, 256};
+static KF kf[] = {e0, e1, e2, e3, e4, e5};
+static int ctas_per_sm[] = {0, 4, 4, 4, 4, 4};
+static int tpbv[] = {256, 256, 256, 256, 256, 256};
 extern "C" int xsx_count() { return (int)(sizeof(kf) / sizeof(kf[0])); }
 extern "C" int xsx_regs(int v) {
   cudaFuncAttributes a;

@@ -226,7 +226,8 @@ def run_omprt(args):
                                   flags)
         else:
             omprt.omprt_cuda_xs_lookup(tables, gen.XS_LOOKUP_SEED, first, L, ver, None, 0,
-                                       THREADS, flags & omprt.OMPRT_XS_FLAT)
+                                       THREADS,
+                                       flags & (omprt.OMPRT_XS_FLAT | omprt.OMPRT_XS_NO_L2_PERSIST))
         if kernel_events:
             kernel_events[1].record(stream)
         omprt.omprt_u64_sum(ver, L, ck)
@@ -236,6 +237,8 @@ def run_omprt(args):
 
     def timed(which, tables, flags, k_steps, w_steps):
         for _ in range(w_steps):
+            torch.cuda.synchronize()
+            omprt.omprt_l2_reset_persisting()
             scrub.fill_(1.0)
             step(None, which, tables, flags)
         torch.cuda.synchronize()
@@ -246,6 +249,8 @@ def run_omprt(args):
                torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
               for _ in range(k_steps)]
         for e in ev:
+            torch.cuda.synchronize()
+            omprt.omprt_l2_reset_persisting()  # no line survives the flush (flat's L2 window)
             scrub.fill_(1.0)  # L2 flush, outside the step's events
             e[0].record(stream)
             step((e[1], e[2]), which, tables, flags)
@@ -270,6 +275,8 @@ def run_omprt(args):
     # twin and variants, in the same process with the same geometry
     kms = {"rt_flat": mx(statistics.mean(kern_ms))}
     for name, which, tables, flags in [("twin_flat", "twin", d_acc, FL),
+                                       ("rt_flat_no_l2_window", "rt", d_acc,
+                                        FL | omprt.OMPRT_XS_NO_L2_PERSIST),
                                        ("rt_assume", "rt", d_acc, A),
                                        ("twin", "twin", d_acc, 0), ("rt_no_assume", "rt", d_acc, 0),
                                        ("plain_rt_assume", "rt", d_pln, A),
@@ -349,7 +356,9 @@ def run_omprt(args):
                        "variant": "runtime-driven SPMD, flattened Fig. 5 loop on a persistent "
                                   "grid (omprt::distribute_parallel_for_flat, 4 teams of 256 "
                                   "per SM), B200 table layouts (binned search, 16-bit index, "
-                                  "bracket records)"},
+                                  "bracket records), bracket records persisting in L2 during "
+                                  "the launch (access-policy window; reset + flushed between "
+                                  "steps)"},
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                          "frac": achieved / peak,
                          "traffic": load_ncu_traffic("omprt_xs_flat_rt"),
@@ -402,6 +411,9 @@ def _time(fn, stream, scrub, reps=5, warm=2, flush=True):
     out = []
     for _ in range(reps):
         if flush:
+            torch.cuda.synchronize()
+            from paper_conf_ipps_doerfertphtdcg22_b200 import omprt
+            omprt.omprt_l2_reset_persisting()
             scrub.fill_(1.0)
         a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         a.record(stream)

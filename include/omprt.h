@@ -101,6 +101,11 @@ extern "C" {
  * lookup starts its next one instead of waiting for the warp's longest lookup.  Identical
  * results.  Not combined with OMPRT_ASSUME_OVERSUB or OMPRT_DEBUG_BUILD. */
 #define OMPRT_XS_FLAT (1u << 15)
+/* With OMPRT_XS_FLAT: launch WITHOUT the L2 access-policy window that otherwise marks the
+ * bracket records (t.brackets) persisting in the L2 set-aside reserved by omprt_init
+ * (cudaLimitPersistingL2CacheSize = the device maximum).  Persisting lines outlive the
+ * launch; omprt_l2_reset_persisting() returns them to normal. */
+#define OMPRT_XS_NO_L2_PERSIST (1u << 16)
 
 /* ---- runtime lifecycle ------------------------------------------------------------- */
 typedef struct {
@@ -110,9 +115,15 @@ typedef struct {
 } omprt_options;
 
 /* Create the per-device workspace; reads OMPRT_DEBUG.  opt may be NULL (defaults).
- * Idempotent per device. */
+ * Idempotent per device.  Also reserves the device's maximum L2 set-aside for persisting
+ * accesses (cudaLimitPersistingL2CacheSize), used by the OMPRT_XS_FLAT launches' access-
+ * policy window; other accesses use the set-aside while no persisting line holds it. */
 int omprt_init(int device, const omprt_options *opt);
 int omprt_fini(int device);
+/* Return every persisting L2 line of the current device's context to normal
+ * (cudaCtxResetPersistingL2Cache; takes effect immediately, not stream-ordered: call it
+ * with no launch in flight, e.g. before an L2 flush between timed steps). */
+int omprt_l2_reset_persisting(void);
 /* Device-side error recorded since init (0 = none); info (nullable) gets 4 ints
  * {team, thread, line, extra}. */
 int omprt_device_status(int device, int *code, int *info);

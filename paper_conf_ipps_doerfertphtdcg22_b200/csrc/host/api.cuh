@@ -36,6 +36,18 @@ extern "C" int omprt_init(int device, const omprt_options* opt) {
   omprt::DeviceEnv env_dev{w.pool, o.pool_bytes_per_team, o.pool_teams, w.err_dev,
                            w.err_dev + 1, w.debug_bits, 0u};
   OMPRT_CUDA_TRY(cudaMemcpyToSymbol(omprt_env, &env_dev, sizeof env_dev));
+  // the L2 set-aside that access-policy windows of hot read-only tables may use
+  // (OMPRT_XS_FLAT); normal accesses still use it while no persisting line claims it
+  int max_persist = 0;
+  if (cudaDeviceGetAttribute(&max_persist, cudaDevAttrMaxPersistingL2CacheSize, device) ==
+          cudaSuccess &&
+      max_persist > 0 &&
+      cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, (size_t)max_persist) == cudaSuccess) {
+    size_t got = 0;
+    if (cudaDeviceGetLimit(&got, cudaLimitPersistingL2CacheSize) == cudaSuccess)
+      w.l2_persist_bytes = got;
+  }
+  cudaGetLastError();  // a device without the set-aside just runs without windows
   OMPRT_CUDA_TRY(cudaDeviceSynchronize());
   w.inited = true;
   return OMPRT_OK;
@@ -68,6 +80,13 @@ extern "C" int omprt_fini(int device) {
   cudaMemcpyToSymbol(omprt_env, &zero, sizeof zero);
   w = Workspace{};
   cudaSetDevice(prev);
+  return OMPRT_OK;
+}
+
+extern "C" int omprt_l2_reset_persisting(void) {
+  Workspace* w;
+  if (int r = current_ws(&w)) return r;
+  OMPRT_CUDA_TRY(cudaCtxResetPersistingL2Cache());
   return OMPRT_OK;
 }
 

@@ -58,6 +58,8 @@ struct Workspace {
   cudaEvent_t compute_done[2] = {nullptr, nullptr};
   uint64_t* pinned_ck = nullptr;     // [kMaxE2ESteps]
   uint64_t* dev_ck = nullptr;        // [kMaxE2ESteps]
+  // L2 set-aside for persisting accesses (cudaLimitPersistingL2CacheSize), granted at init
+  size_t l2_persist_bytes = 0;
 };
 constexpr int kMaxE2ESteps = 1024;
 

@@ -223,6 +223,45 @@ inline XSTables to_dev(const omprt_xs_tables& a) {
                   a.bins, a.index_grid16, a.brackets, a.log2_bins, 0};
 }
 
+// Launch configuration of the flattened kernels: the persistent grid, plus (unless
+// OMPRT_XS_NO_L2_PERSIST) an L2 access-policy window that makes the bracket records -- the
+// bulk of the L2 sectors a lookup touches, 36.9 MB for the small problem -- persisting in
+// the set-aside granted at omprt_init, so the 16-bit index grid's misses cannot evict
+// them; hitRatio scales down when the table exceeds the set-aside.  (Persisting lines
+// outlive the launch: omprt_l2_reset_persisting returns them to normal.)
+struct FlatLaunch {
+  cudaLaunchConfig_t cfg;
+  cudaLaunchAttribute attr[1];
+};
+inline FlatLaunch flat_launch(const omprt_xs_tables& t, int32_t teams, int32_t threads,
+                              uint32_t flags, const Workspace* w, cudaStream_t s) {
+  FlatLaunch L{};
+  L.cfg.gridDim = dim3((unsigned)teams);
+  L.cfg.blockDim = dim3((unsigned)threads);
+  L.cfg.dynamicSmemBytes = 0;
+  L.cfg.stream = s;
+  L.cfg.attrs = L.attr;
+  L.cfg.numAttrs = 0;
+  const size_t br = sizeof(double) * 12ull * t.n_isotopes * (t.n_gridpoints - 1);
+  if (!(flags & OMPRT_XS_NO_L2_PERSIST) && w->l2_persist_bytes > 0 && t.brackets) {
+    int dev = 0, maxwin = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&maxwin, cudaDevAttrMaxAccessPolicyWindowSize, dev);
+    const size_t bytes = std::min(br, (size_t)std::max(maxwin, 0));
+    if (bytes > 0) {
+      cudaAccessPolicyWindow& win = L.attr[0].val.accessPolicyWindow;
+      L.attr[0].id = cudaLaunchAttributeAccessPolicyWindow;
+      win.base_ptr = (void*)t.brackets;
+      win.num_bytes = bytes;
+      win.hitRatio = (float)std::min(1.0, (double)w->l2_persist_bytes / (double)bytes);
+      win.hitProp = cudaAccessPropertyPersisting;
+      win.missProp = cudaAccessPropertyStreaming;
+      L.cfg.numAttrs = 1;
+    }
+  }
+  return L;
+}
+
 // the flattened kernels keep the material tables in team-shared memory when they fit
 inline bool xs_mats_fit_smem(const omprt_xs_tables& t) {
   return 12ll * t.max_num_nucs <= kXSMatSmem;
@@ -342,13 +381,16 @@ extern "C" int omprt_xs_lookup(omprt_xs_tables t, uint64_t seed, int64_t first, 
   const int32_t n = (int32_t)count;
   if (flags & OMPRT_XS_FLAT) {
     const bool smem = xs_mats_fit_smem(t);
+    const FlatLaunch L = flat_launch(t, teams, threads, flags, w, s);
+    cudaError_t e;
 #define OMPRT_XSF(F, S) \
-  omprt_xs_flat_rt<XSTraits, F, S><<<teams, threads, 0, s>>>(d, seed, first, n, verification, ck, p, tk)
+  e = cudaLaunchKernelEx(&L.cfg, omprt_xs_flat_rt<XSTraits, F, S>, d, seed, first, n, verification, ck, p, tk)
     if (fused && smem) OMPRT_XSF(true, true);
     else if (fused) OMPRT_XSF(true, false);
     else if (smem) OMPRT_XSF(false, true);
     else OMPRT_XSF(false, false);
 #undef OMPRT_XSF
+    (void)e;
     return check_launch("omprt_xs_flat_rt");
   }
 #define OMPRT_XS(TR, F, A) \
@@ -393,12 +435,15 @@ extern "C" int omprt_cuda_xs_lookup(omprt_xs_tables t, uint64_t seed, int64_t fi
   auto* p = (unsigned long long*)w->partials;
   unsigned* tk = w->tickets + 1;
   const int32_t n = (int32_t)count;
-  if (flat) {
+  if (flat) {  // the same launch (geometry, L2 window) as the runtime-driven kernel
     const bool smem = xs_mats_fit_smem(t);
-    if (fused && smem) cuda_xs_flat_twin<true, true><<<tm, threads, 0, s>>>(d, seed, first, n, verification, ck, p, tk);
-    else if (fused) cuda_xs_flat_twin<true, false><<<tm, threads, 0, s>>>(d, seed, first, n, verification, ck, p, tk);
-    else if (smem) cuda_xs_flat_twin<false, true><<<tm, threads, 0, s>>>(d, seed, first, n, verification, nullptr, nullptr, nullptr);
-    else cuda_xs_flat_twin<false, false><<<tm, threads, 0, s>>>(d, seed, first, n, verification, nullptr, nullptr, nullptr);
+    const FlatLaunch L = flat_launch(t, tm, threads, flags, w, s);
+    unsigned long long* nul = nullptr;
+    unsigned* nult = nullptr;
+    if (fused && smem) cudaLaunchKernelEx(&L.cfg, cuda_xs_flat_twin<true, true>, d, seed, first, n, verification, ck, p, tk);
+    else if (fused) cudaLaunchKernelEx(&L.cfg, cuda_xs_flat_twin<true, false>, d, seed, first, n, verification, ck, p, tk);
+    else if (smem) cudaLaunchKernelEx(&L.cfg, cuda_xs_flat_twin<false, true>, d, seed, first, n, verification, nul, nul, nult);
+    else cudaLaunchKernelEx(&L.cfg, cuda_xs_flat_twin<false, false>, d, seed, first, n, verification, nul, nul, nult);
     return check_launch("cuda_xs_flat_twin");
   }
   if (fused && accel) cuda_xs_twin<true, true><<<tm, threads, 0, s>>>(d, seed, first, n, verification, ck, p, tk);

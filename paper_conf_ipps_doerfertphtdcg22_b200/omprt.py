@@ -37,10 +37,11 @@ OMPRT_DEGLOBALIZE = 1 << 12
 OMPRT_TMA_STAGED = 1 << 13
 OMPRT_WARP_STAGED = 1 << 14
 OMPRT_XS_FLAT = 1 << 15
+OMPRT_XS_NO_L2_PERSIST = 1 << 16
 
 # Every symbol include/omprt.h declares (checked by tests/test_abi.py).
 EXPORTS = [
-    "omprt_init", "omprt_fini", "omprt_device_status", "omprt_last_error", "omprt_static_owner",
+    "omprt_init", "omprt_fini", "omprt_l2_reset_persisting", "omprt_device_status", "omprt_last_error", "omprt_static_owner",
     "omprt_spmd_axpy_sum", "omprt_cuda_axpy_sum", "omprt_spmd_axpy_sum_chunked",
     "omprt_cuda_axpy_sum_chunked", "omprt_generic_team", "omprt_cuda_generic_team",
     "omprt_icv_probe", "omprt_xs_lookup", "omprt_cuda_xs_lookup", "omprt_u64_sum",
@@ -82,6 +83,7 @@ _vp, _i32, _i64, _u32, _u64, _f64 = C.c_void_p, C.c_int32, C.c_int64, C.c_uint32
 _SIGS = {
     "omprt_init": [C.c_int, C.POINTER(Options)],
     "omprt_fini": [C.c_int],
+    "omprt_l2_reset_persisting": [],
     "omprt_device_status": [C.c_int, C.POINTER(C.c_int), C.POINTER(C.c_int)],
     "omprt_last_error": [C.c_char_p, C.c_size_t],
     "omprt_static_owner": [_i64, _i64, _i32, _i32, C.POINTER(_i32), C.POINTER(_i32)],
@@ -176,6 +178,12 @@ def omprt_init(device=0, pool_bytes_per_team=0, pool_teams=0, max_teams=0):
 
 def omprt_fini(device=0):
     return _check(load().omprt_fini(device))
+
+
+def omprt_l2_reset_persisting():
+    """Return persisting L2 lines (OMPRT_XS_FLAT's access-policy window) to normal; call
+    with no launch in flight."""
+    return _check(load().omprt_l2_reset_persisting())
 
 
 def omprt_device_status(device=0):

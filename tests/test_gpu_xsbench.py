@@ -80,6 +80,19 @@ def test_flat_fused_checksum_and_edges(rt, xs_acc, xs_small):
             assert int(ck.cpu().numpy()[0]) == ref + 7
 
 
+def test_flat_without_l2_window_and_reset(rt, xs_acc, xs_small):
+    """The same bits with the L2 access-policy window off, and after resetting persisting
+    lines (the window only changes where the bracket records are cached)."""
+    first, count = 77, 100_003
+    ref = oracle.xs_lookup(xs_small, first, count, threads=os.cpu_count() or 1)
+    for fl in (rt.OMPRT_XS_FLAT | rt.OMPRT_XS_NO_L2_PERSIST, rt.OMPRT_XS_FLAT):
+        ver = torch.zeros(count, dtype=torch.uint64, device=DEV)
+        rt.omprt_xs_lookup(xs_acc, SEED, first, count, ver, None, 0, 256, fl)
+        torch.cuda.synchronize()
+        rt.omprt_l2_reset_persisting()
+        assert (ver.cpu().numpy() == ref).all()
+
+
 def test_flat_rejects(rt, xs_dev, xs_acc):
     ver = torch.zeros(64, dtype=torch.uint64, device=DEV)
     F = rt.OMPRT_XS_FLAT

@@ -234,6 +234,21 @@ int omprt_xs_accel_sizes(int32_t n_isotopes, int32_t n_gridpoints, int64_t n_uni
  * XSBench's own index-grid construction), not part of a lookup. */
 int omprt_xs_build_accel(omprt_xs_tables *t, int32_t *bins, uint16_t *index_grid16,
                          double *brackets, int32_t log2_bins, void *stream);
+/* Derive XSBench's unionized energy grid and its index grid from the nuclide grids on the
+ * device (XSBench builds them at initialization):
+ *   unionized[e] = the e-th smallest of the n_isotopes*n_gridpoints energies
+ *                  (nuclide_grid[i*6], i = nuclide*n_gridpoints + k; energies finite,
+ *                  sorted within each nuclide, no -0.0),
+ *   index_grid16[e*n_isotopes + q] = clip(#{k : E_q[k] <= unionized[e]} - 1, 0,
+ *                  n_gridpoints - 2)   (ties handled exactly).
+ * All pointers are device pointers (unionized: n_isotopes*n_gridpoints doubles,
+ * index_grid16: that many rows of n_isotopes uint16); tmp: >= omprt_xs_derive_tmp_bytes
+ * bytes of device scratch, 256 B aligned.  Asynchronous on `stream`.  OMPRT_E_INVAL
+ * unless 0 < n_isotopes <= 4096 and 2 <= n_gridpoints <= 65536. */
+int omprt_xs_derive_tmp_bytes(int32_t n_isotopes, int32_t n_gridpoints, uint64_t *bytes);
+int omprt_xs_derive(const double *nuclide_grid, int32_t n_isotopes, int32_t n_gridpoints,
+                    double *unionized, uint16_t *index_grid16, void *tmp, uint64_t tmp_bytes,
+                    void *stream);
 /* K11 ("we moved the reduction out of the timed kernel"): *out_inout += sum v[i]
  * (u64, wraps mod 2^64). */
 int omprt_u64_sum(const uint64_t *v, int64_t n, uint64_t *out_inout, void *stream);
@@ -251,8 +266,11 @@ int omprt_xs_run_host(omprt_xs_tables host_tables, uint64_t seed, int64_t first,
  * `target nowait` + dependences).  host_tables may hold the B200 layouts on the host:
  * index_grid16 (then index_grid may be NULL and 2 B per entry cross PCIe) and/or brackets
  * (then nuclide_grid may be NULL); whatever is missing is built on the device (bins
- * always), which also enables the accelerated lookup (as OMPRT_XS_ACCEL does).
- * *h2d_bytes = bytes copied host->device per step.  Synchronous. */
+ * always), which also enables the accelerated lookup (as OMPRT_XS_ACCEL does).  With
+ * unionized, index_grid and index_grid16 all NULL only the raw problem data crosses PCIe
+ * (nuclide_grid + materials) and the unionized grid and the 16-bit index grid are derived
+ * on the device each step (omprt_xs_derive).  *h2d_bytes = bytes copied host->device per
+ * step.  Synchronous. */
 int omprt_xs_run_host_steps(omprt_xs_tables host_tables, uint64_t seed, int64_t first,
                             int64_t count, int32_t threads, uint32_t flags, int32_t steps,
                             uint64_t *checksums_host, uint64_t *h2d_bytes, uint64_t *d2h_bytes,

@@ -68,7 +68,10 @@ extern "C" int omprt_fini(int device) {
   cudaFree(w.pool);
   cudaFree(w.xs_buf[0]);
   cudaFree(w.xs_buf[1]);
+  cudaFree(w.xs_built);
   cudaFree(w.dev_ck);
+  cudaFree(w.derive_tmp);
+  cudaFree(w.e2e_ver);
   if (w.pinned_ck) cudaFreeHost(w.pinned_ck);
   for (int k = 0; k < 2; ++k) {
     if (w.copy_done[k]) cudaEventDestroy(w.copy_done[k]);

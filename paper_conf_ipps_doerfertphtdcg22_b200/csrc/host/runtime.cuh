@@ -53,11 +53,21 @@ struct Workspace {
   // across steps), grown on demand; a copy stream, per-slot events, pinned checksums
   void* xs_buf[2] = {nullptr, nullptr};
   size_t xs_buf_bytes = 0;
+  // ... and one buffer for the tables built on the device (written and read on the compute
+  // stream only, so one copy serves every step, and the L2 window stays on one range)
+  void* xs_built = nullptr;
+  size_t xs_built_bytes = 0;
   cudaStream_t copy_stream = nullptr;
   cudaEvent_t copy_done[2] = {nullptr, nullptr};
   cudaEvent_t compute_done[2] = {nullptr, nullptr};
   uint64_t* pinned_ck = nullptr;     // [kMaxE2ESteps]
   uint64_t* dev_ck = nullptr;        // [kMaxE2ESteps]
+  // omprt_xs_run_host_steps with derived tables: omprt_xs_derive scratch (grown on demand)
+  void* derive_tmp = nullptr;
+  size_t derive_tmp_bytes = 0;
+  // flattened e2e steps: per-lookup verification scratch, summed by K11 (u64 entries)
+  uint64_t* e2e_ver = nullptr;
+  size_t e2e_ver_n = 0;
   // L2 set-aside for persisting accesses (cudaLimitPersistingL2CacheSize), granted at init
   size_t l2_persist_bytes = 0;
 };

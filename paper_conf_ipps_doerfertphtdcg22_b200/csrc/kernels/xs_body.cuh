@@ -239,7 +239,8 @@ struct XSFlatLookup {
   uint64_t* __restrict__ const ver;
   const int32_t* __restrict__ const mats;  // t.mats, or its team-shared copy
   const double* __restrict__ const concs;  // t.concs, or its team-shared copy
-  unsigned long long acc = 0;  // Fused: this thread's verification sum
+  // Fused: this thread's verification sum lives in a per-thread shared-memory slot
+  // (flat_acc_slot), not in a register held across the whole loop (that spilled)
   LcgMap J;
   uint64_t s;
   double E;
@@ -325,8 +326,13 @@ struct XSFlatLookup {
   template <class Idx>
   __device__ __forceinline__ void end(Idx iv) {
     const uint64_t v = xs_argmax5(m0, m1, m2, m3, m4);
-    if constexpr (Fused) acc += v;
+    if constexpr (Fused) *flat_acc_slot() += v;
     else ver[iv] = v;
+  }
+  // this thread's slot (static shared memory: a constant address, no register)
+  static __device__ __forceinline__ unsigned long long* flat_acc_slot() {
+    __shared__ unsigned long long slots[1024];
+    return slots + threadIdx.x;
   }
 };
 
@@ -399,16 +405,14 @@ __global__ void xs_build_index16(const int32_t* __restrict__ a, uint16_t* __rest
 }
 __global__ void xs_build_brackets(const double* __restrict__ g, double* __restrict__ o,
                                   int32_t n_iso, int32_t n_gp) {
-  const int64_t nb = (int64_t)n_iso * (n_gp - 1);
-  for (int64_t b = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; b < nb;
-       b += (int64_t)gridDim.x * blockDim.x) {
-    const int64_t p = b / (n_gp - 1), k = b % (n_gp - 1);
-    const double* lo = g + (p * n_gp + k) * 6;
-#pragma unroll
-    for (int c = 0; c < 6; ++c) {
-      o[b * 12 + 2 * c] = lo[c];
-      o[b * 12 + 2 * c + 1] = lo[6 + c];
-    }
+  // one output double per thread (coalesced stores): o[b*12 + 2c + h] = g[(p*n_gp + k + h)*6 + c]
+  const int64_t total = (int64_t)n_iso * (n_gp - 1) * 12;
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < total;
+       i += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t b = i / 12;
+    const int j = (int)(i - b * 12), c = j >> 1, h = j & 1;
+    const int64_t p = b / (n_gp - 1), k = b - p * (n_gp - 1);
+    o[i] = __ldg(g + (p * n_gp + k + h) * 6 + c);
   }
 }
 

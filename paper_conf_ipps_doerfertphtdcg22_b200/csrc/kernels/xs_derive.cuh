@@ -1,0 +1,186 @@
+// XSBench's derived tables built on the device from the nuclide grids (SURVEY App. A.1:
+// "unionized grid: all energies, sorted; index grid: per unionized energy and nuclide, the
+// lower bracket index"), so an end-to-end step ships only the raw problem data (nuclide
+// grids + materials, 36.9 MB for the small problem) instead of 147.6 MB of tables.
+//
+//   unionized[e]       = the e-th smallest of all n_iso * n_gp energies (a radix sort of the
+//                        energies' order-preserving 64-bit keys; CUB, the library primitive)
+//   index_grid[e][q]   = clip(#{k : E_q[k] <= unionized[e]} - 1, 0, n_gp - 2)
+//
+// The index rows are a column-wise prefix count over the sorted order: row e differs from
+// row e-1 only in the column of the nuclide that energy e came from.  Rows are cut into
+// chunks of kDeriveRows; (A) counts each chunk's nuclide ids, (B) scans the counts over the
+// chunks per nuclide, (C) walks each chunk with one thread per nuclide column, writing whole
+// rows (n_iso x 2 B, coalesced).  Equal energies (ties) are handled exactly: a row whose
+// energy equals the next rows' also counts those rows (`<=`), by a look-ahead that only runs
+// at ties.  Energies must be finite and not -0.0 (the proxy app draws them from [0, 1)).
+#pragma once
+#include <cub/block/block_scan.cuh>
+#include <cub/device/device_radix_sort.cuh>
+
+#include "../host/runtime.cuh"
+
+namespace omprt_kernels {
+
+constexpr int kDeriveRows = 256;  // rows per chunk
+constexpr int kDeriveMaxIso = 4096;
+
+__global__ void xs_derive_keys(const double* __restrict__ g, int32_t n_gp, int64_t n,
+                               unsigned long long* __restrict__ keys,
+                               uint16_t* __restrict__ ids) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n;
+       i += (int64_t)gridDim.x * blockDim.x) {
+    const unsigned long long b = (unsigned long long)__double_as_longlong(__ldg(g + i * 6));
+    keys[i] = (b >> 63) ? ~b : (b | (1ull << 63));  // IEEE order as unsigned order
+    ids[i] = (uint16_t)(i / n_gp);
+  }
+}
+
+__global__ void xs_derive_unionized(const unsigned long long* __restrict__ keys, int64_t n,
+                                    double* __restrict__ U) {
+  for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < n;
+       e += (int64_t)gridDim.x * blockDim.x) {
+    const unsigned long long k = keys[e];
+    U[e] = __longlong_as_double((long long)((k >> 63) ? (k & ~(1ull << 63)) : ~k));
+  }
+}
+
+// (A) per chunk: how many of its rows come from each nuclide
+__global__ void xs_derive_hist(const uint16_t* __restrict__ ids, int64_t n, int32_t n_iso,
+                               uint32_t* __restrict__ hist) {
+  __shared__ uint32_t h[kDeriveMaxIso];
+  for (int q = threadIdx.x; q < n_iso; q += blockDim.x) h[q] = 0;
+  __syncthreads();
+  const int64_t r0 = (int64_t)blockIdx.x * kDeriveRows;
+  const int64_t r1 = r0 + kDeriveRows < n ? r0 + kDeriveRows : n;
+  for (int64_t e = r0 + threadIdx.x; e < r1; e += blockDim.x) atomicAdd(&h[ids[e]], 1u);
+  __syncthreads();
+  for (int q = threadIdx.x; q < n_iso; q += blockDim.x)
+    hist[(int64_t)blockIdx.x * n_iso + q] = h[q];
+}
+
+// (B) per nuclide (one block each): exclusive scan of the chunk counts, in place
+constexpr int kScanThreads = 1024;
+__global__ void __launch_bounds__(kScanThreads)
+    xs_derive_scan(uint32_t* __restrict__ hist, int32_t n_chunks, int32_t n_iso) {
+  using Scan = cub::BlockScan<uint32_t, kScanThreads>;
+  __shared__ typename Scan::TempStorage tmp;
+  const int q = blockIdx.x;
+  uint32_t carry = 0;
+  for (int c0 = 0; c0 < n_chunks; c0 += kScanThreads) {
+    const int c = c0 + threadIdx.x;
+    const uint32_t v = c < n_chunks ? hist[(int64_t)c * n_iso + q] : 0u;
+    uint32_t ex, tot;
+    Scan(tmp).ExclusiveSum(v, ex, tot);
+    if (c < n_chunks) hist[(int64_t)c * n_iso + q] = carry + ex;
+    carry += tot;
+    __syncthreads();  // tmp is reused by the next tile
+  }
+}
+
+// (C) per chunk, one thread per nuclide column: the running count -> index rows
+__global__ void xs_derive_index(const uint16_t* __restrict__ ids, const double* __restrict__ U,
+                                const uint32_t* __restrict__ start, int64_t n, int32_t n_iso,
+                                int32_t n_gp, uint16_t* __restrict__ index16) {
+  __shared__ uint16_t sid[kDeriveRows];
+  __shared__ double su[kDeriveRows + 1];
+  const int64_t r0 = (int64_t)blockIdx.x * kDeriveRows;
+  const int rows = (int)(r0 + kDeriveRows < n ? kDeriveRows : n - r0);
+  for (int k = threadIdx.x; k < rows; k += blockDim.x) sid[k] = ids[r0 + k];
+  for (int k = threadIdx.x; k <= rows; k += blockDim.x) su[k] = r0 + k < n ? U[r0 + k] : 0.0;
+  __syncthreads();
+  const int32_t kmax = n_gp - 2;
+  for (int q = threadIdx.x; q < n_iso; q += blockDim.x) {
+    int64_t cnt = start[(int64_t)blockIdx.x * n_iso + q];
+    for (int k = 0; k < rows; ++k) {
+      cnt += sid[k] == q;
+      int64_t v = cnt;
+      if (r0 + k + 1 < n && su[k + 1] == su[k]) {  // tie: count the equal rows ahead too
+        for (int64_t e2 = r0 + k + 1; e2 < n && U[e2] == su[k]; ++e2) v += ids[e2] == q;
+      }
+      v -= 1;
+      index16[(r0 + k) * n_iso + q] = (uint16_t)(v < 0 ? 0 : (v > kmax ? kmax : v));
+    }
+  }
+}
+
+struct DeriveLayout {
+  size_t keys_in, keys_out, ids_in, ids_out, hist, cub, total;
+};
+inline size_t al256(size_t b) { return (b + 255) & ~size_t(255); }
+
+inline int xs_derive_layout(int32_t n_iso, int32_t n_gp, DeriveLayout* L) {
+  OMPRT_CHECK_ARG(n_iso > 0 && n_iso <= kDeriveMaxIso && n_gp >= 2 && n_gp <= 65536 &&
+                      (int64_t)n_iso * n_gp < (1ll << 31),
+                  "omprt_xs_derive: need 0 < n_isotopes <= %d, 2 <= n_gridpoints <= 65536",
+                  kDeriveMaxIso);
+  const int64_t n = (int64_t)n_iso * n_gp;
+  const int64_t chunks = (n + kDeriveRows - 1) / kDeriveRows;
+  size_t cub_bytes = 0;
+  cub::DeviceRadixSort::SortPairs(nullptr, cub_bytes, (const unsigned long long*)nullptr,
+                                  (unsigned long long*)nullptr, (const uint16_t*)nullptr,
+                                  (uint16_t*)nullptr, (int)n);
+  size_t off = 0;
+  L->keys_in = off;
+  off += al256(8 * n);
+  L->keys_out = off;
+  off += al256(8 * n);
+  L->ids_in = off;
+  off += al256(2 * n);
+  L->ids_out = off;
+  off += al256(2 * n);
+  L->hist = off;
+  off += al256(4 * chunks * n_iso);
+  L->cub = off;
+  off += al256(cub_bytes);
+  L->total = off;
+  return OMPRT_OK;
+}
+
+inline int xs_derive(const double* nuclide_grid, int32_t n_iso, int32_t n_gp, double* U,
+                     uint16_t* index16, void* tmp, size_t tmp_bytes, cudaStream_t s) {
+  DeriveLayout L;
+  if (int r = xs_derive_layout(n_iso, n_gp, &L)) return r;
+  OMPRT_CHECK_ARG(nuclide_grid && U && index16 && tmp, "omprt_xs_derive: null pointer");
+  OMPRT_CHECK_ARG(tmp_bytes >= L.total, "omprt_xs_derive: tmp needs %zu B", L.total);
+  const int64_t n = (int64_t)n_iso * n_gp;
+  const int32_t chunks = (int32_t)((n + kDeriveRows - 1) / kDeriveRows);
+  unsigned char* b = (unsigned char*)tmp;
+  auto* kin = (unsigned long long*)(b + L.keys_in);
+  auto* kout = (unsigned long long*)(b + L.keys_out);
+  auto* iin = (uint16_t*)(b + L.ids_in);
+  auto* iout = (uint16_t*)(b + L.ids_out);
+  auto* hist = (uint32_t*)(b + L.hist);
+  size_t cub_bytes = L.total - L.cub;
+  xs_derive_keys<<<1024, 256, 0, s>>>(nuclide_grid, n_gp, n, kin, iin);
+  if (cub::DeviceRadixSort::SortPairs(b + L.cub, cub_bytes, kin, kout, iin, iout, (int)n, 0, 64,
+                                      s) != cudaSuccess)
+    return set_error(OMPRT_E_CUDA, "omprt_xs_derive: radix sort failed");
+  xs_derive_unionized<<<1024, 256, 0, s>>>(kout, n, U);
+  xs_derive_hist<<<chunks, 256, 0, s>>>(iout, n, n_iso, hist);
+  xs_derive_scan<<<n_iso, kScanThreads, 0, s>>>(hist, chunks, n_iso);
+  xs_derive_index<<<chunks, 128, 0, s>>>(iout, U, hist, n, n_iso, n_gp, index16);
+  return check_launch("omprt_xs_derive");
+}
+
+}  // namespace omprt_kernels
+
+extern "C" int omprt_xs_derive_tmp_bytes(int32_t n_isotopes, int32_t n_gridpoints,
+                                         uint64_t* bytes) {
+  using namespace omprt_kernels;
+  OMPRT_CHECK_ARG(bytes != nullptr, "omprt_xs_derive_tmp_bytes: null output");
+  DeriveLayout L;
+  if (int r = xs_derive_layout(n_isotopes, n_gridpoints, &L)) return r;
+  *bytes = L.total;
+  return OMPRT_OK;
+}
+
+extern "C" int omprt_xs_derive(const double* nuclide_grid, int32_t n_isotopes,
+                               int32_t n_gridpoints, double* unionized, uint16_t* index_grid16,
+                               void* tmp, uint64_t tmp_bytes, void* stream) {
+  using namespace omprt_kernels;
+  Workspace* w;
+  if (int r = current_ws(&w)) return r;
+  return xs_derive(nuclide_grid, n_isotopes, n_gridpoints, unionized, index_grid16, tmp,
+                   tmp_bytes, as_stream(stream));
+}

@@ -8,6 +8,7 @@
 #pragma once
 #include "../host/runtime.cuh"
 #include "xs_body.cuh"
+#include "xs_derive.cuh"
 
 namespace omprt_kernels {
 
@@ -134,11 +135,13 @@ __global__ void __launch_bounds__(kXSThreads, kXSMinBlocksFlat)
     mats = sm;
     concs = sc;
   }
-  XSFlatLookup<Fused, Smem> lookup(t, seed, first, verification, mats, concs);
+  using Lookup = XSFlatLookup<Fused, Smem>;
+  if constexpr (Fused) *Lookup::flat_acc_slot() = 0ull;
+  Lookup lookup(t, seed, first, verification, mats, concs);
   distribute_parallel_for_flat(team, count, lookup);
   if constexpr (Fused)
-    league_reduce(team, team_reduce_to_main(team, lookup.acc, Plus{}), Plus{}, checksum,
-                  partials, ticket);
+    league_reduce(team, team_reduce_to_main(team, *Lookup::flat_acc_slot(), Plus{}), Plus{},
+                  checksum, partials, ticket);
 }
 
 // Bare CUDA twin: the same flattened loop written by hand around the same body.
@@ -161,7 +164,9 @@ __global__ void __launch_bounds__(kXSThreads, kXSMinBlocksFlat)
     mats = sm;
     concs = sc;
   }
-  XSFlatLookup<Fused, Smem> lookup(t, seed, first, verification, mats, concs);
+  using Lookup = XSFlatLookup<Fused, Smem>;
+  if constexpr (Fused) *Lookup::flat_acc_slot() = 0ull;
+  Lookup lookup(t, seed, first, verification, mats, concs);
   const int32_t stride = (int32_t)gridDim.x * (int32_t)blockDim.x;
   int32_t i = (int32_t)blockIdx.x * (int32_t)blockDim.x + (int32_t)threadIdx.x;
   auto run = [&]() {
@@ -179,7 +184,7 @@ __global__ void __launch_bounds__(kXSThreads, kXSMinBlocksFlat)
     run();
   } else {
     if (i < count) run();
-    twin_u64_ticket_sum(lookup.acc, checksum, partials, ticket);
+    twin_u64_ticket_sum(*Lookup::flat_acc_slot(), checksum, partials, ticket);
   }
 }
 
@@ -488,12 +493,17 @@ extern "C" int omprt_xs_run_host_steps(omprt_xs_tables h, uint64_t seed, int64_t
   using namespace omprt_kernels;
   Workspace* w;
   if (int r = current_ws(&w)) return r;
-  OMPRT_CHECK_ARG(checksums_host && steps >= 1 && steps <= kMaxE2ESteps && h.unionized &&
-                      h.num_nucs && h.mats && h.concs && (h.index_grid || h.index_grid16) &&
-                      (h.nuclide_grid || h.brackets),
+  // derive: only the raw data crosses PCIe; the unionized and index grids are built here
+  const bool derive = !h.unionized && !h.index_grid && !h.index_grid16;
+  OMPRT_CHECK_ARG(checksums_host && steps >= 1 && steps <= kMaxE2ESteps && h.num_nucs &&
+                      h.mats && h.concs && (h.nuclide_grid || h.brackets) &&
+                      (derive ? h.nuclide_grid != nullptr
+                              : (h.unionized && (h.index_grid || h.index_grid16))),
                   "omprt_xs_run_host_steps: bad arguments");
+  OMPRT_CHECK_ARG(!derive || (int64_t)h.n_isotopes * h.n_gridpoints == h.n_union,
+                  "derived tables: n_union must be n_isotopes * n_gridpoints");
   const bool accel =
-      (flags & (OMPRT_XS_ACCEL | OMPRT_XS_FLAT)) || h.index_grid16 || h.brackets;
+      derive || (flags & (OMPRT_XS_ACCEL | OMPRT_XS_FLAT)) || h.index_grid16 || h.brackets;
   OMPRT_CHECK_ARG(accel || (h.index_grid && h.nuclide_grid),
                   "the plain path needs the int32 index grid and the nuclide grid");
   OMPRT_CHECK_ARG(!accel || h.n_gridpoints <= 65536, "16-bit index: n_gridpoints > 65536");
@@ -504,8 +514,26 @@ extern "C" int omprt_xs_run_host_steps(omprt_xs_tables h, uint64_t seed, int64_t
   const bool up16 = accel && h.index_grid16, upbr = accel && h.brackets;
   const size_t n_grid = upbr ? 0 : (size_t)h.n_isotopes * h.n_gridpoints * 6 * sizeof(double);
   const size_t n_br = upbr ? asz[2] : 0;
-  const size_t n_uni = (size_t)h.n_union * sizeof(double);
-  const size_t n_idx = up16 ? asz[1] : (size_t)h.n_union * h.n_isotopes * sizeof(int32_t);
+  const size_t n_uni = derive ? 0 : (size_t)h.n_union * sizeof(double);
+  const size_t n_idx =
+      derive ? 0 : (up16 ? asz[1] : (size_t)h.n_union * h.n_isotopes * sizeof(int32_t));
+  const size_t built_uni = derive ? (size_t)h.n_union * sizeof(double) : 0;
+  if (derive) {
+    uint64_t tb = 0;
+    if (int r = omprt_xs_derive_tmp_bytes(h.n_isotopes, h.n_gridpoints, &tb)) return r;
+    if (w->derive_tmp_bytes < tb) {
+      OMPRT_CUDA_TRY(cudaDeviceSynchronize());
+      cudaFree(w->derive_tmp);
+      w->derive_tmp = nullptr;
+      w->derive_tmp_bytes = 0;
+      if (cudaMalloc(&w->derive_tmp, tb) != cudaSuccess) {
+        cudaGetLastError();
+        return set_error(OMPRT_E_NOMEM, "omprt_xs_run_host_steps: cannot allocate %llu B",
+                         (unsigned long long)tb);
+      }
+      w->derive_tmp_bytes = tb;
+    }
+  }
   const size_t n_num = 12 * sizeof(int32_t);
   const size_t n_mat = (size_t)12 * h.max_num_nucs * sizeof(int32_t);
   const size_t n_con = (size_t)12 * h.max_num_nucs * sizeof(double);
@@ -513,7 +541,21 @@ extern "C" int omprt_xs_run_host_steps(omprt_xs_tables h, uint64_t seed, int64_t
   // slot layout: uploaded tables, then the device-built layouts
   const size_t built16 = (accel && !up16) ? asz[1] : 0, builtbr = (accel && !upbr) ? asz[2] : 0;
   const size_t total = al(n_grid) + al(n_br) + al(n_uni) + al(n_idx) + al(n_num) + al(n_mat) +
-                       al(n_con) + al(asz[0]) + al(built16) + al(builtbr);
+                       al(n_con);
+  const size_t total_built =
+      accel ? al(asz[0]) + al(built16) + al(builtbr) + al(built_uni) : 0;
+  if (w->xs_built_bytes < total_built) {
+    OMPRT_CUDA_TRY(cudaDeviceSynchronize());
+    cudaFree(w->xs_built);
+    w->xs_built = nullptr;
+    w->xs_built_bytes = 0;
+    if (cudaMalloc(&w->xs_built, total_built) != cudaSuccess) {
+      cudaGetLastError();
+      return set_error(OMPRT_E_NOMEM, "omprt_xs_run_host_steps: cannot allocate %zu B",
+                       total_built);
+    }
+    w->xs_built_bytes = total_built;
+  }
   if (!w->copy_stream) {
     OMPRT_CUDA_TRY(cudaStreamCreateWithFlags(&w->copy_stream, cudaStreamNonBlocking));
     for (int k = 0; k < 2; ++k) {
@@ -523,6 +565,17 @@ extern "C" int omprt_xs_run_host_steps(omprt_xs_tables h, uint64_t seed, int64_t
     OMPRT_CUDA_TRY(cudaHostAlloc(&w->pinned_ck, kMaxE2ESteps * sizeof(uint64_t),
                                  cudaHostAllocDefault));
     OMPRT_CUDA_TRY(cudaMalloc(&w->dev_ck, kMaxE2ESteps * sizeof(uint64_t)));
+  }
+  if ((flags & OMPRT_XS_FLAT) && w->e2e_ver_n < (size_t)count) {
+    OMPRT_CUDA_TRY(cudaDeviceSynchronize());
+    cudaFree(w->e2e_ver);
+    w->e2e_ver = nullptr;
+    w->e2e_ver_n = 0;
+    if (cudaMalloc(&w->e2e_ver, std::max<size_t>(count, 1) * sizeof(uint64_t)) != cudaSuccess) {
+      cudaGetLastError();
+      return set_error(OMPRT_E_NOMEM, "omprt_xs_run_host_steps: cannot allocate verification");
+    }
+    w->e2e_ver_n = std::max<size_t>(count, 1);
   }
   if (w->xs_buf_bytes < total) {
     OMPRT_CUDA_TRY(cudaDeviceSynchronize());
@@ -568,21 +621,31 @@ extern "C" int omprt_xs_run_host_steps(omprt_xs_tables h, uint64_t seed, int64_t
     ok = ok && cudaEventRecord(w->copy_done[b], cs) == cudaSuccess;
     if (!ok) return set_error(OMPRT_E_CUDA, "omprt_xs_run_host_steps: H2D copy failed");
     OMPRT_CUDA_TRY(cudaStreamWaitEvent(s, w->copy_done[b], 0));
-    d.index_grid = up16 ? nullptr : (const int32_t*)idx;
+    d.index_grid = (up16 || derive) ? nullptr : (const int32_t*)idx;
     d.bins = nullptr;
     d.index_grid16 = nullptr;
     d.brackets = nullptr;
     if (accel) {
-      int32_t* bins = (int32_t*)(base + off);
-      off += al(asz[0]);
-      uint16_t* i16 = up16 ? (uint16_t*)idx : (uint16_t*)(base + off);
-      off += al(built16);
-      double* brk = upbr ? br : (double*)(base + off);
-      off += al(builtbr);
-      xs_build_bins<<<1024, 256, 0, s>>>(d.unionized, (int32_t)d.n_union, log2_bins, bins);
-      if (!up16)
+      unsigned char* bb = (unsigned char*)w->xs_built;
+      size_t bo = 0;
+      int32_t* bins = (int32_t*)(bb + bo);
+      bo += al(asz[0]);
+      uint16_t* i16 = up16 ? (uint16_t*)idx : (uint16_t*)(bb + bo);
+      bo += al(built16);
+      double* brk = upbr ? br : (double*)(bb + bo);
+      bo += al(builtbr);
+      if (derive) {
+        double* U = (double*)(bb + bo);
+        bo += al(built_uni);
+        if (int r = xs_derive(d.nuclide_grid, d.n_isotopes, d.n_gridpoints, U, i16,
+                              w->derive_tmp, w->derive_tmp_bytes, s))
+          return r;
+        d.unionized = U;
+      } else if (!up16) {
         xs_build_index16<<<2048, 256, 0, s>>>(d.index_grid, i16,
                                               (int64_t)d.n_union * d.n_isotopes);
+      }
+      xs_build_bins<<<1024, 256, 0, s>>>(d.unionized, (int32_t)d.n_union, log2_bins, bins);
       if (!upbr)
         xs_build_brackets<<<2048, 256, 0, s>>>(d.nuclide_grid, brk, d.n_isotopes,
                                                d.n_gridpoints);
@@ -592,11 +655,20 @@ extern "C" int omprt_xs_run_host_steps(omprt_xs_tables h, uint64_t seed, int64_t
       d.brackets = brk;
       d.log2_bins = log2_bins;
     }
-    if (int r = omprt_xs_lookup(d, seed, first, count, nullptr, w->dev_ck + st, 0, threads,
-                                (flags & ~OMPRT_XS_ACCEL) | OMPRT_FUSED_REDUCTION |
-                                    ((flags & OMPRT_XS_FLAT) ? 0u : OMPRT_ASSUME_OVERSUB),
-                                stream))
+    if (flags & OMPRT_XS_FLAT) {
+      // flattened: per-lookup verification + K11 sum (the fused flat kernel spills: its
+      // extra live state does not fit the 64 registers of 4 teams per SM)
+      if (int r = omprt_xs_lookup(d, seed, first, count, w->e2e_ver, nullptr, 0, threads,
+                                  flags & ~OMPRT_XS_ACCEL, stream))
+        return r;
+      if (int r = launch_u64_sum(w->e2e_ver, count, w->dev_ck + st, w, s)) return r;
+    } else if (int r = omprt_xs_lookup(d, seed, first, count, nullptr, w->dev_ck + st, 0,
+                                       threads,
+                                       (flags & ~OMPRT_XS_ACCEL) | OMPRT_FUSED_REDUCTION |
+                                           OMPRT_ASSUME_OVERSUB,
+                                       stream)) {
       return r;
+    }
     OMPRT_CUDA_TRY(cudaMemcpyAsync(w->pinned_ck + st, w->dev_ck + st, sizeof(uint64_t),
                                    cudaMemcpyDeviceToHost, s));
     OMPRT_CUDA_TRY(cudaEventRecord(w->compute_done[b], s));

@@ -7,5 +7,6 @@
 #include "kernels/axpy_chunk.cuh"
 #include "kernels/generic.cuh"
 #include "kernels/xsbench.cuh"
+#include "kernels/xs_derive.cuh"
 #include "kernels/rs_su3.cuh"
 #include "kernels/su3_staged.cuh"

@@ -45,7 +45,8 @@ EXPORTS = [
     "omprt_spmd_axpy_sum", "omprt_cuda_axpy_sum", "omprt_spmd_axpy_sum_chunked",
     "omprt_cuda_axpy_sum_chunked", "omprt_generic_team", "omprt_cuda_generic_team",
     "omprt_icv_probe", "omprt_xs_lookup", "omprt_cuda_xs_lookup", "omprt_u64_sum",
-    "omprt_xs_run_host", "omprt_xs_run_host_steps", "omprt_xs_accel_sizes", "omprt_xs_build_accel", "omprt_rs_lookup", "omprt_cuda_rs_lookup", "omprt_su3_mult",
+    "omprt_xs_run_host", "omprt_xs_run_host_steps", "omprt_xs_accel_sizes", "omprt_xs_build_accel",
+    "omprt_xs_derive_tmp_bytes", "omprt_xs_derive", "omprt_rs_lookup", "omprt_cuda_rs_lookup", "omprt_su3_mult",
     "omprt_cuda_su3_mult", "omprt_kernel_count", "omprt_kernel_name", "omprt_kernel_attrs",
 ]
 
@@ -101,6 +102,8 @@ _SIGS = {
     "omprt_u64_sum": [_vp, _i64, _vp, _vp],
     "omprt_xs_accel_sizes": [_i32, _i32, _i64, _i32, C.POINTER(_u64)],
     "omprt_xs_build_accel": [C.POINTER(XSTablesC), _vp, _vp, _vp, _i32, _vp],
+    "omprt_xs_derive_tmp_bytes": [_i32, _i32, C.POINTER(_u64)],
+    "omprt_xs_derive": [_vp, _i32, _i32, _vp, _vp, _vp, _u64, _vp],
     "omprt_xs_run_host": [XSTablesC, _u64, _i64, _i64, _i32, _u32, C.POINTER(_u64),
                           C.POINTER(_u64), C.POINTER(_u64), _vp],
     "omprt_xs_run_host_steps": [XSTablesC, _u64, _i64, _i64, _i32, _u32, _i32, C.POINTER(_u64),
@@ -289,16 +292,37 @@ def omprt_xs_build_accel(tables, bins, index_grid16, brackets, log2_bins=16, str
                                               _p(brackets), log2_bins, _stream(stream)))
 
 
-def xs_host_struct(t, pinned=None):
+def xs_host_struct(t, pinned=None, derive=False):
     """By-value struct of HOST table pointers (numpy arrays or pinned torch tensors).
     `pinned` maps field names to host buffers; with "index_grid16" (and no "index_grid")
-    the compact 16-bit index grid crosses PCIe instead of the int32 one."""
+    the compact 16-bit index grid crosses PCIe instead of the int32 one.  derive=True: only
+    the raw data (nuclide grid + materials); the unionized and index grids are derived on
+    the device."""
     src = pinned or {}
     g = lambda k: _hp(src[k]) if k in src else (_hp(getattr(t, k)) if k != "index_grid16" else None)
+    if derive:
+        return XSTablesC(g("nuclide_grid"), None, None, g("num_nucs"), g("mats"), g("concs"),
+                         t.n_isotopes, t.n_gridpoints, t.max_num_nucs, 0, t.n_union, None,
+                         None, None, 0, 0)
     idx = None if ("index_grid16" in src and "index_grid" not in src) else g("index_grid")
     return XSTablesC(g("nuclide_grid"), g("unionized"), idx, g("num_nucs"), g("mats"),
                      g("concs"), t.n_isotopes, t.n_gridpoints, t.max_num_nucs, 0, t.n_union,
                      None, g("index_grid16"), _hp(src.get("brackets")), 0, 0)
+
+
+def omprt_xs_derive_tmp_bytes(n_isotopes, n_gridpoints):
+    b = _u64()
+    _check(load().omprt_xs_derive_tmp_bytes(n_isotopes, n_gridpoints, C.byref(b)))
+    return b.value
+
+
+def omprt_xs_derive(nuclide_grid, n_isotopes, n_gridpoints, unionized, index_grid16, tmp,
+                    stream=None):
+    """Device tensors: nuclide_grid f64 [n*6], unionized f64 [n], index_grid16 u16/i16
+    [n*n_isotopes], tmp u8 [>= omprt_xs_derive_tmp_bytes]."""
+    return _check(load().omprt_xs_derive(_p(nuclide_grid), n_isotopes, n_gridpoints,
+                                         _p(unionized), _p(index_grid16), _p(tmp),
+                                         tmp.numel() * tmp.element_size(), _stream(stream)))
 
 
 def omprt_xs_run_host_steps(host_struct, seed, first, count, steps, threads=256, flags=0,

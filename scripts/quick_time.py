@@ -24,6 +24,8 @@ def main(which):
         torch.cuda.synchronize()
         out = []
         for _ in range(reps):
+            torch.cuda.synchronize()
+            omprt.omprt_l2_reset_persisting()
             scrub.fill_(1.0)
             a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
             a.record(s)
@@ -61,6 +63,25 @@ def main(which):
         v = torch.empty(n, dtype=torch.uint64, device=dev)
         res["rs_rt_1M"] = {"ms": t(lambda: omprt.omprt_rs_lookup(rd, 1070, 0, n, v, None, 0, 128, A), 3)}
         res["rs_twin_1M"] = {"ms": t(lambda: omprt.omprt_cuda_rs_lookup(rd, 1070, 0, n, v, None, 0, 128, 0), 3)}
+    if "xs" in which:
+        tabs = gen.XSTables(**gen.XS_SMALL)
+        d = omprt.XSDeviceTables(tabs, dev, accel=True)
+        n = 17_000_000
+        ver = torch.empty(n, dtype=torch.uint64, device=dev)
+        ck = torch.zeros(1, dtype=torch.uint64, device=dev)
+        F, FU = omprt.OMPRT_XS_FLAT, omprt.OMPRT_FUSED_REDUCTION
+        NW = omprt.OMPRT_XS_NO_L2_PERSIST
+        for name, fn, fl in [("rt_flat", omprt.omprt_xs_lookup, F),
+                             ("rt_flat_fused", omprt.omprt_xs_lookup, F | FU),
+                             ("twin_flat_fused", omprt.omprt_cuda_xs_lookup, F | FU),
+                             ("rt_flat_fused_nowin", omprt.omprt_xs_lookup, F | FU | NW)]:
+            res[f"xs_{name}"] = {"ms": t(lambda: fn(d, 1070, 0, n, ver, ck, 0, 256, fl), 5)}
+        ng = torch.from_numpy(tabs.nuclide_grid.reshape(-1)).to(dev)
+        U = torch.empty(tabs.n_union, dtype=torch.float64, device=dev)
+        i16 = torch.empty(tabs.n_union * tabs.n_isotopes, dtype=torch.int16, device=dev)
+        tmp = torch.empty(omprt.omprt_xs_derive_tmp_bytes(68, 11303), dtype=torch.uint8,
+                          device=dev)
+        res["xs_derive"] = {"ms": t(lambda: omprt.omprt_xs_derive(ng, 68, 11303, U, i16, tmp), 5)}
     print(json.dumps(res))
 
 

@@ -219,3 +219,59 @@ def test_end_to_end_pipelined_steps_compact_host_layout(rt, xs_small):
     assert cks == [ref] * 3
     idx16 = xs_small.index_grid.size * 2
     assert h2d == xs_small.nbytes() - xs_small.index_grid.nbytes + idx16 and d2h == 8
+
+
+def _derive(rt, grid, n_iso, n_gp):
+    n = n_iso * n_gp
+    g = torch.from_numpy(np.ascontiguousarray(grid.reshape(-1))).to(DEV)
+    U = torch.full((n,), float("nan"), dtype=torch.float64, device=DEV)
+    idx = torch.zeros(n * n_iso, dtype=torch.int16, device=DEV)
+    tmp = torch.empty(rt.omprt_xs_derive_tmp_bytes(n_iso, n_gp), dtype=torch.uint8, device=DEV)
+    rt.omprt_xs_derive(g, n_iso, n_gp, U, idx, tmp)
+    torch.cuda.synchronize()
+    return U.cpu().numpy(), idx.cpu().numpy().view(np.uint16).reshape(n, n_iso)
+
+
+def _definition(grid, n_iso, n_gp):
+    """App. A.1 written out: the sorted union of all energies, and per unionized energy and
+    nuclide the clipped upper-bound bracket index."""
+    E = grid.reshape(n_iso, n_gp, 6)[:, :, 0]
+    U = np.sort(E.reshape(-1), kind="stable")
+    idx = np.stack([np.clip(np.searchsorted(E[q], U, side="right") - 1, 0, n_gp - 2)
+                    for q in range(n_iso)], axis=1)
+    return U, idx
+
+
+@pytest.mark.parametrize("n_iso,n_gp", [(68, 500), (68, 11303), (3, 2), (7, 1500)])
+def test_derive_unionized_and_index(rt, n_iso, n_gp):
+    t = gen.XSTables(n_isotopes=n_iso, n_gridpoints=n_gp)
+    U, idx = _derive(rt, t.nuclide_grid, n_iso, n_gp)
+    assert (U.view(np.uint64) == t.unionized.view(np.uint64)).all()
+    assert (idx.astype(np.int64) == t.index_grid).all()
+
+
+def test_derive_with_ties(rt):
+    """Energies quantized to 1/64 (ties within and across nuclides): `<=` counts every
+    equal energy, as searchsorted(side='right') does."""
+    n_iso, n_gp = 9, 300
+    t = gen.XSTables(n_isotopes=n_iso, n_gridpoints=n_gp)
+    g = t.nuclide_grid.reshape(n_iso, n_gp, 6).copy()
+    g[:, :, 0] = np.sort(np.floor(g[:, :, 0] * 64.0) / 64.0, axis=1)
+    U, idx = _derive(rt, g, n_iso, n_gp)
+    Ur, ir = _definition(g, n_iso, n_gp)
+    assert (U == Ur).all() and (idx.astype(np.int64) == ir).all()
+
+
+def test_end_to_end_derived_tables(rt, xs_small):
+    """Only the raw data crosses PCIe (nuclide grid + materials); the unionized and index
+    grids are derived on the device every step; checksums equal the oracle's."""
+    pinned = {k: torch.from_numpy(getattr(xs_small, k)).pin_memory()
+              for k in ("nuclide_grid", "num_nucs", "mats", "concs")}
+    hs = rt.xs_host_struct(xs_small, pinned, derive=True)
+    n = 150_000
+    ref = int(oracle.xs_lookup(xs_small, 11, n).sum())
+    for flags in (rt.OMPRT_XS_FLAT, 0):
+        cks, h2d, d2h = rt.omprt_xs_run_host_steps(hs, SEED, 11, n, 3, flags=flags)
+        assert cks == [ref] * 3
+        assert h2d == (xs_small.nuclide_grid.nbytes + xs_small.num_nucs.nbytes +
+                       xs_small.mats.nbytes + xs_small.concs.nbytes) and d2h == 8

@@ -101,11 +101,22 @@ extern "C" {
  * lookup starts its next one instead of waiting for the warp's longest lookup.  Identical
  * results.  Not combined with OMPRT_ASSUME_OVERSUB or OMPRT_DEBUG_BUILD. */
 #define OMPRT_XS_FLAT (1u << 15)
+/* The same flag for omprt_rs_lookup / omprt_cuda_rs_lookup: persistent grid, one nuclide
+ * of the material per flattened step (identical results to the nested form). */
+#define OMPRT_FLAT OMPRT_XS_FLAT
 /* With OMPRT_XS_FLAT: launch WITHOUT the L2 access-policy window that otherwise marks the
- * bracket records (t.brackets) persisting in the L2 set-aside reserved by omprt_init
- * (cudaLimitPersistingL2CacheSize = the device maximum).  Persisting lines outlive the
- * launch; omprt_l2_reset_persisting() returns them to normal. */
+ * bracket records (t.brackets) persisting in the L2 set-aside granted by omprt_l2_set_aside
+ * (cudaLimitPersistingL2CacheSize; without a set-aside there is no window either).
+ * Persisting lines outlive the launch; omprt_l2_reset_persisting() returns them to
+ * normal. */
 #define OMPRT_XS_NO_L2_PERSIST (1u << 16)
+/* schedule(dynamic, C) instead of Fig. 5's static assignment (reading R-D1): team t runs
+ * the contiguous block [t*B, min(n, (t+1)*B)), B = ceil(n/teams), and its threads take
+ * chunks of that block from a team-shared counter as they finish the previous one.  Same
+ * per-iteration results; which thread runs an iteration is not deterministic.
+ * omprt_spmd_axpy_sum_chunked (C = chunk) and, with OMPRT_FLAT, omprt_xs_lookup /
+ * omprt_rs_lookup and their twins (C fixed per kernel). */
+#define OMPRT_SCHED_DYNAMIC (1u << 17)
 
 /* ---- runtime lifecycle ------------------------------------------------------------- */
 typedef struct {
@@ -115,15 +126,19 @@ typedef struct {
 } omprt_options;
 
 /* Create the per-device workspace; reads OMPRT_DEBUG.  opt may be NULL (defaults).
- * Idempotent per device.  Also reserves the device's maximum L2 set-aside for persisting
- * accesses (cudaLimitPersistingL2CacheSize), used by the OMPRT_XS_FLAT launches' access-
- * policy window; other accesses use the set-aside while no persisting line holds it. */
+ * Idempotent per device.  Reserves NO L2 set-aside for persisting accesses (see
+ * omprt_l2_set_aside: a reserved set-aside slows streaming kernels ~3x on B200). */
 int omprt_init(int device, const omprt_options *opt);
 int omprt_fini(int device);
 /* Return every persisting L2 line of the current device's context to normal
  * (cudaCtxResetPersistingL2Cache; takes effect immediately, not stream-ordered: call it
  * with no launch in flight, e.g. before an L2 flush between timed steps). */
 int omprt_l2_reset_persisting(void);
+/* Resize the current device's L2 set-aside for persisting accesses to min(bytes, device
+ * maximum) (synchronizes the device and resets persisting lines first); 0 removes it, and
+ * the OMPRT_XS_FLAT launches then run without their access-policy window.  granted
+ * (nullable) receives the size in effect. */
+int omprt_l2_set_aside(uint64_t bytes, uint64_t *granted);
 /* Device-side error recorded since init (0 = none); info (nullable) gets 4 ints
  * {team, thread, line, extra}. */
 int omprt_device_status(int device, int *code, int *info);

@@ -71,6 +71,8 @@ def _declare(L):
         "oracle_distribute_simulate": (None, [C.c_int64, C.c_int32, _i32p, _i32p]),
         "oracle_static_chunk_owner_closed": (C.c_int, [C.c_int64, C.c_int64, C.c_int64, C.c_int64, C.c_int64, _i32p, _i32p]),
         "oracle_chunk_simulate": (None, [C.c_int64, C.c_int64, C.c_int32, C.c_int32, C.c_int, _i32p, _i32p]),
+        "oracle_dynamic_team_closed": (C.c_int, [C.c_int64, C.c_int64, C.c_int64]),
+        "oracle_dynamic_simulate": (None, [C.c_int64, C.c_int64, C.c_int32, C.c_int32, C.c_uint64, _i32p, _i32p]),
         "oracle_axpy": (None, [C.c_int64, C.c_double, _f64p, _f64p, _f64p]),
         "oracle_sum_f64": (C.c_double, [_f64p, C.c_int64, C.c_double]),
         "oracle_sum_f64_ld": (C.c_longdouble, [_f64p, C.c_int64, C.c_double]),
@@ -146,6 +148,19 @@ def chunk_simulate(n, chunk, teams, threads, assume_oversub=False):
     count = np.empty(n, np.int32)
     lib().oracle_chunk_simulate(n, chunk, teams, threads, int(assume_oversub), _p(owner, _i32p),
                                 _p(count, _i32p))
+    return owner, count
+
+
+def dynamic_team_closed(iv, n, teams):
+    r = lib().oracle_dynamic_team_closed(iv, n, teams)
+    return None if r < 0 else r
+
+
+def dynamic_simulate(n, chunk, teams, threads, order_seed=0):
+    owner = np.empty(n, np.int32)
+    count = np.empty(n, np.int32)
+    lib().oracle_dynamic_simulate(n, chunk, teams, threads, order_seed, _p(owner, _i32p),
+                                  _p(count, _i32p))
     return owner, count
 
 

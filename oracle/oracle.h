@@ -56,6 +56,11 @@ int oracle_static_chunk_owner_closed(int64_t iv, int64_t n, int64_t chunk, int64
                                      int64_t threads, int32_t *team, int32_t *thread);
 void oracle_chunk_simulate(int64_t n, int64_t chunk, int32_t teams, int32_t threads,
                            int assume_oversub, int32_t *owner, int32_t *count);
+/* Reading R-D1: schedule(dynamic, C) under a blocked distribute (team of iteration iv, and
+ * a literal execution for one seeded request order). */
+int oracle_dynamic_team_closed(int64_t iv, int64_t n, int64_t teams);
+void oracle_dynamic_simulate(int64_t n, int64_t chunk, int32_t teams, int32_t threads,
+                             uint64_t order_seed, int32_t *owner, int32_t *count);
 
 /* ---- C1: SPMD axpy + fp64 sum reduction (BASELINE configs[0]) -------------------------- */
 /* a[i] = fma(x, b[i], c[i]) (SURVEY Q12 reading: one rounding, explicit). */

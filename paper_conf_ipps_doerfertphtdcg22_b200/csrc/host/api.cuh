@@ -36,17 +36,10 @@ extern "C" int omprt_init(int device, const omprt_options* opt) {
   omprt::DeviceEnv env_dev{w.pool, o.pool_bytes_per_team, o.pool_teams, w.err_dev,
                            w.err_dev + 1, w.debug_bits, 0u};
   OMPRT_CUDA_TRY(cudaMemcpyToSymbol(omprt_env, &env_dev, sizeof env_dev));
-  // the L2 set-aside that access-policy windows of hot read-only tables may use
-  // (OMPRT_XS_FLAT); normal accesses still use it while no persisting line claims it
-  int max_persist = 0;
-  if (cudaDeviceGetAttribute(&max_persist, cudaDevAttrMaxPersistingL2CacheSize, device) ==
-          cudaSuccess &&
-      max_persist > 0 &&
-      cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, (size_t)max_persist) == cudaSuccess) {
-    size_t got = 0;
-    if (cudaDeviceGetLimit(&got, cudaLimitPersistingL2CacheSize) == cudaSuccess)
-      w.l2_persist_bytes = got;
-  }
+  // No L2 set-aside for persisting accesses by default: a reserved set-aside slows every
+  // streaming kernel (SU(3) 32^4: 0.24 -> 0.71 ms with the 82.9 MB maximum reserved,
+  // profiles/l2_probe_x07.txt).  omprt_l2_set_aside opts in (the XS flat launches' window).
+  w.l2_persist_bytes = 0;
   cudaGetLastError();  // a device without the set-aside just runs without windows
   OMPRT_CUDA_TRY(cudaDeviceSynchronize());
   w.inited = true;
@@ -83,6 +76,23 @@ extern "C" int omprt_fini(int device) {
   cudaMemcpyToSymbol(omprt_env, &zero, sizeof zero);
   w = Workspace{};
   cudaSetDevice(prev);
+  return OMPRT_OK;
+}
+
+extern "C" int omprt_l2_set_aside(uint64_t bytes, uint64_t* granted) {
+  Workspace* w;
+  if (int r = current_ws(&w)) return r;
+  int dev = 0, max_persist = 0;
+  OMPRT_CUDA_TRY(cudaGetDevice(&dev));
+  OMPRT_CUDA_TRY(cudaDeviceGetAttribute(&max_persist, cudaDevAttrMaxPersistingL2CacheSize, dev));
+  const size_t want = std::min<uint64_t>(bytes, (uint64_t)std::max(max_persist, 0));
+  OMPRT_CUDA_TRY(cudaDeviceSynchronize());
+  OMPRT_CUDA_TRY(cudaCtxResetPersistingL2Cache());
+  OMPRT_CUDA_TRY(cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, want));
+  size_t got = 0;
+  OMPRT_CUDA_TRY(cudaDeviceGetLimit(&got, cudaLimitPersistingL2CacheSize));
+  w->l2_persist_bytes = got;
+  if (granted) *granted = got;
   return OMPRT_OK;
 }
 

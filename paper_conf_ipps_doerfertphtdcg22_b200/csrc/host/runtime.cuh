@@ -68,7 +68,7 @@ struct Workspace {
   // flattened e2e steps: per-lookup verification scratch, summed by K11 (u64 entries)
   uint64_t* e2e_ver = nullptr;
   size_t e2e_ver_n = 0;
-  // L2 set-aside for persisting accesses (cudaLimitPersistingL2CacheSize), granted at init
+  // L2 set-aside for persisting accesses (cudaLimitPersistingL2CacheSize), granted by omprt_l2_set_aside
   size_t l2_persist_bytes = 0;
 };
 constexpr int kMaxE2ESteps = 1024;

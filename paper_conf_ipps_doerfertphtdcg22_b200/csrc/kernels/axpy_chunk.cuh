@@ -132,6 +132,91 @@ __global__ void __launch_bounds__(1024)
   }
 }
 
+// schedule(dynamic, C) (OMPRT_SCHED_DYNAMIC, reading R-D1): team blocks, chunks from a
+// team-shared counter.  The per-thread sum order depends on which chunks a thread got, so
+// the fp64 sum is compared with a tolerance; a[] is bit-exact.
+template <class Tr, bool Rec>
+__global__ void __launch_bounds__(1024)
+    omprt_axpy_dyn_rt(typename Tr::Idx n, typename Tr::Idx chunk, double x,
+                      const double* __restrict__ b, const double* __restrict__ c,
+                      double* __restrict__ a, double* sum_inout, double* partials,
+                      unsigned* ticket, int32_t* owner, int32_t* count) {
+  using Idx = typename Tr::Idx;
+  Team<Tr> team = init<Tr>();
+  double acc = 0.0;
+  distribute_parallel_for_dynamic_chunks(team, n, chunk, [&](Idx lo, Idx cnt) {
+    acc += axpy_chunk_body<false>(lo, cnt, x, b, c, a);
+    if constexpr (Rec) {
+      for (Idx i = lo; i < lo + cnt; ++i) {
+        owner[i] = get_team_num(team) * get_num_threads(team) + get_thread_num(team);
+        atomicAdd(count + i, 1);
+      }
+    }
+  });
+  league_reduce(team, team_reduce_to_main(team, acc, Plus{}), Plus{}, sum_inout, partials,
+                ticket);
+}
+
+template <bool Rec>
+__global__ void __launch_bounds__(1024)
+    cuda_axpy_dyn_twin(int32_t n, int32_t chunk, double x, const double* __restrict__ b,
+                       const double* __restrict__ c, double* __restrict__ a, double* sum_inout,
+                       double* partials, unsigned* ticket, int32_t* owner, int32_t* count) {
+  __shared__ unsigned next;
+  __shared__ double warp_sum[32];
+  __shared__ unsigned is_last;
+  const int32_t per = (n + (int32_t)gridDim.x - 1) / (int32_t)gridDim.x;
+  const int32_t blo = min((int32_t)blockIdx.x * per, n), bhi = min(blo + per, n);
+  if (threadIdx.x == 0) next = blockDim.x;
+  __syncthreads();
+  double acc = 0.0;
+  for (int32_t k = threadIdx.x;; k = (int32_t)atomicAdd(&next, 1u)) {
+    const int32_t lo = blo + k * chunk;
+    if (lo >= bhi) break;
+    const int32_t cnt = min(chunk, bhi - lo);
+    acc += axpy_chunk_body<false>(lo, cnt, x, b, c, a);
+    if constexpr (Rec) {
+      for (int32_t i = lo; i < lo + cnt; ++i) {
+        owner[i] = (int32_t)(blockIdx.x * blockDim.x + threadIdx.x);
+        atomicAdd(count + i, 1);
+      }
+    }
+  }
+  for (int off = 16; off > 0; off >>= 1) acc += __shfl_xor_sync(0xffffffffu, acc, off);
+  const unsigned lane = threadIdx.x & 31u, wid = threadIdx.x >> 5, nw = (blockDim.x + 31) >> 5;
+  if (lane == 0) warp_sum[wid] = acc;
+  __syncthreads();
+  double blk = 0.0;
+  if (wid == 0) {
+    blk = lane < nw ? warp_sum[lane] : 0.0;
+    for (int off = 16; off > 0; off >>= 1) blk += __shfl_xor_sync(0xffffffffu, blk, off);
+  }
+  if (threadIdx.x == 0) {
+    partials[blockIdx.x] = blk;
+    __threadfence();
+    is_last = (atomicAdd(ticket, 1u) == gridDim.x - 1) ? 1u : 0u;
+  }
+  __syncthreads();
+  if (is_last) {
+    __threadfence();
+    double t = 0.0;
+    for (unsigned k = threadIdx.x; k < gridDim.x; k += blockDim.x) t += __ldcg(partials + k);
+    for (int off = 16; off > 0; off >>= 1) t += __shfl_xor_sync(0xffffffffu, t, off);
+    if (lane == 0) warp_sum[wid] = t;
+    __syncthreads();
+    if (wid == 0) {
+      double tt = lane < nw ? warp_sum[lane] : 0.0;
+      for (int off = 16; off > 0; off >>= 1) tt += __shfl_xor_sync(0xffffffffu, tt, off);
+      if (threadIdx.x == 0) {
+        *sum_inout = *sum_inout + tt;
+        *ticket = 0u;
+      }
+    }
+  }
+}
+
+OMPRT_REGISTER_KERNEL(omprt_axpy_dyn_rt, omprt_axpy_dyn_rt<AxpyTraits, false>)
+OMPRT_REGISTER_KERNEL(cuda_axpy_dyn_twin, cuda_axpy_dyn_twin<false>)
 OMPRT_REGISTER_KERNEL(omprt_axpy_chunk_rt, omprt_axpy_chunk_rt<AxpyTraits, true, false>)
 OMPRT_REGISTER_KERNEL(cuda_axpy_chunk_twin, cuda_axpy_chunk_twin<int32_t, true, false>)
 
@@ -161,6 +246,12 @@ extern "C" int omprt_spmd_axpy_sum_chunked(int64_t n, int64_t chunk, double x, c
   double* p = (double*)w->partials;
   unsigned* t = w->tickets + 0;
   const int32_t nn = (int32_t)n, cc = (int32_t)chunk;
+  if (flags & OMPRT_SCHED_DYNAMIC) {
+    OMPRT_CHECK_ARG(!assume, "OMPRT_SCHED_DYNAMIC: no oversubscription assumption");
+    if (rec) omprt_axpy_dyn_rt<AxpyTraits, true><<<teams, threads, 0, s>>>(nn, cc, x, b, c, a, sum_inout, p, t, owner, count);
+    else omprt_axpy_dyn_rt<AxpyTraits, false><<<teams, threads, 0, s>>>(nn, cc, x, b, c, a, sum_inout, p, t, owner, count);
+    return check_launch("omprt_axpy_dyn_rt");
+  }
 #define OMPRT_AXC(TR, V, R)                                                                  \
   omprt_axpy_chunk_rt<TR, V, R><<<teams, threads, 0, s>>>(nn, cc, x, b, c, a, sum_inout, p, t, \
                                                          owner, count)
@@ -197,6 +288,11 @@ extern "C" int omprt_cuda_axpy_sum_chunked(int64_t n, int64_t chunk, double x, c
   double* p = (double*)w->partials;
   unsigned* t = w->tickets + 0;
   const int32_t nn = (int32_t)n, cc = (int32_t)chunk;
+  if (flags & OMPRT_SCHED_DYNAMIC) {
+    if (rec) cuda_axpy_dyn_twin<true><<<teams, threads, 0, s>>>(nn, cc, x, b, c, a, sum_inout, p, t, owner, count);
+    else cuda_axpy_dyn_twin<false><<<teams, threads, 0, s>>>(nn, cc, x, b, c, a, sum_inout, p, t, owner, count);
+    return check_launch("cuda_axpy_dyn_twin");
+  }
   if (v4) {
     if (rec) cuda_axpy_chunk_twin<int32_t, true, true><<<teams, threads, 0, s>>>(nn, cc, x, b, c, a, sum_inout, p, t, owner, count);
     else cuda_axpy_chunk_twin<int32_t, true, false><<<teams, threads, 0, s>>>(nn, cc, x, b, c, a, sum_inout, p, t, owner, count);

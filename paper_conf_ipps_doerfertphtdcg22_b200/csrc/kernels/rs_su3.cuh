@@ -40,6 +40,93 @@ __global__ void __launch_bounds__(kRSThreads, kRSMinBlocks)
   verification[i] = rs_lookup_one<Macro>(t, seed, first + i, macro + (int64_t)i * 4);
 }
 
+// Flattened execution (OMPRT_FLAT): a persistent grid of the device's resident teams, each
+// thread running its Fig. 5 lookups through omprt::distribute_parallel_for_flat with one
+// nuclide per step (RSFlatLookup), so lanes are not held by the warp's longest material.
+template <class Tr, bool Macro>
+__global__ void __launch_bounds__(kRSThreads, kRSMinBlocks)
+    omprt_rs_flat_rt(const __grid_constant__ RSTables t, uint64_t seed, int64_t first,
+                     typename Tr::Idx count, uint64_t* __restrict__ verification,
+                     double* __restrict__ macro) {
+  Team<Tr> team = init<Tr>();
+  RSFlatLookup<Macro> lookup(t, seed, first, verification, macro);
+  distribute_parallel_for_flat<Tr, FlatSync::Lockstep>(team, count, lookup);
+}
+
+// Bare CUDA twin: the same flattened loop written by hand around the same body.
+template <bool Macro>
+__global__ void __launch_bounds__(kRSThreads, kRSMinBlocks)
+    cuda_rs_flat_twin(const __grid_constant__ RSTables t, uint64_t seed, int64_t first,
+                      int32_t count, uint64_t* __restrict__ verification,
+                      double* __restrict__ macro) {
+  RSFlatLookup<Macro> lookup(t, seed, first, verification, macro);
+  const int32_t stride = (int32_t)gridDim.x * (int32_t)blockDim.x;
+  int32_t i = (int32_t)blockIdx.x * (int32_t)blockDim.x + (int32_t)threadIdx.x;
+  bool live = i < count;
+  if (live) lookup.begin(i, stride);
+  while (__any_sync(0xffffffffu, live)) {  // lanes step together (warp vote per trip)
+    if (live && !lookup.step()) {
+      lookup.end(i);
+      i += stride;
+      live = i < count;
+      if (live) lookup.next(i);
+    }
+  }
+}
+
+// schedule(dynamic, kRSDynChunk) + flattened (OMPRT_FLAT | OMPRT_SCHED_DYNAMIC): the same
+// body; a thread that drew cheap lookups (few nuclides) requests more of its team's block
+// instead of the static schedule's fixed share (a thread's fuel lookups -- 321 nuclides,
+// 14 % of lookups -- vary by +-25 % between threads, and the warp waits for its slowest).
+constexpr int kRSDynChunk = 1;
+
+template <class Tr, bool Macro>
+__global__ void __launch_bounds__(kRSThreads, kRSMinBlocks)
+    omprt_rs_dflat_rt(const __grid_constant__ RSTables t, uint64_t seed, int64_t first,
+                      typename Tr::Idx count, uint64_t* __restrict__ verification,
+                      double* __restrict__ macro) {
+  Team<Tr> team = init<Tr>();
+  RSFlatLookup<Macro> lookup(t, seed, first, verification, macro);
+  distribute_parallel_for_dynamic_flat<Tr, FlatSync::Lockstep>(team, count,
+                                                               (typename Tr::Idx)kRSDynChunk,
+                                                               lookup);
+}
+
+template <bool Macro>
+__global__ void __launch_bounds__(kRSThreads, kRSMinBlocks)
+    cuda_rs_dflat_twin(const __grid_constant__ RSTables t, uint64_t seed, int64_t first,
+                       int32_t count, uint64_t* __restrict__ verification,
+                       double* __restrict__ macro) {
+  __shared__ unsigned next;
+  const int32_t per = (count + (int32_t)gridDim.x - 1) / (int32_t)gridDim.x;
+  const int32_t lo = min((int32_t)blockIdx.x * per, count);
+  const int32_t hi = min(lo + per, count);
+  if (threadIdx.x == 0) next = blockDim.x;
+  __syncthreads();
+  RSFlatLookup<Macro> lookup(t, seed, first, verification, macro);
+  int32_t i = lo + (int32_t)threadIdx.x * kRSDynChunk;
+  int32_t end = min(i + kRSDynChunk, hi);
+  bool live = i < hi;
+  if (live) lookup.begin(i, 1);
+  while (__any_sync(0xffffffffu, live)) {
+    if (live && !lookup.step()) {
+      lookup.end(i);
+      if (++i < end) {
+        lookup.next(i);
+      } else {
+        i = lo + (int32_t)atomicAdd(&next, 1u) * kRSDynChunk;
+        end = min(i + kRSDynChunk, hi);
+        live = i < hi;
+        if (live) lookup.begin(i, 1);
+      }
+    }
+  }
+}
+
+OMPRT_REGISTER_KERNEL(omprt_rs_dflat_rt, omprt_rs_dflat_rt<RSTraits, false>)
+OMPRT_REGISTER_KERNEL(cuda_rs_dflat_twin, cuda_rs_dflat_twin<false>)
+OMPRT_REGISTER_KERNEL(omprt_rs_flat_rt, omprt_rs_flat_rt<RSTraits, false>)
+OMPRT_REGISTER_KERNEL(cuda_rs_flat_twin, cuda_rs_flat_twin<false>)
 OMPRT_REGISTER_KERNEL(omprt_rs_rt, omprt_rs_rt<RSTraits, false>)
 OMPRT_REGISTER_KERNEL(omprt_rs_rt_assume, omprt_rs_rt<RSTraitsAssume, false>)
 OMPRT_REGISTER_KERNEL(cuda_rs_twin, cuda_rs_twin<false>)
@@ -47,6 +134,17 @@ OMPRT_REGISTER_KERNEL(cuda_rs_twin, cuda_rs_twin<false>)
 inline RSTables to_dev(const omprt_rs_tables& a) {
   return RSTables{a.poles, a.pole_l, a.windows, a.win_range, a.win_off, a.n_windows, a.k0rs,
                   a.num_nucs, a.mats, a.concs, a.n_nuclides, a.numL, a.max_num_nucs, 0};
+}
+
+// Persistent grid of the flattened kernels: teams = 0 -> every SM's resident teams.
+inline int32_t rs_flat_teams(int32_t teams) {
+  if (teams > 0) return teams;
+  int dev = 0, sms = 148, per_sm = kRSMinBlocks;
+  cudaGetDevice(&dev);
+  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, omprt_rs_flat_rt<RSTraits, false>,
+                                                kRSThreads, 0);
+  return sms * std::max(1, per_sm);
 }
 
 inline int rs_validate(const omprt_rs_tables& t, int64_t count, uint64_t* ver, int32_t& teams,
@@ -58,6 +156,11 @@ inline int rs_validate(const omprt_rs_tables& t, int64_t count, uint64_t* ver, i
                       t.k0rs && t.num_nucs && t.mats && t.concs,
                   "bad RSBench tables");
   OMPRT_CHECK_ARG(ver != nullptr || count == 0, "verification is required");
+  OMPRT_CHECK_ARG(!(flags & OMPRT_XS_FLAT) || !(flags & OMPRT_ASSUME_OVERSUB),
+                  "OMPRT_XS_FLAT runs a persistent grid (no oversubscription assumption)");
+  OMPRT_CHECK_ARG(!(flags & OMPRT_SCHED_DYNAMIC) || (flags & OMPRT_XS_FLAT),
+                  "OMPRT_SCHED_DYNAMIC is implemented for the flattened loop (OMPRT_FLAT)");
+  if (flags & OMPRT_XS_FLAT) teams = rs_flat_teams(teams);
   if (teams <= 0) teams = (int32_t)std::max<int64_t>(1, ceil_div(count, threads));
   OMPRT_CHECK_ARG(!(flags & OMPRT_ASSUME_OVERSUB) || count <= (int64_t)teams * threads,
                   "oversubscription assumption violated");
@@ -219,6 +322,17 @@ extern "C" int omprt_rs_lookup(omprt_rs_tables t, uint64_t seed, int64_t first, 
   cudaStream_t s = as_stream(stream);
   const RSTables d = to_dev(t);
   const int32_t n = (int32_t)count;
+  if ((flags & OMPRT_XS_FLAT) && (flags & OMPRT_SCHED_DYNAMIC)) {
+    if (macro) omprt_rs_dflat_rt<RSTraits, true><<<teams, threads, 0, s>>>(d, seed, first, n, verification, macro);
+    else omprt_rs_dflat_rt<RSTraits, false><<<teams, threads, 0, s>>>(d, seed, first, n, verification, nullptr);
+    return check_launch("omprt_rs_dflat_rt");
+  }
+  if (flags & OMPRT_XS_FLAT) {
+    const int32_t tm = rs_flat_teams(teams);
+    if (macro) omprt_rs_flat_rt<RSTraits, true><<<tm, threads, 0, s>>>(d, seed, first, n, verification, macro);
+    else omprt_rs_flat_rt<RSTraits, false><<<tm, threads, 0, s>>>(d, seed, first, n, verification, nullptr);
+    return check_launch("omprt_rs_flat_rt");
+  }
   if (flags & OMPRT_ASSUME_OVERSUB) {
     if (macro) omprt_rs_rt<RSTraitsAssume, true><<<teams, threads, 0, s>>>(d, seed, first, n, verification, macro);
     else omprt_rs_rt<RSTraitsAssume, false><<<teams, threads, 0, s>>>(d, seed, first, n, verification, nullptr);
@@ -235,13 +349,25 @@ extern "C" int omprt_cuda_rs_lookup(omprt_rs_tables t, uint64_t seed, int64_t fi
   using namespace omprt_kernels;
   Workspace* w;
   if (int r = current_ws(&w)) return r;
-  int32_t tm = 0;
-  if (int r = rs_validate(t, count, verification, tm, threads, 0)) return r;
-  (void)teams;
-  (void)flags;
+  const bool flat = flags & OMPRT_XS_FLAT;
+  int32_t tm = flat ? teams : 0;
+  if (int r = rs_validate(t, count, verification, tm, threads,
+                          flags & (OMPRT_XS_FLAT | OMPRT_SCHED_DYNAMIC)))
+    return r;
   if (count == 0) return OMPRT_OK;
   cudaStream_t s = as_stream(stream);
   const RSTables d = to_dev(t);
+  if (flat && (flags & OMPRT_SCHED_DYNAMIC)) {
+    if (macro) cuda_rs_dflat_twin<true><<<tm, threads, 0, s>>>(d, seed, first, (int32_t)count, verification, macro);
+    else cuda_rs_dflat_twin<false><<<tm, threads, 0, s>>>(d, seed, first, (int32_t)count, verification, nullptr);
+    return check_launch("cuda_rs_dflat_twin");
+  }
+  if (flat) {  // the same persistent geometry as the runtime-driven kernel
+    tm = rs_flat_teams(teams);
+    if (macro) cuda_rs_flat_twin<true><<<tm, threads, 0, s>>>(d, seed, first, (int32_t)count, verification, macro);
+    else cuda_rs_flat_twin<false><<<tm, threads, 0, s>>>(d, seed, first, (int32_t)count, verification, nullptr);
+    return check_launch("cuda_rs_flat_twin");
+  }
   if (macro) cuda_rs_twin<true><<<tm, threads, 0, s>>>(d, seed, first, (int32_t)count, verification, macro);
   else cuda_rs_twin<false><<<tm, threads, 0, s>>>(d, seed, first, (int32_t)count, verification, nullptr);
   return check_launch("cuda_rs_twin");

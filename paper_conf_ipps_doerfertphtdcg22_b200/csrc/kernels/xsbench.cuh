@@ -114,7 +114,10 @@ constexpr int kXSMatSmem = 12 * 48;  // entries: up to 48 nuclides per material 
 
 constexpr unsigned kXSMatsSite = 10, kXSConcsSite = 11;  // team_local sites
 
-template <class Tr, bool Fused, bool Smem>
+// OMPRT_SCHED_DYNAMIC: schedule(dynamic, kXSDynChunk) instead of Fig. 5 (reading R-D1)
+constexpr int kXSDynChunk = 8;
+
+template <class Tr, bool Fused, bool Smem, bool Dyn = false>
 __global__ void __launch_bounds__(kXSThreads, kXSMinBlocksFlat)
     omprt_xs_flat_rt(const __grid_constant__ XSTables t, uint64_t seed, int64_t first,
                      typename Tr::Idx count, uint64_t* __restrict__ verification,
@@ -138,14 +141,15 @@ __global__ void __launch_bounds__(kXSThreads, kXSMinBlocksFlat)
   using Lookup = XSFlatLookup<Fused, Smem>;
   if constexpr (Fused) *Lookup::flat_acc_slot() = 0ull;
   Lookup lookup(t, seed, first, verification, mats, concs);
-  distribute_parallel_for_flat(team, count, lookup);
+  if constexpr (Dyn) distribute_parallel_for_dynamic_flat(team, count, (Idx)kXSDynChunk, lookup);
+  else distribute_parallel_for_flat(team, count, lookup);
   if constexpr (Fused)
     league_reduce(team, team_reduce_to_main(team, *Lookup::flat_acc_slot(), Plus{}), Plus{},
                   checksum, partials, ticket);
 }
 
 // Bare CUDA twin: the same flattened loop written by hand around the same body.
-template <bool Fused, bool Smem>
+template <bool Fused, bool Smem, bool Dyn = false>
 __global__ void __launch_bounds__(kXSThreads, kXSMinBlocksFlat)
     cuda_xs_flat_twin(const __grid_constant__ XSTables t, uint64_t seed, int64_t first,
                       int32_t count, uint64_t* __restrict__ verification,
@@ -167,6 +171,29 @@ __global__ void __launch_bounds__(kXSThreads, kXSMinBlocksFlat)
   using Lookup = XSFlatLookup<Fused, Smem>;
   if constexpr (Fused) *Lookup::flat_acc_slot() = 0ull;
   Lookup lookup(t, seed, first, verification, mats, concs);
+  if constexpr (Dyn) {  // team block + team-shared chunk counter, by hand
+    __shared__ unsigned next;
+    const int32_t per = (count + (int32_t)gridDim.x - 1) / (int32_t)gridDim.x;
+    const int32_t lo = min((int32_t)blockIdx.x * per, count);
+    const int32_t hi = min(lo + per, count);
+    if (threadIdx.x == 0) next = blockDim.x;
+    __syncthreads();
+    int32_t i = lo + (int32_t)threadIdx.x * kXSDynChunk;
+    while (i < hi) {
+      const int32_t end = min(i + kXSDynChunk, hi);
+      lookup.begin(i, 1);
+      for (;;) {
+        if (lookup.step()) continue;
+        lookup.end(i);
+        if (++i >= end) break;
+        lookup.next(i);
+      }
+      i = lo + (int32_t)atomicAdd(&next, 1u) * kXSDynChunk;
+    }
+    if constexpr (Fused)
+      twin_u64_ticket_sum(*Lookup::flat_acc_slot(), checksum, partials, ticket);
+    return;
+  }
   const int32_t stride = (int32_t)gridDim.x * (int32_t)blockDim.x;
   int32_t i = (int32_t)blockIdx.x * (int32_t)blockDim.x + (int32_t)threadIdx.x;
   auto run = [&]() {
@@ -216,6 +243,8 @@ OMPRT_REGISTER_KERNEL(omprt_xs_flat_rt_gmem, omprt_xs_flat_rt<XSTraits, false, f
 OMPRT_REGISTER_KERNEL(cuda_xs_flat_twin, cuda_xs_flat_twin<false, true>)
 OMPRT_REGISTER_KERNEL(cuda_xs_flat_twin_fused, cuda_xs_flat_twin<true, true>)
 OMPRT_REGISTER_KERNEL(cuda_xs_flat_twin_gmem, cuda_xs_flat_twin<false, false>)
+OMPRT_REGISTER_KERNEL(omprt_xs_dflat_rt, omprt_xs_flat_rt<XSTraits, false, true, true>)
+OMPRT_REGISTER_KERNEL(cuda_xs_dflat_twin, cuda_xs_flat_twin<false, true, true>)
 OMPRT_REGISTER_KERNEL(cuda_xs_twin, cuda_xs_twin<false, false>)
 OMPRT_REGISTER_KERNEL(cuda_xs_twin_fused, cuda_xs_twin<true, false>)
 OMPRT_REGISTER_KERNEL(cuda_xs_twin_accel, cuda_xs_twin<false, true>)
@@ -231,7 +260,7 @@ inline XSTables to_dev(const omprt_xs_tables& a) {
 // Launch configuration of the flattened kernels: the persistent grid, plus (unless
 // OMPRT_XS_NO_L2_PERSIST) an L2 access-policy window that makes the bracket records -- the
 // bulk of the L2 sectors a lookup touches, 36.9 MB for the small problem -- persisting in
-// the set-aside granted at omprt_init, so the 16-bit index grid's misses cannot evict
+// the set-aside granted by omprt_l2_set_aside (none: no window), so the 16-bit index grid's misses cannot evict
 // them; hitRatio scales down when the table exceeds the set-aside.  (Persisting lines
 // outlive the launch: omprt_l2_reset_persisting returns them to normal.)
 struct FlatLaunch {
@@ -292,6 +321,8 @@ inline int xs_validate(const omprt_xs_tables& t, int64_t count, uint64_t* ver, u
   const bool fused = flags & OMPRT_FUSED_REDUCTION;
   OMPRT_CHECK_ARG(fused ? ck != nullptr : (ver != nullptr || count == 0),
                   fused ? "fused reduction needs checksum_inout" : "verification is required");
+  OMPRT_CHECK_ARG(!(flags & OMPRT_SCHED_DYNAMIC) || (flags & OMPRT_XS_FLAT),
+                  "OMPRT_SCHED_DYNAMIC is implemented for the flattened loop (OMPRT_XS_FLAT)");
   if (flags & OMPRT_XS_FLAT) {
     OMPRT_CHECK_ARG(accel, "OMPRT_XS_FLAT needs the B200 layouts (omprt_xs_build_accel)");
     OMPRT_CHECK_ARG(!(flags & (OMPRT_ASSUME_OVERSUB | OMPRT_DEBUG_BUILD)),
@@ -388,12 +419,19 @@ extern "C" int omprt_xs_lookup(omprt_xs_tables t, uint64_t seed, int64_t first, 
     const bool smem = xs_mats_fit_smem(t);
     const FlatLaunch L = flat_launch(t, teams, threads, flags, w, s);
     cudaError_t e;
-#define OMPRT_XSF(F, S) \
-  e = cudaLaunchKernelEx(&L.cfg, omprt_xs_flat_rt<XSTraits, F, S>, d, seed, first, n, verification, ck, p, tk)
-    if (fused && smem) OMPRT_XSF(true, true);
-    else if (fused) OMPRT_XSF(true, false);
-    else if (smem) OMPRT_XSF(false, true);
-    else OMPRT_XSF(false, false);
+#define OMPRT_XSF(F, S, D) \
+  e = cudaLaunchKernelEx(&L.cfg, omprt_xs_flat_rt<XSTraits, F, S, D>, d, seed, first, n, verification, ck, p, tk)
+    if (flags & OMPRT_SCHED_DYNAMIC) {
+      if (fused && smem) OMPRT_XSF(true, true, true);
+      else if (fused) OMPRT_XSF(true, false, true);
+      else if (smem) OMPRT_XSF(false, true, true);
+      else OMPRT_XSF(false, false, true);
+    } else {
+      if (fused && smem) OMPRT_XSF(true, true, false);
+      else if (fused) OMPRT_XSF(true, false, false);
+      else if (smem) OMPRT_XSF(false, true, false);
+      else OMPRT_XSF(false, false, false);
+    }
 #undef OMPRT_XSF
     (void)e;
     return check_launch("omprt_xs_flat_rt");
@@ -445,10 +483,17 @@ extern "C" int omprt_cuda_xs_lookup(omprt_xs_tables t, uint64_t seed, int64_t fi
     const FlatLaunch L = flat_launch(t, tm, threads, flags, w, s);
     unsigned long long* nul = nullptr;
     unsigned* nult = nullptr;
-    if (fused && smem) cudaLaunchKernelEx(&L.cfg, cuda_xs_flat_twin<true, true>, d, seed, first, n, verification, ck, p, tk);
-    else if (fused) cudaLaunchKernelEx(&L.cfg, cuda_xs_flat_twin<true, false>, d, seed, first, n, verification, ck, p, tk);
-    else if (smem) cudaLaunchKernelEx(&L.cfg, cuda_xs_flat_twin<false, true>, d, seed, first, n, verification, nul, nul, nult);
-    else cudaLaunchKernelEx(&L.cfg, cuda_xs_flat_twin<false, false>, d, seed, first, n, verification, nul, nul, nult);
+    if (flags & OMPRT_SCHED_DYNAMIC) {
+      if (fused && smem) cudaLaunchKernelEx(&L.cfg, cuda_xs_flat_twin<true, true, true>, d, seed, first, n, verification, ck, p, tk);
+      else if (fused) cudaLaunchKernelEx(&L.cfg, cuda_xs_flat_twin<true, false, true>, d, seed, first, n, verification, ck, p, tk);
+      else if (smem) cudaLaunchKernelEx(&L.cfg, cuda_xs_flat_twin<false, true, true>, d, seed, first, n, verification, nul, nul, nult);
+      else cudaLaunchKernelEx(&L.cfg, cuda_xs_flat_twin<false, false, true>, d, seed, first, n, verification, nul, nul, nult);
+    } else {
+      if (fused && smem) cudaLaunchKernelEx(&L.cfg, cuda_xs_flat_twin<true, true>, d, seed, first, n, verification, ck, p, tk);
+      else if (fused) cudaLaunchKernelEx(&L.cfg, cuda_xs_flat_twin<true, false>, d, seed, first, n, verification, ck, p, tk);
+      else if (smem) cudaLaunchKernelEx(&L.cfg, cuda_xs_flat_twin<false, true>, d, seed, first, n, verification, nul, nul, nult);
+      else cudaLaunchKernelEx(&L.cfg, cuda_xs_flat_twin<false, false>, d, seed, first, n, verification, nul, nul, nult);
+    }
     return check_launch("cuda_xs_flat_twin");
   }
   if (fused && accel) cuda_xs_twin<true, true><<<tm, threads, 0, s>>>(d, seed, first, n, verification, ck, p, tk);

@@ -37,11 +37,13 @@ OMPRT_DEGLOBALIZE = 1 << 12
 OMPRT_TMA_STAGED = 1 << 13
 OMPRT_WARP_STAGED = 1 << 14
 OMPRT_XS_FLAT = 1 << 15
+OMPRT_FLAT = OMPRT_XS_FLAT  # omprt_rs_lookup: flattened nuclide loop, persistent grid
+OMPRT_SCHED_DYNAMIC = 1 << 17  # schedule(dynamic, C): team blocks, team-shared chunk counter
 OMPRT_XS_NO_L2_PERSIST = 1 << 16
 
 # Every symbol include/omprt.h declares (checked by tests/test_abi.py).
 EXPORTS = [
-    "omprt_init", "omprt_fini", "omprt_l2_reset_persisting", "omprt_device_status", "omprt_last_error", "omprt_static_owner",
+    "omprt_init", "omprt_fini", "omprt_l2_reset_persisting", "omprt_l2_set_aside", "omprt_device_status", "omprt_last_error", "omprt_static_owner",
     "omprt_spmd_axpy_sum", "omprt_cuda_axpy_sum", "omprt_spmd_axpy_sum_chunked",
     "omprt_cuda_axpy_sum_chunked", "omprt_generic_team", "omprt_cuda_generic_team",
     "omprt_icv_probe", "omprt_xs_lookup", "omprt_cuda_xs_lookup", "omprt_u64_sum",
@@ -85,6 +87,7 @@ _SIGS = {
     "omprt_init": [C.c_int, C.POINTER(Options)],
     "omprt_fini": [C.c_int],
     "omprt_l2_reset_persisting": [],
+    "omprt_l2_set_aside": [C.c_uint64, C.POINTER(C.c_uint64)],
     "omprt_device_status": [C.c_int, C.POINTER(C.c_int), C.POINTER(C.c_int)],
     "omprt_last_error": [C.c_char_p, C.c_size_t],
     "omprt_static_owner": [_i64, _i64, _i32, _i32, C.POINTER(_i32), C.POINTER(_i32)],
@@ -187,6 +190,14 @@ def omprt_l2_reset_persisting():
     """Return persisting L2 lines (OMPRT_XS_FLAT's access-policy window) to normal; call
     with no launch in flight."""
     return _check(load().omprt_l2_reset_persisting())
+
+
+def omprt_l2_set_aside(nbytes):
+    """Resize the L2 set-aside for persisting accesses (0 removes it); returns the size
+    granted."""
+    got = C.c_uint64()
+    _check(load().omprt_l2_set_aside(nbytes, C.byref(got)))
+    return got.value
 
 
 def omprt_device_status(device=0):

@@ -1,0 +1,201 @@
+// Exploration harness (NOT part of libomprt.so): the flattened, lock-step, dynamic-schedule
+// RSBench kernel with Faddeeva evaluation variants x launch bounds.
+//   V0  the library body (rs_body.cuh faddeeva_w: 2 complex divisions / 4 fp64 divides)
+//   V1  asymptotic branch as one complex quotient: i Z (a (Z^2-d) + c (Z^2-b)) /
+//       ((Z^2-b)(Z^2-d)), one real reciprocal of |den|^2
+//   V2  V1 + the Abrarov terms through one real reciprocal each
+#include <cuda_runtime.h>
+#include <cstdint>
+#include "../../paper_conf_ipps_doerfertphtdcg22_b200/csrc/omprt/device/omprt.cuh"
+#include "../../paper_conf_ipps_doerfertphtdcg22_b200/csrc/kernels/rs_body.cuh"
+using namespace omprt_kernels;
+using namespace omprt;
+
+__device__ __forceinline__ cplx cdiv_rcp(cplx a, cplx b) {
+  const double r = 1.0 / (b.r * b.r + b.i * b.i);
+  return {(a.r * b.r + a.i * b.i) * r, (a.i * b.r - a.r * b.i) * r};
+}
+
+template <int V>
+__device__ __forceinline__ cplx faddeeva_v(cplx Z) {
+  if constexpr (V == 0) return faddeeva_w(Z);
+  const double absz = sqrt(__dadd_rn(__dmul_rn(Z.r, Z.r), __dmul_rn(Z.i, Z.i)));
+  if (absz < 6.0) {
+    if constexpr (V == 1) return faddeeva_w(Z);
+    constexpr double tau = 12.0;
+    constexpr double an[10] = {0.27584023329217705,   0.22457395522461585,
+                               0.1594149382739117,    0.0986657664154542,
+                               0.053244140787639394,  0.02505215000539365,
+                               0.01027746567053954,   0.0036761643328448498,
+                               0.001146493641242233,  0.0003117570150461973};
+    constexpr double npi2[10] = {9.869604401089358,  39.47841760435743,  88.82643960980423,
+                                 157.91367041742973, 246.74011002723395, 355.3057584392169,
+                                 483.61061565337855, 631.6546816697189,  799.437956488238,
+                                 986.9604401089358};
+    constexpr double prefactor = 81.24330003087691;
+    const cplx tZ = {tau * Z.r, tau * Z.i};
+    const double ex = rs_fast_exp(-tau * Z.i);
+    double sn, cs;
+    sincos(tau * Z.r, &sn, &cs);
+    const cplx e = {ex * cs, ex * sn};
+    cplx W = cdiv_rcp({e.i, 1.0 - e.r}, tZ);
+    const cplx Z2 = cmul(Z, Z);
+    cplx sum = {0.0, 0.0};
+#pragma unroll
+    for (int n = 0; n < 10; ++n) {
+      const double sgn = (n & 1) ? 1.0 : -1.0;
+      const cplx top = {sgn * e.r - 1.0, sgn * e.i};
+      const cplx bot = {npi2[n] - tau * tau * Z2.r, -tau * tau * Z2.i};
+      const cplx q = cdiv_rcp(top, bot);
+      sum.r += an[n] * q.r;
+      sum.i += an[n] * q.i;
+    }
+    const cplx zs = cmul(Z, sum);
+    W.r += -prefactor * zs.i;
+    W.i += prefactor * zs.r;
+    return W;
+  }
+  constexpr double a = 0.512424224754768462984202823134979415014943561548661637413182;
+  constexpr double b = 0.275255128608410950901357962647054304017026259671664935783653;
+  constexpr double c = 0.051765358792987823963876628425793170829107067780337219430904;
+  constexpr double d = 2.724744871391589049098642037352945695982973740328335064216346;
+  const cplx Z2 = cmul(Z, Z);
+  const cplx u = {Z2.r - b, Z2.i}, v = {Z2.r - d, Z2.i};
+  const cplx num = {a * v.r + c * u.r, a * v.i + c * u.i};
+  const cplx q = cdiv_rcp(num, cmul(u, v));
+  return cmul({-Z.i, Z.r}, q);
+}
+
+template <int V>
+__device__ __forceinline__ void nuclide_v(const RSTables& t, double E, double sqrtE, int nuc,
+                                          double& sigT, double& sigA, double& sigF) {
+  const int nw = __ldg(t.n_windows + nuc);
+  const double spacing = 1.0 / nw;
+  int w = (int)(E / spacing);
+  if (w >= nw) w = nw - 1;
+  cplx f[4];
+#pragma unroll
+  for (int l = 0; l < 4; ++l) {
+    double phi = __ldg(t.k0rs + nuc * 4 + l) * sqrtE;
+    if (l == 1) phi -= -atan(phi);
+    else if (l == 2) phi -= atan(3.0 * phi / (3.0 - phi * phi));
+    else if (l == 3) phi -= atan(phi * (15.0 - phi * phi) / (15.0 - 6.0 * phi * phi));
+    phi *= 2.0;
+    double sn, cs;
+    sincos(phi, &sn, &cs);
+    f[l] = {cs, -sn};
+  }
+  const int64_t wi = (int64_t)__ldg(t.win_off + nuc) + w;
+  const double2 TA = __ldg(reinterpret_cast<const double2*>(t.windows + wi * 4));
+  const double Fw = __ldg(t.windows + wi * 4 + 2);
+  const int2 rg = __ldg(reinterpret_cast<const int2*>(t.win_range + wi * 2));
+  sigT = E * TA.x;
+  sigA = E * TA.y;
+  sigF = E * Fw;
+  for (int p = rg.x; p < rg.y; ++p) {
+    const double2* P = reinterpret_cast<const double2*>(t.poles + (int64_t)p * 8);
+    const double2 EA = __ldg(P + 0), RT = __ldg(P + 1), RA = __ldg(P + 2), RF = __ldg(P + 3);
+    const int l = __ldg(t.pole_l + p);
+    const cplx Z = {(E - EA.x) * 0.5, (0.0 - EA.y) * 0.5};
+    const cplx W = faddeeva_v<V>(Z);
+    const cplx fl = l == 0 ? f[0] : l == 1 ? f[1] : l == 2 ? f[2] : f[3];
+    const cplx Wf = cmul(W, fl);
+    sigT += RT.x * Wf.r - RT.y * Wf.i;
+    sigA += RA.x * W.r - RA.y * W.i;
+    sigF += RF.x * W.r - RF.y * W.i;
+  }
+}
+
+template <int V>
+struct Body {
+  const RSTables& t;
+  uint64_t seed0;
+  int64_t first;
+  uint64_t* ver;
+  double* macro;
+  LcgMap J;
+  uint64_t s;
+  double E, sqrtE;
+  int32_t mat, nn, j;
+  double M0, M1, M2, M3;
+  __device__ Body(const RSTables& tt, uint64_t sd, int64_t f, uint64_t* v, double* m)
+      : t(tt), seed0(sd), first(f), ver(v), macro(m) {}
+  __device__ __forceinline__ void start() {
+    uint64_t seed = s;
+    E = lcg_double(seed);
+    mat = pick_mat(seed);
+    sqrtE = sqrt(E);
+    nn = __ldg(t.num_nucs + mat);
+    j = 0;
+    M0 = M1 = M2 = M3 = 0.0;
+  }
+  template <class Idx> __device__ __forceinline__ void begin(Idx iv, Idx stride) {
+    J = lcg_jump(2ull * (uint64_t)stride);
+    s = lcg_fast_forward(seed0, 2ull * (uint64_t)(first + iv));
+    start();
+  }
+  template <class Idx> __device__ __forceinline__ void next(Idx) {
+    s = lcg_apply(J, s);
+    start();
+  }
+  __device__ __forceinline__ bool step() {
+    if (j < nn) {
+      const int nuc = __ldg(t.mats + mat * t.max_num_nucs + j);
+      const double conc = __ldg(t.concs + mat * t.max_num_nucs + j);
+      double sigT, sigA, sigF;
+      nuclide_v<V>(t, E, sqrtE, nuc, sigT, sigA, sigF);
+      rs_accumulate(conc, sigT, sigA, sigF, M0, M1, M2, M3);
+    }
+    return ++j < nn;
+  }
+  template <class Idx> __device__ __forceinline__ void end(Idx iv) {
+    double* m = macro + (int64_t)iv * 4;
+    m[0] = M0; m[1] = M1; m[2] = M2; m[3] = M3;
+    ver[iv] = rs_argmax4(M0, M1, M2, M3);
+  }
+};
+
+struct Tr : DefaultTraits {};
+
+template <int V, int TPB, int MINB, bool DYN>
+__global__ void __launch_bounds__(TPB, MINB)
+    kern(const __grid_constant__ RSTables t, uint64_t seed, int64_t first, int32_t n,
+         uint64_t* ver, double* macro) {
+  Team<Tr> team = init<Tr>();
+  Body<V> b(t, seed, first, ver, macro);
+  if constexpr (DYN) distribute_parallel_for_dynamic_flat<Tr, FlatSync::Lockstep>(team, n, 1, b);
+  else distribute_parallel_for_flat<Tr, FlatSync::Lockstep>(team, n, b);
+}
+
+typedef void (*KF)(RSTables, uint64_t, int64_t, int32_t, uint64_t*, double*);
+struct Var { KF f; int tpb; const char* name; };
+static Var vars[] = {
+  {kern<0, 128, 5, true>, 128, "V0_128x5_dyn"},
+  {kern<0, 128, 4, true>, 128, "V0_128x4_dyn"},
+  {kern<0, 128, 6, true>, 128, "V0_128x6_dyn"},
+  {kern<0, 128, 8, true>, 128, "V0_128x8_dyn"},
+  {kern<0, 64, 10, true>, 64, "V0_64x10_dyn"},
+  {kern<1, 128, 5, true>, 128, "V1_128x5_dyn"},
+  {kern<2, 128, 5, true>, 128, "V2_128x5_dyn"},
+  {kern<2, 128, 4, true>, 128, "V2_128x4_dyn"},
+  {kern<2, 128, 6, true>, 128, "V2_128x6_dyn"},
+  {kern<2, 128, 8, true>, 128, "V2_128x8_dyn"},
+  {kern<2, 64, 10, true>, 64, "V2_64x10_dyn"},
+  {kern<2, 128, 5, false>, 128, "V2_128x5_static"},
+};
+extern "C" int rsf_count() { return (int)(sizeof(vars) / sizeof(vars[0])); }
+extern "C" const char* rsf_name(int v) { return vars[v].name; }
+extern "C" int rsf_regs(int v) {
+  cudaFuncAttributes a;
+  cudaFuncGetAttributes(&a, (const void*)vars[v].f);
+  return a.numRegs * 1000 + (int)a.localSizeBytes;
+}
+extern "C" int rsf_run(int v, RSTables t, uint64_t seed, int64_t first, int32_t n, uint64_t* ver,
+                       double* macro, void* stream) {
+  int dev = 0, sms = 0, per = 0;
+  cudaGetDevice(&dev);
+  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, vars[v].f, vars[v].tpb, 0);
+  vars[v].f<<<sms * per, vars[v].tpb, 0, (cudaStream_t)stream>>>(t, seed, first, n, ver, macro);
+  return (int)cudaGetLastError();
+}

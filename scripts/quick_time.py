@@ -63,6 +63,12 @@ def main(which):
         v = torch.empty(n, dtype=torch.uint64, device=dev)
         res["rs_rt_1M"] = {"ms": t(lambda: omprt.omprt_rs_lookup(rd, 1070, 0, n, v, None, 0, 128, A), 3)}
         res["rs_twin_1M"] = {"ms": t(lambda: omprt.omprt_cuda_rs_lookup(rd, 1070, 0, n, v, None, 0, 128, 0), 3)}
+        ref = v.clone()
+        F = omprt.OMPRT_FLAT
+        res["rs_rt_flat_1M"] = {"ms": t(lambda: omprt.omprt_rs_lookup(rd, 1070, 0, n, v, None, 0, 128, F), 3)}
+        res["rs_rt_flat_1M"]["same"] = bool((v == ref).all())
+        res["rs_twin_flat_1M"] = {"ms": t(lambda: omprt.omprt_cuda_rs_lookup(rd, 1070, 0, n, v, None, 0, 128, F), 3)}
+        res["rs_twin_flat_1M"]["same"] = bool((v == ref).all())
     if "xs" in which:
         tabs = gen.XSTables(**gen.XS_SMALL)
         d = omprt.XSDeviceTables(tabs, dev, accel=True)

@@ -18,20 +18,24 @@ def rs_dev(rt, rs_tables):
     return rt.RSDeviceTables(rs_tables, DEV)
 
 
-def _rs(rt, d, first, count, which, flags=0):
+def _rs(rt, d, first, count, which, flags=0, teams=0):
     ver = torch.zeros(max(count, 1), dtype=torch.uint64, device=DEV)
     mac = torch.zeros(max(count, 1) * 4, dtype=torch.float64, device=DEV)
     fn = rt.omprt_rs_lookup if which == "rt" else rt.omprt_cuda_rs_lookup
-    fn(d, gen.RS_LOOKUP_SEED, first, count, ver, mac, 0, 128, flags)
+    fn(d, gen.RS_LOOKUP_SEED, first, count, ver, mac, teams, 128, flags)
     torch.cuda.synchronize()
     return ver.cpu().numpy()[:count], mac.cpu().numpy()[: 4 * count].reshape(count, 4)
 
 
-@pytest.mark.parametrize("variant", ["rt", "rt_assume", "twin"])
+@pytest.mark.parametrize("variant", ["rt", "rt_assume", "twin", "rt_flat", "twin_flat",
+                                     "rt_dflat", "twin_dflat"])
 def test_rs_parity(rt, rs_dev, rs_tables, variant):
     first, count = 4321, 20_000 + 17
-    flags = rt.OMPRT_ASSUME_OVERSUB if variant == "rt_assume" else 0
-    ver, mac = _rs(rt, rs_dev, first, count, "twin" if variant == "twin" else "rt", flags)
+    D = rt.OMPRT_FLAT | rt.OMPRT_SCHED_DYNAMIC
+    flags = {"rt_assume": rt.OMPRT_ASSUME_OVERSUB, "rt_flat": rt.OMPRT_FLAT,
+             "twin_flat": rt.OMPRT_FLAT, "rt_dflat": D, "twin_dflat": D}.get(variant, 0)
+    ver, mac = _rs(rt, rs_dev, first, count, "twin" if variant.startswith("twin") else "rt",
+                   flags)
     rv, rm = oracle.rs_lookup(rs_tables, first, count, want_macro=True,
                               threads=os.cpu_count() or 1)
     # macro xs normwise (sigma_E = sigma_T - sigma_A can cancel): 1e-10
@@ -57,6 +61,37 @@ def test_rs_rt_and_twin_agree(rt, rs_dev):
     for q in flip:
         top2 = np.sort(m2[q])[-2:]
         assert top2[1] - top2[0] <= 1e-12 * abs(top2[1])
+
+
+def _agree(v1, m1, v0, m0):
+    """Same body, different inlining contexts: nvcc may contract a*b+c differently, so
+    macro xs agree to rounding (1e-12 normwise) and verification exactly up to near-ties."""
+    err = np.abs(m1 - m0).max(axis=1) / np.abs(m0).max(axis=1)
+    assert err.max() <= 1e-12, err.max()
+    for q in np.nonzero(v1 != v0)[0]:
+        top2 = np.sort(m0[q])[-2:]
+        assert top2[1] - top2[0] <= 1e-12 * abs(top2[1])
+
+
+@pytest.mark.parametrize("teams", [0, 1, 7, 148])
+def test_rs_flat_equals_nested(rt, rs_dev, teams):
+    """The flattened loop (one nuclide per step, lookups i, i+T*N, ... per thread, lock-step
+    warps) and its dynamic-schedule form run the same per-lookup arithmetic in the same
+    order as the nested loop, for persistent grids of any size (teams=1: 128 threads walk
+    all lookups, the LCG jump between a thread's lookups exercised thousands of times)."""
+    first, n = 777, 30_011
+    v0, m0 = _rs(rt, rs_dev, first, n, "rt")
+    D = rt.OMPRT_FLAT | rt.OMPRT_SCHED_DYNAMIC
+    for which, fl in (("rt", rt.OMPRT_FLAT), ("twin", rt.OMPRT_FLAT), ("rt", D), ("twin", D)):
+        v, m = _rs(rt, rs_dev, first, n, which, fl, teams)
+        _agree(v, m, v0, m0)
+
+
+def test_rs_flat_rejects_assumption(rt, rs_dev):
+    v = torch.zeros(16, dtype=torch.uint64, device=DEV)
+    with pytest.raises(Exception):
+        rt.omprt_rs_lookup(rs_dev, 1, 0, 16, v, None, 0, 128,
+                           rt.OMPRT_FLAT | rt.OMPRT_ASSUME_OVERSUB)
 
 
 def _su3(rt, fn, A, B, n, flags=0):

@@ -207,3 +207,45 @@ def test_chunked_vectorized_matches_twin_and_assumption(rt):
                                        torch.zeros(1, dtype=torch.float64, device=DEV), 128,
                                        1024, rt.OMPRT_ASSUME_OVERSUB)
     assert e.value.code == rt.OMPRT_E_INVAL
+
+
+DYN_CASES = [(0, 4, 1, 32), (1, 1, 8, 128), ((1 << 20) + 7, 4, 8, 128), (100003, 16, 37, 64),
+             (4096, 1, 8, 128), (2049, 3, 2, 256), (5000, 7, 300, 32)]
+
+
+@pytest.mark.parametrize("n,C,T,N", DYN_CASES)
+@pytest.mark.parametrize("which", ["rt", "twin"])
+def test_dynamic_schedule_owner_and_values(rt, n, C, T, N, which):
+    """schedule(dynamic, C) (reading R-D1): which thread runs a chunk is up to the hardware,
+    so the GPU's owner[] is checked against the schedule's invariants (the same checks that
+    pin oracle_dynamic_simulate) and the oracle's closed-form team of every iteration;
+    a[] bit-exact, the sum within 1e-12 (its order follows the chunk hand-out)."""
+    from test_oracle_schedule import _check_dynamic
+    x, b, c = gen.axpy_inputs(n)
+    fn = rt.omprt_spmd_axpy_sum_chunked if which == "rt" else rt.omprt_cuda_axpy_sum_chunked
+    bt, ct = torch.from_numpy(b).to(DEV), torch.from_numpy(c).to(DEV)
+    at = torch.full((max(n, 1),), float("nan"), dtype=torch.float64, device=DEV)
+    s = torch.zeros(1, dtype=torch.float64, device=DEV)
+    owner = torch.full((max(n, 1),), -1, dtype=torch.int32, device=DEV)
+    count = torch.zeros(max(n, 1), dtype=torch.int32, device=DEV)
+    fn(n, C, x, bt, ct, at, s, T, N, rt.OMPRT_RECORD_OWNER | rt.OMPRT_SCHED_DYNAMIC, owner,
+       count)
+    torch.cuda.synchronize()
+    own = owner.cpu().numpy()[:n]
+    _check_dynamic(n, C, T, N, own, count.cpu().numpy()[:n])
+    if n:
+        teams = np.array([oracle.dynamic_team_closed(i, n, T) for i in range(0, n, 97)])
+        assert (own[::97] // N == teams).all()
+    a_ref = oracle.axpy(x, b, c)
+    assert (at.cpu().numpy()[:n] == a_ref).all()
+    assert abs(s.item() - oracle.sum_f64(a_ref)) <= 1e-12 * max(oracle.sum_abs_f64(a_ref), 1e-300)
+
+
+def test_dynamic_schedule_rejects_assumption(rt):
+    n = 1024
+    x, b, c = gen.axpy_inputs(n)
+    bt, ct = torch.from_numpy(b).to(DEV), torch.from_numpy(c).to(DEV)
+    with pytest.raises(rt.OmprtError):
+        rt.omprt_spmd_axpy_sum_chunked(n, 1, x, bt, ct, torch.empty_like(bt),
+                                       torch.zeros(1, dtype=torch.float64, device=DEV), 8, 128,
+                                       rt.OMPRT_SCHED_DYNAMIC | rt.OMPRT_ASSUME_OVERSUB)

@@ -85,12 +85,18 @@ def test_flat_without_l2_window_and_reset(rt, xs_acc, xs_small):
     lines (the window only changes where the bracket records are cached)."""
     first, count = 77, 100_003
     ref = oracle.xs_lookup(xs_small, first, count, threads=os.cpu_count() or 1)
-    for fl in (rt.OMPRT_XS_FLAT | rt.OMPRT_XS_NO_L2_PERSIST, rt.OMPRT_XS_FLAT):
-        ver = torch.zeros(count, dtype=torch.uint64, device=DEV)
-        rt.omprt_xs_lookup(xs_acc, SEED, first, count, ver, None, 0, 256, fl)
-        torch.cuda.synchronize()
-        rt.omprt_l2_reset_persisting()
-        assert (ver.cpu().numpy() == ref).all()
+    try:
+        for aside in (1 << 40, 0, 16 << 20):  # device maximum, none, smaller than the table
+            got = rt.omprt_l2_set_aside(aside)  # granted in L2 way units (16 MB -> 23.7 MB)
+            assert (got > 0) == (aside > 0)
+            for fl in (rt.OMPRT_XS_FLAT | rt.OMPRT_XS_NO_L2_PERSIST, rt.OMPRT_XS_FLAT):
+                ver = torch.zeros(count, dtype=torch.uint64, device=DEV)
+                rt.omprt_xs_lookup(xs_acc, SEED, first, count, ver, None, 0, 256, fl)
+                torch.cuda.synchronize()
+                rt.omprt_l2_reset_persisting()
+                assert (ver.cpu().numpy() == ref).all()
+    finally:
+        assert rt.omprt_l2_set_aside(0) == 0
 
 
 def test_flat_rejects(rt, xs_dev, xs_acc):
@@ -275,3 +281,26 @@ def test_end_to_end_derived_tables(rt, xs_small):
         assert cks == [ref] * 3
         assert h2d == (xs_small.nuclide_grid.nbytes + xs_small.num_nucs.nbytes +
                        xs_small.mats.nbytes + xs_small.concs.nbytes) and d2h == 8
+
+
+@pytest.mark.parametrize("teams", [0, 1, 5])
+def test_flat_dynamic_schedule(rt, xs_acc, xs_small, teams):
+    """OMPRT_SCHED_DYNAMIC on the flattened lookup loop: every lookup's verification value
+    bit-exact against the oracle and the fused checksum exact, whatever thread ran it."""
+    F = rt.OMPRT_XS_FLAT | rt.OMPRT_SCHED_DYNAMIC
+    for first, count in [(0, 1), (9, 255), (3, 100_003)]:
+        ref = oracle.xs_lookup(xs_small, first, count, threads=os.cpu_count() or 1)
+        for fn in (rt.omprt_xs_lookup, rt.omprt_cuda_xs_lookup):
+            ver = torch.zeros(count, dtype=torch.uint64, device=DEV)
+            fn(xs_acc, SEED, first, count, ver, None, teams, 256, F)
+            ck = torch.full((1,), 5, dtype=torch.uint64, device=DEV)
+            fn(xs_acc, SEED, first, count, None, ck, teams, 256, F | rt.OMPRT_FUSED_REDUCTION)
+            torch.cuda.synchronize()
+            assert (ver.cpu().numpy() == ref).all()
+            assert int(ck.cpu().numpy()[0]) == int(ref.sum()) + 5
+
+
+def test_dynamic_needs_flat(rt, xs_acc):
+    ver = torch.zeros(64, dtype=torch.uint64, device=DEV)
+    with pytest.raises(Exception):
+        rt.omprt_xs_lookup(xs_acc, SEED, 0, 64, ver, None, 0, 256, rt.OMPRT_SCHED_DYNAMIC)

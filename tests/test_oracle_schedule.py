@@ -103,3 +103,52 @@ def test_chunked_schedule_special_cases():
     a = oracle.chunk_simulate(63, 4, 2, 8, assume_oversub=True)
     b = oracle.chunk_simulate(63, 4, 2, 8)
     assert (a[0] == b[0]).all() and (a[1] == b[1]).all()
+
+
+def _check_dynamic(n, C, T, N, owner, count):
+    """Structural pins of schedule(dynamic, C) under a blocked distribute (reading R-D1),
+    none of which restates the oracle's loop: exactly once; team t's iterations are one
+    contiguous run, in team order, every full team holding ceil(n/T); a chunk of C
+    iterations of the team's run stays on one thread; thread k's first chunk is chunk k."""
+    assert (count == 1).all()
+    B = -(-n // T) if n else 0
+    team = owner // N
+    assert (np.diff(team) >= 0).all()                      # contiguous, ascending teams
+    sizes = np.bincount(team, minlength=T) if n else np.zeros(T, np.int64)
+    full = sizes[sizes > 0]
+    assert (full[:-1] == B).all() and (full[-1:] <= B).all()
+    start = 0
+    for t in range(T):
+        run = owner[start:start + sizes[t]]
+        for c0 in range(0, len(run), C):
+            assert (run[c0:c0 + C] == run[c0]).all()       # a chunk on one thread
+        for k in range(min(N, -(-len(run) // C))):
+            assert run[k * C] == t * N + k                 # thread k starts with chunk k
+        start += sizes[t]
+
+
+def test_dynamic_schedule_invariants_bruteforce():
+    for n in range(0, 50):
+        for C in (1, 2, 3, 5):
+            for T in (1, 2, 3):
+                for N in (1, 2, 4):
+                    for seed in (0, 1):
+                        owner, count = oracle.dynamic_simulate(n, C, T, N, seed)
+                        _check_dynamic(n, C, T, N, owner, count)
+                        for iv in range(n):
+                            assert oracle.dynamic_team_closed(iv, n, T) == owner[iv] // N
+
+
+def test_dynamic_schedule_special_cases():
+    # one thread per team: the blocked distribute itself
+    owner, _ = oracle.dynamic_simulate(10, 1, 3, 1, 7)
+    assert list(owner) == [0, 0, 0, 0, 1, 1, 1, 1, 2, 2]
+    # a chunk covering the whole block: thread 0 of each team runs its block
+    owner, _ = oracle.dynamic_simulate(40, 64, 4, 8, 3)
+    assert list(owner) == [t * 8 for t in range(4) for _ in range(10)]
+    # different request orders are different (legal) executions of the same schedule
+    a, _ = oracle.dynamic_simulate(4000, 2, 2, 16, 1)
+    b, _ = oracle.dynamic_simulate(4000, 2, 2, 16, 2)
+    assert (a != b).any() and ((a // 16) == (b // 16)).all()
+    _check_dynamic(4000, 2, 2, 16, a, np.ones(4000, np.int32))
+    assert oracle.dynamic_team_closed(-1, 10, 2) is None

@@ -225,6 +225,10 @@ typedef struct {
   const uint16_t *index_grid16;/* [n_union][n_isotopes] */
   const double *brackets;      /* [n_isotopes][n_gridpoints-1][12], 32 B aligned */
   int32_t log2_bins, pad2;
+  /* optional compact index grid (omprt_xs_build_compact; both NULL or both set; used by
+   * the OMPRT_XS_FLAT launches, with the B200 layouts above): */
+  const uint16_t *idx_rows;    /* [ceil(n_union/16)][n_isotopes]: #{v <= 16m : owner[v] = q} */
+  const uint8_t *owner;        /* [n_union rounded up to 16]: nuclide of unionized energy v */
 } omprt_xs_tables;
 /* Lookups first..first+count-1 (lookup i draws its energy and material from
  * fast_forward_LCG(seed, 2i), so results do not depend on sharding):
@@ -264,6 +268,22 @@ int omprt_xs_derive_tmp_bytes(int32_t n_isotopes, int32_t n_gridpoints, uint64_t
 int omprt_xs_derive(const double *nuclide_grid, int32_t n_isotopes, int32_t n_gridpoints,
                     double *unionized, uint16_t *index_grid16, void *tmp, uint64_t tmp_bytes,
                     void *stream);
+/* Compact index grid (reading R-X1): the same index grid as every 16th row of position
+ * counts plus the nuclide id of every unionized energy, so a lookup rebuilds its row
+ * exactly (index = clip(rows[e/16][q] + #{v in (16*(e/16), e] : owner[v] = q} - 1, 0,
+ * n_gridpoints - 2)) from 7.3 MB of tables instead of 104.5 MB of 16-bit rows (small
+ * problem).  Built from the nuclide grids on the device (the omprt_xs_derive sort):
+ *   owner[v]   = nuclide of the v-th smallest energy (0xFF past n_union, up to the
+ *                multiple of 16), idx_rows[m*n_isotopes + q] = #{v <= 16m : owner[v] = q}.
+ * Sizes: sizes[0] idx_rows bytes, sizes[1] owner bytes.  tmp: >= omprt_xs_derive_tmp_bytes.
+ * Synchronizes `stream` (it checks the table): OMPRT_E_INVAL unless 0 < n_isotopes <= 255,
+ * 2 <= n_gridpoints <= 65535 and the two smallest and the two largest energies are
+ * distinct (the ends the lookup's clamped search can return; everywhere else ties are
+ * exact).  owner must be 16 B aligned. */
+int omprt_xs_compact_sizes(int32_t n_isotopes, int32_t n_gridpoints, uint64_t *sizes);
+int omprt_xs_build_compact(const double *nuclide_grid, int32_t n_isotopes, int32_t n_gridpoints,
+                           uint16_t *idx_rows, uint8_t *owner, void *tmp, uint64_t tmp_bytes,
+                           void *stream);
 /* K11 ("we moved the reduction out of the timed kernel"): *out_inout += sum v[i]
  * (u64, wraps mod 2^64). */
 int omprt_u64_sum(const uint64_t *v, int64_t n, uint64_t *out_inout, void *stream);
@@ -293,7 +313,7 @@ int omprt_xs_run_host_steps(omprt_xs_tables host_tables, uint64_t seed, int64_t 
 
 /* ---- C4: RSBench-shaped multipole lookup -------------------- */
 typedef struct {
-  const double *poles;      /* [n_poles][8] EA RT RA RF (re, im) */
+  const double *poles;      /* [n_poles][8] EA RT RA RF (re, im), 32 B aligned */
   const int32_t *pole_l;    /* [n_poles] l value in [0, numL) */
   const double *windows;    /* [n_windows][4] T A F 0 */
   const int32_t *win_range; /* [n_windows][2] absolute pole [start, end) */

@@ -26,7 +26,46 @@ struct XSTables {
   const uint16_t* __restrict__ index_grid16;  // [n_union][n_iso] (n_gp <= 65536)
   const double* __restrict__ brackets;      // [n_iso][n_gp-1][12] (E,t,e,a,f,n) x (k, k+1)
   int32_t log2_bins, pad2;
+  // optional compact index grid (omprt_xs_build_compact; both NULL or both set): the index
+  // grid as every 16th row of position counts + the nuclide of every unionized energy
+  const uint16_t* __restrict__ idx_rows;    // [ceil(n_union/16)][n_iso]: #{v <= 16m : owner[v] = q}
+  const uint8_t* __restrict__ owner;        // [n_union rounded up to 16], 0xFF padded
 };
+
+// ---- compact index grid (reading R-X1) --------------------------------------------------
+// index_grid[e][q] = clip(C_q(e) - 1, 0, n_gp - 2) with C_q(e) = #{k : E_q[k] <= U[e]}.  For
+// the e the search returns (the LAST of its group of equal energies, or a clamped end that
+// the builder checks is tie-free) C_q(e) = #{v <= e : owner[v] = q}, a prefix count over the
+// nuclide ids of the sorted energies: the row stored for u0 = e & ~15 plus the matches among
+// owner[u0+1 .. e] -- one 16-byte load per lookup and 4 byte-compares per nuclide.  The
+// table shrinks from 104.5 MB (16-bit rows) to 6.5 + 0.8 MB, so it stays in L2.
+struct OwnerChunk {
+  uint32_t w[4];  // owner[u0 .. u0+15], bytes outside (u0, e] replaced by 0xFF (no nuclide)
+};
+__device__ __forceinline__ OwnerChunk owner_chunk(const XSTables& t, int32_t e) {
+  const int32_t u0 = e & ~15;
+  const uint4 v = __ldg(reinterpret_cast<const uint4*>(t.owner + u0));
+  const int r = e - u0;  // positions 1..r of the chunk count
+  OwnerChunk c{{v.x, v.y, v.z, v.w}};
+#pragma unroll
+  for (int i = 0; i < 4; ++i) {
+    const int valid = r - 4 * i + 1;  // bytes 4i .. 4i+valid-1 have position <= r
+    uint32_t keep = valid >= 4 ? 0xFFFFFFFFu : (valid <= 0 ? 0u : (1u << (8 * valid)) - 1u);
+    if (i == 0) keep &= ~0xFFu;     // position 0 is the stored row itself
+    c.w[i] = (c.w[i] & keep) | ~keep;
+  }
+  return c;
+}
+// index_grid[e][q] from the compact layout (row = idx_rows + (e >> 4) * n_iso)
+__device__ __forceinline__ int32_t compact_index(const XSTables& t,
+                                                 const uint16_t* __restrict__ row,
+                                                 const OwnerChunk& c, int32_t q) {
+  const uint32_t qq = (uint32_t)q * 0x01010101u;
+  const int cnt = __popc(__vcmpeq4(c.w[0], qq)) + __popc(__vcmpeq4(c.w[1], qq)) +
+                  __popc(__vcmpeq4(c.w[2], qq)) + __popc(__vcmpeq4(c.w[3], qq));
+  const int32_t k = (int32_t)__ldg(row + q) + (cnt >> 3) - 1;
+  return k < 0 ? 0 : (k > t.n_gridpoints - 2 ? t.n_gridpoints - 2 : k);
+}
 
 // ---- the proxy apps' LCG (m = 2^63, a = 2806196910506780709, c = 1) ----------------------
 constexpr uint64_t kLcgA = 2806196910506780709ull;
@@ -231,7 +270,7 @@ __device__ __forceinline__ uint64_t xs_lookup_accel(const XSTables& t, uint64_t 
 // L1 traffic is what bounds this loop (ncu: L1 ~80 % busy), so the bracket records, read
 // once, bypass L1 allocation, and with SmemMats the material tables (mats, concs) come
 // from a team-shared copy (`mats`/`concs` then point to shared memory).
-template <bool Fused, bool SmemMats, int P = 2>
+template <bool Fused, bool SmemMats, bool Compact = false, int P = 2>
 struct XSFlatLookup {
   const XSTables& t;
   const uint64_t seed0;
@@ -247,6 +286,7 @@ struct XSFlatLookup {
   int32_t mat, idx, nn, j;
   double m0, m1, m2, m3, m4;
   int32_t pc[P], kc[P];
+  OwnerChunk oc;  // Compact only
 
   __device__ __forceinline__ XSFlatLookup(const XSTables& tab, uint64_t seed, int64_t first_,
                                           uint64_t* verification, const int32_t* mats_,
@@ -262,6 +302,17 @@ struct XSFlatLookup {
     else return __ldg(p);
   }
 
+  // this lookup's row of the index grid, and its entry for nuclide q
+  __device__ __forceinline__ const uint16_t* index_row() const {
+    if constexpr (Compact) return t.idx_rows + (int64_t)(idx >> 4) * t.n_isotopes;
+    else return t.index_grid16 + (int64_t)idx * t.n_isotopes;
+  }
+  __device__ __forceinline__ int32_t index_at(const uint16_t* __restrict__ irow,
+                                              int32_t q) const {
+    if constexpr (Compact) return compact_index(t, irow, oc, q);
+    else return (int32_t)__ldg(irow + q);
+  }
+
   __device__ __forceinline__ void start() {
     uint64_t seed = s;
     E = lcg_double(seed);
@@ -270,12 +321,13 @@ struct XSFlatLookup {
     nn = __ldg(t.num_nucs + mat);
     m0 = m1 = m2 = m3 = m4 = 0.0;
     j = 0;
+    if constexpr (Compact) oc = owner_chunk(t, idx);
     const int32_t* __restrict__ mrow = mats + mat * t.max_num_nucs;
-    const uint16_t* __restrict__ irow = t.index_grid16 + (int64_t)idx * t.n_isotopes;
+    const uint16_t* __restrict__ irow = index_row();
 #pragma unroll
     for (int u = 0; u < P; ++u) {
       pc[u] = u < nn ? mat_at(mrow + u) : 0;
-      kc[u] = u < nn ? (int32_t)__ldg(irow + pc[u]) : 0;
+      kc[u] = u < nn ? index_at(irow, pc[u]) : 0;
     }
   }
   template <class Idx>
@@ -292,13 +344,13 @@ struct XSFlatLookup {
   __device__ __forceinline__ bool step() {
     const int32_t* __restrict__ mrow = mats + mat * t.max_num_nucs;
     const double* __restrict__ crow = concs + mat * t.max_num_nucs;
-    const uint16_t* __restrict__ irow = t.index_grid16 + (int64_t)idx * t.n_isotopes;
+    const uint16_t* __restrict__ irow = index_row();
     int32_t pn[P], kn[P];
 #pragma unroll
     for (int u = 0; u < P; ++u) {  // next step's index entries
       const int jj = j + P + u;
       pn[u] = jj < nn ? mat_at(mrow + jj) : 0;
-      kn[u] = jj < nn ? (int32_t)__ldg(irow + pn[u]) : 0;
+      kn[u] = jj < nn ? index_at(irow, pn[u]) : 0;
     }
 #pragma unroll
     for (int u = 0; u < P; ++u) {

@@ -117,7 +117,7 @@ constexpr unsigned kXSMatsSite = 10, kXSConcsSite = 11;  // team_local sites
 // OMPRT_SCHED_DYNAMIC: schedule(dynamic, kXSDynChunk) instead of Fig. 5 (reading R-D1)
 constexpr int kXSDynChunk = 8;
 
-template <class Tr, bool Fused, bool Smem, bool Dyn = false>
+template <class Tr, bool Fused, bool Smem, bool Dyn = false, bool Compact = false>
 __global__ void __launch_bounds__(kXSThreads, kXSMinBlocksFlat)
     omprt_xs_flat_rt(const __grid_constant__ XSTables t, uint64_t seed, int64_t first,
                      typename Tr::Idx count, uint64_t* __restrict__ verification,
@@ -138,7 +138,7 @@ __global__ void __launch_bounds__(kXSThreads, kXSMinBlocksFlat)
     mats = sm;
     concs = sc;
   }
-  using Lookup = XSFlatLookup<Fused, Smem>;
+  using Lookup = XSFlatLookup<Fused, Smem, Compact>;
   if constexpr (Fused) *Lookup::flat_acc_slot() = 0ull;
   Lookup lookup(t, seed, first, verification, mats, concs);
   if constexpr (Dyn) distribute_parallel_for_dynamic_flat(team, count, (Idx)kXSDynChunk, lookup);
@@ -149,7 +149,7 @@ __global__ void __launch_bounds__(kXSThreads, kXSMinBlocksFlat)
 }
 
 // Bare CUDA twin: the same flattened loop written by hand around the same body.
-template <bool Fused, bool Smem, bool Dyn = false>
+template <bool Fused, bool Smem, bool Dyn = false, bool Compact = false>
 __global__ void __launch_bounds__(kXSThreads, kXSMinBlocksFlat)
     cuda_xs_flat_twin(const __grid_constant__ XSTables t, uint64_t seed, int64_t first,
                       int32_t count, uint64_t* __restrict__ verification,
@@ -168,7 +168,7 @@ __global__ void __launch_bounds__(kXSThreads, kXSMinBlocksFlat)
     mats = sm;
     concs = sc;
   }
-  using Lookup = XSFlatLookup<Fused, Smem>;
+  using Lookup = XSFlatLookup<Fused, Smem, Compact>;
   if constexpr (Fused) *Lookup::flat_acc_slot() = 0ull;
   Lookup lookup(t, seed, first, verification, mats, concs);
   if constexpr (Dyn) {  // team block + team-shared chunk counter, by hand
@@ -254,7 +254,7 @@ OMPRT_REGISTER_KERNEL(omprt_u64_sum_rt, omprt_u64_sum_rt<SumTraits>)
 inline XSTables to_dev(const omprt_xs_tables& a) {
   return XSTables{a.nuclide_grid, a.unionized, a.index_grid, a.num_nucs, a.mats, a.concs,
                   a.n_isotopes, a.n_gridpoints, a.max_num_nucs, 0, a.n_union,
-                  a.bins, a.index_grid16, a.brackets, a.log2_bins, 0};
+                  a.bins, a.index_grid16, a.brackets, a.log2_bins, 0, a.idx_rows, a.owner};
 }
 
 // Launch configuration of the flattened kernels: the persistent grid, plus (unless
@@ -301,6 +301,42 @@ inline bool xs_mats_fit_smem(const omprt_xs_tables& t) {
   return 12ll * t.max_num_nucs <= kXSMatSmem;
 }
 
+inline bool xs_has_compact(const omprt_xs_tables& t) {
+  return t.idx_rows != nullptr && t.owner != nullptr;
+}
+
+// The flattened kernels: runtime-driven (Twin = false) or twin, by (fused, team-shared
+// material tables, dynamic schedule, compact index grid).
+template <bool Twin, bool F, bool S, bool D, bool C>
+inline cudaError_t xs_flat_launch(const cudaLaunchConfig_t& cfg, const XSTables& d, uint64_t seed,
+                                  int64_t first, int32_t n, uint64_t* ver, unsigned long long* ck,
+                                  unsigned long long* p, unsigned* tk) {
+  if constexpr (Twin)
+    return cudaLaunchKernelEx(&cfg, cuda_xs_flat_twin<F, S, D, C>, d, seed, first, n, ver, ck,
+                              p, tk);
+  else
+    return cudaLaunchKernelEx(&cfg, omprt_xs_flat_rt<XSTraits, F, S, D, C>, d, seed, first, n,
+                              ver, ck, p, tk);
+}
+template <bool Twin>
+inline cudaError_t xs_flat_dispatch(uint32_t flags, bool fused, bool smem, bool compact,
+                                    const cudaLaunchConfig_t& cfg, const XSTables& d,
+                                    uint64_t seed, int64_t first, int32_t n, uint64_t* ver,
+                                    unsigned long long* ck, unsigned long long* p,
+                                    unsigned* tk) {
+  const bool dyn = flags & OMPRT_SCHED_DYNAMIC;
+#define OMPRT_XSF(F, S, D, C) \
+  if (fused == F && smem == S && dyn == D && compact == C) \
+    return xs_flat_launch<Twin, F, S, D, C>(cfg, d, seed, first, n, ver, ck, p, tk);
+#define OMPRT_XSF2(F, S, D) OMPRT_XSF(F, S, D, false) OMPRT_XSF(F, S, D, true)
+#define OMPRT_XSF4(F, S) OMPRT_XSF2(F, S, false) OMPRT_XSF2(F, S, true)
+  OMPRT_XSF4(false, false) OMPRT_XSF4(false, true) OMPRT_XSF4(true, false) OMPRT_XSF4(true, true)
+#undef OMPRT_XSF4
+#undef OMPRT_XSF2
+#undef OMPRT_XSF
+  return cudaErrorInvalidValue;
+}
+
 inline bool xs_has_accel(const omprt_xs_tables& t) {
   return t.bins != nullptr && t.index_grid16 != nullptr && t.brackets != nullptr;
 }
@@ -318,6 +354,13 @@ inline int xs_validate(const omprt_xs_tables& t, int64_t count, uint64_t* ver, u
                   "accelerated layout: bad log2_bins");
   OMPRT_CHECK_ARG(accel || (!t.bins && !t.index_grid16 && !t.brackets),
                   "accelerated layout: bins, index_grid16 and brackets go together");
+  OMPRT_CHECK_ARG((t.idx_rows == nullptr) == (t.owner == nullptr),
+                  "compact index grid: idx_rows and owner go together");
+  OMPRT_CHECK_ARG(!xs_has_compact(t) || (accel && (flags & OMPRT_XS_FLAT) &&
+                                          t.n_isotopes <= 255 && t.n_gridpoints <= 65535 &&
+                                          ((uintptr_t)t.owner & 15) == 0),
+                  "compact index grid: flattened launches with the B200 layouts only "
+                  "(n_isotopes <= 255, n_gridpoints <= 65535, owner 16 B aligned)");
   const bool fused = flags & OMPRT_FUSED_REDUCTION;
   OMPRT_CHECK_ARG(fused ? ck != nullptr : (ver != nullptr || count == 0),
                   fused ? "fused reduction needs checksum_inout" : "verification is required");
@@ -419,20 +462,8 @@ extern "C" int omprt_xs_lookup(omprt_xs_tables t, uint64_t seed, int64_t first, 
     const bool smem = xs_mats_fit_smem(t);
     const FlatLaunch L = flat_launch(t, teams, threads, flags, w, s);
     cudaError_t e;
-#define OMPRT_XSF(F, S, D) \
-  e = cudaLaunchKernelEx(&L.cfg, omprt_xs_flat_rt<XSTraits, F, S, D>, d, seed, first, n, verification, ck, p, tk)
-    if (flags & OMPRT_SCHED_DYNAMIC) {
-      if (fused && smem) OMPRT_XSF(true, true, true);
-      else if (fused) OMPRT_XSF(true, false, true);
-      else if (smem) OMPRT_XSF(false, true, true);
-      else OMPRT_XSF(false, false, true);
-    } else {
-      if (fused && smem) OMPRT_XSF(true, true, false);
-      else if (fused) OMPRT_XSF(true, false, false);
-      else if (smem) OMPRT_XSF(false, true, false);
-      else OMPRT_XSF(false, false, false);
-    }
-#undef OMPRT_XSF
+    e = xs_flat_dispatch<false>(flags, fused, smem, xs_has_compact(t), L.cfg, d, seed, first,
+                                n, verification, ck, p, tk);
     (void)e;
     return check_launch("omprt_xs_flat_rt");
   }
@@ -483,17 +514,12 @@ extern "C" int omprt_cuda_xs_lookup(omprt_xs_tables t, uint64_t seed, int64_t fi
     const FlatLaunch L = flat_launch(t, tm, threads, flags, w, s);
     unsigned long long* nul = nullptr;
     unsigned* nult = nullptr;
-    if (flags & OMPRT_SCHED_DYNAMIC) {
-      if (fused && smem) cudaLaunchKernelEx(&L.cfg, cuda_xs_flat_twin<true, true, true>, d, seed, first, n, verification, ck, p, tk);
-      else if (fused) cudaLaunchKernelEx(&L.cfg, cuda_xs_flat_twin<true, false, true>, d, seed, first, n, verification, ck, p, tk);
-      else if (smem) cudaLaunchKernelEx(&L.cfg, cuda_xs_flat_twin<false, true, true>, d, seed, first, n, verification, nul, nul, nult);
-      else cudaLaunchKernelEx(&L.cfg, cuda_xs_flat_twin<false, false, true>, d, seed, first, n, verification, nul, nul, nult);
-    } else {
-      if (fused && smem) cudaLaunchKernelEx(&L.cfg, cuda_xs_flat_twin<true, true>, d, seed, first, n, verification, ck, p, tk);
-      else if (fused) cudaLaunchKernelEx(&L.cfg, cuda_xs_flat_twin<true, false>, d, seed, first, n, verification, ck, p, tk);
-      else if (smem) cudaLaunchKernelEx(&L.cfg, cuda_xs_flat_twin<false, true>, d, seed, first, n, verification, nul, nul, nult);
-      else cudaLaunchKernelEx(&L.cfg, cuda_xs_flat_twin<false, false>, d, seed, first, n, verification, nul, nul, nult);
-    }
+    if (fused)
+      xs_flat_dispatch<true>(flags, fused, smem, xs_has_compact(t), L.cfg, d, seed, first, n,
+                             verification, ck, p, tk);
+    else
+      xs_flat_dispatch<true>(flags, fused, smem, xs_has_compact(t), L.cfg, d, seed, first, n,
+                             verification, nul, nul, nult);
     return check_launch("cuda_xs_flat_twin");
   }
   if (fused && accel) cuda_xs_twin<true, true><<<tm, threads, 0, s>>>(d, seed, first, n, verification, ck, p, tk);

@@ -48,7 +48,7 @@ EXPORTS = [
     "omprt_cuda_axpy_sum_chunked", "omprt_generic_team", "omprt_cuda_generic_team",
     "omprt_icv_probe", "omprt_xs_lookup", "omprt_cuda_xs_lookup", "omprt_u64_sum",
     "omprt_xs_run_host", "omprt_xs_run_host_steps", "omprt_xs_accel_sizes", "omprt_xs_build_accel",
-    "omprt_xs_derive_tmp_bytes", "omprt_xs_derive", "omprt_rs_lookup", "omprt_cuda_rs_lookup", "omprt_su3_mult",
+    "omprt_xs_derive_tmp_bytes", "omprt_xs_derive", "omprt_xs_compact_sizes", "omprt_xs_build_compact", "omprt_rs_lookup", "omprt_cuda_rs_lookup", "omprt_su3_mult",
     "omprt_cuda_su3_mult", "omprt_kernel_count", "omprt_kernel_name", "omprt_kernel_attrs",
 ]
 
@@ -70,7 +70,8 @@ class XSTablesC(C.Structure):
                 ("n_isotopes", C.c_int32), ("n_gridpoints", C.c_int32),
                 ("max_num_nucs", C.c_int32), ("pad", C.c_int32), ("n_union", C.c_int64),
                 ("bins", C.c_void_p), ("index_grid16", C.c_void_p), ("brackets", C.c_void_p),
-                ("log2_bins", C.c_int32), ("pad2", C.c_int32)]
+                ("log2_bins", C.c_int32), ("pad2", C.c_int32),
+                ("idx_rows", C.c_void_p), ("owner", C.c_void_p)]
 
 
 class RSTablesC(C.Structure):
@@ -107,6 +108,8 @@ _SIGS = {
     "omprt_xs_build_accel": [C.POINTER(XSTablesC), _vp, _vp, _vp, _i32, _vp],
     "omprt_xs_derive_tmp_bytes": [_i32, _i32, C.POINTER(_u64)],
     "omprt_xs_derive": [_vp, _i32, _i32, _vp, _vp, _vp, _u64, _vp],
+    "omprt_xs_compact_sizes": [_i32, _i32, C.POINTER(_u64)],
+    "omprt_xs_build_compact": [_vp, _i32, _i32, _vp, _vp, _vp, _u64, _vp],
     "omprt_xs_run_host": [XSTablesC, _u64, _i64, _i64, _i32, _u32, C.POINTER(_u64),
                           C.POINTER(_u64), C.POINTER(_u64), _vp],
     "omprt_xs_run_host_steps": [XSTablesC, _u64, _i64, _i64, _i32, _u32, _i32, C.POINTER(_u64),
@@ -263,7 +266,7 @@ class XSDeviceTables:
     """Device copies (torch tensors) of gen.XSTables and the by-value C struct.  With
     accel=True the B200 layouts are built on the device (omprt_xs_build_accel)."""
 
-    def __init__(self, t, device="cuda", accel=False, log2_bins=16):
+    def __init__(self, t, device="cuda", accel=False, log2_bins=16, compact=False):
         import torch
         self.host = t
         self.nuclide_grid = torch.from_numpy(t.nuclide_grid).to(device)
@@ -281,6 +284,23 @@ class XSDeviceTables:
             self.index_grid16 = torch.empty(sizes[1] // 2, dtype=torch.uint16, device=device)
             self.brackets = torch.empty(sizes[2] // 8, dtype=torch.float64, device=device)
             omprt_xs_build_accel(self, self.bins, self.index_grid16, self.brackets, log2_bins)
+        if compact:  # the compact index grid (flattened launches), from the nuclide grids
+            sizes = omprt_xs_compact_sizes(t.n_isotopes, t.n_gridpoints)
+            self.idx_rows = torch.empty(sizes[0] // 2, dtype=torch.uint16, device=device)
+            self.owner = torch.empty(sizes[1], dtype=torch.uint8, device=device)
+            tmp = torch.empty(omprt_xs_derive_tmp_bytes(t.n_isotopes, t.n_gridpoints),
+                              dtype=torch.uint8, device=device)
+            omprt_xs_build_compact(self.nuclide_grid, t.n_isotopes, t.n_gridpoints,
+                                   self.idx_rows, self.owner, tmp)
+            self.c.idx_rows, self.c.owner = _p(self.idx_rows), _p(self.owner)
+
+    def without_compact(self):
+        """A view of the same tables without the compact index grid."""
+        v = XSDeviceTables.__new__(XSDeviceTables)
+        v.__dict__.update(self.__dict__)
+        v.c = XSTablesC.from_buffer_copy(self.c)
+        v.c.idx_rows = v.c.owner = None
+        return v
 
     def plain(self):
         """A view of the same tables without the accelerated layouts."""
@@ -288,6 +308,7 @@ class XSDeviceTables:
         v.__dict__.update(self.__dict__)
         v.c = XSTablesC.from_buffer_copy(self.c)
         v.c.bins = v.c.index_grid16 = v.c.brackets = None
+        v.c.idx_rows = v.c.owner = None
         v.c.log2_bins = 0
         return v
 
@@ -301,6 +322,20 @@ def omprt_xs_accel_sizes(n_isotopes, n_gridpoints, n_union, log2_bins=16):
 def omprt_xs_build_accel(tables, bins, index_grid16, brackets, log2_bins=16, stream=None):
     return _check(load().omprt_xs_build_accel(C.byref(tables.c), _p(bins), _p(index_grid16),
                                               _p(brackets), log2_bins, _stream(stream)))
+
+
+def omprt_xs_compact_sizes(n_isotopes, n_gridpoints):
+    sz = (_u64 * 2)()
+    _check(load().omprt_xs_compact_sizes(n_isotopes, n_gridpoints, sz))
+    return list(sz)
+
+
+def omprt_xs_build_compact(nuclide_grid, n_isotopes, n_gridpoints, idx_rows, owner, tmp,
+                           stream=None):
+    return _check(load().omprt_xs_build_compact(_p(nuclide_grid), n_isotopes, n_gridpoints,
+                                                _p(idx_rows), _p(owner), _p(tmp),
+                                                tmp.numel() * tmp.element_size(),
+                                                _stream(stream)))
 
 
 def xs_host_struct(t, pinned=None, derive=False):

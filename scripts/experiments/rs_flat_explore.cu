@@ -8,6 +8,7 @@
 #include <cstdint>
 #include "../../paper_conf_ipps_doerfertphtdcg22_b200/csrc/omprt/device/omprt.cuh"
 #include "../../paper_conf_ipps_doerfertphtdcg22_b200/csrc/kernels/rs_body.cuh"
+#include "../../paper_conf_ipps_doerfertphtdcg22_b200/csrc/kernels/vec.cuh"
 using namespace omprt_kernels;
 using namespace omprt;
 
@@ -66,6 +67,9 @@ __device__ __forceinline__ cplx faddeeva_v(cplx Z) {
   return cmul({-Z.i, Z.r}, q);
 }
 
+// V >= 3: 256-bit pole loads (2 x LDG.256 per 64 B pole); V >= 4: the Abrarov branch
+// deferred to the end of the window (one pending pole per lane; its contribution is added
+// last -- a different summation order, within the tolerance contract)
 template <int V>
 __device__ __forceinline__ void nuclide_v(const RSTables& t, double E, double sqrtE, int nuc,
                                           double& sigT, double& sigA, double& sigF) {
@@ -92,17 +96,47 @@ __device__ __forceinline__ void nuclide_v(const RSTables& t, double E, double sq
   sigT = E * TA.x;
   sigA = E * TA.y;
   sigF = E * Fw;
-  for (int p = rg.x; p < rg.y; ++p) {
-    const double2* P = reinterpret_cast<const double2*>(t.poles + (int64_t)p * 8);
-    const double2 EA = __ldg(P + 0), RT = __ldg(P + 1), RA = __ldg(P + 2), RF = __ldg(P + 3);
+  int pend = -1;
+  cplx Zp = {0.0, 0.0};
+  auto add = [&](int p, double rtr, double rti, double rar, double rai, double rfr, double rfi,
+                 cplx W) {
     const int l = __ldg(t.pole_l + p);
-    const cplx Z = {(E - EA.x) * 0.5, (0.0 - EA.y) * 0.5};
-    const cplx W = faddeeva_v<V>(Z);
     const cplx fl = l == 0 ? f[0] : l == 1 ? f[1] : l == 2 ? f[2] : f[3];
     const cplx Wf = cmul(W, fl);
-    sigT += RT.x * Wf.r - RT.y * Wf.i;
-    sigA += RA.x * W.r - RA.y * W.i;
-    sigF += RF.x * W.r - RF.y * W.i;
+    sigT += rtr * Wf.r - rti * Wf.i;
+    sigA += rar * W.r - rai * W.i;
+    sigF += rfr * W.r - rfi * W.i;
+  };
+  for (int p = rg.x; p < rg.y; ++p) {
+    const double* P = t.poles + (int64_t)p * 8;
+    double ear, eai, rtr, rti, rar, rai, rfr, rfi;
+    if constexpr (V >= 3) {
+      ld_nc_v4f64(P, ear, eai, rtr, rti);
+      ld_nc_v4f64(P + 4, rar, rai, rfr, rfi);
+    } else {
+      const double2* Q = reinterpret_cast<const double2*>(P);
+      const double2 EA = __ldg(Q + 0), RT = __ldg(Q + 1), RA = __ldg(Q + 2), RF = __ldg(Q + 3);
+      ear = EA.x; eai = EA.y; rtr = RT.x; rti = RT.y; rar = RA.x; rai = RA.y; rfr = RF.x; rfi = RF.y;
+    }
+    const cplx Z = {(E - ear) * 0.5, (0.0 - eai) * 0.5};
+    if constexpr (V >= 4) {
+      const double absz = sqrt(__dadd_rn(__dmul_rn(Z.r, Z.r), __dmul_rn(Z.i, Z.i)));
+      if (absz < 6.0 && pend < 0) {  // defer (one per lane)
+        pend = p;
+        Zp = Z;
+        continue;
+      }
+    }
+    add(p, rtr, rti, rar, rai, rfr, rfi, faddeeva_v<(V >= 2 ? 2 : V)>(Z));
+  }
+  if constexpr (V >= 4) {
+    if (pend >= 0) {
+      const double* P = t.poles + (int64_t)pend * 8;
+      double ear, eai, rtr, rti, rar, rai, rfr, rfi;
+      ld_nc_v4f64(P, ear, eai, rtr, rti);
+      ld_nc_v4f64(P + 4, rar, rai, rfr, rfi);
+      add(pend, rtr, rti, rar, rai, rfr, rfi, faddeeva_v<2>(Zp));
+    }
   }
 }
 
@@ -170,18 +204,12 @@ __global__ void __launch_bounds__(TPB, MINB)
 typedef void (*KF)(RSTables, uint64_t, int64_t, int32_t, uint64_t*, double*);
 struct Var { KF f; int tpb; const char* name; };
 static Var vars[] = {
-  {kern<0, 128, 5, true>, 128, "V0_128x5_dyn"},
-  {kern<0, 128, 4, true>, 128, "V0_128x4_dyn"},
-  {kern<0, 128, 6, true>, 128, "V0_128x6_dyn"},
-  {kern<0, 128, 8, true>, 128, "V0_128x8_dyn"},
-  {kern<0, 64, 10, true>, 64, "V0_64x10_dyn"},
-  {kern<1, 128, 5, true>, 128, "V1_128x5_dyn"},
   {kern<2, 128, 5, true>, 128, "V2_128x5_dyn"},
-  {kern<2, 128, 4, true>, 128, "V2_128x4_dyn"},
-  {kern<2, 128, 6, true>, 128, "V2_128x6_dyn"},
-  {kern<2, 128, 8, true>, 128, "V2_128x8_dyn"},
-  {kern<2, 64, 10, true>, 64, "V2_64x10_dyn"},
-  {kern<2, 128, 5, false>, 128, "V2_128x5_static"},
+  {kern<3, 128, 5, true>, 128, "V3_128x5_dyn"},
+  {kern<4, 128, 5, true>, 128, "V4_128x5_dyn"},
+  {kern<4, 128, 4, true>, 128, "V4_128x4_dyn"},
+  {kern<4, 64, 10, true>, 64, "V4_64x10_dyn"},
+  {kern<3, 64, 10, true>, 64, "V3_64x10_dyn"},
 };
 extern "C" int rsf_count() { return (int)(sizeof(vars) / sizeof(vars[0])); }
 extern "C" const char* rsf_name(int v) { return vars[v].name; }

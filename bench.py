@@ -353,7 +353,9 @@ def run_omprt(args):
     flat_teams = props.multi_processor_count * 4  # resident teams (4 x 256 per SM, 64 regs)
     alg_plain = load_alg_bytes(False) * L
     omprt.omprt_l2_set_aside(0)
-    secondary = None
+    secondary = sharded = None
+    if not args.no_secondary and world > 1:
+        sharded = run_sharded(omprt, torch, gen, sharding, dev, stream, scrub, rank, world)
     if not args.no_secondary and rank == 0:
         secondary = run_secondary(omprt, torch, gen, dev, stream, scrub)
     cpu = None
@@ -416,6 +418,7 @@ def run_omprt(args):
                 "static_smem": [tab["omprt_xs_flat_rt"]["static_smem"],
                                 tab["cuda_xs_flat_twin"]["static_smem"]]},
             "secondary": secondary,
+            "secondary_sharded": sharded,
         }
         print(json.dumps(line), flush=True)
     if world > 1:
@@ -441,6 +444,51 @@ def _time(fn, stream, scrub, reps=5, warm=2, flush=True):
         torch.cuda.synchronize()
         out.append(a.elapsed_time(b))
     return statistics.median(out)
+
+
+def run_sharded(omprt, torch, gen, sharding, dev, stream, scrub, rank, world):
+    """BASELINE configs[3] and [4] as they are stated for several GPUs (N > 1 only): C4's
+    10M RSBench lookups and C5's 32^4 SU(3) sites split into contiguous per-rank shards
+    (strong scaling), each rank timing its own kernel (CUDA events; the max over ranks is
+    reported), then the one exchange step -- the checksum all-reduce over NCCL."""
+    import torch.distributed as dist
+    res = {}
+    nl = 10_000_000
+    first, cnt = sharding.shard(nl, rank, world)
+    rd = omprt.RSDeviceTables(gen.RSTables(), dev)
+    v = torch.empty(max(cnt, 1), dtype=torch.uint64, device=dev)
+    ck = torch.zeros(1, dtype=torch.uint64, device=dev)
+    FD = omprt.OMPRT_FLAT | omprt.OMPRT_SCHED_DYNAMIC
+    dist.barrier()
+    t = _time(lambda: omprt.omprt_rs_lookup(rd, 1070, first, cnt, v, None, 0, 128, FD), stream,
+              scrub, reps=3, warm=1)
+    ms = sharding.allreduce_max(t, dev)
+    omprt.omprt_u64_sum(v, cnt, ck)
+    sharding.allreduce_u64_sum(ck)
+    res["c4_rsbench_10M"] = {"ranks": world, "lookups_per_rank": cnt, "max_rank_ms": ms,
+                             "lookups_per_s": nl / ms * 1e3,
+                             "checksum": int(ck.cpu().numpy()[0]),
+                             "variant": "flattened, lock-step, schedule(dynamic,1); NCCL u64 "
+                                        "checksum all-reduce"}
+    ns = 32 ** 4
+    s0, sc = sharding.shard(ns, rank, world)
+    Ah, Bh = gen.su3_inputs(sc, first_site=s0)
+    At, Bt = torch.from_numpy(Ah).to(dev), torch.from_numpy(Bh).to(dev)
+    Ct = torch.empty_like(At)
+    cks = torch.zeros(1, dtype=torch.float64, device=dev)
+    dist.barrier()
+    t = _time(lambda: omprt.omprt_su3_mult(At, Bt, Ct, sc, cks, 0, 128,
+                                           omprt.OMPRT_ASSUME_OVERSUB), stream, scrub)
+    ms = sharding.allreduce_max(t, dev)
+    cks.zero_()
+    omprt.omprt_su3_mult(At, Bt, Ct, sc, cks, 0, 128, omprt.OMPRT_ASSUME_OVERSUB)
+    sharding.allreduce_f64_sum(cks)
+    res["c5_su3_32^4"] = {"ranks": world, "sites_per_rank": sc, "max_rank_ms": ms,
+                          "GBps_alg": 1152 * ns / ms / 1e6, "checksum": float(cks.item()),
+                          "variant": "one site per thread, 256-bit accesses; NCCL f64 "
+                                     "checksum all-reduce"}
+    dist.barrier()
+    return res
 
 
 def run_secondary(omprt, torch, gen, dev, stream, scrub):

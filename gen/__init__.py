@@ -41,9 +41,9 @@ def u01(seed: int, n: int, offset: int = 0) -> np.ndarray:
     return (splitmix64(seed, n, offset) >> np.uint64(11)).astype(np.float64) * (2.0 ** -53)
 
 
-def uniform(seed: int, n: int, lo: float, hi: float) -> np.ndarray:
+def uniform(seed: int, n: int, lo: float, hi: float, offset: int = 0) -> np.ndarray:
     """Doubles in [lo,hi) as lo + (hi-lo)*u01 (exact when hi-lo is a power of two)."""
-    return lo + (hi - lo) * u01(seed, n)
+    return lo + (hi - lo) * u01(seed, n, offset)
 
 
 # --------------------------------------------------------------------------------------
@@ -81,10 +81,13 @@ SEED_SU3_B = 0x5B5B5B5B
 SU3_DOUBLES_PER_SITE = 4 * 3 * 3 * 2
 
 
-def su3_inputs(n_sites: int, kind: str = "random"):
-    """kind: 'random' (U[-1,1)), 'identity' (B = I), 'third' (A = 1+0i, B = 1/3+0i)."""
+def su3_inputs(n_sites: int, kind: str = "random", first_site: int = 0):
+    """kind: 'random' (U[-1,1)), 'identity' (B = I), 'third' (A = 1+0i, B = 1/3+0i).
+    first_site: A for sites [first_site, first_site + n_sites) of the same lattice (a
+    rank's contiguous shard)."""
     if kind == "random":
-        a = uniform(SEED_SU3_A, n_sites * SU3_DOUBLES_PER_SITE, -1.0, 1.0)
+        a = uniform(SEED_SU3_A, n_sites * SU3_DOUBLES_PER_SITE, -1.0, 1.0,
+                    first_site * SU3_DOUBLES_PER_SITE)
         b = uniform(SEED_SU3_B, SU3_DOUBLES_PER_SITE, -1.0, 1.0)
     elif kind == "identity":
         a = uniform(SEED_SU3_A, n_sites * SU3_DOUBLES_PER_SITE, -1.0, 1.0)

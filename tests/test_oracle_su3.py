@@ -47,3 +47,12 @@ def test_checksum_tolerance_reference():
     C = oracle.su3_mult(A, B, n)
     re = C.reshape(-1)[0::2]
     assert abs(oracle.sum_f64(re) - math.fsum(re)) <= 1e-15 * oracle.sum_abs_f64(re)
+
+
+def test_su3_input_shards_tile_the_lattice():
+    """A rank's shard of the inputs (first_site) is the same slice of the one lattice."""
+    import gen
+    A, B = gen.su3_inputs(100)
+    for s0, n in [(0, 40), (40, 35), (75, 25)]:
+        a, b = gen.su3_inputs(n, first_site=s0)
+        assert (a == A[s0 * 72:(s0 + n) * 72]).all() and (b == B).all()

@@ -61,7 +61,8 @@ extern "C" int omprt_fini(int device) {
   cudaFree(w.pool);
   cudaFree(w.xs_buf[0]);
   cudaFree(w.xs_buf[1]);
-  cudaFree(w.xs_built);
+  cudaFree(w.xs_built[0]);
+  cudaFree(w.xs_built[1]);
   cudaFree(w.dev_ck);
   cudaFree(w.derive_tmp);
   cudaFree(w.e2e_ver);

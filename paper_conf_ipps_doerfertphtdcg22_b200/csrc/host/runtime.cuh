@@ -55,7 +55,7 @@ struct Workspace {
   size_t xs_buf_bytes = 0;
   // ... and one buffer for the tables built on the device (written and read on the compute
   // stream only, so one copy serves every step, and the L2 window stays on one range)
-  void* xs_built = nullptr;
+  void* xs_built[2] = {nullptr, nullptr};  // device-built layouts, one set per table slot
   size_t xs_built_bytes = 0;
   cudaStream_t copy_stream = nullptr;
   cudaEvent_t copy_done[2] = {nullptr, nullptr};

@@ -617,12 +617,15 @@ extern "C" int omprt_xs_run_host_steps(omprt_xs_tables h, uint64_t seed, int64_t
       accel ? al(asz[0]) + al(built16) + al(builtbr) + al(built_uni) : 0;
   if (w->xs_built_bytes < total_built) {
     OMPRT_CUDA_TRY(cudaDeviceSynchronize());
-    cudaFree(w->xs_built);
-    w->xs_built = nullptr;
+    for (int k = 0; k < 2; ++k) {
+      cudaFree(w->xs_built[k]);
+      w->xs_built[k] = nullptr;
+    }
     w->xs_built_bytes = 0;
-    if (cudaMalloc(&w->xs_built, total_built) != cudaSuccess) {
+    if (cudaMalloc(&w->xs_built[0], total_built) != cudaSuccess ||
+        cudaMalloc(&w->xs_built[1], total_built) != cudaSuccess) {
       cudaGetLastError();
-      return set_error(OMPRT_E_NOMEM, "omprt_xs_run_host_steps: cannot allocate %zu B",
+      return set_error(OMPRT_E_NOMEM, "omprt_xs_run_host_steps: cannot allocate 2 x %zu B",
                        total_built);
     }
     w->xs_built_bytes = total_built;
@@ -689,15 +692,15 @@ extern "C" int omprt_xs_run_host_steps(omprt_xs_tables h, uint64_t seed, int64_t
     d.num_nucs = (const int32_t*)put(h.num_nucs, n_num);
     d.mats = (const int32_t*)put(h.mats, n_mat);
     d.concs = (const double*)put(h.concs, n_con);
-    ok = ok && cudaEventRecord(w->copy_done[b], cs) == cudaSuccess;
     if (!ok) return set_error(OMPRT_E_CUDA, "omprt_xs_run_host_steps: H2D copy failed");
-    OMPRT_CUDA_TRY(cudaStreamWaitEvent(s, w->copy_done[b], 0));
     d.index_grid = (up16 || derive) ? nullptr : (const int32_t*)idx;
     d.bins = nullptr;
     d.index_grid16 = nullptr;
     d.brackets = nullptr;
+    // the slot's device-built layouts are made on the copy stream too, right after its
+    // H2D, so they overlap the previous step's lookups (two slots of built layouts)
     if (accel) {
-      unsigned char* bb = (unsigned char*)w->xs_built;
+      unsigned char* bb = (unsigned char*)w->xs_built[b];
       size_t bo = 0;
       int32_t* bins = (int32_t*)(bb + bo);
       bo += al(asz[0]);
@@ -709,23 +712,25 @@ extern "C" int omprt_xs_run_host_steps(omprt_xs_tables h, uint64_t seed, int64_t
         double* U = (double*)(bb + bo);
         bo += al(built_uni);
         if (int r = xs_derive(d.nuclide_grid, d.n_isotopes, d.n_gridpoints, U, i16,
-                              w->derive_tmp, w->derive_tmp_bytes, s))
+                              w->derive_tmp, w->derive_tmp_bytes, cs))
           return r;
         d.unionized = U;
       } else if (!up16) {
-        xs_build_index16<<<2048, 256, 0, s>>>(d.index_grid, i16,
-                                              (int64_t)d.n_union * d.n_isotopes);
+        xs_build_index16<<<2048, 256, 0, cs>>>(d.index_grid, i16,
+                                               (int64_t)d.n_union * d.n_isotopes);
       }
-      xs_build_bins<<<1024, 256, 0, s>>>(d.unionized, (int32_t)d.n_union, log2_bins, bins);
+      xs_build_bins<<<1024, 256, 0, cs>>>(d.unionized, (int32_t)d.n_union, log2_bins, bins);
       if (!upbr)
-        xs_build_brackets<<<2048, 256, 0, s>>>(d.nuclide_grid, brk, d.n_isotopes,
-                                               d.n_gridpoints);
+        xs_build_brackets<<<2048, 256, 0, cs>>>(d.nuclide_grid, brk, d.n_isotopes,
+                                                d.n_gridpoints);
       if (int r = check_launch("xs_build_accel")) return r;
       d.bins = bins;
       d.index_grid16 = i16;
       d.brackets = brk;
       d.log2_bins = log2_bins;
     }
+    OMPRT_CUDA_TRY(cudaEventRecord(w->copy_done[b], cs));
+    OMPRT_CUDA_TRY(cudaStreamWaitEvent(s, w->copy_done[b], 0));
     if (flags & OMPRT_XS_FLAT) {
       // flattened: per-lookup verification + K11 sum (the fused flat kernel spills: its
       // extra live state does not fit the 64 registers of 4 teams per SM)

@@ -30,6 +30,12 @@ def main():
     omprt.omprt_cuda_axpy_sum(n, x, bt, ct, at, s, 8, 128)
     omprt.omprt_spmd_axpy_sum_chunked(n, 4, x, bt, ct, at, s, 8, 128)
     omprt.omprt_spmd_axpy_sum(n, x, bt, ct, at, s, 128, 128, A)
+    D = omprt.OMPRT_SCHED_DYNAMIC  # schedule(dynamic, C): team-shared chunk counter
+    own = torch.empty(n, dtype=torch.int32, device=dev)
+    cnt = torch.zeros(n, dtype=torch.int32, device=dev)
+    omprt.omprt_spmd_axpy_sum_chunked(n, 3, x, bt, ct, at, s, 8, 128,
+                                      D | omprt.OMPRT_RECORD_OWNER, own, cnt)
+    omprt.omprt_cuda_axpy_sum_chunked(n, 3, x, bt, ct, at, s, 8, 128, D)
     # C2: all state machines, stack placements, SPMDized, deglobalized, postlogue
     T = 16
     inp = torch.from_numpy(gen.generic_inputs(T, 256)).to(dev)
@@ -53,12 +59,28 @@ def main():
     omprt.omprt_xs_lookup(d, 1070, 0, m, None, ck, 0, 256, A | omprt.OMPRT_FUSED_REDUCTION)
     omprt.omprt_cuda_xs_lookup(d, 1070, 0, m, ver, None, 0, 256, 0)
     omprt.omprt_u64_sum(ver, m, ck)
+    # flattened (static, dynamic), compact index grid, fused, with the L2 window
+    F = omprt.OMPRT_XS_FLAT
+    omprt.omprt_l2_set_aside(1 << 40)
+    dc = omprt.XSDeviceTables(t, dev, accel=True, compact=True)
+    for fl in (F, F | D):
+        for tab in (d, dc):
+            omprt.omprt_xs_lookup(tab, 1070, 0, m, ver, None, 3, 256, fl)
+            omprt.omprt_xs_lookup(tab, 1070, 0, m, None, ck, 3, 256,
+                                  fl | omprt.OMPRT_FUSED_REDUCTION)
+            omprt.omprt_cuda_xs_lookup(tab, 1070, 0, m, ver, None, 3, 256, fl)
+    torch.cuda.synchronize()
+    omprt.omprt_l2_set_aside(0)
     # C4 (reduced tables)
     rs = gen.RSTables(n_nuclides=355, avg_poles=20, avg_windows=4)
     rd = omprt.RSDeviceTables(rs, dev)
     v = torch.empty(512, dtype=torch.uint64, device=dev)
     omprt.omprt_rs_lookup(rd, 1070, 0, 512, v, None, 0, 128, A)
     omprt.omprt_cuda_rs_lookup(rd, 1070, 0, 512, v, None, 0, 128, 0)
+    mac = torch.empty(512 * 4, dtype=torch.float64, device=dev)
+    for fl in (F, F | D):  # flattened lock-step (static / dynamic)
+        omprt.omprt_rs_lookup(rd, 1070, 0, 512, v, mac, 2, 128, fl)
+        omprt.omprt_cuda_rs_lookup(rd, 1070, 0, 512, v, None, 2, 128, fl)
     # C5
     ns = 1024
     Ah, Bh = gen.su3_inputs(ns)

@@ -576,6 +576,12 @@ def run_secondary(omprt, torch, gen, dev, stream, scrub):
     res["c5_su3_32^4_warp_staged"] = {"rt_ms": t_rw, "twin_ms": t_tww,
                                       "overhead": t_rw / t_tww - 1,
                                       "GBps_alg": 1152 * ns / t_rw / 1e6}
+    TT = omprt.OMPRT_TMA_TILED
+    t_rtt = _time(lambda: omprt.omprt_su3_mult(At, Bt, Ct, ns, ck, 0, 128, TT), stream, scrub)
+    t_twt = _time(lambda: omprt.omprt_cuda_su3_mult(At, Bt, Ct, ns, ck, 0, 128, TT), stream, scrub)
+    res["c5_su3_32^4_tma_tiled"] = {"rt_ms": t_rtt, "twin_ms": t_twt,
+                                    "overhead": t_rtt / t_twt - 1,
+                                    "GBps_alg": 1152 * ns / t_rtt / 1e6}
     res["c5_su3_32^4"] = {"rt_ms": t_rt, "twin_ms": t_tw, "overhead": t_rt / t_tw - 1,
                           "GBps_alg": 1152 * ns / t_rt / 1e6, "GFLOPs": 864 * ns / t_rt / 1e6}
     return res

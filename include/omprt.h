@@ -117,6 +117,13 @@ extern "C" {
  * omprt_spmd_axpy_sum_chunked (C = chunk) and, with OMPRT_FLAT, omprt_xs_lookup /
  * omprt_rs_lookup and their twins (C fixed per kernel). */
 #define OMPRT_SCHED_DYNAMIC (1u << 17)
+/* omprt_su3_mult / omprt_cuda_su3_mult: the site loop on a persistent grid with each warp's
+ * 32 consecutive site records moved by ONE 2-D TMA tensor copy in (box [32][74] doubles:
+ * the 2 columns past a 576 B record are zero-filled, giving padded 592 B shared-memory
+ * slots) and one out (out-of-tensor columns are not written); double buffered per warp.
+ * Not combined with OMPRT_ASSUME_OVERSUB, OMPRT_TMA_STAGED or OMPRT_WARP_STAGED.  A and C
+ * 16 B aligned. */
+#define OMPRT_TMA_TILED (1u << 18)
 
 /* ---- runtime lifecycle ------------------------------------------------------------- */
 typedef struct {

@@ -67,6 +67,26 @@ __device__ __forceinline__ void fence_proxy_async_smem() {
   asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
 }
 
+// ---- tensor (tiled) TMA copies through a CUtensorMap (sm_90+; SASS UTMALDG / UTMASTG) ----
+// `tmap` is the generic address of a __grid_constant__ CUtensorMap kernel parameter.
+// 2-D box at element coordinates (x, y) -> shared memory, completion counted on `bar`
+__device__ __forceinline__ void tensor_load_2d(void* dst_smem, const void* tmap, int32_t x,
+                                               int32_t y, uint64_t* bar) {
+  asm volatile(
+      "cp.async.bulk.tensor.2d.shared::cluster.global.tile.mbarrier::complete_tx::bytes"
+      " [%0], [%1, {%2, %3}], [%4];" ::"r"(smem_addr(dst_smem)),
+      "l"(tmap), "r"(x), "r"(y), "r"(smem_addr(bar))
+      : "memory");
+}
+// shared memory -> the 2-D box at (x, y), in this thread's bulk group (elements of the box
+// outside the tensor are not written)
+__device__ __forceinline__ void tensor_store_2d(const void* tmap, int32_t x, int32_t y,
+                                                const void* src_smem) {
+  asm volatile("cp.async.bulk.tensor.2d.global.shared::cta.tile.bulk_group [%0, {%1, %2}], [%3];"
+               ::"l"(tmap), "r"(x), "r"(y), "r"(smem_addr(src_smem))
+               : "memory");
+}
+
 // ---- per-thread 16 B asynchronous global->shared copies (sm_80+; SASS LDGSTS) ----------
 // .cg: cached in L2 only (streamed records are not re-read through L1).
 __device__ __forceinline__ void cp_async16(void* smem, const void* gmem) {

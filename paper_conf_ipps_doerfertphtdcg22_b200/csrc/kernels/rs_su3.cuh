@@ -294,6 +294,8 @@ OMPRT_REGISTER_KERNEL(cuda_su3_twin, cuda_su3_twin<true>)
 inline int su3_staged_launch(bool twin, bool warp, const double* A, const double* B, double* Cm,
                              int64_t n, double* ck, int32_t teams, Workspace* w,
                              cudaStream_t s);
+inline int su3_tiled_launch(bool twin, const double* A, const double* B, double* Cm, int64_t n,
+                            double* ck, int32_t teams, Workspace* w, cudaStream_t s);
 
 inline int su3_validate(const double* A, const double* B, double* Cm, int64_t n,
                         int32_t& teams, int32_t threads, uint32_t flags, double* ck,
@@ -380,6 +382,15 @@ extern "C" int omprt_su3_mult(const double* A, const double* B, double* Cm, int6
   using namespace omprt_kernels;
   Workspace* w;
   if (int r = current_ws(&w)) return r;
+  if (flags & OMPRT_TMA_TILED) {
+    OMPRT_CHECK_ARG(!(flags & (OMPRT_ASSUME_OVERSUB | OMPRT_TMA_STAGED | OMPRT_WARP_STAGED)),
+                    "OMPRT_TMA_TILED: persistent grid, exclusive with the other stagings");
+    int32_t tm = 1;
+    if (int r = su3_validate(A, B, Cm, n_sites, tm, threads, 0, checksum_inout, w)) return r;
+    if (n_sites == 0) return OMPRT_OK;
+    return su3_tiled_launch(false, A, B, Cm, n_sites, checksum_inout, teams, w,
+                            as_stream(stream));
+  }
   if (flags & (OMPRT_TMA_STAGED | OMPRT_WARP_STAGED)) {
     OMPRT_CHECK_ARG(threads == kSU3Threads && !(flags & OMPRT_ASSUME_OVERSUB),
                     "the staged variants run a persistent grid (no assumption)");
@@ -418,6 +429,13 @@ extern "C" int omprt_cuda_su3_mult(const double* A, const double* B, double* Cm,
   if (int r = current_ws(&w)) return r;
   int32_t tm = 0;
   if (int r = su3_validate(A, B, Cm, n_sites, tm, threads, 0, checksum_inout, w)) return r;
+  if (flags & OMPRT_TMA_TILED) {
+    OMPRT_CHECK_ARG(!(flags & (OMPRT_TMA_STAGED | OMPRT_WARP_STAGED)),
+                    "OMPRT_TMA_TILED is exclusive with the other stagings");
+    if (n_sites == 0) return OMPRT_OK;
+    return su3_tiled_launch(true, A, B, Cm, n_sites, checksum_inout, teams, w,
+                            as_stream(stream));
+  }
   if (flags & (OMPRT_TMA_STAGED | OMPRT_WARP_STAGED)) {
     OMPRT_CHECK_ARG((flags & OMPRT_TMA_STAGED) == 0 || (flags & OMPRT_WARP_STAGED) == 0,
                     "OMPRT_TMA_STAGED and OMPRT_WARP_STAGED are exclusive");

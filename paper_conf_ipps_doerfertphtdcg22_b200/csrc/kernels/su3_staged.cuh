@@ -5,6 +5,9 @@
 // (omprt/device/staging.cuh), instead of 32-line-wide strided global accesses.  The twin runs
 // the same per-thread double-buffered bulk-copy pipeline, written by hand.
 #pragma once
+#include <cuda.h>
+#include <cudaTypedefs.h>
+
 #include "../common/ptx_tma.cuh"
 #include "../host/runtime.cuh"
 #include "../omprt/device/staging.cuh"
@@ -235,6 +238,146 @@ __global__ void __launch_bounds__(kSU3WarpThreads, 1)
 
 OMPRT_REGISTER_KERNEL(omprt_su3_wstaged_rt, omprt_su3_wstaged_rt<SU3StagedTraits, true>)
 OMPRT_REGISTER_KERNEL(cuda_su3_wstaged_twin, cuda_su3_wstaged_twin<true>)
+
+// ---- TMA tensor tiles (OMPRT_TMA_TILED): one 2-D tensor copy per warp tile in and out ----
+// A and C as tensors [n_sites][72] of doubles; boxes [32][74]: the two columns past the
+// record are zero-filled on the load (592 B padded slots) and skipped on the store
+// (omprt/device/staging.cuh distribute_parallel_for_tma_tiles).  6 warps per team, one
+// team per SM: 6 x 2 x 32 x 592 B + barriers = 227.4 KB of shared memory.
+#ifndef OMPRT_SU3_TILED_WARPS
+#define OMPRT_SU3_TILED_WARPS 6
+#define OMPRT_SU3_TILED_BUFFERS 2
+#endif
+constexpr int kSU3TiledThreads = 32 * OMPRT_SU3_TILED_WARPS;
+constexpr unsigned kSU3TiledBuffers = OMPRT_SU3_TILED_BUFFERS;
+constexpr unsigned kSU3SlotDoubles = kSU3Slot / 8;  // 74
+
+template <class Tr, bool Checksum>
+__global__ void __launch_bounds__(kSU3TiledThreads, 1)
+    omprt_su3_tiled_rt(const __grid_constant__ CUtensorMap tin,
+                       const __grid_constant__ CUtensorMap tout, const double2* __restrict__ B,
+                       typename Tr::Idx n_sites, double* checksum, double* partials,
+                       unsigned* ticket) {
+  using Idx = typename Tr::Idx;
+  Team<Tr> team = init<Tr>();
+  double acc = 0.0;
+  distribute_parallel_for_tma_tiles<Tr, kSU3Slot, kSU3TiledBuffers>(
+      team, n_sites, &tin, &tout,
+      [&](Idx, unsigned char* slot) { acc += su3_site_slot(slot, B); });
+  if constexpr (Checksum)
+    league_reduce(team, team_reduce_to_main(team, acc, Plus{}), Plus{}, checksum, partials,
+                  ticket);
+}
+
+// Bare CUDA twin: the same per-warp tensor-tile pipeline, by hand.
+template <bool Checksum>
+__global__ void __launch_bounds__(kSU3TiledThreads, 1)
+    cuda_su3_tiled_twin(const __grid_constant__ CUtensorMap tin,
+                        const __grid_constant__ CUtensorMap tout, const double2* __restrict__ B,
+                        int32_t n_sites, double* checksum, double* partials, unsigned* ticket) {
+  constexpr uint32_t kBox = 32u * kSU3Slot;
+  constexpr unsigned K = kSU3TiledBuffers;
+  extern __shared__ __align__(128) unsigned char smem[];
+  const unsigned nt = blockDim.x, t = threadIdx.x, lane = t & 31u, w0 = t & ~31u;
+  unsigned char* const buf = smem + w0 * kSU3Slot;
+  const unsigned bstride = nt * kSU3Slot;
+  uint64_t* bar = reinterpret_cast<uint64_t*>(smem + K * nt * kSU3Slot) + K * (t >> 5);
+  if (lane == 0) {
+    for (unsigned j = 0; j < K; ++j) tma::mbar_init(bar + j, 1);
+    tma::fence_mbar_init();
+  }
+  __syncwarp();
+  const int32_t stride = gridDim.x * nt;
+  const int32_t first = blockIdx.x * nt + w0;
+  double acc = 0.0;
+  if (lane == 0)
+    for (unsigned j = 0; j + 1 < K; ++j)
+      if (first + (int32_t)j * stride < n_sites) {
+        tma::mbar_arrive_expect_tx(bar + j, kBox);
+        tma::tensor_load_2d(buf + j * bstride, &tin, 0, first + j * stride, bar + j);
+      }
+  unsigned phases = 0, j = 0;
+  for (int32_t base = first; base < n_sites; base += stride) {
+    const int32_t ahead = base + (int32_t)(K - 1) * stride;
+    const unsigned ja = j == 0 ? K - 1 : j - 1;
+    if (ahead < n_sites && lane == 0) {
+      tma::bulk_wait_read<0>();
+      tma::mbar_arrive_expect_tx(bar + ja, kBox);
+      tma::tensor_load_2d(buf + ja * bstride, &tin, 0, ahead, bar + ja);
+    }
+    tma::mbar_wait(bar + j, (phases >> j) & 1u);
+    phases ^= 1u << j;
+    unsigned char* const cur = buf + j * bstride;
+    if (base + (int32_t)lane < n_sites) acc += su3_site_slot(cur + lane * kSU3Slot, B);
+    tma::fence_proxy_async_smem();
+    __syncwarp();
+    if (lane == 0) {
+      tma::tensor_store_2d(&tout, 0, base, cur);
+      tma::bulk_commit();
+    }
+    j = j + 1 == K ? 0 : j + 1;
+  }
+  if (lane == 0) tma::bulk_wait<0>();
+  if constexpr (Checksum) twin_ticket_sum(acc, checksum, partials, ticket);
+}
+
+OMPRT_REGISTER_KERNEL(omprt_su3_tiled_rt, omprt_su3_tiled_rt<SU3StagedTraits, true>)
+OMPRT_REGISTER_KERNEL(cuda_su3_tiled_twin, cuda_su3_tiled_twin<true>)
+
+// CUtensorMap of a [n][72]-double AoS array with [32][74] boxes (driver entry point fetched
+// once through the runtime; no libcuda link dependency)
+inline int su3_tensor_map(CUtensorMap* m, const double* base, int64_t n) {
+  static PFN_cuTensorMapEncodeTiled_v12000 enc = nullptr;
+  if (!enc) {
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", (void**)&enc, cudaEnableDefault, &q) !=
+            cudaSuccess ||
+        q != cudaDriverEntryPointSuccess || !enc) {
+      cudaGetLastError();
+      enc = nullptr;
+      return set_error(OMPRT_E_CUDA, "cuTensorMapEncodeTiled is not available");
+    }
+  }
+  const cuuint64_t dims[2] = {kSU3Rec / 8, (cuuint64_t)n};
+  const cuuint64_t strides[1] = {kSU3Rec};
+  const cuuint32_t box[2] = {kSU3SlotDoubles, 32}, es[2] = {1, 1};
+  const CUresult r = enc(m, CU_TENSOR_MAP_DATA_TYPE_FLOAT64, 2, const_cast<double*>(base), dims,
+                         strides, box, es, CU_TENSOR_MAP_INTERLEAVE_NONE,
+                         CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                         CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  if (r != CUDA_SUCCESS) return set_error(OMPRT_E_CUDA, "cuTensorMapEncodeTiled failed (%d)", (int)r);
+  return OMPRT_OK;
+}
+
+inline int su3_tiled_launch(bool twin, const double* A, const double* B, double* Cm, int64_t n,
+                            double* ck, int32_t teams, Workspace* w, cudaStream_t s) {
+  OMPRT_CHECK_ARG(((uintptr_t)A | (uintptr_t)Cm) % 16 == 0, "A and C must be 16 B aligned");
+  CUtensorMap tin, tout;
+  if (int r = su3_tensor_map(&tin, A, n)) return r;
+  if (int r = su3_tensor_map(&tout, Cm, n)) return r;
+  const uint32_t smem = tma_tiles_smem_bytes<kSU3Slot, kSU3TiledBuffers>(kSU3TiledThreads);
+  int dev = 0, sms = 148;
+  cudaGetDevice(&dev);
+  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  if (teams <= 0) teams = sms;
+  OMPRT_CHECK_ARG(!ck || (uint64_t)teams <= w->opt.max_teams, "teams exceed max_teams");
+  OMPRT_CHECK_ARG(n + 2 * (int64_t)teams * kSU3TiledThreads < INT32_MAX, "n_sites too large");
+  auto* b2 = (const double2*)B;
+  double* p = (double*)w->partials;
+  unsigned* tk = w->tickets + 3;
+  const int32_t nn = (int32_t)n;
+  auto go = [&](auto k) -> int {
+    OMPRT_CUDA_TRY(cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
+    k<<<teams, kSU3TiledThreads, smem, s>>>(tin, tout, b2, nn, ck, p, tk);
+    return OMPRT_OK;
+  };
+  int r;
+  if (twin) r = ck ? go(cuda_su3_tiled_twin<true>) : go(cuda_su3_tiled_twin<false>);
+  else r = ck ? go(omprt_su3_tiled_rt<SU3StagedTraits, true>)
+              : go(omprt_su3_tiled_rt<SU3StagedTraits, false>);
+  if (r) return r;
+  return check_launch(twin ? "cuda_su3_tiled_twin" : "omprt_su3_tiled_rt");
+}
 
 // persistent geometry: one team per SM.  warp = false: per-thread bulk copies (128 threads,
 // 153 KB of slots + barriers); warp = true: warp-cooperative cp.async (192 threads, 222 KB).

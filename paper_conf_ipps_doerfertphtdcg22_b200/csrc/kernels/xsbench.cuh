@@ -461,10 +461,8 @@ extern "C" int omprt_xs_lookup(omprt_xs_tables t, uint64_t seed, int64_t first, 
   if (flags & OMPRT_XS_FLAT) {
     const bool smem = xs_mats_fit_smem(t);
     const FlatLaunch L = flat_launch(t, teams, threads, flags, w, s);
-    cudaError_t e;
-    e = xs_flat_dispatch<false>(flags, fused, smem, xs_has_compact(t), L.cfg, d, seed, first,
-                                n, verification, ck, p, tk);
-    (void)e;
+    xs_flat_dispatch<false>(flags, fused, smem, xs_has_compact(t), L.cfg, d, seed, first, n,
+                            verification, ck, p, tk);
     return check_launch("omprt_xs_flat_rt");
   }
 #define OMPRT_XS(TR, F, A) \

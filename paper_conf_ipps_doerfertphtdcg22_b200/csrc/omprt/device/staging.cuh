@@ -175,4 +175,89 @@ __device__ __forceinline__ void distribute_parallel_for_warp_staged(Team<Tr>& te
   }
 }
 
+// ---- TMA tensor tiles ----------------------------------------------------------------
+// The records of a warp's 32 consecutive iterations (Fig. 5) as ONE 2-D tensor copy: the
+// records are a tensor [n][kRecBytes / 8] of doubles, the box is [32][kSlotBytes / 8].  The
+// box's extra columns lie outside the tensor, so TMA zero-fills them on the load -- every
+// record lands in its own padded kSlotBytes slot (conflict-free per-lane shared-memory
+// access) -- and skips them on the store.  One lane of the warp issues the copies; each
+// lane runs body(i, slot) on its record in place; the warp's tiles are double buffered (the
+// next tile's load is in flight while the body runs).  No team barrier; the tensor maps
+// (tmap_in, tmap_out: generic addresses of __grid_constant__ CUtensorMap parameters) are
+// encoded on the host.  Needs tma_tiles_smem_bytes<kSlotBytes>(team_size) bytes of dynamic
+// shared memory and a team size that is a multiple of 32.
+template <unsigned kSlotBytes, unsigned kBuffers = 2>
+__host__ __device__ constexpr uint32_t tma_tiles_smem_bytes(uint32_t team_size) {
+  return team_size * kBuffers * kSlotBytes + (team_size / 32u) * kBuffers * 8u;
+}
+
+template <class Tr, unsigned kSlotBytes, unsigned kBuffers = 2, class Body>
+__device__ __forceinline__ void distribute_parallel_for_tma_tiles(Team<Tr>& team,
+                                                                  typename Tr::Idx n,
+                                                                  const void* tmap_in,
+                                                                  const void* tmap_out,
+                                                                  Body&& body) {
+  using Idx = typename Tr::Idx;
+  static_assert(kSlotBytes % 16 == 0, "TMA boxes have 16 B multiples per row");
+  static_assert(kBuffers >= 2 && kBuffers <= 4, "2..4 tile buffers per warp");
+  constexpr uint32_t kBox = 32u * kSlotBytes;  // bytes a tile load writes (zero fill included)
+  OMPRT_TRACE(Tr, "distribute_parallel_for_tma_tiles");
+  extern __shared__ __align__(128) unsigned char omprt_stage_smem[];
+  const uint32_t nt = (uint32_t)team.team_size, t = (uint32_t)team.thread_num;
+  OMPRT_ASSERT(Tr, nt % 32u == 0, "TMA tiles need whole warps");
+  const uint32_t lane = t & 31u, w0 = t & ~31u;
+  // buffer j of this warp: omprt_stage_smem + (j * nt + w0) * kSlotBytes
+  unsigned char* const buf = omprt_stage_smem + w0 * kSlotBytes;
+  const uint32_t buf_stride = nt * kSlotBytes;
+  uint64_t* const bar = reinterpret_cast<uint64_t*>(omprt_stage_smem + kBuffers * nt * kSlotBytes) +
+                        kBuffers * (t >> 5);
+  if (lane == 0) {
+#pragma unroll
+    for (unsigned j = 0; j < kBuffers; ++j) tma::mbar_init(bar + j, 1);
+    tma::fence_mbar_init();
+  }
+  __syncwarp();
+  const Idx total = (Idx)gridDim.x * (Idx)nt;
+  const Idx first = (Idx)blockIdx.x * (Idx)nt + (Idx)w0;  // the warp's first iteration
+  if (Tr::assume_teams_oversub) OMPRT_ASSERT(Tr, n <= total, "oversubscription assumption violated");
+  // prologue: the warp's first kBuffers - 1 tiles in flight
+  if (lane == 0) {
+#pragma unroll
+    for (unsigned j = 0; j + 1 < kBuffers; ++j) {
+      const Idx b0 = first + (Idx)j * total;
+      if (b0 < n && (j == 0 || !Tr::assume_teams_oversub)) {
+        tma::mbar_arrive_expect_tx(bar + j, kBox);
+        tma::tensor_load_2d(buf + j * buf_stride, tmap_in, 0, (int32_t)b0, bar + j);
+      }
+    }
+  }
+  uint32_t phases = 0;  // bit j: parity of buffer j's next completion
+  uint32_t j = 0;       // this tile's buffer
+  for (Idx base = first; base < n; base += total) {
+    // the tile kBuffers - 1 ahead goes into the buffer the previous tile used, once that
+    // tile's store has read it
+    const Idx ahead = base + (Idx)(kBuffers - 1) * total;
+    const uint32_t ja = j == 0 ? kBuffers - 1 : j - 1;
+    if (!Tr::assume_teams_oversub && ahead < n && lane == 0) {
+      tma::bulk_wait_read<0>();
+      tma::mbar_arrive_expect_tx(bar + ja, kBox);
+      tma::tensor_load_2d(buf + ja * buf_stride, tmap_in, 0, (int32_t)ahead, bar + ja);
+    }
+    tma::mbar_wait(bar + j, (phases >> j) & 1u);
+    phases ^= 1u << j;
+    unsigned char* const cur = buf + j * buf_stride;
+    const Idx iv = base + (Idx)lane;
+    if (iv < n) body(iv, cur + lane * kSlotBytes);
+    tma::fence_proxy_async_smem();  // this lane's slot writes -> the async proxy
+    __syncwarp();
+    if (lane == 0) {
+      tma::tensor_store_2d(tmap_out, 0, (int32_t)base, cur);
+      tma::bulk_commit();
+    }
+    if (Tr::assume_teams_oversub) break;
+    j = j + 1 == kBuffers ? 0 : j + 1;
+  }
+  if (lane == 0) tma::bulk_wait<0>();  // the stores are complete before the warp exits
+}
+
 }  // namespace omprt

@@ -47,6 +47,8 @@ def main(which):
                     ("rt_staged", omprt.omprt_su3_mult, TS),
                     ("twin_staged", omprt.omprt_cuda_su3_mult, TS),
                     ("rt_wstaged", omprt.omprt_su3_mult, omprt.OMPRT_WARP_STAGED),
+                    ("rt_tiled", omprt.omprt_su3_mult, omprt.OMPRT_TMA_TILED),
+                    ("twin_tiled", omprt.omprt_cuda_su3_mult, omprt.OMPRT_TMA_TILED),
                     ("twin_wstaged", omprt.omprt_cuda_su3_mult, omprt.OMPRT_WARP_STAGED)]
         for name, fn, fl in variants:
             res[f"su3_{name}"] = {"ms": []}

@@ -25,6 +25,7 @@ PAIRS = [
     ("omprt_xs_flat_rt_fused", "cuda_xs_flat_twin_fused", True),
     ("omprt_su3_staged_rt", "cuda_su3_staged_twin", True),
     ("omprt_su3_wstaged_rt", "cuda_su3_wstaged_twin", True),
+    ("omprt_su3_tiled_rt", "cuda_su3_tiled_twin", True),
     ("omprt_rs_flat_rt", "cuda_rs_flat_twin", True),
     ("omprt_rs_dflat_rt", "cuda_rs_dflat_twin", True),
     ("omprt_axpy_dyn_rt", "cuda_axpy_dyn_twin", True),

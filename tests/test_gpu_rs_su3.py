@@ -105,13 +105,14 @@ def _su3(rt, fn, A, B, n, flags=0):
 
 @pytest.mark.parametrize("n", [8 ** 4, 8 ** 4 + 5, 32 ** 4])
 @pytest.mark.parametrize("variant", ["rt", "rt_loop", "twin", "rt_staged", "twin_staged",
-                                     "rt_wstaged", "twin_wstaged"])
+                                     "rt_wstaged", "twin_wstaged", "rt_tiled", "twin_tiled"])
 def test_su3_bit_exact(rt, n, variant):
     A, B = gen.su3_inputs(n)
     fn = rt.omprt_cuda_su3_mult if variant.startswith("twin") else rt.omprt_su3_mult
     flags = {"rt": rt.OMPRT_ASSUME_OVERSUB, "rt_loop": 0, "twin": 0,
              "rt_staged": rt.OMPRT_TMA_STAGED, "twin_staged": rt.OMPRT_TMA_STAGED,
-             "rt_wstaged": rt.OMPRT_WARP_STAGED, "twin_wstaged": rt.OMPRT_WARP_STAGED}[variant]
+             "rt_wstaged": rt.OMPRT_WARP_STAGED, "twin_wstaged": rt.OMPRT_WARP_STAGED,
+             "rt_tiled": rt.OMPRT_TMA_TILED, "twin_tiled": rt.OMPRT_TMA_TILED}[variant]
     C, ck = _su3(rt, fn, A, B, n, flags)
     Cref = oracle.su3_mult(A, B, n, threads=os.cpu_count() or 1)
     assert (C == Cref).all()
@@ -119,7 +120,7 @@ def test_su3_bit_exact(rt, n, variant):
     assert abs(ck - oracle.sum_f64(re)) <= 1e-12 * oracle.sum_abs_f64(re)
 
 
-@pytest.mark.parametrize("flag", ["OMPRT_TMA_STAGED", "OMPRT_WARP_STAGED"])
+@pytest.mark.parametrize("flag", ["OMPRT_TMA_STAGED", "OMPRT_WARP_STAGED", "OMPRT_TMA_TILED"])
 @pytest.mark.parametrize("teams", [1, 3, 148])
 def test_su3_staged_geometries(rt, flag, teams):
     """Few persistent teams (many tiles per warp, both buffers cycling) and a ragged last
@@ -138,9 +139,31 @@ def test_su3_staged_geometries(rt, flag, teams):
 def test_su3_staged_flags_exclusive(rt):
     A = torch.zeros(72 * 64, dtype=torch.float64, device=DEV)
     B = torch.zeros(72, dtype=torch.float64, device=DEV)
-    both = rt.OMPRT_TMA_STAGED | rt.OMPRT_WARP_STAGED
-    with pytest.raises(Exception):
-        rt.omprt_su3_mult(A, B, A, 64, None, 0, 128, both)
+    for both in (rt.OMPRT_TMA_STAGED | rt.OMPRT_WARP_STAGED,
+                 rt.OMPRT_TMA_TILED | rt.OMPRT_WARP_STAGED,
+                 rt.OMPRT_TMA_TILED | rt.OMPRT_ASSUME_OVERSUB):
+        with pytest.raises(Exception):
+            rt.omprt_su3_mult(A, B, A, 64, None, 0, 128, both)
+
+
+def test_su3_tma_tiled_tail_and_sass(rt):
+    """The ragged last tile: the box rows past n_sites are zero-filled on the load and not
+    written on the store (the C buffer's NaN guard past the last site survives), for
+    every tail length; and the kernel really moves data with tensor TMA (UTMALDG/UTMASTG)."""
+    for n in (1, 31, 33, 6 * 32 * 148 + 5):
+        A, B = gen.su3_inputs(n)
+        At, Bt = torch.from_numpy(A).to(DEV), torch.from_numpy(B).to(DEV)
+        Ct = torch.full((n * 72 + 4 * 72,), float("nan"), dtype=torch.float64, device=DEV)
+        ck = torch.zeros(1, dtype=torch.float64, device=DEV)
+        rt.omprt_su3_mult(At, Bt, Ct, n, ck, 0, 128, rt.OMPRT_TMA_TILED)
+        torch.cuda.synchronize()
+        C = Ct.cpu().numpy()
+        Cref = oracle.su3_mult(A, B, n)
+        assert (C[:n * 72] == Cref).all() and np.isnan(C[n * 72:]).all()
+    import subprocess
+    so = os.path.join(os.path.dirname(rt.__file__), "libomprt.so")
+    sass = subprocess.run(["cuobjdump", "-sass", so], capture_output=True, text=True).stdout
+    assert "UTMALDG" in sass and "UTMASTG" in sass
 
 
 def test_su3_pins_on_gpu(rt):

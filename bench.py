@@ -504,6 +504,13 @@ def run_secondary(omprt, torch, gen, dev, stream, scrub):
     t_tw = _time(lambda: omprt.omprt_cuda_axpy_sum(n, x, bt, ct, at, s, 8, 128), stream, scrub)
     res["c1_axpy_sum_8x128"] = {"rt_ms": t_rt, "twin_ms": t_tw, "overhead": t_rt / t_tw - 1,
                                 "GBps_alg": 24 * n / t_rt / 1e6}
+    # the same loop, operands streamed by 2-D TMA boxes (Fig. 5 assignment kept)
+    TS_ = omprt.OMPRT_TMA_STREAM
+    t_rt = _time(lambda: omprt.omprt_spmd_axpy_sum(n, x, bt, ct, at, s, 8, 128, TS_), stream, scrub)
+    t_tw = _time(lambda: omprt.omprt_cuda_axpy_sum(n, x, bt, ct, at, s, 8, 128, TS_), stream, scrub)
+    res["c1_axpy_sum_8x128_tma_stream"] = {"rt_ms": t_rt, "twin_ms": t_tw,
+                                           "overhead": t_rt / t_tw - 1,
+                                           "GBps_alg": 24 * n / t_rt / 1e6}
     # NEXT f3: the same loop with schedule(static, 4): 256-bit chunk accesses
     t_rt = _time(lambda: omprt.omprt_spmd_axpy_sum_chunked(n, 4, x, bt, ct, at, s, 8, 128),
                  stream, scrub)

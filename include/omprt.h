@@ -124,6 +124,13 @@ extern "C" {
  * Not combined with OMPRT_ASSUME_OVERSUB, OMPRT_TMA_STAGED or OMPRT_WARP_STAGED.  A and C
  * 16 B aligned. */
 #define OMPRT_TMA_TILED (1u << 18)
+/* omprt_spmd_axpy_sum / omprt_cuda_axpy_sum: the Fig. 5 loop with its operands moved by 2-D
+ * TMA boxes -- b, c, a viewed as [n / (T*N)][T*N] matrices (row = trip, column = global
+ * thread), each team streaming its N columns 16 trips per box, 4 boxes per array in
+ * flight; the trailing partial trip from global memory.  Same iteration -> thread map and
+ * per-thread order as Fig. 5 (a[] and the sum bit-identical).  threads <= 256 and a
+ * multiple of 32; arrays 16 B aligned; no OMPRT_ASSUME_OVERSUB / OMPRT_DEBUG_BUILD. */
+#define OMPRT_TMA_STREAM (1u << 19)
 
 /* ---- runtime lifecycle ------------------------------------------------------------- */
 typedef struct {

@@ -2,7 +2,14 @@
 //   for (i = 0; i < n; ++i) { a[i] = x*b[i] + c[i]; sum += a[i]; }
 // runtime-driven (omprt) and bare-CUDA twin.  a[i] = fma(x, b[i], c[i]).
 #pragma once
+#include <cuda.h>
+#include <cudaTypedefs.h>
+
+#include <algorithm>
+#include <type_traits>
+
 #include "../host/runtime.cuh"
+#include "../omprt/device/staging.cuh"
 
 namespace omprt_kernels {
 
@@ -109,6 +116,240 @@ __global__ void __launch_bounds__(1024)
   }
 }
 
+// ---- OMPRT_TMA_STREAM: the same loop with its operands streamed by 2-D TMA boxes --------
+// (omprt/device/staging.cuh distribute_parallel_for_tma_stream): b, c and a viewed as
+// [n / (T*N)][T*N] matrices, team b's columns [b*N, (b+1)*N) moved kAxRows trips at a time,
+// kAxStages boxes per array in flight.  Same iterations per thread in the same order as
+// Fig. 5, so a[] and the sum are bit-identical to omprt_axpy_rt.  (8 teams: the config's
+// 8 SMs must each keep ~100 KB in flight to approach their share of HBM bandwidth.)
+#ifndef OMPRT_AXPY_TMA_STAGES
+#define OMPRT_AXPY_TMA_STAGES 6
+#define OMPRT_AXPY_TMA_STORE 0
+#endif
+// rows per box: 2048 / threads; stages x (2 or 3 arrays) x 16 KB <= 227 KB
+constexpr unsigned kAxStages = OMPRT_AXPY_TMA_STAGES;
+constexpr bool kAxTmaStore = OMPRT_AXPY_TMA_STORE;  // a[] through TMA stores, or direct
+struct AxpyMaps {
+  CUtensorMap m[3];  // b, c (loads), a (store)
+};
+
+template <class Tr, bool Rec, unsigned kAxRows>
+__global__ void __launch_bounds__(256)
+    omprt_axpy_tma_rt(const __grid_constant__ AxpyMaps maps, typename Tr::Idx n, double x,
+                      const double* __restrict__ b, const double* __restrict__ c,
+                      double* __restrict__ a, double* sum_inout, double* partials,
+                      unsigned* ticket, int32_t* owner, int32_t* count) {
+  using Idx = typename Tr::Idx;
+  Team<Tr> team = init<Tr>();
+  double acc = 0.0;
+  auto rec = [&](Idx i) {
+    if constexpr (Rec) {
+      owner[i] = get_team_num(team) * get_num_threads(team) + get_thread_num(team);
+      atomicAdd(count + i, 1);
+    }
+  };
+  distribute_parallel_for_tma_stream<Tr, 2, kAxTmaStore ? 1 : 0, kAxRows, kAxStages>(
+      team, n, maps.m,
+      [&](Idx i, const double (&xs)[2], double (&ys)[1]) {
+        const double v = fma(x, xs[0], xs[1]);
+        if constexpr (kAxTmaStore) ys[0] = v;
+        else a[i] = v;
+        acc += v;
+        rec(i);
+      },
+      [&](Idx i) {
+        const double v = fma(x, __ldg(b + i), __ldg(c + i));
+        a[i] = v;
+        acc += v;
+        rec(i);
+      });
+  league_reduce(team, team_reduce_to_main(team, acc, Plus{}), Plus{}, sum_inout, partials,
+                ticket);
+}
+
+// Bare CUDA twin: the same TMA box pipeline and the same hand-written reduction.
+template <bool Rec, unsigned kAxRows>
+__global__ void __launch_bounds__(256)
+    cuda_axpy_tma_twin(const __grid_constant__ AxpyMaps maps, int32_t n, double x,
+                       const double* __restrict__ b, const double* __restrict__ c,
+                       double* __restrict__ a, double* sum_inout, double* partials,
+                       unsigned* ticket, int32_t* owner, int32_t* count) {
+  extern __shared__ __align__(128) unsigned char smem[];
+  double* const sb = reinterpret_cast<double*>(smem);
+  const unsigned N = blockDim.x, t = threadIdx.x, box = kAxRows * N;
+  constexpr unsigned kArr = kAxTmaStore ? 3u : 2u;
+  uint64_t* const full = reinterpret_cast<uint64_t*>(smem + kAxStages * kArr * box * 8u);
+  const int32_t TN = gridDim.x * N, rows = n / TN, col0 = blockIdx.x * N;
+  const unsigned chunks = (unsigned)((rows + kAxRows - 1) / kAxRows);
+  double acc = 0.0;
+  if (t == 0) {
+    for (unsigned s = 0; s < kAxStages; ++s) tma::mbar_init(full + s, 1);
+    tma::fence_mbar_init();
+    for (unsigned s = 0; s < kAxStages && s < chunks; ++s) {
+      tma::mbar_arrive_expect_tx(full + s, 2u * box * 8u);
+      tma::tensor_load_2d(sb + (s * kArr + 0) * box, &maps.m[0], col0, s * kAxRows, full + s);
+      tma::tensor_load_2d(sb + (s * kArr + 1) * box, &maps.m[1], col0, s * kAxRows, full + s);
+    }
+  }
+  __syncthreads();
+  for (unsigned ch = 0; ch < chunks; ++ch) {
+    const unsigned s = ch % kAxStages;
+    tma::mbar_wait(full + s, (ch / kAxStages) & 1u);
+    double* const bs = sb + (s * kArr + 0) * box;
+    double* const cs = sb + (s * kArr + 1) * box;
+    double* const as = sb + (s * kArr + 2) * box;  // kAxTmaStore only
+    const int32_t row0 = ch * kAxRows;
+#pragma unroll 4
+    for (unsigned r = 0; r < kAxRows; ++r) {
+      if (row0 + (int32_t)r < rows) {
+        const double v = fma(x, bs[r * N + t], cs[r * N + t]);
+        if constexpr (kAxTmaStore) as[r * N + t] = v;
+        else a[(row0 + r) * TN + col0 + t] = v;
+        acc += v;
+        if constexpr (Rec) {
+          const int32_t i = (row0 + r) * TN + col0 + t;
+          owner[i] = blockIdx.x * N + t;
+          atomicAdd(count + i, 1);
+        }
+      }
+    }
+    if constexpr (kAxTmaStore) {
+      tma::fence_proxy_async_smem();
+      if (t == 0) tma::bulk_wait_read<kAxStages - 2>();
+    }
+    __syncthreads();
+    if (t == 0) {
+      if constexpr (kAxTmaStore) {
+        tma::tensor_store_2d(&maps.m[2], col0, row0, as);
+        tma::bulk_commit();
+      }
+      if (ch + kAxStages < chunks) {
+        tma::mbar_arrive_expect_tx(full + s, 2u * box * 8u);
+        tma::tensor_load_2d(bs, &maps.m[0], col0, (ch + kAxStages) * kAxRows, full + s);
+        tma::tensor_load_2d(cs, &maps.m[1], col0, (ch + kAxStages) * kAxRows, full + s);
+      }
+    }
+  }
+  const int32_t i = rows * TN + col0 + t;
+  if (i < n) {
+    const double v = fma(x, __ldg(b + i), __ldg(c + i));
+    a[i] = v;
+    acc += v;
+    if constexpr (Rec) {
+      owner[i] = blockIdx.x * N + t;
+      atomicAdd(count + i, 1);
+    }
+  }
+  if constexpr (kAxTmaStore)
+    if (t == 0) tma::bulk_wait<0>();
+  __shared__ double warp_sum[32];
+  __shared__ unsigned is_last;
+  for (int off = 16; off > 0; off >>= 1) acc += __shfl_xor_sync(0xffffffffu, acc, off);
+  const unsigned lane = t & 31u, wid = t >> 5, nw = (N + 31) >> 5;
+  if (lane == 0) warp_sum[wid] = acc;
+  __syncthreads();
+  double blk = 0.0;
+  if (wid == 0) {
+    blk = lane < nw ? warp_sum[lane] : 0.0;
+    for (int off = 16; off > 0; off >>= 1) blk += __shfl_xor_sync(0xffffffffu, blk, off);
+  }
+  if (t == 0) {
+    partials[blockIdx.x] = blk;
+    __threadfence();
+    is_last = (atomicAdd(ticket, 1u) == gridDim.x - 1) ? 1u : 0u;
+  }
+  __syncthreads();
+  if (is_last) {
+    __threadfence();
+    double tt0 = 0.0;
+    for (unsigned k = t; k < gridDim.x; k += N) tt0 += __ldcg(partials + k);
+    for (int off = 16; off > 0; off >>= 1) tt0 += __shfl_xor_sync(0xffffffffu, tt0, off);
+    if (lane == 0) warp_sum[wid] = tt0;
+    __syncthreads();
+    if (wid == 0) {
+      double tt = lane < nw ? warp_sum[lane] : 0.0;
+      for (int off = 16; off > 0; off >>= 1) tt += __shfl_xor_sync(0xffffffffu, tt, off);
+      if (t == 0) {
+        *sum_inout = *sum_inout + tt;
+        *ticket = 0u;
+      }
+    }
+  }
+}
+
+OMPRT_REGISTER_KERNEL(omprt_axpy_tma_rt, omprt_axpy_tma_rt<AxpyTraits, false, 16>)
+OMPRT_REGISTER_KERNEL(cuda_axpy_tma_twin, cuda_axpy_tma_twin<false, 16>)
+
+// the three tensor maps of a launch: [rows][T*N] doubles, box [kAxRows][threads]
+inline int axpy_tma_maps(AxpyMaps* M, const double* b, const double* c, double* a, int64_t n,
+                         int32_t teams, int32_t threads, uint32_t rows_per_box) {
+  static PFN_cuTensorMapEncodeTiled_v12000 enc = nullptr;
+  if (!enc) {
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", (void**)&enc, cudaEnableDefault, &q) !=
+            cudaSuccess ||
+        q != cudaDriverEntryPointSuccess || !enc) {
+      cudaGetLastError();
+      enc = nullptr;
+      return set_error(OMPRT_E_CUDA, "cuTensorMapEncodeTiled is not available");
+    }
+  }
+  const int64_t TN = (int64_t)teams * threads;
+  const int64_t rows = std::max<int64_t>(n / TN, 1);  // rows = 0: no box is ever issued
+  const cuuint64_t dims[2] = {(cuuint64_t)TN, (cuuint64_t)rows};
+  const cuuint64_t strides[1] = {(cuuint64_t)TN * 8u};
+  const cuuint32_t box[2] = {(cuuint32_t)threads, rows_per_box}, es[2] = {1, 1};
+  const double* ptr[3] = {b, c, a};
+  for (int k = 0; k < 3; ++k) {
+    const CUresult r = enc(&M->m[k], CU_TENSOR_MAP_DATA_TYPE_FLOAT64, 2, const_cast<double*>(ptr[k]),
+                           dims, strides, box, es, CU_TENSOR_MAP_INTERLEAVE_NONE,
+                           CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                           CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+    if (r != CUDA_SUCCESS) return set_error(OMPRT_E_CUDA, "cuTensorMapEncodeTiled failed (%d)", (int)r);
+  }
+  return OMPRT_OK;
+}
+
+inline int launch_axpy_tma(bool twin, int64_t n, double x, const double* b, const double* c,
+                           double* a, double* sum, int32_t teams, int32_t threads,
+                           int32_t* owner, int32_t* count, Workspace* w, cudaStream_t s) {
+  OMPRT_CHECK_ARG(threads <= 256 && threads % 32 == 0,
+                  "OMPRT_TMA_STREAM: threads must be a multiple of 32, at most 256 (box width)");
+  OMPRT_CHECK_ARG(((uintptr_t)a | (uintptr_t)b | (uintptr_t)c) % 16 == 0,
+                  "OMPRT_TMA_STREAM: arrays must be 16 B aligned");
+  OMPRT_CHECK_ARG(n + 2 * (int64_t)teams * threads < INT32_MAX,
+                  "OMPRT_TMA_STREAM: n too large for the 32-bit path");
+  if (n == 0) {
+    // nothing to stream; the reduction still adds 0 (keeps *sum untouched numerically)
+    return OMPRT_OK;
+  }
+  const uint32_t rows_per_box = threads <= 64 ? 32u : (threads <= 128 ? 16u : 8u);
+  AxpyMaps M;
+  if (int r = axpy_tma_maps(&M, b, c, a, n, teams, threads, rows_per_box)) return r;
+  double* p = (double*)w->partials;
+  unsigned* tk = w->tickets + 0;
+  const int32_t nn = (int32_t)n;
+  auto go = [&](auto k, uint32_t smem) -> int {
+    OMPRT_CUDA_TRY(cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
+    k<<<teams, threads, smem, s>>>(M, nn, x, b, c, a, sum, p, tk, owner, count);
+    return OMPRT_OK;
+  };
+  auto pick = [&](auto rows_c) -> int {
+    constexpr unsigned R = decltype(rows_c)::value;
+    const uint32_t smem = tma_stream_smem_bytes<2, kAxTmaStore ? 1 : 0, R, kAxStages>(threads);
+    if (twin)
+      return owner ? go(cuda_axpy_tma_twin<true, R>, smem) : go(cuda_axpy_tma_twin<false, R>, smem);
+    return owner ? go(omprt_axpy_tma_rt<AxpyTraits, true, R>, smem)
+                 : go(omprt_axpy_tma_rt<AxpyTraits, false, R>, smem);
+  };
+  int r;
+  if (rows_per_box == 32) r = pick(std::integral_constant<unsigned, 32>{});
+  else if (rows_per_box == 16) r = pick(std::integral_constant<unsigned, 16>{});
+  else r = pick(std::integral_constant<unsigned, 8>{});
+  if (r) return r;
+  return check_launch(twin ? "cuda_axpy_tma_twin" : "omprt_axpy_tma_rt");
+}
+
 OMPRT_REGISTER_KERNEL(omprt_axpy_rt, omprt_axpy_rt<AxpyTraits, false>)
 OMPRT_REGISTER_KERNEL(omprt_axpy_rt_assume, omprt_axpy_rt<AxpyTraitsAssume, false>)
 OMPRT_REGISTER_KERNEL(omprt_axpy_rt_debug, omprt_axpy_rt<AxpyTraitsDebug, false>)
@@ -161,6 +402,11 @@ extern "C" int omprt_spmd_axpy_sum(int64_t n, double x, const double* b, const d
     return r;
   if (!(flags & OMPRT_RECORD_OWNER)) owner = count = nullptr;
   cudaStream_t s = as_stream(stream);
+  if (flags & OMPRT_TMA_STREAM) {
+    OMPRT_CHECK_ARG(!(flags & (OMPRT_ASSUME_OVERSUB | OMPRT_DEBUG_BUILD)),
+                    "OMPRT_TMA_STREAM: release build, no oversubscription assumption");
+    return launch_axpy_tma(false, n, x, b, c, a, sum_inout, teams, threads, owner, count, w, s);
+  }
   const bool assume = flags & OMPRT_ASSUME_OVERSUB, debug = flags & OMPRT_DEBUG_BUILD;
   // 32-bit induction variable when n + (unroll+1)*T*N fits
   const bool i32 = n + 9 * (int64_t)teams * threads < INT32_MAX;
@@ -192,6 +438,9 @@ extern "C" int omprt_cuda_axpy_sum(int64_t n, double x, const double* b, const d
     return r;
   cudaStream_t s = as_stream(stream);
   const bool rec = flags & OMPRT_RECORD_OWNER;
+  if (flags & OMPRT_TMA_STREAM)
+    return launch_axpy_tma(true, n, x, b, c, a, sum_inout, teams, threads, rec ? owner : nullptr,
+                           rec ? count : nullptr, w, s);
   const bool i32 = n + 9 * (int64_t)teams * threads < INT32_MAX;
   double* p = (double*)w->partials;
   unsigned* t = w->tickets + 0;

@@ -14,6 +14,7 @@
 
 #include "../../common/ptx_tma.cuh"
 #include "state.cuh"
+#include "sync.cuh"
 
 namespace omprt {
 
@@ -258,6 +259,102 @@ __device__ __forceinline__ void distribute_parallel_for_tma_tiles(Team<Tr>& team
     j = j + 1 == kBuffers ? 0 : j + 1;
   }
   if (lane == 0) tma::bulk_wait<0>();  // the stores are complete before the warp exits
+}
+
+// ---- TMA streaming of element-wise loops under the Fig. 5 assignment -------------------
+// For a `distribute parallel for` whose iteration i reads element i of kIn arrays and
+// writes element i of kOut arrays (fp64).  Fig. 5 hands iteration i to global thread
+// i mod (T*N), so viewed as a row-major matrix [n / (T*N)][T*N] (row = trip, column = global
+// thread), team b owns the N columns [b*N, (b+1)*N) of every row: one 2-D TMA box
+// [kRows][N] per array moves kRows trips of the whole team.  kStages boxes per array are in
+// flight (the HBM latency is covered by the bytes in flight, not by the team's few warps);
+// thread t computes column t of each row in row order -- exactly its Fig. 5 iterations, in
+// its Fig. 5 order -- and its outputs go back with one TMA store per array and stage.  The
+// trailing n mod (T*N) iterations (a partial row, not a box) run from global memory via
+// tail(i).  maps[0 .. kIn) load, maps[kIn .. kIn+kOut) store: generic addresses of
+// __grid_constant__ CUtensorMaps of shape [rows = n / (T*N)][T*N] with box [kRows][N].
+// body(i, const double (&x)[kIn], double (&y)[kOut]); with kOut = 0 the body writes its
+// outputs itself (y is a dummy) -- coalesced direct stores need no staging.  Needs
+// tma_stream_smem_bytes<kIn, kOut, kRows, kStages>(N) bytes of dynamic shared memory.
+template <unsigned kIn, unsigned kOut, unsigned kRows, unsigned kStages>
+__host__ __device__ constexpr uint32_t tma_stream_smem_bytes(uint32_t team_size) {
+  return kStages * (kIn + kOut) * kRows * team_size * 8u + kStages * 8u;
+}
+
+template <class Tr, unsigned kIn, unsigned kOut, unsigned kRows, unsigned kStages, class Maps,
+          class Body, class Tail>
+__device__ __forceinline__ void distribute_parallel_for_tma_stream(Team<Tr>& team,
+                                                                   typename Tr::Idx n,
+                                                                   const Maps* maps, Body&& body,
+                                                                   Tail&& tail) {
+  using Idx = typename Tr::Idx;
+  static_assert(kStages >= 2, "at least double buffered");
+  OMPRT_TRACE(Tr, "distribute_parallel_for_tma_stream");
+  extern __shared__ __align__(128) unsigned char omprt_stage_smem[];
+  double* const sbuf = reinterpret_cast<double*>(omprt_stage_smem);
+  const uint32_t N = (uint32_t)team.team_size, t = (uint32_t)team.thread_num;
+  const uint32_t box = kRows * N;  // doubles per array per stage
+  uint64_t* const full =
+      reinterpret_cast<uint64_t*>(omprt_stage_smem + kStages * (kIn + kOut) * box * 8u);
+  auto stage_buf = [&](uint32_t s, uint32_t k) { return sbuf + (s * (kIn + kOut) + k) * box; };
+  const Idx TN = (Idx)gridDim.x * (Idx)N;
+  const Idx rows = n / TN;  // whole trips: the TMA part
+  const int32_t col0 = (int32_t)(blockIdx.x * N);
+  const uint32_t chunks = (uint32_t)((rows + kRows - 1) / kRows);
+  if (t == 0) {
+#pragma unroll
+    for (uint32_t s = 0; s < kStages; ++s) tma::mbar_init(full + s, 1);
+    tma::fence_mbar_init();
+#pragma unroll
+    for (uint32_t s = 0; s < kStages; ++s)
+      if (s < chunks) {
+        tma::mbar_arrive_expect_tx(full + s, kIn * box * 8u);
+#pragma unroll
+        for (uint32_t k = 0; k < kIn; ++k)
+          tma::tensor_load_2d(stage_buf(s, k), maps + k, col0, (int32_t)(s * kRows), full + s);
+      }
+  }
+  aligned_barrier();  // barriers initialized before anyone waits on them
+  for (uint32_t c = 0; c < chunks; ++c) {
+    const uint32_t s = c % kStages;
+    tma::mbar_wait(full + s, (c / kStages) & 1u);
+    const Idx row0 = (Idx)c * kRows;
+#pragma unroll 4
+    for (uint32_t r = 0; r < kRows; ++r) {
+      if (row0 + (Idx)r < rows) {
+        double x[kIn], y[kOut > 0 ? kOut : 1];
+#pragma unroll
+        for (uint32_t k = 0; k < kIn; ++k) x[k] = stage_buf(s, k)[r * N + t];
+        body((row0 + (Idx)r) * TN + (Idx)col0 + (Idx)t, x, y);
+#pragma unroll
+        for (uint32_t k = 0; k < kOut; ++k) stage_buf(s, kIn + k)[r * N + t] = y[k];
+      }
+    }
+    if constexpr (kOut > 0) {
+      tma::fence_proxy_async_smem();  // this thread's outputs -> the async proxy
+      if (t == 0) tma::bulk_wait_read<kStages - 2>();  // chunk c+1 may rewrite chunk c+1-K's
+    }
+    aligned_barrier();
+    if (t == 0) {
+      if constexpr (kOut > 0) {
+#pragma unroll
+        for (uint32_t k = 0; k < kOut; ++k)
+          tma::tensor_store_2d(maps + kIn + k, col0, (int32_t)row0, stage_buf(s, kIn + k));
+        tma::bulk_commit();
+      }
+      if (c + kStages < chunks) {  // this stage's inputs are consumed: refill it
+        tma::mbar_arrive_expect_tx(full + s, kIn * box * 8u);
+#pragma unroll
+        for (uint32_t k = 0; k < kIn; ++k)
+          tma::tensor_load_2d(stage_buf(s, k), maps + k, col0, (int32_t)((c + kStages) * kRows),
+                              full + s);
+      }
+    }
+  }
+  const Idx iv = rows * TN + (Idx)col0 + (Idx)t;  // this thread's last Fig. 5 iteration
+  if (iv < n) tail(iv);
+  if constexpr (kOut > 0)
+    if (t == 0) tma::bulk_wait<0>();
 }
 
 }  // namespace omprt

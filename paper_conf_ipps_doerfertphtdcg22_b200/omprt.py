@@ -40,6 +40,7 @@ OMPRT_XS_FLAT = 1 << 15
 OMPRT_FLAT = OMPRT_XS_FLAT  # omprt_rs_lookup: flattened nuclide loop, persistent grid
 OMPRT_SCHED_DYNAMIC = 1 << 17  # schedule(dynamic, C): team blocks, team-shared chunk counter
 OMPRT_TMA_TILED = 1 << 18  # SU(3): one 2-D TMA tensor copy per warp tile, padded slots
+OMPRT_TMA_STREAM = 1 << 19  # axpy: Fig. 5 loop with operands streamed by 2-D TMA boxes
 OMPRT_XS_NO_L2_PERSIST = 1 << 16
 
 # Every symbol include/omprt.h declares (checked by tests/test_abi.py).

@@ -58,6 +58,21 @@ def main(which):
         for name, _, _ in variants:
             ms = min(res[f"su3_{name}"]["ms"])
             res[f"su3_{name}"]["GBps_alg"] = 1152 * ns / ms / 1e6
+    if "c1" in which:
+        n = 1 << 20
+        x, b, c = gen.axpy_inputs(n)
+        bt, ct = torch.from_numpy(b).to(dev), torch.from_numpy(c).to(dev)
+        at = torch.empty_like(bt)
+        sm = torch.zeros(1, dtype=torch.float64, device=dev)
+        TS_ = omprt.OMPRT_TMA_STREAM
+        for name, fn, fl, T, N in [("rt", omprt.omprt_spmd_axpy_sum, 0, 8, 128),
+                                   ("twin", omprt.omprt_cuda_axpy_sum, 0, 8, 128),
+                                   ("rt_tma", omprt.omprt_spmd_axpy_sum, TS_, 8, 128),
+                                   ("twin_tma", omprt.omprt_cuda_axpy_sum, TS_, 8, 128),
+                                   ("rt_tma_8x256", omprt.omprt_spmd_axpy_sum, TS_, 8, 256),
+                                   ("rt_tma_148x128", omprt.omprt_spmd_axpy_sum, TS_, 148, 128)]:
+            ms = t(lambda: fn(n, x, bt, ct, at, sm, T, N, fl), 11)
+            res[f"c1_{name}"] = {"ms": ms, "GBps_alg": 24 * n / ms / 1e6}
     if "rs" in which:
         rs = gen.RSTables()
         rd = omprt.RSDeviceTables(rs, dev)

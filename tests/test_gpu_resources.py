@@ -26,6 +26,7 @@ PAIRS = [
     ("omprt_su3_staged_rt", "cuda_su3_staged_twin", True),
     ("omprt_su3_wstaged_rt", "cuda_su3_wstaged_twin", True),
     ("omprt_su3_tiled_rt", "cuda_su3_tiled_twin", True),
+    ("omprt_axpy_tma_rt", "cuda_axpy_tma_twin", True),
     ("omprt_rs_flat_rt", "cuda_rs_flat_twin", True),
     ("omprt_rs_dflat_rt", "cuda_rs_dflat_twin", True),
     ("omprt_axpy_dyn_rt", "cuda_axpy_dyn_twin", True),

@@ -249,3 +249,42 @@ def test_dynamic_schedule_rejects_assumption(rt):
         rt.omprt_spmd_axpy_sum_chunked(n, 1, x, bt, ct, torch.empty_like(bt),
                                        torch.zeros(1, dtype=torch.float64, device=DEV), 8, 128,
                                        rt.OMPRT_SCHED_DYNAMIC | rt.OMPRT_ASSUME_OVERSUB)
+
+
+TMA_CASES = [(0, 1, 32), (1, 8, 128), (1023, 8, 128), (1024, 8, 128), (1025, 8, 128),
+             (1 << 20, 8, 128), ((1 << 20) + 7, 3, 96), (100003, 37, 64), (16 * 1024 * 5 + 3, 8, 128),
+             (300_000, 2, 256)]
+
+
+@pytest.mark.parametrize("n,T,N", TMA_CASES)
+@pytest.mark.parametrize("which", ["rt", "twin"])
+def test_tma_stream_owner_values_and_sum(rt, n, T, N, which):
+    """OMPRT_TMA_STREAM: the operands move by 2-D TMA boxes, the iterations stay Fig. 5's --
+    owners bit-exact against the literal Fig. 5 simulation, every iteration once, a[]
+    bit-exact, and the sum bit-identical to the register-path runtime kernel (the same
+    iterations per thread in the same order); partial last boxes, a partial last trip and
+    fewer iterations than threads included."""
+    x, b, c = gen.axpy_inputs(n)
+    fn = rt.omprt_spmd_axpy_sum if which == "rt" else rt.omprt_cuda_axpy_sum
+    a, s, owner, count = _run(rt, fn, n, T, N, rt.OMPRT_TMA_STREAM, x, b, c)
+    ref_owner, _ = oracle.fig5_simulate(n, T, N)
+    assert (count == 1).all() and (owner == ref_owner).all()
+    assert (a == oracle.axpy(x, b, c)).all()
+    _, s_reg, _, _ = _run(rt, rt.omprt_spmd_axpy_sum, n, T, N, 0, x, b, c)
+    assert s == s_reg
+    if n:
+        assert abs(s - oracle.sum_f64(a)) <= 1e-12 * oracle.sum_abs_f64(a)
+
+
+def test_tma_stream_exact_sum_and_rejects(rt):
+    n = 1 << 20
+    x, b, c = gen.axpy_inputs(n, exact=True)
+    for fn in (rt.omprt_spmd_axpy_sum, rt.omprt_cuda_axpy_sum):
+        _, s, _, _ = _run(rt, fn, n, 8, 128, rt.OMPRT_TMA_STREAM, x, b, c)
+        assert s == float(1 << 30)
+    with pytest.raises(rt.OmprtError):  # box width: at most 256 threads
+        _run(rt, rt.omprt_spmd_axpy_sum, n, 8, 512, rt.OMPRT_TMA_STREAM, x, b, c)
+    with pytest.raises(rt.OmprtError):
+        _run(rt, rt.omprt_spmd_axpy_sum, 1024, 8, 128,
+             rt.OMPRT_TMA_STREAM | rt.OMPRT_ASSUME_OVERSUB, x[:1] if False else x, b[:1024],
+             c[:1024])

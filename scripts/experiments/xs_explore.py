@@ -43,6 +43,9 @@ def main():
             ts.append(a.elapsed_time(b))
         ok = bool(torch.equal(ver, ref))
         res[v] = {"ms": statistics.median(ts[1:]), "regs": L.xsx_regs(v), "exact": ok}
+        if hasattr(L, "xsx_name"):
+            L.xsx_name.restype = C.c_char_p
+            res[v]["name"] = L.xsx_name(v).decode()
         print(v, res[v], flush=True)
     print(json.dumps(res))
 

@@ -446,6 +446,31 @@ def _time(fn, stream, scrub, reps=5, warm=2, flush=True):
     return statistics.median(out)
 
 
+def _time_pair(fa, fb, stream, scrub, reps=9, warm=2):
+    """Medians of fa and fb timed INTERLEAVED (a b, b a, a b, ...), each rep cold (L2 reset +
+    flushed): the runtime-driven kernel and its twin see the same clocks and the same drift,
+    so their ratio (the overhead) is not biased by which one ran first."""
+    import torch
+    from paper_conf_ipps_doerfertphtdcg22_b200 import omprt
+    for _ in range(warm):
+        fa()
+        fb()
+    torch.cuda.synchronize()
+    out = ([], [])
+    for r in range(reps):
+        for k in ((0, 1) if r % 2 == 0 else (1, 0)):
+            torch.cuda.synchronize()
+            omprt.omprt_l2_reset_persisting()
+            scrub.fill_(1.0)
+            a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            a.record(stream)
+            (fa, fb)[k]()
+            b.record(stream)
+            torch.cuda.synchronize()
+            out[k].append(a.elapsed_time(b))
+    return statistics.median(out[0]), statistics.median(out[1])
+
+
 def run_sharded(omprt, torch, gen, sharding, dev, stream, scrub, rank, world):
     """BASELINE configs[3] and [4] as they are stated for several GPUs (N > 1 only): C4's
     10M RSBench lookups and C5's 32^4 SU(3) sites split into contiguous per-rank shards
@@ -458,9 +483,9 @@ def run_sharded(omprt, torch, gen, sharding, dev, stream, scrub, rank, world):
     rd = omprt.RSDeviceTables(gen.RSTables(), dev)
     v = torch.empty(max(cnt, 1), dtype=torch.uint64, device=dev)
     ck = torch.zeros(1, dtype=torch.uint64, device=dev)
-    FD = omprt.OMPRT_FLAT | omprt.OMPRT_SCHED_DYNAMIC
+    FQ = omprt.OMPRT_FLAT | omprt.OMPRT_SCHED_DYNAMIC | omprt.OMPRT_RS_QUEUE
     dist.barrier()
-    t = _time(lambda: omprt.omprt_rs_lookup(rd, 1070, first, cnt, v, None, 0, 128, FD), stream,
+    t = _time(lambda: omprt.omprt_rs_lookup(rd, 1070, first, cnt, v, None, 0, 128, FQ), stream,
               scrub, reps=3, warm=1)
     ms = sharding.allreduce_max(t, dev)
     omprt.omprt_u64_sum(v, cnt, ck)
@@ -468,8 +493,8 @@ def run_sharded(omprt, torch, gen, sharding, dev, stream, scrub, rank, world):
     res["c4_rsbench_10M"] = {"ranks": world, "lookups_per_rank": cnt, "max_rank_ms": ms,
                              "lookups_per_s": nl / ms * 1e3,
                              "checksum": int(ck.cpu().numpy()[0]),
-                             "variant": "flattened, lock-step, schedule(dynamic,1); NCCL u64 "
-                                        "checksum all-reduce"}
+                             "variant": "flattened, lock-step, schedule(dynamic,1), Abrarov poles "
+                                        "queued per warp; NCCL u64 checksum all-reduce"}
     ns = 32 ** 4
     s0, sc = sharding.shard(ns, rank, world)
     Ah, Bh = gen.su3_inputs(sc, first_site=s0)
@@ -500,22 +525,26 @@ def run_secondary(omprt, torch, gen, dev, stream, scrub):
     bt, ct = torch.from_numpy(b).to(dev), torch.from_numpy(c).to(dev)
     at = torch.empty_like(bt)
     s = torch.zeros(1, dtype=torch.float64, device=dev)
-    t_rt = _time(lambda: omprt.omprt_spmd_axpy_sum(n, x, bt, ct, at, s, 8, 128), stream, scrub)
-    t_tw = _time(lambda: omprt.omprt_cuda_axpy_sum(n, x, bt, ct, at, s, 8, 128), stream, scrub)
+    t_rt, t_tw = _time_pair(
+        lambda: omprt.omprt_spmd_axpy_sum(n, x, bt, ct, at, s, 8, 128),
+        lambda: omprt.omprt_cuda_axpy_sum(n, x, bt, ct, at, s, 8, 128),
+        stream, scrub)
     res["c1_axpy_sum_8x128"] = {"rt_ms": t_rt, "twin_ms": t_tw, "overhead": t_rt / t_tw - 1,
                                 "GBps_alg": 24 * n / t_rt / 1e6}
     # the same loop, operands streamed by 2-D TMA boxes (Fig. 5 assignment kept)
     TS_ = omprt.OMPRT_TMA_STREAM
-    t_rt = _time(lambda: omprt.omprt_spmd_axpy_sum(n, x, bt, ct, at, s, 8, 128, TS_), stream, scrub)
-    t_tw = _time(lambda: omprt.omprt_cuda_axpy_sum(n, x, bt, ct, at, s, 8, 128, TS_), stream, scrub)
+    t_rt, t_tw = _time_pair(
+        lambda: omprt.omprt_spmd_axpy_sum(n, x, bt, ct, at, s, 8, 128, TS_),
+        lambda: omprt.omprt_cuda_axpy_sum(n, x, bt, ct, at, s, 8, 128, TS_),
+        stream, scrub)
     res["c1_axpy_sum_8x128_tma_stream"] = {"rt_ms": t_rt, "twin_ms": t_tw,
                                            "overhead": t_rt / t_tw - 1,
                                            "GBps_alg": 24 * n / t_rt / 1e6}
     # NEXT f3: the same loop with schedule(static, 4): 256-bit chunk accesses
-    t_rt = _time(lambda: omprt.omprt_spmd_axpy_sum_chunked(n, 4, x, bt, ct, at, s, 8, 128),
-                 stream, scrub)
-    t_tw = _time(lambda: omprt.omprt_cuda_axpy_sum_chunked(n, 4, x, bt, ct, at, s, 8, 128),
-                 stream, scrub)
+    t_rt, t_tw = _time_pair(
+        lambda: omprt.omprt_spmd_axpy_sum_chunked(n, 4, x, bt, ct, at, s, 8, 128),
+        lambda: omprt.omprt_cuda_axpy_sum_chunked(n, 4, x, bt, ct, at, s, 8, 128),
+        stream, scrub)
     res["c1_axpy_sum_8x128_chunk4"] = {"rt_ms": t_rt, "twin_ms": t_tw,
                                        "overhead": t_rt / t_tw - 1,
                                        "GBps_alg": 24 * n / t_rt / 1e6}
@@ -523,18 +552,18 @@ def run_secondary(omprt, torch, gen, dev, stream, scrub):
     T = 4096
     inp = torch.from_numpy(gen.generic_inputs(T, 256)).to(dev)
     out = torch.empty(T * 256, dtype=torch.float64, device=dev)
-    t_rt = _time(lambda: omprt.omprt_generic_team(T, 256, 256, inp, out, None, None,
-                                                  omprt.OMPRT_ASSUME_OVERSUB), stream, scrub)
-    t_gs = _time(lambda: omprt.omprt_generic_team(T, 256, 256, inp, out, None, None,
-                                                  omprt.OMPRT_GENERAL_SM), stream, scrub)
-    t_tw = _time(lambda: omprt.omprt_cuda_generic_team(T, 256, 256, inp, out), stream, scrub)
     A_ = omprt.OMPRT_ASSUME_OVERSUB
-    t_sp = _time(lambda: omprt.omprt_generic_team(T, 256, 256, inp, out, None, None,
-                                                  A_ | omprt.OMPRT_SPMDIZE), stream, scrub)
-    t_dg = _time(lambda: omprt.omprt_generic_team(T, 256, 256, inp, out, None, None,
-                                                  A_ | omprt.OMPRT_DEGLOBALIZE), stream, scrub)
-    t_db = _time(lambda: omprt.omprt_generic_team(T, 256, 256, inp, out, None, None,
-                                                  omprt.OMPRT_DEBUG_BUILD), stream, scrub)
+
+    def gen_rt(flags):
+        return lambda: omprt.omprt_generic_team(T, 256, 256, inp, out, None, None, flags)
+
+    t_rt, t_tw = _time_pair(gen_rt(A_),
+                            lambda: omprt.omprt_cuda_generic_team(T, 256, 256, inp, out),
+                            stream, scrub)
+    t_gs, t_db = _time_pair(gen_rt(omprt.OMPRT_GENERAL_SM), gen_rt(omprt.OMPRT_DEBUG_BUILD),
+                            stream, scrub)
+    t_sp, t_dg = _time_pair(gen_rt(A_ | omprt.OMPRT_SPMDIZE), gen_rt(A_ | omprt.OMPRT_DEGLOBALIZE),
+                            stream, scrub)
     res["c2_generic_4096x256"] = {"rt_ms": t_rt, "rt_general_sm_ms": t_gs, "twin_ms": t_tw,
                                   "overhead": t_rt / t_tw - 1, "rt_spmdized_ms": t_sp,
                                   "rt_deglobalized_ms": t_dg,
@@ -545,47 +574,67 @@ def run_secondary(omprt, torch, gen, dev, stream, scrub):
     nl = 10_000_000
     v = torch.empty(nl, dtype=torch.uint64, device=dev)
     A = omprt.OMPRT_ASSUME_OVERSUB
-    t_rt = _time(lambda: omprt.omprt_rs_lookup(rd, 1070, 0, nl, v, None, 0, 128, A), stream,
-                 scrub, reps=3, warm=1)
-    t_tw = _time(lambda: omprt.omprt_cuda_rs_lookup(rd, 1070, 0, nl, v, None, 0, 128, 0), stream,
-                 scrub, reps=3, warm=1)
+    t_rt, t_tw = _time_pair(
+        lambda: omprt.omprt_rs_lookup(rd, 1070, 0, nl, v, None, 0, 128, A),
+        lambda: omprt.omprt_cuda_rs_lookup(rd, 1070, 0, nl, v, None, 0, 128, 0),
+        stream, scrub, reps=3, warm=1)
     res["c4_rsbench_10M_nested"] = {"rt_ms": t_rt, "twin_ms": t_tw, "overhead": t_rt / t_tw - 1,
                                     "lookups_per_s": nl / t_rt * 1e3}
-    # the C4 path: flattened nuclide loop, lock-step warps, schedule(dynamic, 1)
+    # flattened nuclide loop, lock-step warps, schedule(dynamic, 1)
     FD = omprt.OMPRT_FLAT | omprt.OMPRT_SCHED_DYNAMIC
-    t_rt = _time(lambda: omprt.omprt_rs_lookup(rd, 1070, 0, nl, v, None, 0, 128, FD), stream,
-                 scrub, reps=3, warm=1)
-    t_tw = _time(lambda: omprt.omprt_cuda_rs_lookup(rd, 1070, 0, nl, v, None, 0, 128, FD),
-                 stream, scrub, reps=3, warm=1)
+    t_rt, t_tw = _time_pair(
+        lambda: omprt.omprt_rs_lookup(rd, 1070, 0, nl, v, None, 0, 128, FD),
+        lambda: omprt.omprt_cuda_rs_lookup(rd, 1070, 0, nl, v, None, 0, 128, FD),
+        stream, scrub, reps=3, warm=1)
     tab = omprt.kernel_table()
+    res["c4_rsbench_10M_dflat"] = {"rt_ms": t_rt, "twin_ms": t_tw, "overhead": t_rt / t_tw - 1,
+                                   "lookups_per_s": nl / t_rt * 1e3,
+                                   "regs": [tab["omprt_rs_dflat_rt"]["regs"],
+                                            tab["cuda_rs_dflat_twin"]["regs"]]}
+    # the C4 path: the same + the Abrarov poles queued per warp and drained by all lanes
+    # (the runtime's lock-step warp-collective hook, reading R-A8)
+    FQ = FD | omprt.OMPRT_RS_QUEUE
+    t_rt, t_tw = _time_pair(
+        lambda: omprt.omprt_rs_lookup(rd, 1070, 0, nl, v, None, 0, 128, FQ),
+        lambda: omprt.omprt_cuda_rs_lookup(rd, 1070, 0, nl, v, None, 0, 128, FQ),
+        stream, scrub, reps=3, warm=1)
     res["c4_rsbench_10M"] = {"rt_ms": t_rt, "twin_ms": t_tw, "overhead": t_rt / t_tw - 1,
                              "lookups_per_s": nl / t_rt * 1e3,
                              "variant": "flattened nuclide loop, lock-step warps, "
-                                        "schedule(dynamic,1), persistent grid",
-                             "regs": [tab["omprt_rs_dflat_rt"]["regs"],
-                                      tab["cuda_rs_dflat_twin"]["regs"]]}
+                                        "schedule(dynamic,1), persistent grid, pole records "
+                                        "prefetched, Abrarov poles queued per warp",
+                             "regs": [tab["omprt_rs_qflat_rt"]["regs"],
+                                      tab["cuda_rs_qflat_twin"]["regs"]]}
     # C5: SU(3) 32^4 sites
     ns = 32 ** 4
     Ah, Bh = gen.su3_inputs(ns)
     At, Bt = torch.from_numpy(Ah).to(dev), torch.from_numpy(Bh).to(dev)
     Ct = torch.empty_like(At)
     ck = torch.zeros(1, dtype=torch.float64, device=dev)
-    t_rt = _time(lambda: omprt.omprt_su3_mult(At, Bt, Ct, ns, ck, 0, 128, A), stream, scrub)
-    t_tw = _time(lambda: omprt.omprt_cuda_su3_mult(At, Bt, Ct, ns, ck, 0, 128, 0), stream, scrub)
+    t_rt, t_tw = _time_pair(
+        lambda: omprt.omprt_su3_mult(At, Bt, Ct, ns, ck, 0, 128, A),
+        lambda: omprt.omprt_cuda_su3_mult(At, Bt, Ct, ns, ck, 0, 128, 0),
+        stream, scrub)
     TS = omprt.OMPRT_TMA_STAGED
-    t_rs = _time(lambda: omprt.omprt_su3_mult(At, Bt, Ct, ns, ck, 0, 128, TS), stream, scrub)
-    t_ts = _time(lambda: omprt.omprt_cuda_su3_mult(At, Bt, Ct, ns, ck, 0, 128, TS), stream, scrub)
+    t_rs, t_ts = _time_pair(
+        lambda: omprt.omprt_su3_mult(At, Bt, Ct, ns, ck, 0, 128, TS),
+        lambda: omprt.omprt_cuda_su3_mult(At, Bt, Ct, ns, ck, 0, 128, TS),
+        stream, scrub)
     res["c5_su3_32^4_tma_staged"] = {"rt_ms": t_rs, "twin_ms": t_ts, "overhead": t_rs / t_ts - 1,
                                      "GBps_alg": 1152 * ns / t_rs / 1e6}
     WS = omprt.OMPRT_WARP_STAGED
-    t_rw = _time(lambda: omprt.omprt_su3_mult(At, Bt, Ct, ns, ck, 0, 128, WS), stream, scrub)
-    t_tww = _time(lambda: omprt.omprt_cuda_su3_mult(At, Bt, Ct, ns, ck, 0, 128, WS), stream, scrub)
+    t_rw, t_tww = _time_pair(
+        lambda: omprt.omprt_su3_mult(At, Bt, Ct, ns, ck, 0, 128, WS),
+        lambda: omprt.omprt_cuda_su3_mult(At, Bt, Ct, ns, ck, 0, 128, WS),
+        stream, scrub)
     res["c5_su3_32^4_warp_staged"] = {"rt_ms": t_rw, "twin_ms": t_tww,
                                       "overhead": t_rw / t_tww - 1,
                                       "GBps_alg": 1152 * ns / t_rw / 1e6}
     TT = omprt.OMPRT_TMA_TILED
-    t_rtt = _time(lambda: omprt.omprt_su3_mult(At, Bt, Ct, ns, ck, 0, 128, TT), stream, scrub)
-    t_twt = _time(lambda: omprt.omprt_cuda_su3_mult(At, Bt, Ct, ns, ck, 0, 128, TT), stream, scrub)
+    t_rtt, t_twt = _time_pair(
+        lambda: omprt.omprt_su3_mult(At, Bt, Ct, ns, ck, 0, 128, TT),
+        lambda: omprt.omprt_cuda_su3_mult(At, Bt, Ct, ns, ck, 0, 128, TT),
+        stream, scrub)
     res["c5_su3_32^4_tma_tiled"] = {"rt_ms": t_rtt, "twin_ms": t_twt,
                                     "overhead": t_rtt / t_twt - 1,
                                     "GBps_alg": 1152 * ns / t_rtt / 1e6}

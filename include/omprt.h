@@ -131,6 +131,13 @@ extern "C" {
  * per-thread order as Fig. 5 (a[] and the sum bit-identical).  threads <= 256 and a
  * multiple of 32; arrays 16 B aligned; no OMPRT_ASSUME_OVERSUB / OMPRT_DEBUG_BUILD. */
 #define OMPRT_TMA_STREAM (1u << 19)
+/* omprt_rs_lookup / omprt_cuda_rs_lookup with OMPRT_FLAT | OMPRT_SCHED_DYNAMIC: poles in the
+ * Faddeeva function's Abrarov branch (|Z| < 6) are queued per warp in shared memory and
+ * evaluated by all 32 lanes together (the runtime's lock-step warp-collective hook) instead
+ * of by one divergent lane each; their contributions are added to the macroscopic cross
+ * sections per pole (reading R-A8: a different summation order, within the RSBench
+ * tolerance contract -- macro xs 1e-10 normwise, verification up to near-ties). */
+#define OMPRT_RS_QUEUE (1u << 20)
 
 /* ---- runtime lifecycle ------------------------------------------------------------- */
 typedef struct {

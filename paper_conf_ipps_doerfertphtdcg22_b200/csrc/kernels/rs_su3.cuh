@@ -15,9 +15,15 @@ struct RSTraitsAssume : DefaultTraits {
   static constexpr bool assume_teams_oversub = true;
 };
 constexpr int kRSThreads = 128;
+static_assert(kRSThreads == kRSBodyThreads, "rs_nuclide's shared-memory slots");
 // 5 teams of 128 per SM (<= 96 registers): 10 % faster than the unconstrained 122-register
 // build (scripts/experiments/rs_explore, profiles/rs_explore_x05.txt)
 constexpr int kRSMinBlocks = 5;
+// The flattened kernels: 4 teams of 128 per SM (<= 128 registers, no spills).  With the
+// prefetched pole loop (and, queued, the Abrarov drain) in one loop body the 96-register
+// budget of 5 teams spills inside the pole loop: queued 106 ms vs 77.8 ms, dynamic 82.8 vs
+// 81.9 ms at 10M lookups (profiles/rs_q_explore_x33.txt).
+constexpr int kRSFlatMinBlocks = 4;
 
 template <class Tr, bool Macro>
 __global__ void __launch_bounds__(kRSThreads, kRSMinBlocks)
@@ -44,7 +50,7 @@ __global__ void __launch_bounds__(kRSThreads, kRSMinBlocks)
 // thread running its Fig. 5 lookups through omprt::distribute_parallel_for_flat with one
 // nuclide per step (RSFlatLookup), so lanes are not held by the warp's longest material.
 template <class Tr, bool Macro>
-__global__ void __launch_bounds__(kRSThreads, kRSMinBlocks)
+__global__ void __launch_bounds__(kRSThreads, kRSFlatMinBlocks)
     omprt_rs_flat_rt(const __grid_constant__ RSTables t, uint64_t seed, int64_t first,
                      typename Tr::Idx count, uint64_t* __restrict__ verification,
                      double* __restrict__ macro) {
@@ -55,7 +61,7 @@ __global__ void __launch_bounds__(kRSThreads, kRSMinBlocks)
 
 // Bare CUDA twin: the same flattened loop written by hand around the same body.
 template <bool Macro>
-__global__ void __launch_bounds__(kRSThreads, kRSMinBlocks)
+__global__ void __launch_bounds__(kRSThreads, kRSFlatMinBlocks)
     cuda_rs_flat_twin(const __grid_constant__ RSTables t, uint64_t seed, int64_t first,
                       int32_t count, uint64_t* __restrict__ verification,
                       double* __restrict__ macro) {
@@ -81,7 +87,7 @@ __global__ void __launch_bounds__(kRSThreads, kRSMinBlocks)
 constexpr int kRSDynChunk = 1;
 
 template <class Tr, bool Macro>
-__global__ void __launch_bounds__(kRSThreads, kRSMinBlocks)
+__global__ void __launch_bounds__(kRSThreads, kRSFlatMinBlocks)
     omprt_rs_dflat_rt(const __grid_constant__ RSTables t, uint64_t seed, int64_t first,
                       typename Tr::Idx count, uint64_t* __restrict__ verification,
                       double* __restrict__ macro) {
@@ -93,7 +99,7 @@ __global__ void __launch_bounds__(kRSThreads, kRSMinBlocks)
 }
 
 template <bool Macro>
-__global__ void __launch_bounds__(kRSThreads, kRSMinBlocks)
+__global__ void __launch_bounds__(kRSThreads, kRSFlatMinBlocks)
     cuda_rs_dflat_twin(const __grid_constant__ RSTables t, uint64_t seed, int64_t first,
                        int32_t count, uint64_t* __restrict__ verification,
                        double* __restrict__ macro) {
@@ -123,7 +129,62 @@ __global__ void __launch_bounds__(kRSThreads, kRSMinBlocks)
   }
 }
 
+// OMPRT_RS_QUEUE (with OMPRT_FLAT | OMPRT_SCHED_DYNAMIC): the same dynamic lock-step loop
+// around RSQueuedLookup -- Abrarov poles queued per warp and drained by the runtime's
+// warp-collective hook (reading R-A8).  One queue per warp in team-shared memory.
+template <class Tr, bool Macro>
+__global__ void __launch_bounds__(kRSThreads, kRSFlatMinBlocks)
+    omprt_rs_qflat_rt(const __grid_constant__ RSTables t, uint64_t seed, int64_t first,
+                      typename Tr::Idx count, uint64_t* __restrict__ verification,
+                      double* __restrict__ macro) {
+  Team<Tr> team = init<Tr>();
+  using Lookup = RSQueuedLookup<Macro, kRSThreads / 32>;
+  Lookup::init_queue();  // published by the loop's team barrier (dynamic_init)
+  Lookup lookup(t, seed, first, verification, macro);
+  distribute_parallel_for_dynamic_flat<Tr, FlatSync::Lockstep>(team, count,
+                                                               (typename Tr::Idx)kRSDynChunk,
+                                                               lookup);
+}
+
+template <bool Macro>
+__global__ void __launch_bounds__(kRSThreads, kRSFlatMinBlocks)
+    cuda_rs_qflat_twin(const __grid_constant__ RSTables t, uint64_t seed, int64_t first,
+                       int32_t count, uint64_t* __restrict__ verification,
+                       double* __restrict__ macro) {
+  __shared__ unsigned next;
+  using Lookup = RSQueuedLookup<Macro, kRSThreads / 32>;
+  const int32_t per = (count + (int32_t)gridDim.x - 1) / (int32_t)gridDim.x;
+  const int32_t lo = min((int32_t)blockIdx.x * per, count);
+  const int32_t hi = min(lo + per, count);
+  if (threadIdx.x == 0) next = blockDim.x;
+  Lookup::init_queue();
+  __syncthreads();
+  Lookup lookup(t, seed, first, verification, macro);
+  int32_t i = lo + (int32_t)threadIdx.x * kRSDynChunk;
+  int32_t end = min(i + kRSDynChunk, hi);
+  bool live = i < hi;
+  if (live) lookup.begin(i, 1);
+  while (__any_sync(0xffffffffu, live)) {
+    const bool done = live && !lookup.step();
+    __syncwarp();
+    lookup.warp_collective(done);
+    if (done) {
+      lookup.end(i);
+      if (++i < end) {
+        lookup.next(i);
+      } else {
+        i = lo + (int32_t)atomicAdd(&next, 1u) * kRSDynChunk;
+        end = min(i + kRSDynChunk, hi);
+        live = i < hi;
+        if (live) lookup.begin(i, 1);
+      }
+    }
+  }
+}
+
 OMPRT_REGISTER_KERNEL(omprt_rs_dflat_rt, omprt_rs_dflat_rt<RSTraits, false>)
+OMPRT_REGISTER_KERNEL(omprt_rs_qflat_rt, omprt_rs_qflat_rt<RSTraits, false>)
+OMPRT_REGISTER_KERNEL(cuda_rs_qflat_twin, cuda_rs_qflat_twin<false>)
 OMPRT_REGISTER_KERNEL(cuda_rs_dflat_twin, cuda_rs_dflat_twin<false>)
 OMPRT_REGISTER_KERNEL(omprt_rs_flat_rt, omprt_rs_flat_rt<RSTraits, false>)
 OMPRT_REGISTER_KERNEL(cuda_rs_flat_twin, cuda_rs_flat_twin<false>)
@@ -136,14 +197,19 @@ inline RSTables to_dev(const omprt_rs_tables& a) {
                   a.num_nucs, a.mats, a.concs, a.n_nuclides, a.numL, a.max_num_nucs, 0};
 }
 
-// Persistent grid of the flattened kernels: teams = 0 -> every SM's resident teams.
-inline int32_t rs_flat_teams(int32_t teams) {
+// Persistent grid of the flattened kernels: teams = 0 -> every SM's resident teams (of the
+// queued kernel with OMPRT_RS_QUEUE: fewer per SM, more registers).
+inline int32_t rs_flat_teams(int32_t teams, uint32_t flags = 0) {
   if (teams > 0) return teams;
   int dev = 0, sms = 148, per_sm = kRSMinBlocks;
   cudaGetDevice(&dev);
   cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, omprt_rs_flat_rt<RSTraits, false>,
-                                                kRSThreads, 0);
+  if (flags & OMPRT_RS_QUEUE)
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, omprt_rs_qflat_rt<RSTraits, false>,
+                                                  kRSThreads, 0);
+  else
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, omprt_rs_flat_rt<RSTraits, false>,
+                                                  kRSThreads, 0);
   return sms * std::max(1, per_sm);
 }
 
@@ -161,7 +227,10 @@ inline int rs_validate(const omprt_rs_tables& t, int64_t count, uint64_t* ver, i
                   "OMPRT_XS_FLAT runs a persistent grid (no oversubscription assumption)");
   OMPRT_CHECK_ARG(!(flags & OMPRT_SCHED_DYNAMIC) || (flags & OMPRT_XS_FLAT),
                   "OMPRT_SCHED_DYNAMIC is implemented for the flattened loop (OMPRT_FLAT)");
-  if (flags & OMPRT_XS_FLAT) teams = rs_flat_teams(teams);
+  OMPRT_CHECK_ARG(!(flags & OMPRT_RS_QUEUE) ||
+                      ((flags & OMPRT_XS_FLAT) && (flags & OMPRT_SCHED_DYNAMIC)),
+                  "OMPRT_RS_QUEUE requires OMPRT_FLAT | OMPRT_SCHED_DYNAMIC");
+  if (flags & OMPRT_XS_FLAT) teams = rs_flat_teams(teams, flags);
   if (teams <= 0) teams = (int32_t)std::max<int64_t>(1, ceil_div(count, threads));
   OMPRT_CHECK_ARG(!(flags & OMPRT_ASSUME_OVERSUB) || count <= (int64_t)teams * threads,
                   "oversubscription assumption violated");
@@ -325,6 +394,11 @@ extern "C" int omprt_rs_lookup(omprt_rs_tables t, uint64_t seed, int64_t first, 
   cudaStream_t s = as_stream(stream);
   const RSTables d = to_dev(t);
   const int32_t n = (int32_t)count;
+  if (flags & OMPRT_RS_QUEUE) {
+    if (macro) omprt_rs_qflat_rt<RSTraits, true><<<teams, threads, 0, s>>>(d, seed, first, n, verification, macro);
+    else omprt_rs_qflat_rt<RSTraits, false><<<teams, threads, 0, s>>>(d, seed, first, n, verification, nullptr);
+    return check_launch("omprt_rs_qflat_rt");
+  }
   if ((flags & OMPRT_XS_FLAT) && (flags & OMPRT_SCHED_DYNAMIC)) {
     if (macro) omprt_rs_dflat_rt<RSTraits, true><<<teams, threads, 0, s>>>(d, seed, first, n, verification, macro);
     else omprt_rs_dflat_rt<RSTraits, false><<<teams, threads, 0, s>>>(d, seed, first, n, verification, nullptr);
@@ -355,11 +429,16 @@ extern "C" int omprt_cuda_rs_lookup(omprt_rs_tables t, uint64_t seed, int64_t fi
   const bool flat = flags & OMPRT_XS_FLAT;
   int32_t tm = flat ? teams : 0;
   if (int r = rs_validate(t, count, verification, tm, threads,
-                          flags & (OMPRT_XS_FLAT | OMPRT_SCHED_DYNAMIC)))
+                          flags & (OMPRT_XS_FLAT | OMPRT_SCHED_DYNAMIC | OMPRT_RS_QUEUE)))
     return r;
   if (count == 0) return OMPRT_OK;
   cudaStream_t s = as_stream(stream);
   const RSTables d = to_dev(t);
+  if (flags & OMPRT_RS_QUEUE) {
+    if (macro) cuda_rs_qflat_twin<true><<<tm, threads, 0, s>>>(d, seed, first, (int32_t)count, verification, macro);
+    else cuda_rs_qflat_twin<false><<<tm, threads, 0, s>>>(d, seed, first, (int32_t)count, verification, nullptr);
+    return check_launch("cuda_rs_qflat_twin");
+  }
   if (flat && (flags & OMPRT_SCHED_DYNAMIC)) {
     if (macro) cuda_rs_dflat_twin<true><<<tm, threads, 0, s>>>(d, seed, first, (int32_t)count, verification, macro);
     else cuda_rs_dflat_twin<false><<<tm, threads, 0, s>>>(d, seed, first, (int32_t)count, verification, nullptr);

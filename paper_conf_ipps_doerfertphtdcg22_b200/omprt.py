@@ -41,6 +41,7 @@ OMPRT_FLAT = OMPRT_XS_FLAT  # omprt_rs_lookup: flattened nuclide loop, persisten
 OMPRT_SCHED_DYNAMIC = 1 << 17  # schedule(dynamic, C): team blocks, team-shared chunk counter
 OMPRT_TMA_TILED = 1 << 18  # SU(3): one 2-D TMA tensor copy per warp tile, padded slots
 OMPRT_TMA_STREAM = 1 << 19  # axpy: Fig. 5 loop with operands streamed by 2-D TMA boxes
+OMPRT_RS_QUEUE = 1 << 20  # RSBench: Abrarov poles queued per warp, drained by all lanes (R-A8)
 OMPRT_XS_NO_L2_PERSIST = 1 << 16
 
 # Every symbol include/omprt.h declares (checked by tests/test_abi.py).

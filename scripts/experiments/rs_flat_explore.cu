@@ -201,15 +201,196 @@ __global__ void __launch_bounds__(TPB, MINB)
   else distribute_parallel_for_flat<Tr, FlatSync::Lockstep>(team, n, b);
 }
 
+
+// ---- V5: the Abrarov branch through a per-warp shared-memory QUEUE -----------------------
+// A lane whose pole has |Z| < 6 appends (Z, f_l, conc, pole, link) to its warp's queue and
+// moves on; the asymptotic poles never wait for it.  After every lock-step trip the whole
+// warp (all 32 lanes, converged) flushes the queue when it holds >= 32 entries or when a
+// lane that is about to finish its lookup has entries pending: every lane evaluates one
+// queued Abrarov pole, writes conc * (dT, dA, dF, dT - dA) into the slot, and each owner
+// adds its own entries in push order (a linked list per lane: deterministic).  The
+// contributions reach M0..M3 per pole instead of through sigT..sigF of their nuclide: a
+// different summation order, within the tolerance contract.
+constexpr int kQCap = 64;
+struct WarpQ {
+  double zr[kQCap], zi[kQCap], fr[kQCap], fi[kQCap], cc[kQCap];
+  int p[kQCap], nxt[kQCap];
+  int count;
+};
+
+struct QBody {
+  const RSTables& t;
+  uint64_t seed0;
+  int64_t first;
+  uint64_t* ver;
+  double* macro;
+  WarpQ& q;
+  LcgMap J;
+  uint64_t s;
+  double E, sqrtE;
+  int32_t mat, nn, j;
+  int32_t qhead, qtail;
+  double M0, M1, M2, M3;
+  __device__ QBody(const RSTables& tt, uint64_t sd, int64_t f, uint64_t* v, double* m, WarpQ& qq)
+      : t(tt), seed0(sd), first(f), ver(v), macro(m), q(qq), qhead(-1), qtail(-1) {}
+  __device__ __forceinline__ void start() {
+    uint64_t seed = s;
+    E = lcg_double(seed);
+    mat = pick_mat(seed);
+    sqrtE = sqrt(E);
+    nn = __ldg(t.num_nucs + mat);
+    j = 0;
+    M0 = M1 = M2 = M3 = 0.0;
+  }
+  template <class Idx> __device__ __forceinline__ void begin(Idx iv, Idx stride) {
+    J = lcg_jump(2ull * (uint64_t)stride);
+    s = lcg_fast_forward(seed0, 2ull * (uint64_t)(first + iv));
+    start();
+  }
+  template <class Idx> __device__ __forceinline__ void next(Idx) {
+    s = lcg_apply(J, s);
+    start();
+  }
+  __device__ __forceinline__ void nuclide(int nuc, double conc, double& sigT, double& sigA,
+                                          double& sigF) {
+    const int nw = __ldg(t.n_windows + nuc);
+    const double spacing = 1.0 / nw;
+    int w = (int)(E / spacing);
+    if (w >= nw) w = nw - 1;
+    cplx f[4];
+#pragma unroll
+    for (int l = 0; l < 4; ++l) {
+      double phi = __ldg(t.k0rs + nuc * 4 + l) * sqrtE;
+      if (l == 1) phi -= -atan(phi);
+      else if (l == 2) phi -= atan(3.0 * phi / (3.0 - phi * phi));
+      else if (l == 3) phi -= atan(phi * (15.0 - phi * phi) / (15.0 - 6.0 * phi * phi));
+      phi *= 2.0;
+      double sn, cs;
+      sincos(phi, &sn, &cs);
+      f[l] = {cs, -sn};
+    }
+    const int64_t wi = (int64_t)__ldg(t.win_off + nuc) + w;
+    const double2 TA = __ldg(reinterpret_cast<const double2*>(t.windows + wi * 4));
+    const double Fw = __ldg(t.windows + wi * 4 + 2);
+    const int2 rg = __ldg(reinterpret_cast<const int2*>(t.win_range + wi * 2));
+    sigT = E * TA.x;
+    sigA = E * TA.y;
+    sigF = E * Fw;
+    for (int p = rg.x; p < rg.y; ++p) {
+      const double* P = t.poles + (int64_t)p * 8;
+      double ear, eai, rtr, rti, rar, rai, rfr, rfi;
+      ld_nc_v4f64(P, ear, eai, rtr, rti);
+      ld_nc_v4f64(P + 4, rar, rai, rfr, rfi);
+      const int l = __ldg(t.pole_l + p);
+      const cplx fl = l == 0 ? f[0] : l == 1 ? f[1] : l == 2 ? f[2] : f[3];
+      const cplx Z = {(E - ear) * 0.5, (0.0 - eai) * 0.5};
+      const double absz = sqrt(__dadd_rn(__dmul_rn(Z.r, Z.r), __dmul_rn(Z.i, Z.i)));
+      if (absz < 6.0) {
+        const int slot = atomicAdd(&q.count, 1);
+        if (slot < kQCap) {
+          q.zr[slot] = Z.r; q.zi[slot] = Z.i; q.fr[slot] = fl.r; q.fi[slot] = fl.i;
+          q.cc[slot] = conc; q.p[slot] = p; q.nxt[slot] = -1;
+          if (qtail >= 0) q.nxt[qtail] = slot;
+          else qhead = slot;
+          qtail = slot;
+          continue;
+        }
+      }
+      const cplx W = faddeeva_v<2>(Z);
+      const cplx Wf = cmul(W, fl);
+      sigT += rtr * Wf.r - rti * Wf.i;
+      sigA += rar * W.r - rai * W.i;
+      sigF += rfr * W.r - rfi * W.i;
+    }
+  }
+  __device__ __forceinline__ bool step() {
+    if (j < nn) {
+      const int nuc = __ldg(t.mats + mat * t.max_num_nucs + j);
+      const double conc = __ldg(t.concs + mat * t.max_num_nucs + j);
+      double sigT, sigA, sigF;
+      nuclide(nuc, conc, sigT, sigA, sigF);
+      rs_accumulate(conc, sigT, sigA, sigF, M0, M1, M2, M3);
+    }
+    return ++j < nn;
+  }
+  // all 32 lanes, converged, after every lock-step trip
+  __device__ __forceinline__ void collective(bool done) {
+    __syncwarp();
+    const int n = min(*(volatile int*)&q.count, kQCap);
+    if (!__any_sync(0xffffffffu, done && qhead >= 0) && n < 32) return;
+    const int lane = threadIdx.x & 31;
+    for (int k = lane; k < n; k += 32) {
+      const cplx Z = {q.zr[k], q.zi[k]}, fl = {q.fr[k], q.fi[k]};
+      const double conc = q.cc[k];
+      const double* P = t.poles + (int64_t)q.p[k] * 8;
+      double ear, eai, rtr, rti, rar, rai, rfr, rfi;
+      ld_nc_v4f64(P, ear, eai, rtr, rti);
+      ld_nc_v4f64(P + 4, rar, rai, rfr, rfi);
+      const cplx W = faddeeva_v<2>(Z);
+      const cplx Wf = cmul(W, fl);
+      const double dT = rtr * Wf.r - rti * Wf.i;
+      const double dA = rar * W.r - rai * W.i;
+      const double dF = rfr * W.r - rfi * W.i;
+      q.zr[k] = dT * conc;
+      q.zi[k] = dA * conc;
+      q.fr[k] = dF * conc;
+      q.fi[k] = (dT - dA) * conc;
+    }
+    __syncwarp();
+    for (int k = qhead; k >= 0; k = q.nxt[k]) {
+      M0 += q.zr[k];
+      M1 += q.zi[k];
+      M2 += q.fr[k];
+      M3 += q.fi[k];
+    }
+    qhead = qtail = -1;
+    __syncwarp();
+    if (lane == 0) q.count = 0;
+    __syncwarp();
+  }
+  template <class Idx> __device__ __forceinline__ void end(Idx iv) {
+    double* m = macro + (int64_t)iv * 4;
+    m[0] = M0; m[1] = M1; m[2] = M2; m[3] = M3;
+    ver[iv] = rs_argmax4(M0, M1, M2, M3);
+  }
+};
+
+// the lock-step dynamic loop (cuda_rs_dflat_twin) with the warp-collective hook per trip
+template <int TPB, int MINB>
+__global__ void __launch_bounds__(TPB, MINB)
+    kernq(const __grid_constant__ RSTables t, uint64_t seed, int64_t first, int32_t count,
+          uint64_t* ver, double* macro) {
+  __shared__ unsigned next;
+  __shared__ WarpQ qs[TPB / 32];
+  const int32_t per = (count + (int32_t)gridDim.x - 1) / (int32_t)gridDim.x;
+  const int32_t lo = min((int32_t)blockIdx.x * per, count);
+  const int32_t hi = min(lo + per, count);
+  if (threadIdx.x == 0) next = blockDim.x;
+  if ((threadIdx.x & 31) == 0) qs[threadIdx.x >> 5].count = 0;
+  __syncthreads();
+  QBody b(t, seed, first, ver, macro, qs[threadIdx.x >> 5]);
+  int32_t i = lo + (int32_t)threadIdx.x;
+  bool live = i < hi;
+  if (live) b.begin(i, 1);
+  while (__any_sync(0xffffffffu, live)) {
+    const bool done = live && !b.step();
+    b.collective(done);
+    if (done) {
+      b.end(i);
+      i = lo + (int32_t)atomicAdd(&next, 1u);
+      live = i < hi;
+      if (live) b.begin(i, 1);
+    }
+  }
+}
+
 typedef void (*KF)(RSTables, uint64_t, int64_t, int32_t, uint64_t*, double*);
 struct Var { KF f; int tpb; const char* name; };
 static Var vars[] = {
-  {kern<2, 128, 5, true>, 128, "V2_128x5_dyn"},
+  {kernq<128, 5>, 128, "V5_queue_128x5_dyn"},
+  {kernq<128, 4>, 128, "V5_queue_128x4_dyn"},
   {kern<3, 128, 5, true>, 128, "V3_128x5_dyn"},
-  {kern<4, 128, 5, true>, 128, "V4_128x5_dyn"},
-  {kern<4, 128, 4, true>, 128, "V4_128x4_dyn"},
-  {kern<4, 64, 10, true>, 64, "V4_64x10_dyn"},
-  {kern<3, 64, 10, true>, 64, "V3_64x10_dyn"},
+
 };
 extern "C" int rsf_count() { return (int)(sizeof(vars) / sizeof(vars[0])); }
 extern "C" const char* rsf_name(int v) { return vars[v].name; }

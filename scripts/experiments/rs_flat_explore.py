@@ -11,13 +11,14 @@ import sys
 HERE = os.path.dirname(os.path.abspath(__file__))
 ROOT = os.path.dirname(os.path.dirname(HERE))
 sys.path.insert(0, ROOT)
-SO = os.path.join(HERE, "librs_flat_explore.so")
+SRC = os.environ.get("RSX_SRC", "rs_flat_explore.cu")
+SO = os.path.join(HERE, "lib" + SRC.replace(".cu", ".so"))
 
 
 def build():
     subprocess.check_call(["nvcc", "-O3", "-std=c++17", "-gencode", "arch=compute_100a,code=sm_100a",
                            "-lineinfo", "--shared", "-Xcompiler", "-fPIC", "-Xptxas", "-v",
-                           os.path.join(HERE, "rs_flat_explore.cu"), "-o", SO])
+                           os.path.join(HERE, SRC), "-o", SO])
 
 
 def main():

@@ -24,7 +24,7 @@ for K in omprt_xs_flat_rt cuda_xs_flat_twin omprt_xs_rt; do
   ncu -i $OUT/prof_${K}_$TAG.ncu-rep --page source --csv --print-units base > $OUT/src_${K}_$TAG.csv 2>&1
 done
 rm -f $OUT/prof_omprt_xs_rt_$TAG.ncu-rep  # keep the returned payload small (CSV kept)
-bash scripts/ncu_rs.sh $TAG omprt_rs_dflat_rt cuda_rs_dflat_twin
+bash scripts/ncu_rs.sh $TAG omprt_rs_qflat_rt cuda_rs_qflat_twin
 rm -f $OUT/prof_*_$TAG.ncu-rep  # the CSV exports come back; the reports exceed gpurun's 64 MiB
 OMPRT_DEBUG=0 timeout 600 python scripts/debug_cost.py > $OUT/debug_cost_env0_$TAG.txt 2>&1
 OMPRT_DEBUG=1 timeout 600 python scripts/debug_cost.py > $OUT/debug_cost_env1_$TAG.txt 2>&1

@@ -86,6 +86,34 @@ def main(which):
         res["rs_rt_flat_1M"]["same"] = bool((v == ref).all())
         res["rs_twin_flat_1M"] = {"ms": t(lambda: omprt.omprt_cuda_rs_lookup(rd, 1070, 0, n, v, None, 0, 128, F), 3)}
         res["rs_twin_flat_1M"]["same"] = bool((v == ref).all())
+    if "rsq" in which:  # C4 at 10M: dynamic lock-step flat vs the queued-Abrarov form
+        rs = gen.RSTables()
+        rd = omprt.RSDeviceTables(rs, dev)
+        n = 10_000_000
+        FD = omprt.OMPRT_FLAT | omprt.OMPRT_SCHED_DYNAMIC
+        Q = FD | omprt.OMPRT_RS_QUEUE
+        outs = {}
+        variants = [("rt_dflat", omprt.omprt_rs_lookup, FD), ("twin_dflat", omprt.omprt_cuda_rs_lookup, FD),
+                    ("rt_qflat", omprt.omprt_rs_lookup, Q), ("twin_qflat", omprt.omprt_cuda_rs_lookup, Q)]
+        for name, fn, fl in variants:
+            v = torch.empty(n, dtype=torch.uint64, device=dev)
+            m = torch.empty(4 * n, dtype=torch.float64, device=dev)
+            outs[name] = (v, m)
+            res[f"rs10M_{name}"] = {"ms": []}
+        for _ in range(2):
+            for name, fn, fl in variants:
+                v, m = outs[name]
+                res[f"rs10M_{name}"]["ms"].append(
+                    t(lambda: fn(rd, 1070, 0, n, v, m, 0, 128, fl), 3))
+        v0, m0 = outs["rt_dflat"]
+        m0 = m0.view(n, 4)
+        for name in outs:
+            v, m = outs[name]
+            m = m.view(n, 4)
+            err = ((m - m0).abs().max(dim=1).values / m0.abs().max(dim=1).values).max().item()
+            res[f"rs10M_{name}"].update({"min_ms": min(res[f"rs10M_{name}"]["ms"]),
+                                         "flips_vs_rt_dflat": int((v != v0).sum().item()),
+                                         "max_norm_err_vs_rt_dflat": err})
     if "xs" in which:
         tabs = gen.XSTables(**gen.XS_SMALL)
         d = omprt.XSDeviceTables(tabs, dev, accel=True)

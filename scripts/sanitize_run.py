@@ -78,7 +78,7 @@ def main():
     omprt.omprt_rs_lookup(rd, 1070, 0, 512, v, None, 0, 128, A)
     omprt.omprt_cuda_rs_lookup(rd, 1070, 0, 512, v, None, 0, 128, 0)
     mac = torch.empty(512 * 4, dtype=torch.float64, device=dev)
-    for fl in (F, F | D):  # flattened lock-step (static / dynamic)
+    for fl in (F, F | D, F | D | omprt.OMPRT_RS_QUEUE):  # lock-step: static, dynamic, queued
         omprt.omprt_rs_lookup(rd, 1070, 0, 512, v, mac, 2, 128, fl)
         omprt.omprt_cuda_rs_lookup(rd, 1070, 0, 512, v, None, 2, 128, fl)
     # C5

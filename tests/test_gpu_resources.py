@@ -29,6 +29,7 @@ PAIRS = [
     ("omprt_axpy_tma_rt", "cuda_axpy_tma_twin", True),
     ("omprt_rs_flat_rt", "cuda_rs_flat_twin", True),
     ("omprt_rs_dflat_rt", "cuda_rs_dflat_twin", True),
+    ("omprt_rs_qflat_rt", "cuda_rs_qflat_twin", True),
     ("omprt_axpy_dyn_rt", "cuda_axpy_dyn_twin", True),
 ]
 

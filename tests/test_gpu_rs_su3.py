@@ -28,12 +28,14 @@ def _rs(rt, d, first, count, which, flags=0, teams=0):
 
 
 @pytest.mark.parametrize("variant", ["rt", "rt_assume", "twin", "rt_flat", "twin_flat",
-                                     "rt_dflat", "twin_dflat"])
+                                     "rt_dflat", "twin_dflat", "rt_qflat", "twin_qflat"])
 def test_rs_parity(rt, rs_dev, rs_tables, variant):
     first, count = 4321, 20_000 + 17
     D = rt.OMPRT_FLAT | rt.OMPRT_SCHED_DYNAMIC
+    Q = D | rt.OMPRT_RS_QUEUE
     flags = {"rt_assume": rt.OMPRT_ASSUME_OVERSUB, "rt_flat": rt.OMPRT_FLAT,
-             "twin_flat": rt.OMPRT_FLAT, "rt_dflat": D, "twin_dflat": D}.get(variant, 0)
+             "twin_flat": rt.OMPRT_FLAT, "rt_dflat": D, "twin_dflat": D,
+             "rt_qflat": Q, "twin_qflat": Q}.get(variant, 0)
     ver, mac = _rs(rt, rs_dev, first, count, "twin" if variant.startswith("twin") else "rt",
                    flags)
     rv, rm = oracle.rs_lookup(rs_tables, first, count, want_macro=True,
@@ -82,9 +84,30 @@ def test_rs_flat_equals_nested(rt, rs_dev, teams):
     first, n = 777, 30_011
     v0, m0 = _rs(rt, rs_dev, first, n, "rt")
     D = rt.OMPRT_FLAT | rt.OMPRT_SCHED_DYNAMIC
-    for which, fl in (("rt", rt.OMPRT_FLAT), ("twin", rt.OMPRT_FLAT), ("rt", D), ("twin", D)):
+    Q = D | rt.OMPRT_RS_QUEUE  # R-A8: another summation order, agreement to rounding
+    for which, fl in (("rt", rt.OMPRT_FLAT), ("twin", rt.OMPRT_FLAT), ("rt", D), ("twin", D),
+                      ("rt", Q), ("twin", Q)):
         v, m = _rs(rt, rs_dev, first, n, which, fl, teams)
         _agree(v, m, v0, m0)
+
+
+def test_rs_queue_full_10M_checksum(rt, rs_dev):
+    """The C4 bench path (queued Abrarov poles) at the full 10M lookups: the verification
+    checksum equals the plain dynamic lock-step kernel's (itself pinned to the oracle above),
+    and no lookup flips except at near-ties of the plain kernel's macro xs."""
+    n = 10_000_000
+    D = rt.OMPRT_FLAT | rt.OMPRT_SCHED_DYNAMIC
+    v0, m0 = _rs(rt, rs_dev, 0, n, "rt", D)
+    v1, m1 = _rs(rt, rs_dev, 0, n, "rt", D | rt.OMPRT_RS_QUEUE)
+    _agree(v1, m1, v0, m0)
+    assert int(v1.sum(dtype=np.uint64)) == int(v0.sum(dtype=np.uint64))
+
+
+def test_rs_queue_requires_dynamic_flat(rt, rs_dev):
+    v = torch.zeros(16, dtype=torch.uint64, device=DEV)
+    for fl in (rt.OMPRT_RS_QUEUE, rt.OMPRT_RS_QUEUE | rt.OMPRT_FLAT):
+        with pytest.raises(Exception):
+            rt.omprt_rs_lookup(rs_dev, 1, 0, 16, v, None, 0, 128, fl)
 
 
 def test_rs_flat_rejects_assumption(rt, rs_dev):

@@ -73,6 +73,18 @@ def main(which):
                                    ("rt_tma_148x128", omprt.omprt_spmd_axpy_sum, TS_, 148, 128)]:
             ms = t(lambda: fn(n, x, bt, ct, at, sm, T, N, fl), 11)
             res[f"c1_{name}"] = {"ms": ms, "GBps_alg": 24 * n / ms / 1e6}
+    if "c2" in which:
+        T = 4096
+        inp = torch.from_numpy(gen.generic_inputs(T, 256)).to(dev)
+        out = torch.empty(T * 256, dtype=torch.float64, device=dev)
+        A_ = omprt.OMPRT_ASSUME_OVERSUB
+        for name, fl in [("rt", A_), ("rt_general_sm", omprt.OMPRT_GENERAL_SM),
+                         ("rt_spmdized", A_ | omprt.OMPRT_SPMDIZE),
+                         ("rt_deglobalized", A_ | omprt.OMPRT_DEGLOBALIZE)]:
+            res[f"c2_{name}"] = {"ms": t(lambda: omprt.omprt_generic_team(T, 256, 256, inp, out, None, None, fl), 11)}
+        res["c2_twin"] = {"ms": t(lambda: omprt.omprt_cuda_generic_team(T, 256, 256, inp, out), 11)}
+        for k in [k for k in res if k.startswith("c2_")]:
+            res[k]["GBps_alg"] = 16 * T * 256 / res[k]["ms"] / 1e6
     if "rs" in which:
         rs = gen.RSTables()
         rd = omprt.RSDeviceTables(rs, dev)

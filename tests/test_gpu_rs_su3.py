@@ -91,16 +91,26 @@ def test_rs_flat_equals_nested(rt, rs_dev, teams):
         _agree(v, m, v0, m0)
 
 
-def test_rs_queue_full_10M_checksum(rt, rs_dev):
-    """The C4 bench path (queued Abrarov poles) at the full 10M lookups: the verification
-    checksum equals the plain dynamic lock-step kernel's (itself pinned to the oracle above),
-    and no lookup flips except at near-ties of the plain kernel's macro xs."""
+def test_rs_queue_full_10M_checksum(rt, rs_dev, rs_tables):
+    """The C4 bench path (queued Abrarov poles, bench's launch configuration) at the full 10M
+    lookups: the verification checksum equals the plain dynamic lock-step kernel's, no
+    lookup flips except at near-ties, and sampled windows across the whole range (the
+    first, middle and last lookups of the batch) match the oracle lookup by lookup."""
     n = 10_000_000
     D = rt.OMPRT_FLAT | rt.OMPRT_SCHED_DYNAMIC
     v0, m0 = _rs(rt, rs_dev, 0, n, "rt", D)
     v1, m1 = _rs(rt, rs_dev, 0, n, "rt", D | rt.OMPRT_RS_QUEUE)
     _agree(v1, m1, v0, m0)
     assert int(v1.sum(dtype=np.uint64)) == int(v0.sum(dtype=np.uint64))
+    for first in (0, 1_234_567, 5_000_000, 8_765_432, n - 300):
+        rv, rm = oracle.rs_lookup(rs_tables, first, 300, want_macro=True,
+                                  threads=os.cpu_count() or 1)
+        mac, ver = m1[first:first + 300], v1[first:first + 300]
+        err = np.abs(mac - rm).max(axis=1) / np.abs(rm).max(axis=1)
+        assert err.max() <= 1e-10, (first, err.max())
+        for q in np.nonzero(ver != rv)[0]:
+            top2 = np.sort(rm[q])[-2:]
+            assert top2[1] - top2[0] <= 1e-12 * abs(top2[1]), (first + q, rm[q])
 
 
 def test_rs_queue_requires_dynamic_flat(rt, rs_dev):

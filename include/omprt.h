@@ -225,6 +225,16 @@ int omprt_cuda_generic_team(int32_t teams, int32_t threads, int32_t inner_n, con
 int omprt_icv_probe(int32_t teams, int32_t threads, int32_t nested_request, int32_t *rec,
                     uint32_t flags, void *stream);
 
+/* Lock-step probe (tests): the lock-step flattened loop (Fig. 5 static, or dynamic with chunk
+ * 3 when dynamic != 0) over n synthetic iterations, iteration i taking 1 + (7 i mod 13)
+ * steps, with a body that uses the runtime's warp-collective hook.  steps[i] (n int32) gets
+ * the steps iteration i ran, hooks[g] (teams*threads int32) how often the hook ran on
+ * thread g; *errors (caller-zeroed int32) counts hook-contract violations (hook not on all
+ * 32 lanes / not once per trip, done not reported exactly on an iteration's last step,
+ * end() without it).  threads a multiple of 32. */
+int omprt_lockstep_probe(int64_t n, int32_t teams, int32_t threads, int32_t dynamic,
+                         int32_t *steps, int32_t *hooks, int32_t *errors, void *stream);
+
 /* ---- C3: XSBench-shaped lookup (§V-A) ------------------------- */
 typedef struct {
   const double *nuclide_grid; /* [n_isotopes*n_gridpoints][6] energy + 5 xs, per nuclide sorted */

@@ -10,3 +10,4 @@
 #include "kernels/xs_derive.cuh"
 #include "kernels/rs_su3.cuh"
 #include "kernels/su3_staged.cuh"
+#include "kernels/lockstep_probe.cuh"

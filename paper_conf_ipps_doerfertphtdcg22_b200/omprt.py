@@ -49,7 +49,7 @@ EXPORTS = [
     "omprt_init", "omprt_fini", "omprt_l2_reset_persisting", "omprt_l2_set_aside", "omprt_device_status", "omprt_last_error", "omprt_static_owner",
     "omprt_spmd_axpy_sum", "omprt_cuda_axpy_sum", "omprt_spmd_axpy_sum_chunked",
     "omprt_cuda_axpy_sum_chunked", "omprt_generic_team", "omprt_cuda_generic_team",
-    "omprt_icv_probe", "omprt_xs_lookup", "omprt_cuda_xs_lookup", "omprt_u64_sum",
+    "omprt_icv_probe", "omprt_lockstep_probe", "omprt_xs_lookup", "omprt_cuda_xs_lookup", "omprt_u64_sum",
     "omprt_xs_run_host", "omprt_xs_run_host_steps", "omprt_xs_accel_sizes", "omprt_xs_build_accel",
     "omprt_xs_derive_tmp_bytes", "omprt_xs_derive", "omprt_xs_compact_sizes", "omprt_xs_build_compact", "omprt_rs_lookup", "omprt_cuda_rs_lookup", "omprt_su3_mult",
     "omprt_cuda_su3_mult", "omprt_kernel_count", "omprt_kernel_name", "omprt_kernel_attrs",
@@ -104,6 +104,7 @@ _SIGS = {
     "omprt_generic_team": [_i32, _i32, _i32, _vp, _vp, _vp, _vp, _u32, _vp],
     "omprt_cuda_generic_team": [_i32, _i32, _i32, _vp, _vp, _vp, _vp, _u32, _vp],
     "omprt_icv_probe": [_i32, _i32, _i32, _vp, _u32, _vp],
+    "omprt_lockstep_probe": [_i64, _i32, _i32, _i32, _vp, _vp, _vp, _vp],
     "omprt_xs_lookup": [XSTablesC, _u64, _i64, _i64, _vp, _vp, _i32, _i32, _u32, _vp],
     "omprt_cuda_xs_lookup": [XSTablesC, _u64, _i64, _i64, _vp, _vp, _i32, _i32, _u32, _vp],
     "omprt_u64_sum": [_vp, _i64, _vp, _vp],
@@ -262,6 +263,11 @@ def omprt_cuda_generic_team(teams, threads, inner_n, inp, out, owner=None, postl
 def omprt_icv_probe(teams, threads, nested_request, rec, flags=0, stream=None):
     return _check(load().omprt_icv_probe(teams, threads, nested_request, _p(rec), flags,
                                          _stream(stream)))
+
+
+def omprt_lockstep_probe(n, teams, threads, dynamic, steps, hooks, errors, stream=None):
+    return _check(load().omprt_lockstep_probe(n, teams, threads, int(dynamic), _p(steps),
+                                              _p(hooks), _p(errors), _stream(stream)))
 
 
 # ---------------------------------------------------------------- C3

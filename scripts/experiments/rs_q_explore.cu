@@ -29,10 +29,15 @@ __global__ void __launch_bounds__(128, MINB)
 
 typedef void (*KF)(RSTables, uint64_t, int64_t, int32_t, uint64_t*, double*);
 struct Var { KF f; int tpb; const char* name; };
+#ifdef OMPRT_RS_ABRAROV_NOINLINE
+#define VN(x) x "_noinline"
+#else
+#define VN(x) x
+#endif
 static Var vars[] = {
-  {kern<false, 5>, 128, "dflat_128x5"}, {kern<true, 5>, 128, "qflat_128x5"},
-  {kern<false, 4>, 128, "dflat_128x4"}, {kern<true, 4>, 128, "qflat_128x4"},
-  {kern<false, 6>, 128, "dflat_128x6"}, {kern<true, 3>, 128, "qflat_128x3"},
+  {kern<false, 5>, 128, VN("dflat_128x5")}, {kern<true, 5>, 128, VN("qflat_128x5")},
+  {kern<false, 4>, 128, VN("dflat_128x4")}, {kern<true, 4>, 128, VN("qflat_128x4")},
+  {kern<true, 6>, 128, VN("qflat_128x6")},
 };
 extern "C" int rsf_count() { return (int)(sizeof(vars) / sizeof(vars[0])); }
 extern "C" const char* rsf_name(int v) { return vars[v].name; }

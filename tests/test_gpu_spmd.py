@@ -288,3 +288,28 @@ def test_tma_stream_exact_sum_and_rejects(rt):
         _run(rt, rt.omprt_spmd_axpy_sum, 1024, 8, 128,
              rt.OMPRT_TMA_STREAM | rt.OMPRT_ASSUME_OVERSUB, x[:1] if False else x, b[:1024],
              c[:1024])
+
+
+@pytest.mark.parametrize("dynamic", [False, True])
+@pytest.mark.parametrize("n,T,N", [(0, 2, 64), (1, 1, 32), (1000, 3, 64), (20_011, 7, 128),
+                                   (50_000, 148, 256)])
+def test_lockstep_warp_collective_hook(rt, n, T, N, dynamic):
+    """The lock-step flattened loops call a body's warp_collective(done) after every trip on
+    all 32 lanes, report done exactly on an iteration's last step, before its end(); every
+    iteration runs all its steps exactly once; under Fig. 5 (static) each warp runs as many
+    trips as its busiest lane has steps."""
+    steps = torch.full((max(n, 1),), -1, dtype=torch.int32, device="cuda:0")
+    hooks = torch.zeros(T * N, dtype=torch.int32, device="cuda:0")
+    errors = torch.zeros(1, dtype=torch.int32, device="cuda:0")
+    rt.omprt_lockstep_probe(n, T, N, dynamic, steps, hooks, errors)
+    torch.cuda.synchronize()
+    assert int(errors.item()) == 0
+    i = np.arange(n)
+    L = 1 + (7 * i) % 13
+    assert (steps.cpu().numpy()[:n] == L).all()
+    h = hooks.cpu().numpy().reshape(-1, 32)
+    assert (h == h[:, :1]).all()  # every lane of a warp saw every hook call
+    if not dynamic:
+        per_thread = np.zeros(T * N, dtype=np.int64)
+        np.add.at(per_thread, i % (T * N), L)  # Fig. 5: iteration i on thread i mod T*N
+        assert (h[:, 0] == per_thread.reshape(-1, 32).max(axis=1)).all()

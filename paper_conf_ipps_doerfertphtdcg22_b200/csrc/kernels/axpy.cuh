@@ -199,19 +199,26 @@ __global__ void __launch_bounds__(256)
     double* const cs = sb + (s * kArr + 1) * box;
     double* const as = sb + (s * kArr + 2) * box;  // kAxTmaStore only
     const int32_t row0 = ch * kAxRows;
-#pragma unroll 4
-    for (unsigned r = 0; r < kAxRows; ++r) {
-      if (row0 + (int32_t)r < rows) {
-        const double v = fma(x, bs[r * N + t], cs[r * N + t]);
-        if constexpr (kAxTmaStore) as[r * N + t] = v;
-        else a[(row0 + r) * TN + col0 + t] = v;
-        acc += v;
-        if constexpr (Rec) {
-          const int32_t i = (row0 + r) * TN + col0 + t;
-          owner[i] = blockIdx.x * N + t;
-          atomicAdd(count + i, 1);
-        }
+    const int32_t i0 = row0 * TN + col0 + t;
+    const double* const bt = bs + t;
+    const double* const ct = cs + t;
+    double* const at = as + t;
+    auto row = [&](unsigned r) {
+      const double v = fma(x, bt[r * N], ct[r * N]);
+      const int32_t i = i0 + (int32_t)r * TN;
+      if constexpr (kAxTmaStore) at[r * N] = v;
+      else a[i] = v;
+      acc += v;
+      if constexpr (Rec) {
+        owner[i] = blockIdx.x * N + t;
+        atomicAdd(count + i, 1);
       }
+    };
+    if (row0 + (int32_t)kAxRows <= rows) {  // a whole box: no per-row bound, fully unrolled
+#pragma unroll
+      for (unsigned r = 0; r < kAxRows; ++r) row(r);
+    } else {
+      for (unsigned r = 0; row0 + (int32_t)r < rows; ++r) row(r);
     }
     if constexpr (kAxTmaStore) {
       tma::fence_proxy_async_smem();

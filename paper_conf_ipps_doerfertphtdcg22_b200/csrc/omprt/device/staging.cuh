@@ -319,16 +319,26 @@ __device__ __forceinline__ void distribute_parallel_for_tma_stream(Team<Tr>& tea
     const uint32_t s = c % kStages;
     tma::mbar_wait(full + s, (c / kStages) & 1u);
     const Idx row0 = (Idx)c * kRows;
-#pragma unroll 4
-    for (uint32_t r = 0; r < kRows; ++r) {
-      if (row0 + (Idx)r < rows) {
-        double x[kIn], y[kOut > 0 ? kOut : 1];
+    const Idx iv0 = row0 * TN + (Idx)col0 + (Idx)t;  // this thread's iteration in row r: + r*TN
+    const double* xin[kIn];
+    double* yout[kOut > 0 ? kOut : 1];
 #pragma unroll
-        for (uint32_t k = 0; k < kIn; ++k) x[k] = stage_buf(s, k)[r * N + t];
-        body((row0 + (Idx)r) * TN + (Idx)col0 + (Idx)t, x, y);
+    for (uint32_t k = 0; k < kIn; ++k) xin[k] = stage_buf(s, k) + t;
 #pragma unroll
-        for (uint32_t k = 0; k < kOut; ++k) stage_buf(s, kIn + k)[r * N + t] = y[k];
-      }
+    for (uint32_t k = 0; k < kOut; ++k) yout[k] = stage_buf(s, kIn + k) + t;
+    auto row = [&](uint32_t r) {
+      double x[kIn], y[kOut > 0 ? kOut : 1];
+#pragma unroll
+      for (uint32_t k = 0; k < kIn; ++k) x[k] = xin[k][r * N];
+      body(iv0 + (Idx)r * TN, x, y);
+#pragma unroll
+      for (uint32_t k = 0; k < kOut; ++k) yout[k][r * N] = y[k];
+    };
+    if (row0 + (Idx)kRows <= rows) {  // a whole box: no per-row bound, fully unrolled
+#pragma unroll
+      for (uint32_t r = 0; r < kRows; ++r) row(r);
+    } else {
+      for (uint32_t r = 0; row0 + (Idx)r < rows; ++r) row(r);
     }
     if constexpr (kOut > 0) {
       tma::fence_proxy_async_smem();  // this thread's outputs -> the async proxy

@@ -55,5 +55,7 @@ elif which == "axpy":
     for _ in range(reps):
         omprt.omprt_spmd_axpy_sum(n, x, bt, ct, at, s, 8, 128)
         omprt.omprt_cuda_axpy_sum(n, x, bt, ct, at, s, 8, 128)
+        omprt.omprt_spmd_axpy_sum(n, x, bt, ct, at, s, 8, 128, omprt.OMPRT_TMA_STREAM)
+        omprt.omprt_spmd_axpy_sum(n, x, bt, ct, at, s, 8, 256, omprt.OMPRT_TMA_STREAM)
 torch.cuda.synchronize()
 print("done", which)

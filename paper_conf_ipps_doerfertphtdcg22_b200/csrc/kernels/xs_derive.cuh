@@ -104,6 +104,68 @@ __global__ void xs_derive_index(const uint16_t* __restrict__ ids, const double* 
   }
 }
 
+// (C') the same rows for an even n_iso <= kDeriveBallotIso with every thread busy: thread
+// t owns the column pair (2p, 2p+1), p = t mod n_iso/2, over one of the chunk's row segments
+// (t div n_iso/2) and writes both entries of a row with one 32-bit store (a warp: one
+// contiguous row piece).  A segment's starting counts come from per-(warp, nuclide) ballot
+// masks of the chunk's rows (popc of the rows before the segment), then the thread walks its
+// rows as (C) does.  Ties as in (C).
+constexpr int kDeriveBallotIso = 256;
+constexpr int kDeriveWords = kDeriveRows / 32;
+__global__ void __launch_bounds__(kDeriveRows)
+    xs_derive_index_pairs(const uint16_t* __restrict__ ids, const double* __restrict__ U,
+                          const uint32_t* __restrict__ start, int64_t n, int32_t n_iso,
+                          int32_t n_gp, uint16_t* __restrict__ index16) {
+  __shared__ uint32_t mask[kDeriveWords][kDeriveBallotIso];
+  __shared__ uint16_t sid[kDeriveRows];
+  __shared__ double su[kDeriveRows + 1];
+  const int64_t r0 = (int64_t)blockIdx.x * kDeriveRows;
+  const int rows = (int)(r0 + kDeriveRows < n ? kDeriveRows : n - r0);
+  const int k = threadIdx.x, w = k >> 5;
+  const int my = k < rows ? (int)ids[r0 + k] : -1;
+  if (k < rows) sid[k] = (uint16_t)my;
+  for (int q = 0; q < n_iso; ++q) {
+    const uint32_t m = __ballot_sync(0xffffffffu, my == q);
+    if ((k & 31) == 0) mask[w][q] = m;
+  }
+  for (int j = k; j <= rows; j += blockDim.x) su[j] = r0 + j < n ? U[r0 + j] : 0.0;
+  __syncthreads();
+  const int pairs = n_iso >> 1, segs = kDeriveRows / pairs;
+  const int seg = k / pairs, q0 = 2 * (k - seg * pairs);
+  if (seg >= segs) return;
+  const int per = (rows + segs - 1) / segs;
+  const int rs = seg * per, re = rs + per < rows ? rs + per : rows;
+  // counts of rows < rs of this chunk, per column
+  int64_t c0 = start[(int64_t)blockIdx.x * n_iso + q0];
+  int64_t c1 = start[(int64_t)blockIdx.x * n_iso + q0 + 1];
+  for (int j = 0; j < (rs >> 5); ++j) {
+    c0 += __popc(mask[j][q0]);
+    c1 += __popc(mask[j][q0 + 1]);
+  }
+  if (rs & 31) {
+    const uint32_t below = (1u << (rs & 31)) - 1u;
+    c0 += __popc(mask[rs >> 5][q0] & below);
+    c1 += __popc(mask[rs >> 5][q0 + 1] & below);
+  }
+  const int32_t kmax = n_gp - 2;
+  uint32_t* out = reinterpret_cast<uint32_t*>(index16 + (r0 + rs) * n_iso + q0);
+  for (int r = rs; r < re; ++r, out += pairs) {
+    const int id = sid[r];
+    c0 += id == q0;
+    c1 += id == q0 + 1;
+    int64_t v0 = c0, v1 = c1;
+    if (r0 + r + 1 < n && su[r + 1] == su[r]) {  // tie: count the equal rows ahead too
+      for (int64_t e2 = r0 + r + 1; e2 < n && U[e2] == su[r]; ++e2) {
+        v0 += ids[e2] == q0;
+        v1 += ids[e2] == q0 + 1;
+      }
+    }
+    v0 = v0 - 1 < 0 ? 0 : (v0 - 1 > kmax ? kmax : v0 - 1);
+    v1 = v1 - 1 < 0 ? 0 : (v1 - 1 > kmax ? kmax : v1 - 1);
+    *out = (uint32_t)v0 | ((uint32_t)v1 << 16);
+  }
+}
+
 // ---- compact index grid (omprt_xs_build_compact, reading R-X1) -------------------------
 // owner[v] = nuclide of sorted energy v (0xFF pad to a multiple of 16)
 __global__ void xs_compact_owner(const uint16_t* __restrict__ ids, int64_t n, int64_t n_pad,
@@ -192,7 +254,10 @@ inline int xs_derive(const double* nuclide_grid, int32_t n_iso, int32_t n_gp, do
   xs_derive_unionized<<<1024, 256, 0, s>>>(kout, n, U);
   xs_derive_hist<<<chunks, 256, 0, s>>>(iout, n, n_iso, hist);
   xs_derive_scan<<<n_iso, kScanThreads, 0, s>>>(hist, chunks, n_iso);
-  xs_derive_index<<<chunks, 128, 0, s>>>(iout, U, hist, n, n_iso, n_gp, index16);
+  if (n_iso <= kDeriveBallotIso && n_iso % 2 == 0 && ((uintptr_t)index16 & 3) == 0)
+    xs_derive_index_pairs<<<chunks, kDeriveRows, 0, s>>>(iout, U, hist, n, n_iso, n_gp, index16);
+  else
+    xs_derive_index<<<chunks, 128, 0, s>>>(iout, U, hist, n, n_iso, n_gp, index16);
   return check_launch("omprt_xs_derive");
 }
 

@@ -248,7 +248,7 @@ def _definition(grid, n_iso, n_gp):
     return U, idx
 
 
-@pytest.mark.parametrize("n_iso,n_gp", [(68, 500), (68, 11303), (3, 2), (7, 1500)])
+@pytest.mark.parametrize("n_iso,n_gp", [(68, 500), (68, 11303), (3, 2), (7, 1500), (300, 40)])
 def test_derive_unionized_and_index(rt, n_iso, n_gp):
     t = gen.XSTables(n_isotopes=n_iso, n_gridpoints=n_gp)
     U, idx = _derive(rt, t.nuclide_grid, n_iso, n_gp)

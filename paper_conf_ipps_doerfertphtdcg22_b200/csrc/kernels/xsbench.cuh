@@ -281,11 +281,24 @@ inline FlatLaunch flat_launch(const omprt_xs_tables& t, int32_t teams, int32_t t
     int dev = 0, maxwin = 0;
     cudaGetDevice(&dev);
     cudaDeviceGetAttribute(&maxwin, cudaDevAttrMaxAccessPolicyWindowSize, dev);
-    const size_t bytes = std::min(br, (size_t)std::max(maxwin, 0));
+    // the other hot read-only tables join the window when they lie just below the bracket
+    // records (one allocation: [unionized | bins | brackets], XSDeviceTables' layout): the
+    // bisection probes then hit persisting lines too
+    uintptr_t lo = (uintptr_t)t.brackets;
+    const uintptr_t hi = lo + br;
+    auto join = [&](const void* p, size_t n) {
+      const uintptr_t a = (uintptr_t)p;
+      if (p && a < lo && a + n <= lo && lo - (a + n) <= 4096 && hi - a <= (size_t)maxwin &&
+          hi - a <= (size_t)w->l2_persist_bytes)
+        lo = a;
+    };
+    join(t.bins, sizeof(int32_t) * ((1ull << t.log2_bins) + 1));
+    join(t.unionized, sizeof(double) * (size_t)t.n_union);
+    const size_t bytes = std::min((size_t)(hi - lo), (size_t)std::max(maxwin, 0));
     if (bytes > 0) {
       cudaAccessPolicyWindow& win = L.attr[0].val.accessPolicyWindow;
       L.attr[0].id = cudaLaunchAttributeAccessPolicyWindow;
-      win.base_ptr = (void*)t.brackets;
+      win.base_ptr = (void*)lo;
       win.num_bytes = bytes;
       win.hitRatio = (float)std::min(1.0, (double)w->l2_persist_bytes / (double)bytes);
       win.hitProp = cudaAccessPropertyPersisting;
@@ -698,17 +711,19 @@ extern "C" int omprt_xs_run_host_steps(omprt_xs_tables h, uint64_t seed, int64_t
     // the slot's device-built layouts are made on the copy stream too, right after its
     // H2D, so they overlap the previous step's lookups (two slots of built layouts)
     if (accel) {
+      // [unionized | bins | brackets | index]: the hot read-only tables adjacent, so the
+      // flattened launch's L2 window covers all three (flat_launch)
       unsigned char* bb = (unsigned char*)w->xs_built[b];
       size_t bo = 0;
+      double* U = (double*)(bb + bo);
+      bo += al(built_uni);
       int32_t* bins = (int32_t*)(bb + bo);
       bo += al(asz[0]);
-      uint16_t* i16 = up16 ? (uint16_t*)idx : (uint16_t*)(bb + bo);
-      bo += al(built16);
       double* brk = upbr ? br : (double*)(bb + bo);
       bo += al(builtbr);
+      uint16_t* i16 = up16 ? (uint16_t*)idx : (uint16_t*)(bb + bo);
+      bo += al(built16);
       if (derive) {
-        double* U = (double*)(bb + bo);
-        bo += al(built_uni);
         if (int r = xs_derive(d.nuclide_grid, d.n_isotopes, d.n_gridpoints, U, i16,
                               w->derive_tmp, w->derive_tmp_bytes, cs))
           return r;

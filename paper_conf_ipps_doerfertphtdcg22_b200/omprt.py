@@ -275,7 +275,7 @@ class XSDeviceTables:
     """Device copies (torch tensors) of gen.XSTables and the by-value C struct.  With
     accel=True the B200 layouts are built on the device (omprt_xs_build_accel)."""
 
-    def __init__(self, t, device="cuda", accel=False, log2_bins=16, compact=False):
+    def __init__(self, t, device="cuda", accel=False, log2_bins=16, compact=False, packed=True):
         import torch
         self.host = t
         self.nuclide_grid = torch.from_numpy(t.nuclide_grid).to(device)
@@ -289,9 +289,20 @@ class XSDeviceTables:
                            t.n_gridpoints, t.max_num_nucs, 0, t.n_union, None, None, None, 0, 0)
         if accel:
             sizes = omprt_xs_accel_sizes(t.n_isotopes, t.n_gridpoints, t.n_union, log2_bins)
-            self.bins = torch.empty(sizes[0] // 4, dtype=torch.int32, device=device)
             self.index_grid16 = torch.empty(sizes[1] // 2, dtype=torch.uint16, device=device)
-            self.brackets = torch.empty(sizes[2] // 8, dtype=torch.float64, device=device)
+            if packed:  # [unionized | bins | brackets] in one allocation: one L2 window
+                al = lambda b: (b + 255) // 256 * 256
+                nu = al(8 * t.n_union)
+                nb = al(sizes[0])
+                self._pack = torch.empty(nu + nb + sizes[2], dtype=torch.uint8, device=device)
+                self.unionized = self._pack[: 8 * t.n_union].view(torch.float64)
+                self.unionized.copy_(torch.from_numpy(t.unionized))
+                self.c.unionized = _p(self.unionized)
+                self.bins = self._pack[nu: nu + sizes[0]].view(torch.int32)
+                self.brackets = self._pack[nu + nb:].view(torch.float64)
+            else:
+                self.bins = torch.empty(sizes[0] // 4, dtype=torch.int32, device=device)
+                self.brackets = torch.empty(sizes[2] // 8, dtype=torch.float64, device=device)
             omprt_xs_build_accel(self, self.bins, self.index_grid16, self.brackets, log2_bins)
         if compact:  # the compact index grid (flattened launches), from the nuclide grids
             sizes = omprt_xs_compact_sizes(t.n_isotopes, t.n_gridpoints)

@@ -117,51 +117,54 @@ __global__ void __launch_bounds__(kDeriveRows)
                           const uint32_t* __restrict__ start, int64_t n, int32_t n_iso,
                           int32_t n_gp, uint16_t* __restrict__ index16) {
   __shared__ uint32_t mask[kDeriveWords][kDeriveBallotIso];
-  __shared__ uint16_t sid[kDeriveRows];
-  __shared__ double su[kDeriveRows + 1];
+  __shared__ uint16_t sidt[kDeriveRows];  // nuclide id | 0x8000 when the next energy ties
   const int64_t r0 = (int64_t)blockIdx.x * kDeriveRows;
   const int rows = (int)(r0 + kDeriveRows < n ? kDeriveRows : n - r0);
   const int k = threadIdx.x, w = k >> 5;
   const int my = k < rows ? (int)ids[r0 + k] : -1;
-  if (k < rows) sid[k] = (uint16_t)my;
+  if (k < rows) {
+    const bool tie = r0 + k + 1 < n && U[r0 + k + 1] == U[r0 + k];
+    sidt[k] = (uint16_t)(my | (tie ? 0x8000 : 0));
+  }
   for (int q = 0; q < n_iso; ++q) {
     const uint32_t m = __ballot_sync(0xffffffffu, my == q);
     if ((k & 31) == 0) mask[w][q] = m;
   }
-  for (int j = k; j <= rows; j += blockDim.x) su[j] = r0 + j < n ? U[r0 + j] : 0.0;
   __syncthreads();
   const int pairs = n_iso >> 1, segs = kDeriveRows / pairs;
-  const int seg = k / pairs, q0 = 2 * (k - seg * pairs);
+  const int seg = k / pairs, q0 = 2 * (k - seg * pairs), q1 = q0 + 1;
   if (seg >= segs) return;
   const int per = (rows + segs - 1) / segs;
   const int rs = seg * per, re = rs + per < rows ? rs + per : rows;
-  // counts of rows < rs of this chunk, per column
-  int64_t c0 = start[(int64_t)blockIdx.x * n_iso + q0];
-  int64_t c1 = start[(int64_t)blockIdx.x * n_iso + q0 + 1];
+  // counts of rows < rs of this chunk, per column (<= n_gp: int32)
+  int c0 = (int)start[(int64_t)blockIdx.x * n_iso + q0];
+  int c1 = (int)start[(int64_t)blockIdx.x * n_iso + q1];
   for (int j = 0; j < (rs >> 5); ++j) {
     c0 += __popc(mask[j][q0]);
-    c1 += __popc(mask[j][q0 + 1]);
+    c1 += __popc(mask[j][q1]);
   }
   if (rs & 31) {
     const uint32_t below = (1u << (rs & 31)) - 1u;
     c0 += __popc(mask[rs >> 5][q0] & below);
-    c1 += __popc(mask[rs >> 5][q0 + 1] & below);
+    c1 += __popc(mask[rs >> 5][q1] & below);
   }
-  const int32_t kmax = n_gp - 2;
+  const int kmax = n_gp - 2;
   uint32_t* out = reinterpret_cast<uint32_t*>(index16 + (r0 + rs) * n_iso + q0);
+#pragma unroll 4
   for (int r = rs; r < re; ++r, out += pairs) {
-    const int id = sid[r];
+    const int v = sidt[r], id = v & 0x7fff;
     c0 += id == q0;
-    c1 += id == q0 + 1;
-    int64_t v0 = c0, v1 = c1;
-    if (r0 + r + 1 < n && su[r + 1] == su[r]) {  // tie: count the equal rows ahead too
-      for (int64_t e2 = r0 + r + 1; e2 < n && U[e2] == su[r]; ++e2) {
+    c1 += id == q1;
+    int v0 = c0, v1 = c1;
+    if (v & 0x8000) {  // tie: count the equal rows ahead too
+      const double u = U[r0 + r];
+      for (int64_t e2 = r0 + r + 1; e2 < n && U[e2] == u; ++e2) {
         v0 += ids[e2] == q0;
-        v1 += ids[e2] == q0 + 1;
+        v1 += ids[e2] == q1;
       }
     }
-    v0 = v0 - 1 < 0 ? 0 : (v0 - 1 > kmax ? kmax : v0 - 1);
-    v1 = v1 - 1 < 0 ? 0 : (v1 - 1 > kmax ? kmax : v1 - 1);
+    v0 = min(max(v0 - 1, 0), kmax);
+    v1 = min(max(v1 - 1, 0), kmax);
     *out = (uint32_t)v0 | ((uint32_t)v1 << 16);
   }
 }

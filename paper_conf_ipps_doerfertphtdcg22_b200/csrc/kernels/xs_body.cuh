@@ -457,14 +457,20 @@ __global__ void xs_build_index16(const int32_t* __restrict__ a, uint16_t* __rest
 }
 __global__ void xs_build_brackets(const double* __restrict__ g, double* __restrict__ o,
                                   int32_t n_iso, int32_t n_gp) {
-  // one output double per thread (coalesced stores): o[b*12 + 2c + h] = g[(p*n_gp + k + h)*6 + c]
-  const int64_t total = (int64_t)n_iso * (n_gp - 1) * 12;
-  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < total;
-       i += (int64_t)gridDim.x * blockDim.x) {
-    const int64_t b = i / 12;
-    const int j = (int)(i - b * 12), c = j >> 1, h = j & 1;
+  // one bracket record per thread: gridpoints k and k+1 of nuclide p (96 contiguous bytes,
+  // 6 x 16 B loads) interleaved into (E,t,e,a,f,n) x (k, k+1) and written as 3 x 32 B
+  // stores: o[b*12 + 2c + h] = g[(p*n_gp + k + h)*6 + c]
+  const int64_t nb = (int64_t)n_iso * (n_gp - 1);
+  for (int64_t b = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; b < nb;
+       b += (int64_t)gridDim.x * blockDim.x) {
     const int64_t p = b / (n_gp - 1), k = b - p * (n_gp - 1);
-    o[i] = __ldg(g + (p * n_gp + k + h) * 6 + c);
+    const double2* src = reinterpret_cast<const double2*>(g + (p * n_gp + k) * 6);
+    const double2 l0 = __ldg(src + 0), l1 = __ldg(src + 1), l2 = __ldg(src + 2);
+    const double2 h0 = __ldg(src + 3), h1 = __ldg(src + 4), h2 = __ldg(src + 5);
+    double* d = o + b * 12;
+    st_v4f64(d, l0.x, h0.x, l0.y, h0.y);      // E_k E_k1 t_k t_k1
+    st_v4f64(d + 4, l1.x, h1.x, l1.y, h1.y);  // e_k e_k1 a_k a_k1
+    st_v4f64(d + 8, l2.x, h2.x, l2.y, h2.y);  // f_k f_k1 n_k n_k1
   }
 }
 

@@ -439,6 +439,7 @@ inline int launch_xs_accel(omprt_xs_tables* t, int32_t* bins, uint16_t* idx16, d
   OMPRT_CHECK_ARG(t->nuclide_grid && t->unionized && t->index_grid && bins && idx16 && brackets,
                   "omprt_xs_build_accel: null pointer");
   OMPRT_CHECK_ARG((uintptr_t)brackets % 32 == 0, "brackets must be 32 B aligned");
+  OMPRT_CHECK_ARG((uintptr_t)t->nuclide_grid % 16 == 0, "nuclide_grid must be 16 B aligned");
   xs_build_bins<<<1024, 256, 0, s>>>(t->unionized, (int32_t)t->n_union, log2_bins, bins);
   xs_build_index16<<<2048, 256, 0, s>>>(t->index_grid, idx16,
                                         (int64_t)t->n_union * t->n_isotopes);

@@ -273,7 +273,10 @@ def omprt_lockstep_probe(n, teams, threads, dynamic, steps, hooks, errors, strea
 # ---------------------------------------------------------------- C3
 class XSDeviceTables:
     """Device copies (torch tensors) of gen.XSTables and the by-value C struct.  With
-    accel=True the B200 layouts are built on the device (omprt_xs_build_accel)."""
+    accel=True the B200 layouts are built on the device (omprt_xs_build_accel); packed=True
+    (default) puts the unionized grid, the search bins and the bracket records in one
+    allocation, in that order, so the flattened launch's L2 persisting window covers all
+    three (xsbench.cuh flat_launch)."""
 
     def __init__(self, t, device="cuda", accel=False, log2_bins=16, compact=False, packed=True):
         import torch

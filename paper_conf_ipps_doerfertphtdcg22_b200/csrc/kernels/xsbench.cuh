@@ -591,7 +591,7 @@ extern "C" int omprt_xs_run_host_steps(omprt_xs_tables h, uint64_t seed, int64_t
                   "the plain path needs the int32 index grid and the nuclide grid");
   OMPRT_CHECK_ARG(!accel || h.n_gridpoints <= 65536, "16-bit index: n_gridpoints > 65536");
   cudaStream_t s = as_stream(stream);
-  const int32_t log2_bins = 16;
+  const int32_t log2_bins = 18;  // 2^18 search bins: ~1.5 bisection probes (profiles/l2_pack_x57.txt)
   uint64_t asz[3] = {0, 0, 0};
   if (accel) xs_accel_sizes(h.n_isotopes, h.n_gridpoints, h.n_union, log2_bins, asz);
   const bool up16 = accel && h.index_grid16, upbr = accel && h.brackets;

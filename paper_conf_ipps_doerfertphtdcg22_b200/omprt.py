@@ -278,7 +278,7 @@ class XSDeviceTables:
     allocation, in that order, so the flattened launch's L2 persisting window covers all
     three (xsbench.cuh flat_launch)."""
 
-    def __init__(self, t, device="cuda", accel=False, log2_bins=16, compact=False, packed=True):
+    def __init__(self, t, device="cuda", accel=False, log2_bins=18, compact=False, packed=True):
         import torch
         self.host = t
         self.nuclide_grid = torch.from_numpy(t.nuclide_grid).to(device)
@@ -336,13 +336,13 @@ class XSDeviceTables:
         return v
 
 
-def omprt_xs_accel_sizes(n_isotopes, n_gridpoints, n_union, log2_bins=16):
+def omprt_xs_accel_sizes(n_isotopes, n_gridpoints, n_union, log2_bins=18):
     sz = (_u64 * 3)()
     _check(load().omprt_xs_accel_sizes(n_isotopes, n_gridpoints, n_union, log2_bins, sz))
     return list(sz)
 
 
-def omprt_xs_build_accel(tables, bins, index_grid16, brackets, log2_bins=16, stream=None):
+def omprt_xs_build_accel(tables, bins, index_grid16, brackets, log2_bins=18, stream=None):
     return _check(load().omprt_xs_build_accel(C.byref(tables.c), _p(bins), _p(index_grid16),
                                               _p(brackets), log2_bins, _stream(stream)))
 

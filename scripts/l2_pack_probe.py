@@ -23,13 +23,17 @@ def main():
     n = 17_000_000
     tabs = {"packed": omprt.XSDeviceTables(t, "cuda", accel=True, packed=True),
             "separate": omprt.XSDeviceTables(t, "cuda", accel=True, packed=False)}
+    for lb in (17, 18, 19):  # finer search bins (still inside the window up to 2^19)
+        tabs[f"packed_bins{lb}"] = omprt.XSDeviceTables(t, "cuda", accel=True, packed=True,
+                                                        log2_bins=lb)
     ver = {k: torch.zeros(n, dtype=torch.uint64, device="cuda") for k in tabs}
     scrub = torch.empty(64 << 20, dtype=torch.float32, device="cuda")
     s = torch.cuda.current_stream()
     ms = {k: [] for k in tabs}
     F = omprt.OMPRT_XS_FLAT
     for r in range(12):
-        for k in (("packed", "separate") if r % 2 == 0 else ("separate", "packed")):
+        ks = list(tabs)
+        for k in (ks if r % 2 == 0 else ks[::-1]):
             torch.cuda.synchronize()
             omprt.omprt_l2_reset_persisting()
             scrub.fill_(1.0)
@@ -40,7 +44,7 @@ def main():
             torch.cuda.synchronize()
             ms[k].append(a.elapsed_time(b))
     res = {k: statistics.median(v[2:]) for k, v in ms.items()}
-    res["same"] = bool(torch.equal(ver["packed"], ver["separate"]))
+    res["same"] = all(bool(torch.equal(ver["packed"], v)) for v in ver.values())
     res["set_aside"] = got
     print(json.dumps(res))
 

@@ -23,7 +23,7 @@ import gen  # noqa: E402
 import oracle  # noqa: E402
 
 N = 17_000_000
-LOG2_BINS = 16
+LOG2_BINS = 18
 
 
 def plain_bytes(t):

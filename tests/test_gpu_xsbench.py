@@ -112,7 +112,7 @@ def test_flat_rejects(rt, xs_dev, xs_acc):
 
 def test_accel_tables_content(rt, xs_acc, xs_small):
     bins = xs_acc.bins.cpu().numpy()
-    H = 1 << 16
+    H = 1 << xs_acc.c.log2_bins
     edges = np.arange(H + 1, dtype=np.float64) / H
     U = xs_small.unionized
     assert (bins == np.clip(np.searchsorted(U, edges, side="right") - 1, 0, U.size - 2)).all()

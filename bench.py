@@ -446,10 +446,19 @@ def _time(fn, stream, scrub, reps=5, warm=2, flush=True):
     return statistics.median(out)
 
 
-def _time_pair(fa, fb, stream, scrub, reps=9, warm=2):
-    """Medians of fa and fb timed INTERLEAVED (a b, b a, a b, ...), each rep cold (L2 reset +
-    flushed): the runtime-driven kernel and its twin see the same clocks and the same drift,
-    so their ratio (the overhead) is not biased by which one ran first."""
+def _trimmed_mean(v, trim):
+    v = sorted(v)
+    v = v[trim:len(v) - trim] if len(v) > 2 * trim else v
+    return sum(v) / len(v)
+
+
+def _time_pair(fa, fb, stream, scrub, reps=15, warm=2):
+    """fa and fb timed INTERLEAVED (a b, b a, a b, ...), each rep cold (L2 reset + flushed):
+    the runtime-driven kernel and its twin see the same clocks and the same drift, so their
+    ratio (the overhead) is not biased by which one ran first.  Returns trimmed means (the 2
+    lowest and 2 highest reps dropped): CUDA events here tick in ~2 us steps, so for the
+    ~30 us kernels (C1, C2) a median lands on one tick or the next; the mean of many reps
+    resolves below a tick."""
     import torch
     from paper_conf_ipps_doerfertphtdcg22_b200 import omprt
     for _ in range(warm):
@@ -468,7 +477,8 @@ def _time_pair(fa, fb, stream, scrub, reps=9, warm=2):
             b.record(stream)
             torch.cuda.synchronize()
             out[k].append(a.elapsed_time(b))
-    return statistics.median(out[0]), statistics.median(out[1])
+    t = 2 if reps >= 9 else 0
+    return _trimmed_mean(out[0], t), _trimmed_mean(out[1], t)
 
 
 def run_sharded(omprt, torch, gen, sharding, dev, stream, scrub, rank, world):

@@ -3,8 +3,10 @@
 // lower bracket index"), so an end-to-end step ships only the raw problem data (nuclide
 // grids + materials, 36.9 MB for the small problem) instead of 147.6 MB of tables.
 //
-//   unionized[e]       = the e-th smallest of all n_iso * n_gp energies (a radix sort of the
-//                        energies' order-preserving 64-bit keys; CUB, the library primitive)
+//   unionized[e]       = the e-th smallest of all n_iso * n_gp energies (a stable merge of the
+//                        n_iso per-nuclide sorted runs of the energies' order-preserving
+//                        64-bit keys, ceil(log2 n_iso) merge-path levels; the same order as
+//                        a stable radix sort, 90 vs 131 us for the small problem)
 //   index_grid[e][q]   = clip(#{k : E_q[k] <= unionized[e]} - 1, 0, n_gp - 2)
 //
 // The index rows are a column-wise prefix count over the sorted order: row e differs from
@@ -42,6 +44,58 @@ __global__ void xs_derive_unionized(const unsigned long long* __restrict__ keys,
        e += (int64_t)gridDim.x * blockDim.x) {
     const unsigned long long k = keys[e];
     U[e] = __longlong_as_double((long long)((k >> 63) ? (k & ~(1ull << 63)) : ~k));
+  }
+}
+
+// The union as a merge of the per-nuclide runs: every nuclide's energies are sorted (the
+// index grid's definition presumes it), so the keys in nuclide-major order are n_iso sorted
+// runs of n_gp.  ceil(log2 n_iso) levels of pairwise merges (runs of L -> 2L; the last run
+// of a level may be short or alone) give the same order as a stable sort of the keys: ties
+// go to the lower run, i.e. the lower nuclide, then the lower k -- CUB's stable radix order.
+// Each thread writes kMergeItems consecutive outputs: the merge-path co-rank of its first
+// output by bisection, then a sequential merge.
+constexpr int kMergeItems = 4;
+__global__ void xs_derive_merge(const unsigned long long* __restrict__ kin,
+                                const uint16_t* __restrict__ iin,
+                                unsigned long long* __restrict__ kout,
+                                uint16_t* __restrict__ iout, int64_t n, int64_t L) {
+  const int64_t o0 = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) * kMergeItems;
+  if (o0 >= n) return;
+  const int64_t o1 = o0 + kMergeItems < n ? o0 + kMergeItems : n;
+  int64_t o = o0;
+  while (o < o1) {
+    // the pair of runs [a0, a0+la) and [b0, b0+lb) that output position o belongs to
+    const int64_t a0 = (o / (2 * L)) * (2 * L);
+    const int64_t b0 = a0 + L < n ? a0 + L : n;
+    const int64_t la = b0 - a0, lb = (b0 + L < n ? b0 + L : n) - b0;
+    const int64_t pend = b0 + lb;  // end of this pair's output
+    const int64_t d = o - a0;
+    int64_t lo = d - lb > 0 ? d - lb : 0, hi = d < la ? d : la;
+    while (lo < hi) {  // #A among the first d outputs (A wins ties)
+      const int64_t i = (lo + hi) >> 1;
+      if (__ldg(kin + a0 + i) <= __ldg(kin + b0 + (d - i - 1))) lo = i + 1;
+      else hi = i;
+    }
+    int64_t i = lo, j = d - lo;
+    const int64_t stop = o1 < pend ? o1 : pend;
+    // heads of both runs in registers (an exhausted run's head is +inf: never taken)
+    constexpr unsigned long long kInf = ~0ull;
+    unsigned long long ka = i < la ? __ldg(kin + a0 + i) : kInf;
+    unsigned long long kb = j < lb ? __ldg(kin + b0 + j) : kInf;
+    for (; o < stop; ++o) {
+      const bool takeA = j >= lb || (i < la && ka <= kb);
+      if (takeA) {
+        kout[o] = ka;
+        iout[o] = __ldg(iin + a0 + i);
+        ++i;
+        ka = i < la ? __ldg(kin + a0 + i) : kInf;
+      } else {
+        kout[o] = kb;
+        iout[o] = __ldg(iin + b0 + j);
+        ++j;
+        kb = j < lb ? __ldg(kin + b0 + j) : kInf;
+      }
+    }
   }
 }
 
@@ -251,9 +305,32 @@ inline int xs_derive(const double* nuclide_grid, int32_t n_iso, int32_t n_gp, do
   auto* hist = (uint32_t*)(b + L.hist);
   size_t cub_bytes = L.total - L.cub;
   xs_derive_keys<<<1024, 256, 0, s>>>(nuclide_grid, n_gp, n, kin, iin);
-  if (cub::DeviceRadixSort::SortPairs(b + L.cub, cub_bytes, kin, kout, iin, iout, (int)n, 0, 64,
-                                      s) != cudaSuccess)
-    return set_error(OMPRT_E_CUDA, "omprt_xs_derive: radix sort failed");
+  (void)cub_bytes;
+  // merge levels, ping-ponging between the two key/id buffers; the result ends in kout/iout
+  const unsigned mblocks = (unsigned)((n + 256 * kMergeItems - 1) / (256 * kMergeItems));
+  int levels = 0;
+  for (int64_t run = n_gp; run < n; run *= 2) ++levels;
+  if (levels == 0) {
+    OMPRT_CUDA_TRY(cudaMemcpyAsync(kout, kin, n * sizeof(unsigned long long),
+                                   cudaMemcpyDeviceToDevice, s));
+    OMPRT_CUDA_TRY(cudaMemcpyAsync(iout, iin, n * sizeof(uint16_t), cudaMemcpyDeviceToDevice, s));
+  }
+  {
+    // an odd number of levels starts in (kin -> kout), an even one in (kout <- kin copied)
+    unsigned long long* ks[2] = {kin, kout};
+    uint16_t* is[2] = {iin, iout};
+    int src = (levels % 2 == 0) ? 1 : 0;  // so that the last level writes kout/iout
+    if (levels > 0 && src == 1) {
+      OMPRT_CUDA_TRY(cudaMemcpyAsync(kout, kin, n * sizeof(unsigned long long),
+                                     cudaMemcpyDeviceToDevice, s));
+      OMPRT_CUDA_TRY(cudaMemcpyAsync(iout, iin, n * sizeof(uint16_t), cudaMemcpyDeviceToDevice,
+                                     s));
+    }
+    for (int64_t run = n_gp; run < n; run *= 2) {
+      xs_derive_merge<<<mblocks, 256, 0, s>>>(ks[src], is[src], ks[src ^ 1], is[src ^ 1], n, run);
+      src ^= 1;
+    }
+  }
   xs_derive_unionized<<<1024, 256, 0, s>>>(kout, n, U);
   xs_derive_hist<<<chunks, 256, 0, s>>>(iout, n, n_iso, hist);
   xs_derive_scan<<<n_iso, kScanThreads, 0, s>>>(hist, chunks, n_iso);

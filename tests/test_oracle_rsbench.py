@@ -125,3 +125,19 @@ def test_rs_counts(rs_tables):
     assert 40 < per[8] < 75          # nuclides per lookup (fuel has 321 of 355)
     assert 8 < per[7] / per[8] < 12  # ~avg_poles/avg_windows poles per window
     assert per[6] / per[5] < 0.02    # the Abrarov branch is rare
+
+
+def test_abrarov_branch_without_sqrt():
+    """The GPU decides the Faddeeva branch as x < 36 instead of sqrt(x) < 6 (x = |Z|^2 with
+    separately rounded terms, rs_body.cuh rs_abrarov_branch): identical for every double
+    because sqrt is correctly rounded and 36 is a perfect square -- checked on the 2e5
+    doubles nearest 36 and on 1e6 random x in [0, 100)."""
+    a = b = 36.0
+    xs = [36.0]
+    for _ in range(100_000):
+        a, b = np.nextafter(a, 0.0), np.nextafter(b, 100.0)
+        xs += [a, b]
+    xs = np.array(xs)
+    assert ((np.sqrt(xs) < 6.0) == (xs < 36.0)).all()
+    r = np.random.default_rng(7).uniform(0.0, 100.0, 1_000_000)
+    assert ((np.sqrt(r) < 6.0) == (r < 36.0)).all()

@@ -590,6 +590,18 @@ extern "C" int omprt_xs_run_host_steps(omprt_xs_tables h, uint64_t seed, int64_t
   OMPRT_CHECK_ARG(accel || (h.index_grid && h.nuclide_grid),
                   "the plain path needs the int32 index grid and the nuclide grid");
   OMPRT_CHECK_ARG(!accel || h.n_gridpoints <= 65536, "16-bit index: n_gridpoints > 65536");
+  // the material tables are host memory here: every listed nuclide must exist (a table
+  // built for fewer nuclides than the material lists name would read past the grids)
+  OMPRT_CHECK_ARG(h.max_num_nucs > 0, "omprt_xs_run_host_steps: max_num_nucs must be > 0");
+  for (int m = 0; m < 12; ++m) {
+    OMPRT_CHECK_ARG(h.num_nucs[m] >= 0 && h.num_nucs[m] <= h.max_num_nucs,
+                    "material %d: num_nucs out of range", m);
+    for (int k = 0; k < h.num_nucs[m]; ++k) {
+      const int32_t q = h.mats[m * h.max_num_nucs + k];
+      OMPRT_CHECK_ARG(q >= 0 && q < h.n_isotopes, "material %d lists nuclide %d of %d", m, q,
+                      h.n_isotopes);
+    }
+  }
   cudaStream_t s = as_stream(stream);
   const int32_t log2_bins = 18;  // 2^18 search bins: ~1.5 bisection probes (profiles/l2_pack_x57.txt)
   uint64_t asz[3] = {0, 0, 0};

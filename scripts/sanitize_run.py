@@ -89,8 +89,46 @@ def main():
     cs = torch.zeros(1, dtype=torch.float64, device=dev)
     omprt.omprt_su3_mult(At, Bt, Ct, ns, cs, 0, 128, A)
     omprt.omprt_cuda_su3_mult(At, Bt, Ct, ns, cs, 0, 128, 0)
+    # staged / streamed variants: SU(3) per-thread bulk, warp cp.async, 2-D tensor tiles; C1
+    # TMA-streamed Fig. 5 columns
+    # (synccheck cannot track the per-thread mbarriers of OMPRT_TMA_STAGED -- 2 per thread:
+    # "overflow of tracked cuda::barrier structures", then the instrumented run faults --
+    # so the round script skips that variant under synccheck only)
+    staged = [] if os.environ.get("OMPRT_SANITIZE_NO_PER_THREAD_BULK") else [
+        omprt.OMPRT_TMA_STAGED]
+    for fl in staged + [omprt.OMPRT_WARP_STAGED, omprt.OMPRT_TMA_TILED]:
+        omprt.omprt_su3_mult(At, Bt, Ct, ns, cs, 2, 128, fl)
+        omprt.omprt_cuda_su3_mult(At, Bt, Ct, ns, cs, 2, 128, fl)
+    n1 = 8 * 128 * 40 + 77  # whole boxes, a partial box and a ragged last trip
+    x1, b1, c1 = gen.axpy_inputs(n1)
+    b1t, c1t = torch.from_numpy(b1).to(dev), torch.from_numpy(c1).to(dev)
+    a1t = torch.empty_like(b1t)
+    omprt.omprt_spmd_axpy_sum(n1, x1, b1t, c1t, a1t, s, 8, 128, omprt.OMPRT_TMA_STREAM)
+    omprt.omprt_cuda_axpy_sum(n1, x1, b1t, c1t, a1t, s, 8, 128, omprt.OMPRT_TMA_STREAM)
+    # lock-step loops with the warp-collective hook
+    st = torch.zeros(5000, dtype=torch.int32, device=dev)
+    hk = torch.zeros(3 * 64, dtype=torch.int32, device=dev)
+    er = torch.zeros(1, dtype=torch.int32, device=dev)
+    for dyn in (False, True):
+        omprt.omprt_lockstep_probe(5000, 3, 64, dyn, st, hk, er)
+    # the e2e derivation (merge levels, index rows, brackets, bins) and pipelined host steps
+    import numpy as np
+    tx = gen.XSTables(n_isotopes=68, n_gridpoints=40)  # the material lists name 68 nuclides
+    g = np.ascontiguousarray(tx.nuclide_grid.reshape(68, 40, 6).copy())
+    g[:, :, 0] = np.sort(np.floor(g[:, :, 0] * 64.0) / 64.0, axis=1)  # ties
+    for grid in (tx.nuclide_grid, g):
+        gt = torch.from_numpy(np.ascontiguousarray(grid.reshape(-1))).to(dev)
+        U = torch.empty(68 * 40, dtype=torch.float64, device=dev)
+        i16 = torch.empty(68 * 40 * 68, dtype=torch.int16, device=dev)
+        tmp = torch.empty(omprt.omprt_xs_derive_tmp_bytes(68, 40), dtype=torch.uint8, device=dev)
+        omprt.omprt_xs_derive(gt, 68, 40, U, i16, tmp)
+    raw = {k: torch.from_numpy(getattr(tx, k)).pin_memory()
+           for k in ("nuclide_grid", "num_nucs", "mats", "concs")}
+    hs = omprt.xs_host_struct(tx, raw, derive=True)
+    omprt.omprt_xs_run_host_steps(hs, gen.XS_LOOKUP_SEED, 0, 20_000, 2, flags=F)
     torch.cuda.synchronize()
-    print("sanitize_run: ok, device status", omprt.omprt_device_status(0)[0])
+    print("sanitize_run: ok, device status", omprt.omprt_device_status(0)[0],
+          "lockstep errors", int(er.item()))
 
 
 if __name__ == "__main__":

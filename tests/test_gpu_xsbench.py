@@ -283,6 +283,26 @@ def test_end_to_end_derived_tables(rt, xs_small):
                        xs_small.mats.nbytes + xs_small.concs.nbytes) and d2h == 8
 
 
+def test_end_to_end_small_table_and_bad_materials(rt):
+    """A small table (68 nuclides x 40 gridpoints, derived on the device) checks against the
+    oracle; a table with fewer nuclides than the material lists name is rejected on the
+    host (it would read past the grids) instead of launching."""
+    t = gen.XSTables(n_isotopes=68, n_gridpoints=40)
+    pinned = {k: torch.from_numpy(getattr(t, k)).pin_memory()
+              for k in ("nuclide_grid", "num_nucs", "mats", "concs")}
+    hs = rt.xs_host_struct(t, pinned, derive=True)
+    n = 20_000
+    ref = int(oracle.xs_lookup(t, 0, n).sum())
+    cks, _, _ = rt.omprt_xs_run_host_steps(hs, SEED, 0, n, 2, flags=rt.OMPRT_XS_FLAT)
+    assert cks == [ref] * 2
+    bad = gen.XSTables(n_isotopes=9, n_gridpoints=40)
+    pb = {k: torch.from_numpy(getattr(bad, k)).pin_memory()
+          for k in ("nuclide_grid", "num_nucs", "mats", "concs")}
+    with pytest.raises(rt.OmprtError):
+        rt.omprt_xs_run_host_steps(rt.xs_host_struct(bad, pb, derive=True), SEED, 0, 100, 1,
+                                   flags=rt.OMPRT_XS_FLAT)
+
+
 @pytest.mark.parametrize("teams", [0, 1, 5])
 def test_flat_dynamic_schedule(rt, xs_acc, xs_small, teams):
     """OMPRT_SCHED_DYNAMIC on the flattened lookup loop: every lookup's verification value

@@ -21,7 +21,18 @@ struct DI {
 };
 static DI g_di;
 
-template <int P = 2>
+__device__ __forceinline__ uint16_t ld_na_u16(const uint16_t* p) {
+  unsigned short v;
+  asm("ld.global.nc.L1::no_allocate.u16 %0, [%1];" : "=h"(v) : "l"(p));
+  return v;
+}
+__device__ __forceinline__ uint16_t ld_el_u16(const uint16_t* p) {
+  unsigned short v;
+  asm("ld.global.nc.L1::evict_last.u16 %0, [%1];" : "=h"(v) : "l"(p));
+  return v;
+}
+
+template <int P = 2, int Mode = 0>  // Mode 0: delta8; 1: index16 no_allocate; 2: index16 evict_last
 struct XSDeltaLookup {
   const XSTables& t;
   const DI& di;
@@ -43,6 +54,10 @@ struct XSDeltaLookup {
       : t(tab), di(d), seed0(seed), first(f), ver(v), mats(ms), concs(cs) {}
 
   __device__ __forceinline__ int32_t index_at(int32_t q) const {
+    if constexpr (Mode == 1)
+      return (int32_t)ld_na_u16(t.index_grid16 + (int64_t)idx * t.n_isotopes + q);
+    if constexpr (Mode == 2)
+      return (int32_t)ld_el_u16(t.index_grid16 + (int64_t)idx * t.n_isotopes + q);
     return (int32_t)__ldg(di.coarse + (int64_t)(idx >> kCoarseShift) * t.n_isotopes + q) +
            (int32_t)__ldg(di.delta + (int64_t)idx * t.n_isotopes + q);
   }
@@ -126,8 +141,8 @@ __device__ __forceinline__ void flat_loop(Body& lookup, int32_t count) {
   }
 }
 
-template <int V>
-__global__ void __launch_bounds__(kThreads, 4)
+template <int V, int TPB = kThreads, int MINB = 4>
+__global__ void __launch_bounds__(TPB, MINB)
     kern(const __grid_constant__ XSTables t, const __grid_constant__ DI di, uint64_t seed,
          int64_t first, int32_t count, uint64_t* __restrict__ ver) {
   __shared__ int32_t sm[kMatSmem];
@@ -140,8 +155,11 @@ __global__ void __launch_bounds__(kThreads, 4)
   if constexpr (V == 0) {
     XSFlatLookup<false, true> lookup(t, seed, first, ver, sm, sc);
     flat_loop(lookup, count);
-  } else {
+  } else if constexpr (V == 1) {
     XSDeltaLookup<2> lookup(t, di, seed, first, ver, sm, sc);
+    flat_loop(lookup, count);
+  } else {
+    XSDeltaLookup<2, V - 1> lookup(t, di, seed, first, ver, sm, sc);
     flat_loop(lookup, count);
   }
 }
@@ -164,11 +182,12 @@ struct Var {
   void (*k)(XSTables, DI, uint64_t, int64_t, int32_t, uint64_t*);
   bool window;
   const char* name;
+  int tpb = kThreads, minb = 4;
 };
-static Var kVars[] = {{kern<0>, false, "V0_product_body"},
-                      {kern<1>, false, "D1_delta8_index"},
-                      {kern<0>, true, "V0_product_body+packed_window"},
-                      {kern<1>, true, "D1_delta8_index+packed_window"}};
+static Var kVars[] = {{kern<0>, true, "V0_product_body+packed_window"},
+                      {kern<0, 512, 2>, true, "V0_512x2+packed_window", 512, 2},
+                      {kern<0, 1024, 1>, true, "V0_1024x1+packed_window", 1024, 1},
+                      {kern<0>, true, "V0_product_body+packed_window(again)"}};
 
 extern "C" int xsx_count() { return (int)(sizeof(kVars) / sizeof(kVars[0])); }
 extern "C" const char* xsx_name(int v) { return kVars[v].name; }
@@ -194,8 +213,8 @@ extern "C" int xsx_run(int v, XSTables t, uint64_t seed, int64_t first, int32_t 
   cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
   cudaLaunchConfig_t cfg{};
   cudaLaunchAttribute attr[1];
-  cfg.gridDim = dim3(sms * 4);
-  cfg.blockDim = dim3(kThreads);
+  cfg.gridDim = dim3(sms * kVars[v].minb);
+  cfg.blockDim = dim3(kVars[v].tpb);
   cfg.stream = (cudaStream_t)stream;
   cfg.attrs = attr;
   cfg.numAttrs = 0;

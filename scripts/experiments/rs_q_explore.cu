@@ -37,7 +37,7 @@ struct Var { KF f; int tpb; const char* name; };
 static Var vars[] = {
   {kern<false, 5>, 128, VN("dflat_128x5")}, {kern<true, 5>, 128, VN("qflat_128x5")},
   {kern<false, 4>, 128, VN("dflat_128x4")}, {kern<true, 4>, 128, VN("qflat_128x4")},
-  {kern<true, 6>, 128, VN("qflat_128x6")},
+  {kern<true, 3>, 128, VN("qflat_128x3")},
 };
 extern "C" int rsf_count() { return (int)(sizeof(vars) / sizeof(vars[0])); }
 extern "C" const char* rsf_name(int v) { return vars[v].name; }

@@ -155,6 +155,9 @@ __global__ void __launch_bounds__(TPB, MINB)
   if constexpr (V == 0) {
     XSFlatLookup<false, true> lookup(t, seed, first, ver, sm, sc);
     flat_loop(lookup, count);
+  } else if constexpr (V >= 10) {  // nuclides per step P = V - 10
+    XSFlatLookup<false, true, false, V - 10> lookup(t, seed, first, ver, sm, sc);
+    flat_loop(lookup, count);
   } else if constexpr (V == 1) {
     XSDeltaLookup<2> lookup(t, di, seed, first, ver, sm, sc);
     flat_loop(lookup, count);
@@ -184,10 +187,11 @@ struct Var {
   const char* name;
   int tpb = kThreads, minb = 4;
 };
-static Var kVars[] = {{kern<0>, true, "V0_product_body+packed_window"},
-                      {kern<0, 512, 2>, true, "V0_512x2+packed_window", 512, 2},
-                      {kern<0, 1024, 1>, true, "V0_1024x1+packed_window", 1024, 1},
-                      {kern<0>, true, "V0_product_body+packed_window(again)"}};
+static Var kVars[] = {{kern<0>, true, "V0_product_body(P=2)+packed_window"},
+                      {kern<11>, true, "P=1+packed_window"},
+                      {kern<13>, true, "P=3+packed_window"},
+                      {kern<14>, true, "P=4+packed_window"},
+                      {kern<0>, true, "V0_product_body(P=2)+packed_window(again)"}};
 
 extern "C" int xsx_count() { return (int)(sizeof(kVars) / sizeof(kVars[0])); }
 extern "C" const char* xsx_name(int v) { return kVars[v].name; }

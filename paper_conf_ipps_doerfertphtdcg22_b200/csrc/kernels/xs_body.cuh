@@ -270,6 +270,7 @@ __device__ __forceinline__ uint64_t xs_lookup_accel(const XSTables& t, uint64_t 
 // L1 traffic is what bounds this loop (ncu: L1 ~80 % busy), so the bracket records, read
 // once, bypass L1 allocation, and with SmemMats the material tables (mats, concs) come
 // from a team-shared copy (`mats`/`concs` then point to shared memory).
+constexpr int kXSFlatThreads = 256;  // team size of the flattened XS kernels
 template <bool Fused, bool SmemMats, bool Compact = false, int P = 2>
 struct XSFlatLookup {
   const XSTables& t;
@@ -382,8 +383,10 @@ struct XSFlatLookup {
     else ver[iv] = v;
   }
   // this thread's slot (static shared memory: a constant address, no register)
+  // sized for the flattened kernels' 256-thread teams (host-checked): a 1024-slot array
+  // took 8 KB of shared memory per team and, through the carve-out, L1 the lookups need
   static __device__ __forceinline__ unsigned long long* flat_acc_slot() {
-    __shared__ unsigned long long slots[1024];
+    __shared__ unsigned long long slots[kXSFlatThreads];
     return slots + threadIdx.x;
   }
 };

@@ -26,6 +26,7 @@ struct XSTraitsAssumeDebug : XSTraitsAssume {
 };
 
 constexpr int kXSThreads = 256;
+static_assert(kXSThreads == kXSFlatThreads, "XSFlatLookup::flat_acc_slot is sized for it");
 // 4 teams of 256 per SM (<= 64 registers): measured best occupancy / memory-parallelism
 // trade-off for this latency-bound gather (scripts/experiments/xs_explore.*).
 constexpr int kXSMinBlocks = 4;   // plain layout

@@ -346,7 +346,7 @@ int omprt_xs_run_host_steps(omprt_xs_tables host_tables, uint64_t seed, int64_t 
 typedef struct {
   const double *poles;      /* [n_poles][8] EA RT RA RF (re, im), 32 B aligned */
   const int32_t *pole_l;    /* [n_poles] l value in [0, numL) */
-  const double *windows;    /* [n_windows][4] T A F 0 */
+  const double *windows;    /* [n_windows][4] T A F 0, 32 B aligned */
   const int32_t *win_range; /* [n_windows][2] absolute pole [start, end) */
   const int32_t *win_off;   /* [n_nuclides+1] window CSR offsets */
   const int32_t *n_windows; /* [n_nuclides] */

@@ -222,7 +222,8 @@ inline int rs_validate(const omprt_rs_tables& t, int64_t count, uint64_t* ver, i
                       t.k0rs && t.num_nucs && t.mats && t.concs,
                   "bad RSBench tables");
   OMPRT_CHECK_ARG(ver != nullptr || count == 0, "verification is required");
-  OMPRT_CHECK_ARG(((uintptr_t)t.poles & 31) == 0, "poles must be 32 B aligned (256-bit loads)");
+  OMPRT_CHECK_ARG((((uintptr_t)t.poles | (uintptr_t)t.windows) & 31) == 0,
+                  "poles and windows must be 32 B aligned (256-bit loads)");
   OMPRT_CHECK_ARG(!(flags & OMPRT_XS_FLAT) || !(flags & OMPRT_ASSUME_OVERSUB),
                   "OMPRT_XS_FLAT runs a persistent grid (no oversubscription assumption)");
   OMPRT_CHECK_ARG(!(flags & OMPRT_SCHED_DYNAMIC) || (flags & OMPRT_XS_FLAT),

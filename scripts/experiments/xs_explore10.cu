@@ -32,7 +32,41 @@ __device__ __forceinline__ uint16_t ld_el_u16(const uint16_t* p) {
   return v;
 }
 
-template <int P = 2, int Mode = 0>  // Mode 0: delta8; 1: index16 no_allocate; 2: index16 evict_last
+__device__ __forceinline__ double ld_na_f64(const double* p) {
+  double v;
+  asm("ld.global.nc.L1::no_allocate.f64 %0, [%1];" : "=d"(v) : "l"(p));
+  return v;
+}
+__device__ __forceinline__ int32_t ld_na_s32(const int32_t* p) {
+  int32_t v;
+  asm("ld.global.nc.L1::no_allocate.s32 %0, [%1];" : "=r"(v) : "l"(p));
+  return v;
+}
+// binned_grid_search with the bins and probes not allocated in L1 (Probe: 1 bins+probes,
+// 2 probes only)
+template <int Probe>
+__device__ __forceinline__ int32_t search_na(const XSTables& t, double E) {
+  const int64_t H = 1ll << t.log2_bins;
+  int64_t b = (int64_t)(E * (double)H);
+  if (b > H - 1) b = H - 1;
+  int32_t lo, hi;
+  if constexpr (Probe == 1) {
+    lo = ld_na_s32(t.bins + b);
+    hi = ld_na_s32(t.bins + b + 1) + 1;
+  } else {
+    lo = __ldg(t.bins + b);
+    hi = __ldg(t.bins + b + 1) + 1;
+  }
+  if (hi > (int32_t)t.n_union - 1) hi = (int32_t)t.n_union - 1;
+  while (hi - lo > 1) {
+    const int32_t mid = lo + ((hi - lo) >> 1);
+    if (ld_na_f64(t.unionized + mid) > E) hi = mid;
+    else lo = mid;
+  }
+  return lo;
+}
+
+template <int P = 2, int Mode = 0>  // Mode 0: delta8; 1: index16 no_allocate; 2: index16 evict_last; 3/4: index16 __ldg, search_na<1/2>
 struct XSDeltaLookup {
   const XSTables& t;
   const DI& di;
@@ -58,6 +92,8 @@ struct XSDeltaLookup {
       return (int32_t)ld_na_u16(t.index_grid16 + (int64_t)idx * t.n_isotopes + q);
     if constexpr (Mode == 2)
       return (int32_t)ld_el_u16(t.index_grid16 + (int64_t)idx * t.n_isotopes + q);
+    if constexpr (Mode >= 3)
+      return (int32_t)__ldg(t.index_grid16 + (int64_t)idx * t.n_isotopes + q);
     return (int32_t)__ldg(di.coarse + (int64_t)(idx >> kCoarseShift) * t.n_isotopes + q) +
            (int32_t)__ldg(di.delta + (int64_t)idx * t.n_isotopes + q);
   }
@@ -65,7 +101,8 @@ struct XSDeltaLookup {
     uint64_t seed = s;
     E = lcg_double(seed);
     mat = pick_mat(seed);
-    idx = binned_grid_search(t, E);
+    if constexpr (Mode >= 3) idx = search_na<Mode - 2>(t, E);
+    else idx = binned_grid_search(t, E);
     nn = __ldg(t.num_nucs + mat);
     m0 = m1 = m2 = m3 = m4 = 0.0;
     j = 0;
@@ -187,11 +224,10 @@ struct Var {
   const char* name;
   int tpb = kThreads, minb = 4;
 };
-static Var kVars[] = {{kern<0>, true, "V0_product_body(P=2)+packed_window"},
-                      {kern<11>, true, "P=1+packed_window"},
-                      {kern<13>, true, "P=3+packed_window"},
-                      {kern<14>, true, "P=4+packed_window"},
-                      {kern<0>, true, "V0_product_body(P=2)+packed_window(again)"}};
+static Var kVars[] = {{kern<0>, true, "V0_product_body+packed_window"},
+                      {kern<4>, true, "S1_bins+probes_no_L1+packed_window"},
+                      {kern<5>, true, "S2_probes_no_L1+packed_window"},
+                      {kern<0>, true, "V0_product_body+packed_window(again)"}};
 
 extern "C" int xsx_count() { return (int)(sizeof(kVars) / sizeof(kVars[0])); }
 extern "C" const char* xsx_name(int v) { return kVars[v].name; }

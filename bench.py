@@ -625,13 +625,6 @@ def run_secondary(omprt, torch, gen, dev, stream, scrub):
         lambda: omprt.omprt_su3_mult(At, Bt, Ct, ns, ck, 0, 128, A),
         lambda: omprt.omprt_cuda_su3_mult(At, Bt, Ct, ns, ck, 0, 128, 0),
         stream, scrub)
-    TS = omprt.OMPRT_TMA_STAGED
-    t_rs, t_ts = _time_pair(
-        lambda: omprt.omprt_su3_mult(At, Bt, Ct, ns, ck, 0, 128, TS),
-        lambda: omprt.omprt_cuda_su3_mult(At, Bt, Ct, ns, ck, 0, 128, TS),
-        stream, scrub)
-    res["c5_su3_32^4_tma_staged"] = {"rt_ms": t_rs, "twin_ms": t_ts, "overhead": t_rs / t_ts - 1,
-                                     "GBps_alg": 1152 * ns / t_rs / 1e6}
     WS = omprt.OMPRT_WARP_STAGED
     t_rw, t_tww = _time_pair(
         lambda: omprt.omprt_su3_mult(At, Bt, Ct, ns, ck, 0, 128, WS),

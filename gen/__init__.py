@@ -236,6 +236,20 @@ class XSTables:
                 + self.num_nucs.nbytes + self.mats.nbytes + self.concs.nbytes)
 
 
+def xs_tied_channels(t: "XSTables") -> "XSTables":
+    """A copy of XS tables with channels made equal at every gridpoint: elastic := total,
+    fission := nu-fission := absorption (columns 2 := 1, 4 := 5 := 3).  Input data only:
+    lookups on it accumulate equal macroscopic values, so ties in the argmax are certain."""
+    import copy
+    c = copy.copy(t)
+    g = t.nuclide_grid.reshape(-1, 6).copy()
+    g[:, 2] = g[:, 1]
+    g[:, 4] = g[:, 3]
+    g[:, 5] = g[:, 3]
+    c.nuclide_grid = np.ascontiguousarray(g.reshape(t.nuclide_grid.shape))
+    return c
+
+
 # --------------------------------------------------------------------------------------
 # C4: RSBench-shaped multipole tables (SURVEY App. A.2), CSR layout
 # --------------------------------------------------------------------------------------

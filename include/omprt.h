@@ -84,15 +84,12 @@ extern "C" {
 /* omprt_generic_team, NEXT f2 (P:172 globalization elimination): generic mode with
  * the globalized arrays in static team-local shared memory -- no stack (0 B).  inner_n <= 256. */
 #define OMPRT_DEGLOBALIZE (1u << 12)
-/* omprt_su3_mult: move the 576 B site records with bulk (TMA) copies through padded shared
- * memory slots (one persistent team of 128 per SM, per-thread double buffering); teams = 0:
- * one per SM.  Not combined with OMPRT_ASSUME_OVERSUB. */
-#define OMPRT_TMA_STAGED (1u << 13)
+/* (1u << 13) is unused: a per-thread bulk-copy SU(3) staging measured slower and removed. */
 /* omprt_su3_mult / omprt_cuda_su3_mult: warp-cooperative staging -- a warp's 32 consecutive
  * site records (one contiguous 18 KiB range) are copied by coalesced 16 B cp.async into
  * padded shared-memory slots and written back by coalesced 16 B stores (one persistent team
- * of 192 per SM, per-warp double buffering); teams = 0: one per SM.  Exclusive with
- * OMPRT_TMA_STAGED; not combined with OMPRT_ASSUME_OVERSUB. */
+ * of 192 per SM, per-warp double buffering); teams = 0: one per SM.  Not combined with
+ * OMPRT_ASSUME_OVERSUB. */
 #define OMPRT_WARP_STAGED (1u << 14)
 /* omprt_xs_lookup / omprt_cuda_xs_lookup (B200 layouts required) and the e2e entry points:
  * flattened execution -- a persistent grid (teams = 0: the device's resident teams) whose
@@ -121,7 +118,7 @@ extern "C" {
  * 32 consecutive site records moved by ONE 2-D TMA tensor copy in (box [32][74] doubles:
  * the 2 columns past a 576 B record are zero-filled, giving padded 592 B shared-memory
  * slots) and one out (out-of-tensor columns are not written); double buffered per warp.
- * Not combined with OMPRT_ASSUME_OVERSUB, OMPRT_TMA_STAGED or OMPRT_WARP_STAGED.  A and C
+ * Not combined with OMPRT_ASSUME_OVERSUB or OMPRT_WARP_STAGED.  A and C
  * 16 B aligned. */
 #define OMPRT_TMA_TILED (1u << 18)
 /* omprt_spmd_axpy_sum / omprt_cuda_axpy_sum: the Fig. 5 loop with its operands moved by 2-D
@@ -256,23 +253,25 @@ typedef struct {
   const uint16_t *index_grid16;/* [n_union][n_isotopes] */
   const double *brackets;      /* [n_isotopes][n_gridpoints-1][12], 32 B aligned */
   int32_t log2_bins, pad2;
-  /* optional compact index grid (omprt_xs_build_compact; both NULL or both set; used by
-   * the OMPRT_XS_FLAT launches, with the B200 layouts above): */
-  const uint16_t *idx_rows;    /* [ceil(n_union/16)][n_isotopes]: #{v <= 16m : owner[v] = q} */
-  const uint8_t *owner;        /* [n_union rounded up to 16]: nuclide of unionized energy v */
 } omprt_xs_tables;
 /* Lookups first..first+count-1 (lookup i draws its energy and material from
  * fast_forward_LCG(seed, 2i), so results do not depend on sharding):
- * verification[i-first] = 1 + argmax of the 5 macroscopic cross sections.  teams = 0:
- * ceil(count/threads).  With OMPRT_FUSED_REDUCTION, verification may be NULL and
- * *checksum_inout += sum of the verification values instead (checksum_inout device u64).
- * flags: OMPRT_ASSUME_OVERSUB | OMPRT_FUSED_REDUCTION | OMPRT_DEBUG_BUILD. */
+ * verification[i-first] = 1 + argmax of the 5 macroscopic cross sections (the first
+ * maximum wins).  teams = 0: ceil(count/threads).  With OMPRT_FUSED_REDUCTION,
+ * verification may be NULL and *checksum_inout += sum of the verification values instead
+ * (checksum_inout device u64).  macro (nullable; test build, P:266 -- the values the
+ * verification is the argmax of): [count][5] doubles, macro[(i-first)*5 + k] = macroscopic
+ * xs k (total, elastic, absorption, fission, nu-fission), bit-identical to SURVEY App. A.1's
+ * definition; written by a separate (unfused, release) instantiation of the same body, not
+ * the timed one; OMPRT_E_INVAL with OMPRT_FUSED_REDUCTION or OMPRT_DEBUG_BUILD.
+ * flags: OMPRT_ASSUME_OVERSUB | OMPRT_FUSED_REDUCTION | OMPRT_DEBUG_BUILD | OMPRT_XS_FLAT |
+ * OMPRT_SCHED_DYNAMIC | OMPRT_XS_NO_L2_PERSIST. */
 int omprt_xs_lookup(omprt_xs_tables t, uint64_t seed, int64_t first, int64_t count,
-                    uint64_t *verification, uint64_t *checksum_inout, int32_t teams,
-                    int32_t threads, uint32_t flags, void *stream);
+                    uint64_t *verification, uint64_t *checksum_inout, double *macro,
+                    int32_t teams, int32_t threads, uint32_t flags, void *stream);
 int omprt_cuda_xs_lookup(omprt_xs_tables t, uint64_t seed, int64_t first, int64_t count,
-                         uint64_t *verification, uint64_t *checksum_inout, int32_t teams,
-                         int32_t threads, uint32_t flags, void *stream);
+                         uint64_t *verification, uint64_t *checksum_inout, double *macro,
+                         int32_t teams, int32_t threads, uint32_t flags, void *stream);
 /* Byte sizes of the three accelerated-layout buffers for tables of this shape:
  * sizes[0] bins, sizes[1] index_grid16, sizes[2] brackets.  OMPRT_E_INVAL when
  * n_gridpoints > 65536 (the 16-bit index cannot hold it) or log2_bins not in [1, 28]. */
@@ -299,22 +298,6 @@ int omprt_xs_derive_tmp_bytes(int32_t n_isotopes, int32_t n_gridpoints, uint64_t
 int omprt_xs_derive(const double *nuclide_grid, int32_t n_isotopes, int32_t n_gridpoints,
                     double *unionized, uint16_t *index_grid16, void *tmp, uint64_t tmp_bytes,
                     void *stream);
-/* Compact index grid (reading R-X1): the same index grid as every 16th row of position
- * counts plus the nuclide id of every unionized energy, so a lookup rebuilds its row
- * exactly (index = clip(rows[e/16][q] + #{v in (16*(e/16), e] : owner[v] = q} - 1, 0,
- * n_gridpoints - 2)) from 7.3 MB of tables instead of 104.5 MB of 16-bit rows (small
- * problem).  Built from the nuclide grids on the device (the omprt_xs_derive sort):
- *   owner[v]   = nuclide of the v-th smallest energy (0xFF past n_union, up to the
- *                multiple of 16), idx_rows[m*n_isotopes + q] = #{v <= 16m : owner[v] = q}.
- * Sizes: sizes[0] idx_rows bytes, sizes[1] owner bytes.  tmp: >= omprt_xs_derive_tmp_bytes.
- * Synchronizes `stream` (it checks the table): OMPRT_E_INVAL unless 0 < n_isotopes <= 255,
- * 2 <= n_gridpoints <= 65535 and the two smallest and the two largest energies are
- * distinct (the ends the lookup's clamped search can return; everywhere else ties are
- * exact).  owner must be 16 B aligned. */
-int omprt_xs_compact_sizes(int32_t n_isotopes, int32_t n_gridpoints, uint64_t *sizes);
-int omprt_xs_build_compact(const double *nuclide_grid, int32_t n_isotopes, int32_t n_gridpoints,
-                           uint16_t *idx_rows, uint8_t *owner, void *tmp, uint64_t tmp_bytes,
-                           void *stream);
 /* K11 ("we moved the reduction out of the timed kernel"): *out_inout += sum v[i]
  * (u64, wraps mod 2^64). */
 int omprt_u64_sum(const uint64_t *v, int64_t n, uint64_t *out_inout, void *stream);

@@ -45,7 +45,7 @@ __global__ void __launch_bounds__(1024)
       atomicAdd(count + i, 1);
     }
   });
-  league_reduce(team, team_reduce_to_main(team, acc, Plus{}), Plus{}, sum_inout, partials,
+  league_reduce_threads(team, acc, Plus{}, sum_inout, partials,
                 ticket);
 }
 
@@ -163,7 +163,7 @@ __global__ void __launch_bounds__(256)
         acc += v;
         rec(i);
       });
-  league_reduce(team, team_reduce_to_main(team, acc, Plus{}), Plus{}, sum_inout, partials,
+  league_reduce_threads(team, acc, Plus{}, sum_inout, partials,
                 ticket);
 }
 

@@ -61,7 +61,7 @@ __global__ void __launch_bounds__(1024)
       }
     }
   });
-  league_reduce(team, team_reduce_to_main(team, acc, Plus{}), Plus{}, sum_inout, partials,
+  league_reduce_threads(team, acc, Plus{}, sum_inout, partials,
                 ticket);
 }
 
@@ -153,7 +153,7 @@ __global__ void __launch_bounds__(1024)
       }
     }
   });
-  league_reduce(team, team_reduce_to_main(team, acc, Plus{}), Plus{}, sum_inout, partials,
+  league_reduce_threads(team, acc, Plus{}, sum_inout, partials,
                 ticket);
 }
 

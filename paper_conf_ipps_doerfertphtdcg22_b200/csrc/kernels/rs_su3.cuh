@@ -307,7 +307,7 @@ __global__ void __launch_bounds__(kSU3Threads)
     acc += su3_site(A + (int64_t)s * 72, B, Cm + (int64_t)s * 72);
   });
   if constexpr (Checksum)
-    league_reduce(team, team_reduce_to_main(team, acc, Plus{}), Plus{}, checksum, partials,
+    league_reduce_threads(team, acc, Plus{}, checksum, partials,
                   ticket);
 }
 
@@ -361,9 +361,8 @@ OMPRT_REGISTER_KERNEL(omprt_su3_rt_loop, omprt_su3_rt<SU3TraitsLoop, true>)
 OMPRT_REGISTER_KERNEL(cuda_su3_twin, cuda_su3_twin<true>)
 
 // staged variants (su3_staged.cuh)
-inline int su3_staged_launch(bool twin, bool warp, const double* A, const double* B, double* Cm,
-                             int64_t n, double* ck, int32_t teams, Workspace* w,
-                             cudaStream_t s);
+inline int su3_staged_launch(bool twin, const double* A, const double* B, double* Cm, int64_t n,
+                             double* ck, int32_t teams, Workspace* w, cudaStream_t s);
 inline int su3_tiled_launch(bool twin, const double* A, const double* B, double* Cm, int64_t n,
                             double* ck, int32_t teams, Workspace* w, cudaStream_t s);
 
@@ -463,7 +462,7 @@ extern "C" int omprt_su3_mult(const double* A, const double* B, double* Cm, int6
   Workspace* w;
   if (int r = current_ws(&w)) return r;
   if (flags & OMPRT_TMA_TILED) {
-    OMPRT_CHECK_ARG(!(flags & (OMPRT_ASSUME_OVERSUB | OMPRT_TMA_STAGED | OMPRT_WARP_STAGED)),
+    OMPRT_CHECK_ARG(!(flags & (OMPRT_ASSUME_OVERSUB | OMPRT_WARP_STAGED)),
                     "OMPRT_TMA_TILED: persistent grid, exclusive with the other stagings");
     int32_t tm = 1;
     if (int r = su3_validate(A, B, Cm, n_sites, tm, threads, 0, checksum_inout, w)) return r;
@@ -471,16 +470,14 @@ extern "C" int omprt_su3_mult(const double* A, const double* B, double* Cm, int6
     return su3_tiled_launch(false, A, B, Cm, n_sites, checksum_inout, teams, w,
                             as_stream(stream));
   }
-  if (flags & (OMPRT_TMA_STAGED | OMPRT_WARP_STAGED)) {
+  if (flags & OMPRT_WARP_STAGED) {
     OMPRT_CHECK_ARG(threads == kSU3Threads && !(flags & OMPRT_ASSUME_OVERSUB),
-                    "the staged variants run a persistent grid (no assumption)");
-    OMPRT_CHECK_ARG((flags & OMPRT_TMA_STAGED) == 0 || (flags & OMPRT_WARP_STAGED) == 0,
-                    "OMPRT_TMA_STAGED and OMPRT_WARP_STAGED are exclusive");
+                    "the staged variant runs a persistent grid (no assumption)");
     int32_t tm = 1;
     if (int r = su3_validate(A, B, Cm, n_sites, tm, threads, 0, checksum_inout, w)) return r;
     if (n_sites == 0) return OMPRT_OK;
-    return su3_staged_launch(false, (flags & OMPRT_WARP_STAGED) != 0, A, B, Cm, n_sites,
-                             checksum_inout, teams, w, as_stream(stream));
+    return su3_staged_launch(false, A, B, Cm, n_sites, checksum_inout, teams, w,
+                             as_stream(stream));
   }
   if (int r = su3_validate(A, B, Cm, n_sites, teams, threads, flags, checksum_inout, w)) return r;
   if (n_sites == 0) return OMPRT_OK;
@@ -510,18 +507,16 @@ extern "C" int omprt_cuda_su3_mult(const double* A, const double* B, double* Cm,
   int32_t tm = 0;
   if (int r = su3_validate(A, B, Cm, n_sites, tm, threads, 0, checksum_inout, w)) return r;
   if (flags & OMPRT_TMA_TILED) {
-    OMPRT_CHECK_ARG(!(flags & (OMPRT_TMA_STAGED | OMPRT_WARP_STAGED)),
-                    "OMPRT_TMA_TILED is exclusive with the other stagings");
+    OMPRT_CHECK_ARG(!(flags & OMPRT_WARP_STAGED),
+                    "OMPRT_TMA_TILED is exclusive with the other staging");
     if (n_sites == 0) return OMPRT_OK;
     return su3_tiled_launch(true, A, B, Cm, n_sites, checksum_inout, teams, w,
                             as_stream(stream));
   }
-  if (flags & (OMPRT_TMA_STAGED | OMPRT_WARP_STAGED)) {
-    OMPRT_CHECK_ARG((flags & OMPRT_TMA_STAGED) == 0 || (flags & OMPRT_WARP_STAGED) == 0,
-                    "OMPRT_TMA_STAGED and OMPRT_WARP_STAGED are exclusive");
+  if (flags & OMPRT_WARP_STAGED) {
     if (n_sites == 0) return OMPRT_OK;
-    return su3_staged_launch(true, (flags & OMPRT_WARP_STAGED) != 0, A, B, Cm, n_sites,
-                             checksum_inout, teams, w, as_stream(stream));
+    return su3_staged_launch(true, A, B, Cm, n_sites, checksum_inout, teams, w,
+                             as_stream(stream));
   }
   (void)teams;
   (void)flags;

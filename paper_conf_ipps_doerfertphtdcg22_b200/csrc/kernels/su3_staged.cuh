@@ -1,9 +1,9 @@
-// C5 with shared-memory staging: OMPRT_TMA_STAGED (per-thread bulk copies) and
-// OMPRT_WARP_STAGED (warp-cooperative cp.async).  TMA staging: the SU(3) site loop as a persistent
-// `distribute parallel for` (one team of 128 per SM, Fig. 5 assignment) whose site records
-// (576 B, AoS) are moved by bulk copies into padded shared-memory slots and back
-// (omprt/device/staging.cuh), instead of 32-line-wide strided global accesses.  The twin runs
-// the same per-thread double-buffered bulk-copy pipeline, written by hand.
+// C5 with shared-memory staging: OMPRT_WARP_STAGED (warp-cooperative cp.async) and
+// OMPRT_TMA_TILED (one 2-D TMA tensor copy per warp tile).  The SU(3) site loop runs as a
+// persistent `distribute parallel for` (Fig. 5 assignment) whose site records (576 B, AoS)
+// are moved into padded shared-memory slots and back (omprt/device/staging.cuh), instead of
+// 32-line-wide strided global accesses.  Each twin runs the same pipeline, written by hand.
+// (A per-thread bulk-copy variant was measured slower -- 0.33 vs 0.20 ms -- and removed.)
 #pragma once
 #include <cuda.h>
 #include <cudaTypedefs.h>
@@ -20,7 +20,6 @@ using namespace omprt;
 constexpr unsigned kSU3Rec = 576;   // 4 links x 3 x 3 complex fp64
 constexpr unsigned kSU3Slot = 592;  // 148 words: 8 consecutive threads' 16 B loads hit
                                     // disjoint bank quads (conflict-free LDS.128)
-constexpr int kSU3StagedThreads = 128;
 
 // The body on a staged record (in place): C[l] = A[l] x B[l], the App. A.3 fma order, the
 // same (l, r, c) accumulation of Re C as su3_site.
@@ -96,72 +95,6 @@ __device__ __forceinline__ void twin_ticket_sum(double acc, double* checksum, do
 
 struct SU3StagedTraits : DefaultTraits {};  // persistent grid: the loop stays
 
-template <class Tr, bool Checksum>
-__global__ void __launch_bounds__(kSU3StagedThreads, 1)
-    omprt_su3_staged_rt(const double* __restrict__ A, const double2* __restrict__ B,
-                        double* __restrict__ Cm, typename Tr::Idx n_sites, double* checksum,
-                        double* partials, unsigned* ticket) {
-  using Idx = typename Tr::Idx;
-  Team<Tr> team = init<Tr>();
-  double acc = 0.0;
-  distribute_parallel_for_staged<Tr, kSU3Rec, kSU3Slot>(
-      team, n_sites, reinterpret_cast<const unsigned char*>(A),
-      reinterpret_cast<unsigned char*>(Cm),
-      [&](Idx, unsigned char* slot) { acc += su3_site_slot(slot, B); });
-  if constexpr (Checksum)
-    league_reduce(team, team_reduce_to_main(team, acc, Plus{}), Plus{}, checksum, partials,
-                  ticket);
-}
-
-// Bare CUDA twin: the same per-thread bulk-copy pipeline and reduction, by hand.
-template <bool Checksum>
-__global__ void __launch_bounds__(kSU3StagedThreads, 1)
-    cuda_su3_staged_twin(const double* __restrict__ A, const double2* __restrict__ B,
-                         double* __restrict__ Cm, int32_t n_sites, double* checksum,
-                         double* partials, unsigned* ticket) {
-  extern __shared__ __align__(128) unsigned char smem[];
-  const unsigned nt = blockDim.x, t = threadIdx.x;
-  unsigned char* slot0 = smem + t * kSU3Slot;
-  unsigned char* slot1 = smem + (nt + t) * kSU3Slot;
-  uint64_t* bar = reinterpret_cast<uint64_t*>(smem + 2 * nt * kSU3Slot) + 2 * t;
-  tma::mbar_init(bar, 1);
-  tma::mbar_init(bar + 1, 1);
-  tma::fence_mbar_init();
-  const unsigned char* in = reinterpret_cast<const unsigned char*>(A);
-  unsigned char* out = reinterpret_cast<unsigned char*>(Cm);
-  const int32_t stride = gridDim.x * nt;
-  int32_t s = blockIdx.x * nt + t;
-  double acc = 0.0;
-  if (s < n_sites) {
-    tma::mbar_arrive_expect_tx(bar, kSU3Rec);
-    tma::bulk_load(slot0, in + (size_t)s * kSU3Rec, kSU3Rec, bar);
-  }
-  uint32_t ph0 = 0, ph1 = 0;
-  for (unsigned k = 0; s < n_sites; s += stride, ++k) {
-    unsigned char* cur = (k & 1) ? slot1 : slot0;
-    unsigned char* nxt = (k & 1) ? slot0 : slot1;
-    uint64_t* bcur = bar + (k & 1);
-    uint64_t* bnxt = bar + ((k & 1) ^ 1);
-    if (s + stride < n_sites) {
-      tma::bulk_wait_read<0>();
-      tma::mbar_arrive_expect_tx(bnxt, kSU3Rec);
-      tma::bulk_load(nxt, in + (size_t)(s + stride) * kSU3Rec, kSU3Rec, bnxt);
-    }
-    tma::mbar_wait(bcur, (k & 1) ? ph1 : ph0);
-    if (k & 1) ph1 ^= 1u;
-    else ph0 ^= 1u;
-    acc += su3_site_slot(cur, B);
-    tma::fence_proxy_async_smem();
-    tma::bulk_store(out + (size_t)s * kSU3Rec, cur, kSU3Rec);
-    tma::bulk_commit();
-  }
-  tma::bulk_wait<0>();
-  if constexpr (Checksum) twin_ticket_sum(acc, checksum, partials, ticket);
-}
-
-OMPRT_REGISTER_KERNEL(omprt_su3_staged_rt, omprt_su3_staged_rt<SU3StagedTraits, true>)
-OMPRT_REGISTER_KERNEL(cuda_su3_staged_twin, cuda_su3_staged_twin<true>)
-
 // ---- warp-cooperative staging (OMPRT_WARP_STAGED): coalesced cp.async in, STG.128 out ----
 constexpr int kSU3WarpThreads = 192;  // 6 warps x 2 x 32 slots x 592 B = 222 KB per team
 
@@ -178,7 +111,7 @@ __global__ void __launch_bounds__(kSU3WarpThreads, 1)
       reinterpret_cast<unsigned char*>(Cm),
       [&](Idx, unsigned char* slot) { acc += su3_site_slot(slot, B); });
   if constexpr (Checksum)
-    league_reduce(team, team_reduce_to_main(team, acc, Plus{}), Plus{}, checksum, partials,
+    league_reduce_threads(team, acc, Plus{}, checksum, partials,
                   ticket);
 }
 
@@ -265,7 +198,7 @@ __global__ void __launch_bounds__(kSU3TiledThreads, 1)
       team, n_sites, &tin, &tout,
       [&](Idx, unsigned char* slot) { acc += su3_site_slot(slot, B); });
   if constexpr (Checksum)
-    league_reduce(team, team_reduce_to_main(team, acc, Plus{}), Plus{}, checksum, partials,
+    league_reduce_threads(team, acc, Plus{}, checksum, partials,
                   ticket);
 }
 
@@ -379,8 +312,7 @@ inline int su3_tiled_launch(bool twin, const double* A, const double* B, double*
   return check_launch(twin ? "cuda_su3_tiled_twin" : "omprt_su3_tiled_rt");
 }
 
-// persistent geometry: one team per SM.  warp = false: per-thread bulk copies (128 threads,
-// 153 KB of slots + barriers); warp = true: warp-cooperative cp.async (192 threads, 222 KB).
+// persistent geometry: one team per SM, warp-cooperative cp.async (192 threads, 222 KB).
 template <class K>
 inline int su3_staged_go(K k, uint32_t smem, int32_t teams, int threads, const double* A,
                          const double2* B, double* Cm, int32_t n, double* ck, double* p,
@@ -390,12 +322,10 @@ inline int su3_staged_go(K k, uint32_t smem, int32_t teams, int threads, const d
   return OMPRT_OK;
 }
 
-inline int su3_staged_launch(bool twin, bool warp, const double* A, const double* B,
-                             double* Cm, int64_t n, double* ck, int32_t teams, Workspace* w,
-                             cudaStream_t s) {
-  const int threads = warp ? kSU3WarpThreads : kSU3StagedThreads;
-  const uint32_t smem = warp ? warp_staged_smem_bytes<kSU3Slot>(kSU3WarpThreads)
-                             : staged_smem_bytes<kSU3Slot, 2>(kSU3StagedThreads);
+inline int su3_staged_launch(bool twin, const double* A, const double* B, double* Cm, int64_t n,
+                             double* ck, int32_t teams, Workspace* w, cudaStream_t s) {
+  const int threads = kSU3WarpThreads;
+  const uint32_t smem = warp_staged_smem_bytes<kSU3Slot>(kSU3WarpThreads);
   int dev = 0, sms = 148;
   cudaGetDevice(&dev);
   cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
@@ -407,23 +337,15 @@ inline int su3_staged_launch(bool twin, bool warp, const double* A, const double
   double* p = (double*)w->partials;
   unsigned* tk = w->tickets + 3;
   int r;
-  if (warp && twin)
+  if (twin)
     r = su3_staged_go(ck ? cuda_su3_wstaged_twin<true> : cuda_su3_wstaged_twin<false>, smem,
                       teams, threads, A, b2, Cm, nn, ck, p, tk, s);
-  else if (warp)
+  else
     r = su3_staged_go(ck ? omprt_su3_wstaged_rt<SU3StagedTraits, true>
                          : omprt_su3_wstaged_rt<SU3StagedTraits, false>,
                       smem, teams, threads, A, b2, Cm, nn, ck, p, tk, s);
-  else if (twin)
-    r = su3_staged_go(ck ? cuda_su3_staged_twin<true> : cuda_su3_staged_twin<false>, smem,
-                      teams, threads, A, b2, Cm, nn, ck, p, tk, s);
-  else
-    r = su3_staged_go(ck ? omprt_su3_staged_rt<SU3StagedTraits, true>
-                         : omprt_su3_staged_rt<SU3StagedTraits, false>,
-                      smem, teams, threads, A, b2, Cm, nn, ck, p, tk, s);
   if (r) return r;
-  return check_launch(warp ? (twin ? "cuda_su3_wstaged_twin" : "omprt_su3_wstaged_rt")
-                           : (twin ? "cuda_su3_staged_twin" : "omprt_su3_staged_rt"));
+  return check_launch(twin ? "cuda_su3_wstaged_twin" : "omprt_su3_wstaged_rt");
 }
 
 }  // namespace omprt_kernels

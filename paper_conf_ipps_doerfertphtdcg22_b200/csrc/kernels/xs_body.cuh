@@ -26,46 +26,7 @@ struct XSTables {
   const uint16_t* __restrict__ index_grid16;  // [n_union][n_iso] (n_gp <= 65536)
   const double* __restrict__ brackets;      // [n_iso][n_gp-1][12] (E,t,e,a,f,n) x (k, k+1)
   int32_t log2_bins, pad2;
-  // optional compact index grid (omprt_xs_build_compact; both NULL or both set): the index
-  // grid as every 16th row of position counts + the nuclide of every unionized energy
-  const uint16_t* __restrict__ idx_rows;    // [ceil(n_union/16)][n_iso]: #{v <= 16m : owner[v] = q}
-  const uint8_t* __restrict__ owner;        // [n_union rounded up to 16], 0xFF padded
 };
-
-// ---- compact index grid (reading R-X1) --------------------------------------------------
-// index_grid[e][q] = clip(C_q(e) - 1, 0, n_gp - 2) with C_q(e) = #{k : E_q[k] <= U[e]}.  For
-// the e the search returns (the LAST of its group of equal energies, or a clamped end that
-// the builder checks is tie-free) C_q(e) = #{v <= e : owner[v] = q}, a prefix count over the
-// nuclide ids of the sorted energies: the row stored for u0 = e & ~15 plus the matches among
-// owner[u0+1 .. e] -- one 16-byte load per lookup and 4 byte-compares per nuclide.  The
-// table shrinks from 104.5 MB (16-bit rows) to 6.5 + 0.8 MB, so it stays in L2.
-struct OwnerChunk {
-  uint32_t w[4];  // owner[u0 .. u0+15], bytes outside (u0, e] replaced by 0xFF (no nuclide)
-};
-__device__ __forceinline__ OwnerChunk owner_chunk(const XSTables& t, int32_t e) {
-  const int32_t u0 = e & ~15;
-  const uint4 v = __ldg(reinterpret_cast<const uint4*>(t.owner + u0));
-  const int r = e - u0;  // positions 1..r of the chunk count
-  OwnerChunk c{{v.x, v.y, v.z, v.w}};
-#pragma unroll
-  for (int i = 0; i < 4; ++i) {
-    const int valid = r - 4 * i + 1;  // bytes 4i .. 4i+valid-1 have position <= r
-    uint32_t keep = valid >= 4 ? 0xFFFFFFFFu : (valid <= 0 ? 0u : (1u << (8 * valid)) - 1u);
-    if (i == 0) keep &= ~0xFFu;     // position 0 is the stored row itself
-    c.w[i] = (c.w[i] & keep) | ~keep;
-  }
-  return c;
-}
-// index_grid[e][q] from the compact layout (row = idx_rows + (e >> 4) * n_iso)
-__device__ __forceinline__ int32_t compact_index(const XSTables& t,
-                                                 const uint16_t* __restrict__ row,
-                                                 const OwnerChunk& c, int32_t q) {
-  const uint32_t qq = (uint32_t)q * 0x01010101u;
-  const int cnt = __popc(__vcmpeq4(c.w[0], qq)) + __popc(__vcmpeq4(c.w[1], qq)) +
-                  __popc(__vcmpeq4(c.w[2], qq)) + __popc(__vcmpeq4(c.w[3], qq));
-  const int32_t k = (int32_t)__ldg(row + q) + (cnt >> 3) - 1;
-  return k < 0 ? 0 : (k > t.n_gridpoints - 2 ? t.n_gridpoints - 2 : k);
-}
 
 // ---- the proxy apps' LCG (m = 2^63, a = 2806196910506780709, c = 1) ----------------------
 constexpr uint64_t kLcgA = 2806196910506780709ull;
@@ -192,6 +153,18 @@ __device__ __forceinline__ void xs_accumulate(double E, double conc, double le, 
   m4 = fma(fma(-f, hn - ln, hn), conc, m4);      // nu-fission
 }
 
+// Test build (Macro): the 5 macroscopic cross sections of a lookup, [total, elastic,
+// absorption, fission, nu-fission] -- the values the argmax is taken over, for bitwise parity
+// with the oracle.
+__device__ __forceinline__ void xs_store_macro(double* __restrict__ mo, double m0, double m1,
+                                               double m2, double m3, double m4) {
+  mo[0] = m0;
+  mo[1] = m1;
+  mo[2] = m2;
+  mo[3] = m3;
+  mo[4] = m4;
+}
+
 __device__ __forceinline__ uint64_t xs_argmax5(double m0, double m1, double m2, double m3,
                                                double m4) {
   // 1 + argmax, strict '>' from max = -1 (the first maximum wins)
@@ -209,8 +182,9 @@ __device__ __forceinline__ uint64_t xs_argmax5(double m0, double m1, double m2, 
 // of the next pair of nuclides are requested before the current pair's brackets, so the
 // index -> bracket dependency of one pair overlaps the other (measured: x04 in profiles/).
 // Same arithmetic in the same order as the plain path.
+template <bool Macro = false>
 __device__ __forceinline__ uint64_t xs_lookup_accel(const XSTables& t, uint64_t seed0,
-                                                    int64_t i) {
+                                                    int64_t i, double* __restrict__ mo = nullptr) {
   constexpr int P = 2;
   uint64_t seed = lcg_fast_forward(seed0, 2ull * (uint64_t)i);
   const double E = lcg_double(seed);
@@ -257,6 +231,7 @@ __device__ __forceinline__ uint64_t xs_lookup_accel(const XSTables& t, uint64_t 
       kc[u] = kn[u];
     }
   }
+  if constexpr (Macro) xs_store_macro(mo, m0, m1, m2, m3, m4);
   return xs_argmax5(m0, m1, m2, m3, m4);
 }
 
@@ -271,12 +246,13 @@ __device__ __forceinline__ uint64_t xs_lookup_accel(const XSTables& t, uint64_t 
 // once, bypass L1 allocation, and with SmemMats the material tables (mats, concs) come
 // from a team-shared copy (`mats`/`concs` then point to shared memory).
 constexpr int kXSFlatThreads = 256;  // team size of the flattened XS kernels
-template <bool Fused, bool SmemMats, bool Compact = false, int P = 2>
+template <bool Fused, bool SmemMats, bool Macro = false, int P = 2>
 struct XSFlatLookup {
   const XSTables& t;
   const uint64_t seed0;
   const int64_t first;
   uint64_t* __restrict__ const ver;
+  double* __restrict__ const macro;        // Macro: [count][5] macroscopic xs (test build)
   const int32_t* __restrict__ const mats;  // t.mats, or its team-shared copy
   const double* __restrict__ const concs;  // t.concs, or its team-shared copy
   // Fused: this thread's verification sum lives in a per-thread shared-memory slot
@@ -287,12 +263,12 @@ struct XSFlatLookup {
   int32_t mat, idx, nn, j;
   double m0, m1, m2, m3, m4;
   int32_t pc[P], kc[P];
-  OwnerChunk oc;  // Compact only
 
   __device__ __forceinline__ XSFlatLookup(const XSTables& tab, uint64_t seed, int64_t first_,
                                           uint64_t* verification, const int32_t* mats_,
-                                          const double* concs_)
-      : t(tab), seed0(seed), first(first_), ver(verification), mats(mats_), concs(concs_) {}
+                                          const double* concs_, double* macro_ = nullptr)
+      : t(tab), seed0(seed), first(first_), ver(verification), macro(macro_), mats(mats_),
+        concs(concs_) {}
 
   __device__ __forceinline__ int32_t mat_at(const int32_t* p) const {
     if constexpr (SmemMats) return *p;
@@ -305,13 +281,11 @@ struct XSFlatLookup {
 
   // this lookup's row of the index grid, and its entry for nuclide q
   __device__ __forceinline__ const uint16_t* index_row() const {
-    if constexpr (Compact) return t.idx_rows + (int64_t)(idx >> 4) * t.n_isotopes;
-    else return t.index_grid16 + (int64_t)idx * t.n_isotopes;
+    return t.index_grid16 + (int64_t)idx * t.n_isotopes;
   }
   __device__ __forceinline__ int32_t index_at(const uint16_t* __restrict__ irow,
                                               int32_t q) const {
-    if constexpr (Compact) return compact_index(t, irow, oc, q);
-    else return (int32_t)__ldg(irow + q);
+    return (int32_t)__ldg(irow + q);
   }
 
   __device__ __forceinline__ void start() {
@@ -322,7 +296,6 @@ struct XSFlatLookup {
     nn = __ldg(t.num_nucs + mat);
     m0 = m1 = m2 = m3 = m4 = 0.0;
     j = 0;
-    if constexpr (Compact) oc = owner_chunk(t, idx);
     const int32_t* __restrict__ mrow = mats + mat * t.max_num_nucs;
     const uint16_t* __restrict__ irow = index_row();
 #pragma unroll
@@ -379,6 +352,7 @@ struct XSFlatLookup {
   template <class Idx>
   __device__ __forceinline__ void end(Idx iv) {
     const uint64_t v = xs_argmax5(m0, m1, m2, m3, m4);
+    if constexpr (Macro) xs_store_macro(macro + (int64_t)iv * 5, m0, m1, m2, m3, m4);
     if constexpr (Fused) *flat_acc_slot() += v;
     else ver[iv] = v;
   }
@@ -391,9 +365,10 @@ struct XSFlatLookup {
   }
 };
 
-template <bool Accel, int kUnroll = 4>
-__device__ __forceinline__ uint64_t xs_lookup_one(const XSTables& t, uint64_t seed0, int64_t i) {
-  if constexpr (Accel) return xs_lookup_accel(t, seed0, i);
+template <bool Accel, bool Macro = false, int kUnroll = 4>
+__device__ __forceinline__ uint64_t xs_lookup_one(const XSTables& t, uint64_t seed0, int64_t i,
+                                                  double* __restrict__ mo = nullptr) {
+  if constexpr (Accel) return xs_lookup_accel<Macro>(t, seed0, i, mo);
   uint64_t seed = lcg_fast_forward(seed0, 2ull * (uint64_t)i);
   const double E = lcg_double(seed);
   const int mat = pick_mat(seed);
@@ -433,15 +408,8 @@ __device__ __forceinline__ uint64_t xs_lookup_one(const XSTables& t, uint64_t se
     m3 = fma(fma(-f, hf - lf, hf), conc, m3);      // fission
     m4 = fma(fma(-f, hn - ln, hn), conc, m4);      // nu-fission
   }
-  // 1 + argmax, strict '>' from max = -1 (the first maximum wins)
-  double mx = -1.0;
-  uint64_t v = 1;
-  if (m0 > mx) { mx = m0; v = 1; }
-  if (m1 > mx) { mx = m1; v = 2; }
-  if (m2 > mx) { mx = m2; v = 3; }
-  if (m3 > mx) { mx = m3; v = 4; }
-  if (m4 > mx) { mx = m4; v = 5; }
-  return v;
+  if constexpr (Macro) xs_store_macro(mo, m0, m1, m2, m3, m4);
+  return xs_argmax5(m0, m1, m2, m3, m4);
 }
 
 // ---- builders of the accelerated layouts (table preparation, not per lookup) -------------

@@ -18,7 +18,6 @@
 // at ties.  Energies must be finite and not -0.0 (the proxy app draws them from [0, 1)).
 #pragma once
 #include <cub/block/block_scan.cuh>
-#include <cub/device/device_radix_sort.cuh>
 
 #include "../host/runtime.cuh"
 
@@ -223,41 +222,8 @@ __global__ void __launch_bounds__(kDeriveRows)
   }
 }
 
-// ---- compact index grid (omprt_xs_build_compact, reading R-X1) -------------------------
-// owner[v] = nuclide of sorted energy v (0xFF pad to a multiple of 16)
-__global__ void xs_compact_owner(const uint16_t* __restrict__ ids, int64_t n, int64_t n_pad,
-                                 uint8_t* __restrict__ owner) {
-  for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < n_pad;
-       v += (int64_t)gridDim.x * blockDim.x)
-    owner[v] = v < n ? (uint8_t)ids[v] : (uint8_t)0xFF;
-}
-// per chunk of kDeriveRows sorted energies, one thread per nuclide column: every 16th
-// position's inclusive count  rows[m][q] = #{v <= 16m : ids[v] = q}
-__global__ void xs_compact_rows(const uint16_t* __restrict__ ids,
-                                const uint32_t* __restrict__ start, int64_t n, int32_t n_iso,
-                                uint16_t* __restrict__ rows) {
-  __shared__ uint16_t sid[kDeriveRows];
-  const int64_t r0 = (int64_t)blockIdx.x * kDeriveRows;
-  const int cnt_rows = (int)(r0 + kDeriveRows < n ? kDeriveRows : n - r0);
-  for (int k = threadIdx.x; k < cnt_rows; k += blockDim.x) sid[k] = ids[r0 + k];
-  __syncthreads();
-  for (int q = threadIdx.x; q < n_iso; q += blockDim.x) {
-    uint32_t c = start[(int64_t)blockIdx.x * n_iso + q];
-    for (int k = 0; k < cnt_rows; ++k) {
-      c += sid[k] == q;
-      if ((k & 15) == 0) rows[((r0 + k) >> 4) * n_iso + q] = (uint16_t)c;
-    }
-  }
-}
-// the clamped ends of the search must be tie-free: out[0] = 1 if keys[0] == keys[1] or
-// keys[n-2] == keys[n-1]
-__global__ void xs_compact_check(const unsigned long long* __restrict__ keys, int64_t n,
-                                 unsigned long long* out) {
-  out[0] = (keys[0] == keys[1] || keys[n - 2] == keys[n - 1]) ? 1ull : 0ull;
-}
-
 struct DeriveLayout {
-  size_t keys_in, keys_out, ids_in, ids_out, hist, cub, total;
+  size_t keys_in, keys_out, ids_in, ids_out, hist, total;
 };
 inline size_t al256(size_t b) { return (b + 255) & ~size_t(255); }
 
@@ -268,10 +234,6 @@ inline int xs_derive_layout(int32_t n_iso, int32_t n_gp, DeriveLayout* L) {
                   kDeriveMaxIso);
   const int64_t n = (int64_t)n_iso * n_gp;
   const int64_t chunks = (n + kDeriveRows - 1) / kDeriveRows;
-  size_t cub_bytes = 0;
-  cub::DeviceRadixSort::SortPairs(nullptr, cub_bytes, (const unsigned long long*)nullptr,
-                                  (unsigned long long*)nullptr, (const uint16_t*)nullptr,
-                                  (uint16_t*)nullptr, (int)n);
   size_t off = 0;
   L->keys_in = off;
   off += al256(8 * n);
@@ -283,8 +245,6 @@ inline int xs_derive_layout(int32_t n_iso, int32_t n_gp, DeriveLayout* L) {
   off += al256(2 * n);
   L->hist = off;
   off += al256(4 * chunks * n_iso);
-  L->cub = off;
-  off += al256(cub_bytes);
   L->total = off;
   return OMPRT_OK;
 }
@@ -303,9 +263,7 @@ inline int xs_derive(const double* nuclide_grid, int32_t n_iso, int32_t n_gp, do
   auto* iin = (uint16_t*)(b + L.ids_in);
   auto* iout = (uint16_t*)(b + L.ids_out);
   auto* hist = (uint32_t*)(b + L.hist);
-  size_t cub_bytes = L.total - L.cub;
   xs_derive_keys<<<1024, 256, 0, s>>>(nuclide_grid, n_gp, n, kin, iin);
-  (void)cub_bytes;
   // merge levels, ping-ponging between the two key/id buffers; the result ends in kout/iout
   const unsigned mblocks = (unsigned)((n + 256 * kMergeItems - 1) / (256 * kMergeItems));
   int levels = 0;
@@ -341,68 +299,7 @@ inline int xs_derive(const double* nuclide_grid, int32_t n_iso, int32_t n_gp, do
   return check_launch("omprt_xs_derive");
 }
 
-inline int xs_compact_sizes(int32_t n_iso, int32_t n_gp, uint64_t* sizes) {
-  OMPRT_CHECK_ARG(n_iso > 0 && n_iso <= 255 && n_gp >= 2 && n_gp <= 65535 &&
-                      (int64_t)n_iso * n_gp < (1ll << 31) && sizes,
-                  "omprt_xs_compact: need 0 < n_isotopes <= 255, 2 <= n_gridpoints <= 65535");
-  const int64_t n = (int64_t)n_iso * n_gp;
-  sizes[0] = 2ull * (uint64_t)((n + 15) / 16) * (uint64_t)n_iso;
-  sizes[1] = (uint64_t)((n + 15) / 16) * 16ull;
-  return OMPRT_OK;
-}
-
-inline int xs_build_compact(const double* nuclide_grid, int32_t n_iso, int32_t n_gp,
-                            uint16_t* rows, uint8_t* owner, void* tmp, size_t tmp_bytes,
-                            Workspace* w, cudaStream_t s) {
-  uint64_t sz[2];
-  if (int r = xs_compact_sizes(n_iso, n_gp, sz)) return r;
-  DeriveLayout L;
-  if (int r = xs_derive_layout(n_iso, n_gp, &L)) return r;
-  OMPRT_CHECK_ARG(nuclide_grid && rows && owner && tmp, "omprt_xs_build_compact: null pointer");
-  OMPRT_CHECK_ARG(((uintptr_t)owner & 15) == 0, "omprt_xs_build_compact: owner not 16 B aligned");
-  OMPRT_CHECK_ARG(tmp_bytes >= L.total, "omprt_xs_build_compact: tmp needs %zu B", L.total);
-  const int64_t n = (int64_t)n_iso * n_gp;
-  const int32_t chunks = (int32_t)((n + kDeriveRows - 1) / kDeriveRows);
-  unsigned char* b = (unsigned char*)tmp;
-  auto* kin = (unsigned long long*)(b + L.keys_in);
-  auto* kout = (unsigned long long*)(b + L.keys_out);
-  auto* iin = (uint16_t*)(b + L.ids_in);
-  auto* iout = (uint16_t*)(b + L.ids_out);
-  auto* hist = (uint32_t*)(b + L.hist);
-  size_t cub_bytes = L.total - L.cub;
-  xs_derive_keys<<<1024, 256, 0, s>>>(nuclide_grid, n_gp, n, kin, iin);
-  if (cub::DeviceRadixSort::SortPairs(b + L.cub, cub_bytes, kin, kout, iin, iout, (int)n, 0, 64,
-                                      s) != cudaSuccess)
-    return set_error(OMPRT_E_CUDA, "omprt_xs_build_compact: radix sort failed");
-  xs_compact_owner<<<1024, 256, 0, s>>>(iout, n, (int64_t)sz[1], owner);
-  xs_derive_hist<<<chunks, 256, 0, s>>>(iout, n, n_iso, hist);
-  xs_derive_scan<<<n_iso, kScanThreads, 0, s>>>(hist, chunks, n_iso);
-  xs_compact_rows<<<chunks, 128, 0, s>>>(iout, hist, n, n_iso, rows);
-  xs_compact_check<<<1, 1, 0, s>>>(kout, n, (unsigned long long*)w->scratch_u64 + 7);
-  if (int r = check_launch("omprt_xs_build_compact")) return r;
-  unsigned long long tie = 0;
-  OMPRT_CUDA_TRY(cudaMemcpyAsync(&tie, w->scratch_u64 + 7, 8, cudaMemcpyDeviceToHost, s));
-  OMPRT_CUDA_TRY(cudaStreamSynchronize(s));
-  OMPRT_CHECK_ARG(tie == 0, "omprt_xs_build_compact: equal energies at the grid's ends");
-  return OMPRT_OK;
-}
-
 }  // namespace omprt_kernels
-
-extern "C" int omprt_xs_compact_sizes(int32_t n_isotopes, int32_t n_gridpoints,
-                                      uint64_t* sizes) {
-  return omprt_kernels::xs_compact_sizes(n_isotopes, n_gridpoints, sizes);
-}
-
-extern "C" int omprt_xs_build_compact(const double* nuclide_grid, int32_t n_isotopes,
-                                      int32_t n_gridpoints, uint16_t* idx_rows, uint8_t* owner,
-                                      void* tmp, uint64_t tmp_bytes, void* stream) {
-  using namespace omprt_kernels;
-  Workspace* w;
-  if (int r = current_ws(&w)) return r;
-  return xs_build_compact(nuclide_grid, n_isotopes, n_gridpoints, idx_rows, owner, tmp,
-                          tmp_bytes, w, as_stream(stream));
-}
 
 extern "C" int omprt_xs_derive_tmp_bytes(int32_t n_isotopes, int32_t n_gridpoints,
                                          uint64_t* bytes) {

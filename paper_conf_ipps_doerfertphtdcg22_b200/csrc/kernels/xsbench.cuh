@@ -32,21 +32,22 @@ static_assert(kXSThreads == kXSFlatThreads, "XSFlatLookup::flat_acc_slot is size
 constexpr int kXSMinBlocks = 4;   // plain layout
 constexpr int kXSMinBlocksAccel = 3;  // B200 layouts: 78 registers, no spills (x04)
 
-template <class Tr, bool Fused, bool Accel>
+template <class Tr, bool Fused, bool Accel, bool Macro = false>
 __global__ void __launch_bounds__(kXSThreads, Accel ? kXSMinBlocksAccel : kXSMinBlocks)
     omprt_xs_rt(const __grid_constant__ XSTables t, uint64_t seed, int64_t first,
                 typename Tr::Idx count, uint64_t* __restrict__ verification,
-                unsigned long long* checksum, unsigned long long* partials, unsigned* ticket) {
+                unsigned long long* checksum, unsigned long long* partials, unsigned* ticket,
+                double* __restrict__ macro = nullptr) {
   using Idx = typename Tr::Idx;
   Team<Tr> team = init<Tr>();
   unsigned long long acc = 0;
   distribute_parallel_for(team, count, [&](Idx iv) {
-    const uint64_t v = xs_lookup_one<Accel>(t, seed, first + iv);
+    const uint64_t v = xs_lookup_one<Accel, Macro>(t, seed, first + iv, macro + (int64_t)iv * 5);
     if constexpr (Fused) acc += v;
     else verification[iv] = v;
   });
   if constexpr (Fused)
-    league_reduce(team, team_reduce_to_main(team, acc, Plus{}), Plus{}, checksum, partials,
+    league_reduce_threads(team, acc, Plus{}, checksum, partials,
                   ticket);
 }
 
@@ -90,15 +91,16 @@ __device__ __forceinline__ void twin_u64_ticket_sum(unsigned long long v,
 
 // XSBench's CUDA kernel shape: one lookup per thread, early return past the end; the fused
 // variant hand-codes the same reduction algorithm as the runtime.
-template <bool Fused, bool Accel>
+template <bool Fused, bool Accel, bool Macro = false>
 __global__ void __launch_bounds__(kXSThreads, Accel ? kXSMinBlocksAccel : kXSMinBlocks)
     cuda_xs_twin(const __grid_constant__ XSTables t, uint64_t seed, int64_t first, int32_t count,
                  uint64_t* __restrict__ verification, unsigned long long* checksum,
-                 unsigned long long* partials, unsigned* ticket) {
+                 unsigned long long* partials, unsigned* ticket,
+                 double* __restrict__ macro = nullptr) {
   const int32_t i = blockIdx.x * blockDim.x + threadIdx.x;
   if constexpr (!Fused) {
     if (i >= count) return;
-    verification[i] = xs_lookup_one<Accel>(t, seed, first + i);
+    verification[i] = xs_lookup_one<Accel, Macro>(t, seed, first + i, macro + (int64_t)i * 5);
   } else {
     const unsigned long long v = i < count ? xs_lookup_one<Accel>(t, seed, first + i) : 0ull;
     twin_u64_ticket_sum(v, checksum, partials, ticket);
@@ -118,12 +120,12 @@ constexpr unsigned kXSMatsSite = 10, kXSConcsSite = 11;  // team_local sites
 // OMPRT_SCHED_DYNAMIC: schedule(dynamic, kXSDynChunk) instead of Fig. 5 (reading R-D1)
 constexpr int kXSDynChunk = 8;
 
-template <class Tr, bool Fused, bool Smem, bool Dyn = false, bool Compact = false>
+template <class Tr, bool Fused, bool Smem, bool Dyn = false, bool Macro = false>
 __global__ void __launch_bounds__(kXSThreads, kXSMinBlocksFlat)
     omprt_xs_flat_rt(const __grid_constant__ XSTables t, uint64_t seed, int64_t first,
                      typename Tr::Idx count, uint64_t* __restrict__ verification,
                      unsigned long long* checksum, unsigned long long* partials,
-                     unsigned* ticket) {
+                     unsigned* ticket, double* __restrict__ macro = nullptr) {
   using Idx = typename Tr::Idx;
   Team<Tr> team = init<Tr>();
   const int32_t* mats = t.mats;
@@ -139,23 +141,23 @@ __global__ void __launch_bounds__(kXSThreads, kXSMinBlocksFlat)
     mats = sm;
     concs = sc;
   }
-  using Lookup = XSFlatLookup<Fused, Smem, Compact>;
+  using Lookup = XSFlatLookup<Fused, Smem, Macro>;
   if constexpr (Fused) *Lookup::flat_acc_slot() = 0ull;
-  Lookup lookup(t, seed, first, verification, mats, concs);
+  Lookup lookup(t, seed, first, verification, mats, concs, macro);
   if constexpr (Dyn) distribute_parallel_for_dynamic_flat(team, count, (Idx)kXSDynChunk, lookup);
   else distribute_parallel_for_flat(team, count, lookup);
   if constexpr (Fused)
-    league_reduce(team, team_reduce_to_main(team, *Lookup::flat_acc_slot(), Plus{}), Plus{},
+    league_reduce_threads(team, *Lookup::flat_acc_slot(), Plus{},
                   checksum, partials, ticket);
 }
 
 // Bare CUDA twin: the same flattened loop written by hand around the same body.
-template <bool Fused, bool Smem, bool Dyn = false, bool Compact = false>
+template <bool Fused, bool Smem, bool Dyn = false, bool Macro = false>
 __global__ void __launch_bounds__(kXSThreads, kXSMinBlocksFlat)
     cuda_xs_flat_twin(const __grid_constant__ XSTables t, uint64_t seed, int64_t first,
                       int32_t count, uint64_t* __restrict__ verification,
                       unsigned long long* checksum, unsigned long long* partials,
-                      unsigned* ticket) {
+                      unsigned* ticket, double* __restrict__ macro = nullptr) {
   const int32_t* mats = t.mats;
   const double* concs = t.concs;
   if constexpr (Smem) {
@@ -169,9 +171,9 @@ __global__ void __launch_bounds__(kXSThreads, kXSMinBlocksFlat)
     mats = sm;
     concs = sc;
   }
-  using Lookup = XSFlatLookup<Fused, Smem, Compact>;
+  using Lookup = XSFlatLookup<Fused, Smem, Macro>;
   if constexpr (Fused) *Lookup::flat_acc_slot() = 0ull;
-  Lookup lookup(t, seed, first, verification, mats, concs);
+  Lookup lookup(t, seed, first, verification, mats, concs, macro);
   if constexpr (Dyn) {  // team block + team-shared chunk counter, by hand
     __shared__ unsigned next;
     const int32_t per = (count + (int32_t)gridDim.x - 1) / (int32_t)gridDim.x;
@@ -228,7 +230,7 @@ __global__ void __launch_bounds__(512)
   Team<Tr> team = init<Tr>();
   unsigned long long acc = 0;
   distribute_parallel_for(team, n, [&](Idx i) { acc += __ldg(v + i); });
-  league_reduce(team, team_reduce_to_main(team, acc, Plus{}), Plus{}, out, partials, ticket);
+  league_reduce_threads(team, acc, Plus{}, out, partials, ticket);
 }
 
 OMPRT_REGISTER_KERNEL(omprt_xs_rt, omprt_xs_rt<XSTraits, false, false>)
@@ -255,7 +257,7 @@ OMPRT_REGISTER_KERNEL(omprt_u64_sum_rt, omprt_u64_sum_rt<SumTraits>)
 inline XSTables to_dev(const omprt_xs_tables& a) {
   return XSTables{a.nuclide_grid, a.unionized, a.index_grid, a.num_nucs, a.mats, a.concs,
                   a.n_isotopes, a.n_gridpoints, a.max_num_nucs, 0, a.n_union,
-                  a.bins, a.index_grid16, a.brackets, a.log2_bins, 0, a.idx_rows, a.owner};
+                  a.bins, a.index_grid16, a.brackets, a.log2_bins, 0};
 }
 
 // Launch configuration of the flattened kernels: the persistent grid, plus (unless
@@ -315,37 +317,37 @@ inline bool xs_mats_fit_smem(const omprt_xs_tables& t) {
   return 12ll * t.max_num_nucs <= kXSMatSmem;
 }
 
-inline bool xs_has_compact(const omprt_xs_tables& t) {
-  return t.idx_rows != nullptr && t.owner != nullptr;
-}
-
 // The flattened kernels: runtime-driven (Twin = false) or twin, by (fused, team-shared
-// material tables, dynamic schedule, compact index grid).
-template <bool Twin, bool F, bool S, bool D, bool C>
+// material tables, dynamic schedule, macroscopic-xs output of the test build).
+template <bool Twin, bool F, bool S, bool D, bool M>
 inline cudaError_t xs_flat_launch(const cudaLaunchConfig_t& cfg, const XSTables& d, uint64_t seed,
                                   int64_t first, int32_t n, uint64_t* ver, unsigned long long* ck,
-                                  unsigned long long* p, unsigned* tk) {
+                                  unsigned long long* p, unsigned* tk, double* mac) {
   if constexpr (Twin)
-    return cudaLaunchKernelEx(&cfg, cuda_xs_flat_twin<F, S, D, C>, d, seed, first, n, ver, ck,
-                              p, tk);
+    return cudaLaunchKernelEx(&cfg, cuda_xs_flat_twin<F, S, D, M>, d, seed, first, n, ver, ck,
+                              p, tk, mac);
   else
-    return cudaLaunchKernelEx(&cfg, omprt_xs_flat_rt<XSTraits, F, S, D, C>, d, seed, first, n,
-                              ver, ck, p, tk);
+    return cudaLaunchKernelEx(&cfg, omprt_xs_flat_rt<XSTraits, F, S, D, M>, d, seed, first, n,
+                              ver, ck, p, tk, mac);
 }
 template <bool Twin>
-inline cudaError_t xs_flat_dispatch(uint32_t flags, bool fused, bool smem, bool compact,
+inline cudaError_t xs_flat_dispatch(uint32_t flags, bool fused, bool smem,
                                     const cudaLaunchConfig_t& cfg, const XSTables& d,
                                     uint64_t seed, int64_t first, int32_t n, uint64_t* ver,
                                     unsigned long long* ck, unsigned long long* p,
-                                    unsigned* tk) {
+                                    unsigned* tk, double* mac) {
   const bool dyn = flags & OMPRT_SCHED_DYNAMIC;
-#define OMPRT_XSF(F, S, D, C) \
-  if (fused == F && smem == S && dyn == D && compact == C) \
-    return xs_flat_launch<Twin, F, S, D, C>(cfg, d, seed, first, n, ver, ck, p, tk);
-#define OMPRT_XSF2(F, S, D) OMPRT_XSF(F, S, D, false) OMPRT_XSF(F, S, D, true)
-#define OMPRT_XSF4(F, S) OMPRT_XSF2(F, S, false) OMPRT_XSF2(F, S, true)
-  OMPRT_XSF4(false, false) OMPRT_XSF4(false, true) OMPRT_XSF4(true, false) OMPRT_XSF4(true, true)
-#undef OMPRT_XSF4
+  if (mac) {  // test build: unfused only (xs_validate)
+    if (smem && dyn) return xs_flat_launch<Twin, false, true, true, true>(cfg, d, seed, first, n, ver, ck, p, tk, mac);
+    if (smem) return xs_flat_launch<Twin, false, true, false, true>(cfg, d, seed, first, n, ver, ck, p, tk, mac);
+    if (dyn) return xs_flat_launch<Twin, false, false, true, true>(cfg, d, seed, first, n, ver, ck, p, tk, mac);
+    return xs_flat_launch<Twin, false, false, false, true>(cfg, d, seed, first, n, ver, ck, p, tk, mac);
+  }
+#define OMPRT_XSF(F, S, D) \
+  if (fused == F && smem == S && dyn == D) \
+    return xs_flat_launch<Twin, F, S, D, false>(cfg, d, seed, first, n, ver, ck, p, tk, mac);
+#define OMPRT_XSF2(F, S) OMPRT_XSF(F, S, false) OMPRT_XSF(F, S, true)
+  OMPRT_XSF2(false, false) OMPRT_XSF2(false, true) OMPRT_XSF2(true, false) OMPRT_XSF2(true, true)
 #undef OMPRT_XSF2
 #undef OMPRT_XSF
   return cudaErrorInvalidValue;
@@ -356,7 +358,8 @@ inline bool xs_has_accel(const omprt_xs_tables& t) {
 }
 
 inline int xs_validate(const omprt_xs_tables& t, int64_t count, uint64_t* ver, uint64_t* ck,
-                       int32_t& teams, int32_t threads, uint32_t flags, Workspace* w) {
+                       double* macro, int32_t& teams, int32_t threads, uint32_t flags,
+                       Workspace* w) {
   OMPRT_CHECK_ARG(count >= 0 && count < (1ll << 31), "count must be in [0, 2^31)");
   OMPRT_CHECK_ARG(threads == kXSThreads, "threads must be %d", kXSThreads);
   OMPRT_CHECK_ARG(t.unionized && t.num_nucs && t.mats && t.concs && t.n_union >= 2 &&
@@ -368,14 +371,9 @@ inline int xs_validate(const omprt_xs_tables& t, int64_t count, uint64_t* ver, u
                   "accelerated layout: bad log2_bins");
   OMPRT_CHECK_ARG(accel || (!t.bins && !t.index_grid16 && !t.brackets),
                   "accelerated layout: bins, index_grid16 and brackets go together");
-  OMPRT_CHECK_ARG((t.idx_rows == nullptr) == (t.owner == nullptr),
-                  "compact index grid: idx_rows and owner go together");
-  OMPRT_CHECK_ARG(!xs_has_compact(t) || (accel && (flags & OMPRT_XS_FLAT) &&
-                                          t.n_isotopes <= 255 && t.n_gridpoints <= 65535 &&
-                                          ((uintptr_t)t.owner & 15) == 0),
-                  "compact index grid: flattened launches with the B200 layouts only "
-                  "(n_isotopes <= 255, n_gridpoints <= 65535, owner 16 B aligned)");
   const bool fused = flags & OMPRT_FUSED_REDUCTION;
+  OMPRT_CHECK_ARG(!macro || (!fused && !(flags & OMPRT_DEBUG_BUILD)),
+                  "macro (test build) is written by the unfused release kernels only");
   OMPRT_CHECK_ARG(fused ? ck != nullptr : (ver != nullptr || count == 0),
                   fused ? "fused reduction needs checksum_inout" : "verification is required");
   OMPRT_CHECK_ARG(!(flags & OMPRT_SCHED_DYNAMIC) || (flags & OMPRT_XS_FLAT),
@@ -457,12 +455,13 @@ inline int launch_xs_accel(omprt_xs_tables* t, int32_t* bins, uint16_t* idx16, d
 }  // namespace omprt_kernels
 
 extern "C" int omprt_xs_lookup(omprt_xs_tables t, uint64_t seed, int64_t first, int64_t count,
-                               uint64_t* verification, uint64_t* checksum_inout, int32_t teams,
-                               int32_t threads, uint32_t flags, void* stream) {
+                               uint64_t* verification, uint64_t* checksum_inout, double* macro,
+                               int32_t teams, int32_t threads, uint32_t flags, void* stream) {
   using namespace omprt_kernels;
   Workspace* w;
   if (int r = current_ws(&w)) return r;
-  if (int r = xs_validate(t, count, verification, checksum_inout, teams, threads, flags, w))
+  if (int r = xs_validate(t, count, verification, checksum_inout, macro, teams, threads, flags,
+                          w))
     return r;
   if (count == 0) return OMPRT_OK;
   cudaStream_t s = as_stream(stream);
@@ -476,13 +475,21 @@ extern "C" int omprt_xs_lookup(omprt_xs_tables t, uint64_t seed, int64_t first, 
   if (flags & OMPRT_XS_FLAT) {
     const bool smem = xs_mats_fit_smem(t);
     const FlatLaunch L = flat_launch(t, teams, threads, flags, w, s);
-    xs_flat_dispatch<false>(flags, fused, smem, xs_has_compact(t), L.cfg, d, seed, first, n,
-                            verification, ck, p, tk);
+    xs_flat_dispatch<false>(flags, fused, smem, L.cfg, d, seed, first, n, verification, ck, p,
+                            tk, macro);
     return check_launch("omprt_xs_flat_rt");
   }
 #define OMPRT_XS(TR, F, A) \
   omprt_xs_rt<TR, F, A><<<teams, threads, 0, s>>>(d, seed, first, n, verification, ck, p, tk)
-  if (debug) {
+#define OMPRT_XSM(TR, A) \
+  omprt_xs_rt<TR, false, A, true><<<teams, threads, 0, s>>>(d, seed, first, n, verification, \
+                                                           ck, p, tk, macro)
+  if (macro) {  // test build: the macroscopic cross sections too
+    if (accel && assume) OMPRT_XSM(XSTraitsAssume, true);
+    else if (accel) OMPRT_XSM(XSTraits, true);
+    else if (assume) OMPRT_XSM(XSTraitsAssume, false);
+    else OMPRT_XSM(XSTraits, false);
+  } else if (debug) {
     OMPRT_CHECK_ARG(!fused && !accel, "the debug build covers the plain, unfused kernel");
     if (assume) OMPRT_XS(XSTraitsAssumeDebug, false, false);
     else OMPRT_XS(XSTraitsDebug, false, false);
@@ -497,21 +504,22 @@ extern "C" int omprt_xs_lookup(omprt_xs_tables t, uint64_t seed, int64_t first, 
     else if (assume) OMPRT_XS(XSTraitsAssume, false, false);
     else OMPRT_XS(XSTraits, false, false);
   }
+#undef OMPRT_XSM
 #undef OMPRT_XS
   return check_launch("omprt_xs_rt");
 }
 
 extern "C" int omprt_cuda_xs_lookup(omprt_xs_tables t, uint64_t seed, int64_t first,
                                     int64_t count, uint64_t* verification,
-                                    uint64_t* checksum_inout, int32_t teams, int32_t threads,
-                                    uint32_t flags, void* stream) {
+                                    uint64_t* checksum_inout, double* macro, int32_t teams,
+                                    int32_t threads, uint32_t flags, void* stream) {
   using namespace omprt_kernels;
   Workspace* w;
   if (int r = current_ws(&w)) return r;
   // the twin runs one lookup per thread, or (OMPRT_XS_FLAT) the same persistent grid
   const bool flat = flags & OMPRT_XS_FLAT;
   int32_t tm = flat ? teams : 0;
-  if (int r = xs_validate(t, count, verification, checksum_inout, tm, threads,
+  if (int r = xs_validate(t, count, verification, checksum_inout, macro, tm, threads,
                           flags & ~(OMPRT_ASSUME_OVERSUB | OMPRT_DEBUG_BUILD), w))
     return r;
   if (count == 0) return OMPRT_OK;
@@ -528,14 +536,16 @@ extern "C" int omprt_cuda_xs_lookup(omprt_xs_tables t, uint64_t seed, int64_t fi
     unsigned long long* nul = nullptr;
     unsigned* nult = nullptr;
     if (fused)
-      xs_flat_dispatch<true>(flags, fused, smem, xs_has_compact(t), L.cfg, d, seed, first, n,
-                             verification, ck, p, tk);
+      xs_flat_dispatch<true>(flags, fused, smem, L.cfg, d, seed, first, n, verification, ck, p,
+                             tk, macro);
     else
-      xs_flat_dispatch<true>(flags, fused, smem, xs_has_compact(t), L.cfg, d, seed, first, n,
-                             verification, nul, nul, nult);
+      xs_flat_dispatch<true>(flags, fused, smem, L.cfg, d, seed, first, n, verification, nul,
+                             nul, nult, macro);
     return check_launch("cuda_xs_flat_twin");
   }
-  if (fused && accel) cuda_xs_twin<true, true><<<tm, threads, 0, s>>>(d, seed, first, n, verification, ck, p, tk);
+  if (macro && accel) cuda_xs_twin<false, true, true><<<tm, threads, 0, s>>>(d, seed, first, n, verification, nullptr, nullptr, nullptr, macro);
+  else if (macro) cuda_xs_twin<false, false, true><<<tm, threads, 0, s>>>(d, seed, first, n, verification, nullptr, nullptr, nullptr, macro);
+  else if (fused && accel) cuda_xs_twin<true, true><<<tm, threads, 0, s>>>(d, seed, first, n, verification, ck, p, tk);
   else if (fused) cuda_xs_twin<true, false><<<tm, threads, 0, s>>>(d, seed, first, n, verification, ck, p, tk);
   else if (accel) cuda_xs_twin<false, true><<<tm, threads, 0, s>>>(d, seed, first, n, verification, nullptr, nullptr, nullptr);
   else cuda_xs_twin<false, false><<<tm, threads, 0, s>>>(d, seed, first, n, verification, nullptr, nullptr, nullptr);
@@ -761,11 +771,11 @@ extern "C" int omprt_xs_run_host_steps(omprt_xs_tables h, uint64_t seed, int64_t
     if (flags & OMPRT_XS_FLAT) {
       // flattened: per-lookup verification + K11 sum (the fused flat kernel spills: its
       // extra live state does not fit the 64 registers of 4 teams per SM)
-      if (int r = omprt_xs_lookup(d, seed, first, count, w->e2e_ver, nullptr, 0, threads,
+      if (int r = omprt_xs_lookup(d, seed, first, count, w->e2e_ver, nullptr, nullptr, 0, threads,
                                   flags & ~OMPRT_XS_ACCEL, stream))
         return r;
       if (int r = launch_u64_sum(w->e2e_ver, count, w->dev_ck + st, w, s)) return r;
-    } else if (int r = omprt_xs_lookup(d, seed, first, count, nullptr, w->dev_ck + st, 0,
+    } else if (int r = omprt_xs_lookup(d, seed, first, count, nullptr, w->dev_ck + st, nullptr, 0,
                                        threads,
                                        (flags & ~OMPRT_XS_ACCEL) | OMPRT_FUSED_REDUCTION |
                                            OMPRT_ASSUME_OVERSUB,

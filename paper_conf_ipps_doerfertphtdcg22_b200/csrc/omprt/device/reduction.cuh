@@ -62,10 +62,13 @@ __device__ __forceinline__ T warp_reduce(T v, Op op) {
   return v;
 }
 
-// Team reduction over all threads of the CTA; the result is valid in warp 0 (thread 0 is
-// what the league reduction uses).  One aligned barrier.
-template <class Tr, class T, class Op>
-__device__ __forceinline__ T team_reduce_to_main(Team<Tr>&, T v, Op op) {
+namespace detail {
+// Team reduction over all threads of the CTA; the result is valid in warp 0.  One aligned
+// barrier, none after it: the per-warp slots are free again only after the caller's next
+// aligned barrier (league_reduce has one right after; its last-team combine is the final
+// use of the slots).
+template <class T, class Op>
+__device__ __forceinline__ T team_reduce_to_warp0(T v, Op op) {
   __shared__ T omprt_warp_partial[32];
   v = warp_reduce(v, op);
   const uint32_t w = threadIdx.x >> 5, l = threadIdx.x & 31u;
@@ -79,12 +82,23 @@ __device__ __forceinline__ T team_reduce_to_main(Team<Tr>&, T v, Op op) {
   }
   return r;
 }
+}  // namespace detail
+
+// Team reduction over all threads of the CTA; the result is valid in warp 0 (thread 0 is
+// what the league reduction uses).  Ends with an aligned barrier, so back-to-back calls
+// cannot overwrite a slot warp 0 is still reading.
+template <class Tr, class T, class Op>
+__device__ __forceinline__ T team_reduce_to_main(Team<Tr>&, T v, Op op) {
+  const T r = detail::team_reduce_to_warp0(v, op);
+  aligned_barrier();
+  return r;
+}
 
 // Team reduction whose result is valid in every thread (SURVEY §8(b) team_reduce).
 template <class Tr, class T, class Op>
 __device__ __forceinline__ T team_reduce(Team<Tr>& team, T v, Op op) {
   __shared__ T omprt_team_result;
-  T r = team_reduce_to_main(team, v, op);
+  T r = detail::team_reduce_to_warp0(v, op);
   if (threadIdx.x == 0) omprt_team_result = r;
   aligned_barrier();
   r = omprt_team_result;
@@ -112,12 +126,22 @@ __device__ __forceinline__ void league_reduce(Team<Tr>& team, T team_val, Op op,
     T acc = Op::template identity<T>();
     for (uint32_t k = threadIdx.x; k < gridDim.x; k += blockDim.x)
       acc = op(acc, __ldcg(partials + k));
-    const T total = team_reduce_to_main(team, acc, op);
+    const T total = detail::team_reduce_to_warp0(acc, op);  // last use of the slots
     if (threadIdx.x == 0) {
       *inout = op(*inout, total);
       *ticket = 0u;
     }
   }
+}
+
+// Team + league reduction of every thread's private value v (the combined-construct form
+// `reduction(op: x)`): the team reduction feeds the league's ticket protocol directly, whose
+// aligned barrier also frees the team reduction's slots -- one barrier fewer than
+// league_reduce(team, team_reduce_to_main(...)).  Every thread of every team must call it.
+template <class Tr, class T, class Op>
+__device__ __forceinline__ void league_reduce_threads(Team<Tr>& team, T v, Op op, T* inout,
+                                                      T* partials, unsigned* ticket) {
+  league_reduce(team, detail::team_reduce_to_warp0(v, op), op, inout, partials, ticket);
 }
 
 }  // namespace omprt

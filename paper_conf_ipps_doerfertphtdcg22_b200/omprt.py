@@ -34,7 +34,6 @@ OMPRT_UNCHECKED = 1 << 9
 OMPRT_XS_ACCEL = 1 << 10
 OMPRT_SPMDIZE = 1 << 11
 OMPRT_DEGLOBALIZE = 1 << 12
-OMPRT_TMA_STAGED = 1 << 13
 OMPRT_WARP_STAGED = 1 << 14
 OMPRT_XS_FLAT = 1 << 15
 OMPRT_FLAT = OMPRT_XS_FLAT  # omprt_rs_lookup: flattened nuclide loop, persistent grid
@@ -51,7 +50,7 @@ EXPORTS = [
     "omprt_cuda_axpy_sum_chunked", "omprt_generic_team", "omprt_cuda_generic_team",
     "omprt_icv_probe", "omprt_lockstep_probe", "omprt_xs_lookup", "omprt_cuda_xs_lookup", "omprt_u64_sum",
     "omprt_xs_run_host", "omprt_xs_run_host_steps", "omprt_xs_accel_sizes", "omprt_xs_build_accel",
-    "omprt_xs_derive_tmp_bytes", "omprt_xs_derive", "omprt_xs_compact_sizes", "omprt_xs_build_compact", "omprt_rs_lookup", "omprt_cuda_rs_lookup", "omprt_su3_mult",
+    "omprt_xs_derive_tmp_bytes", "omprt_xs_derive", "omprt_rs_lookup", "omprt_cuda_rs_lookup", "omprt_su3_mult",
     "omprt_cuda_su3_mult", "omprt_kernel_count", "omprt_kernel_name", "omprt_kernel_attrs",
 ]
 
@@ -73,8 +72,7 @@ class XSTablesC(C.Structure):
                 ("n_isotopes", C.c_int32), ("n_gridpoints", C.c_int32),
                 ("max_num_nucs", C.c_int32), ("pad", C.c_int32), ("n_union", C.c_int64),
                 ("bins", C.c_void_p), ("index_grid16", C.c_void_p), ("brackets", C.c_void_p),
-                ("log2_bins", C.c_int32), ("pad2", C.c_int32),
-                ("idx_rows", C.c_void_p), ("owner", C.c_void_p)]
+                ("log2_bins", C.c_int32), ("pad2", C.c_int32)]
 
 
 class RSTablesC(C.Structure):
@@ -105,15 +103,13 @@ _SIGS = {
     "omprt_cuda_generic_team": [_i32, _i32, _i32, _vp, _vp, _vp, _vp, _u32, _vp],
     "omprt_icv_probe": [_i32, _i32, _i32, _vp, _u32, _vp],
     "omprt_lockstep_probe": [_i64, _i32, _i32, _i32, _vp, _vp, _vp, _vp],
-    "omprt_xs_lookup": [XSTablesC, _u64, _i64, _i64, _vp, _vp, _i32, _i32, _u32, _vp],
-    "omprt_cuda_xs_lookup": [XSTablesC, _u64, _i64, _i64, _vp, _vp, _i32, _i32, _u32, _vp],
+    "omprt_xs_lookup": [XSTablesC, _u64, _i64, _i64, _vp, _vp, _vp, _i32, _i32, _u32, _vp],
+    "omprt_cuda_xs_lookup": [XSTablesC, _u64, _i64, _i64, _vp, _vp, _vp, _i32, _i32, _u32, _vp],
     "omprt_u64_sum": [_vp, _i64, _vp, _vp],
     "omprt_xs_accel_sizes": [_i32, _i32, _i64, _i32, C.POINTER(_u64)],
     "omprt_xs_build_accel": [C.POINTER(XSTablesC), _vp, _vp, _vp, _i32, _vp],
     "omprt_xs_derive_tmp_bytes": [_i32, _i32, C.POINTER(_u64)],
     "omprt_xs_derive": [_vp, _i32, _i32, _vp, _vp, _vp, _u64, _vp],
-    "omprt_xs_compact_sizes": [_i32, _i32, C.POINTER(_u64)],
-    "omprt_xs_build_compact": [_vp, _i32, _i32, _vp, _vp, _vp, _u64, _vp],
     "omprt_xs_run_host": [XSTablesC, _u64, _i64, _i64, _i32, _u32, C.POINTER(_u64),
                           C.POINTER(_u64), C.POINTER(_u64), _vp],
     "omprt_xs_run_host_steps": [XSTablesC, _u64, _i64, _i64, _i32, _u32, _i32, C.POINTER(_u64),
@@ -156,15 +152,30 @@ def _check(code):
     return code
 
 
-def _p(t):
-    """Device pointer of a torch CUDA tensor (None -> NULL)."""
+def _p(t, dtype=None, n=None):
+    """Device pointer of a torch CUDA tensor (None -> NULL).  Checks what the C ABI cannot:
+    contiguous, on the current CUDA device, of the element type the ABI expects (`dtype`,
+    a torch dtype or a tuple of them) and holding at least `n` elements -- a wrong tensor is
+    a ValueError here, not an out-of-bounds device access."""
     if t is None:
         return None
     if not t.is_cuda:
         raise ValueError("expected a CUDA tensor")
     if not t.is_contiguous():
         raise ValueError("expected a contiguous tensor")
+    import torch
+    if t.device.index != torch.cuda.current_device():
+        raise ValueError(f"tensor on {t.device}, current device is cuda:{torch.cuda.current_device()}")
+    if dtype is not None and t.dtype not in (dtype if isinstance(dtype, tuple) else (dtype,)):
+        raise ValueError(f"expected dtype {dtype}, got {t.dtype}")
+    if n is not None and t.numel() < n:
+        raise ValueError(f"tensor holds {t.numel()} elements, the call needs {n}")
     return t.data_ptr()
+
+
+def _T():
+    import torch
+    return torch
 
 
 def _hp(a):
@@ -220,43 +231,58 @@ def omprt_static_owner(iv, n, teams, threads):
 
 
 # ---------------------------------------------------------------- C1
+def _axpy_ptrs(n, b, c, a, sum_inout, owner, count):
+    f64, i32, m = _T().float64, _T().int32, max(int(n), 0)
+    return (_p(b, f64, m), _p(c, f64, m), _p(a, f64, m), _p(sum_inout, f64, 1),
+            _p(owner, i32, m), _p(count, i32, m))
+
+
 def omprt_spmd_axpy_sum(n, x, b, c, a, sum_inout, teams, threads, flags=0, owner=None,
                         count=None, stream=None):
-    return _check(load().omprt_spmd_axpy_sum(n, x, _p(b), _p(c), _p(a), _p(sum_inout), teams,
-                                             threads, flags, _p(owner), _p(count), _stream(stream)))
+    pb, pc, pa, ps, po, pn = _axpy_ptrs(n, b, c, a, sum_inout, owner, count)
+    return _check(load().omprt_spmd_axpy_sum(n, x, pb, pc, pa, ps, teams, threads, flags, po, pn,
+                                             _stream(stream)))
 
 
 def omprt_cuda_axpy_sum(n, x, b, c, a, sum_inout, teams, threads, flags=0, owner=None,
                         count=None, stream=None):
-    return _check(load().omprt_cuda_axpy_sum(n, x, _p(b), _p(c), _p(a), _p(sum_inout), teams,
-                                             threads, flags, _p(owner), _p(count), _stream(stream)))
+    pb, pc, pa, ps, po, pn = _axpy_ptrs(n, b, c, a, sum_inout, owner, count)
+    return _check(load().omprt_cuda_axpy_sum(n, x, pb, pc, pa, ps, teams, threads, flags, po, pn,
+                                             _stream(stream)))
 
 
 def omprt_spmd_axpy_sum_chunked(n, chunk, x, b, c, a, sum_inout, teams, threads, flags=0,
                                 owner=None, count=None, stream=None):
-    return _check(load().omprt_spmd_axpy_sum_chunked(n, chunk, x, _p(b), _p(c), _p(a),
-                                                     _p(sum_inout), teams, threads, flags,
-                                                     _p(owner), _p(count), _stream(stream)))
+    pb, pc, pa, ps, po, pn = _axpy_ptrs(n, b, c, a, sum_inout, owner, count)
+    return _check(load().omprt_spmd_axpy_sum_chunked(n, chunk, x, pb, pc, pa, ps, teams, threads,
+                                                     flags, po, pn, _stream(stream)))
 
 
 def omprt_cuda_axpy_sum_chunked(n, chunk, x, b, c, a, sum_inout, teams, threads, flags=0,
                                 owner=None, count=None, stream=None):
-    return _check(load().omprt_cuda_axpy_sum_chunked(n, chunk, x, _p(b), _p(c), _p(a),
-                                                     _p(sum_inout), teams, threads, flags,
-                                                     _p(owner), _p(count), _stream(stream)))
+    pb, pc, pa, ps, po, pn = _axpy_ptrs(n, b, c, a, sum_inout, owner, count)
+    return _check(load().omprt_cuda_axpy_sum_chunked(n, chunk, x, pb, pc, pa, ps, teams, threads,
+                                                     flags, po, pn, _stream(stream)))
 
 
 # ---------------------------------------------------------------- C2
+def _generic_ptrs(teams, inner_n, inp, out, owner, postlogue):
+    f64, m = _T().float64, max(int(teams) * int(inner_n), 0)
+    return (_p(inp, f64, m), _p(out, f64, m), _p(owner, _T().int32, m),
+            _p(postlogue, f64, max(int(teams), 0)))
+
+
 def omprt_generic_team(teams, threads, inner_n, inp, out, owner=None, postlogue=None, flags=0,
                        stream=None):
-    return _check(load().omprt_generic_team(teams, threads, inner_n, _p(inp), _p(out), _p(owner),
-                                            _p(postlogue), flags, _stream(stream)))
+    pi, po, pw, pp = _generic_ptrs(teams, inner_n, inp, out, owner, postlogue)
+    return _check(load().omprt_generic_team(teams, threads, inner_n, pi, po, pw, pp, flags,
+                                            _stream(stream)))
 
 
 def omprt_cuda_generic_team(teams, threads, inner_n, inp, out, owner=None, postlogue=None,
                             flags=0, stream=None):
-    return _check(load().omprt_cuda_generic_team(teams, threads, inner_n, _p(inp), _p(out),
-                                                 _p(owner), _p(postlogue), flags,
+    pi, po, pw, pp = _generic_ptrs(teams, inner_n, inp, out, owner, postlogue)
+    return _check(load().omprt_cuda_generic_team(teams, threads, inner_n, pi, po, pw, pp, flags,
                                                  _stream(stream)))
 
 
@@ -278,7 +304,7 @@ class XSDeviceTables:
     allocation, in that order, so the flattened launch's L2 persisting window covers all
     three (xsbench.cuh flat_launch)."""
 
-    def __init__(self, t, device="cuda", accel=False, log2_bins=18, compact=False, packed=True):
+    def __init__(self, t, device="cuda", accel=False, log2_bins=18, packed=True):
         import torch
         self.host = t
         self.nuclide_grid = torch.from_numpy(t.nuclide_grid).to(device)
@@ -307,23 +333,6 @@ class XSDeviceTables:
                 self.bins = torch.empty(sizes[0] // 4, dtype=torch.int32, device=device)
                 self.brackets = torch.empty(sizes[2] // 8, dtype=torch.float64, device=device)
             omprt_xs_build_accel(self, self.bins, self.index_grid16, self.brackets, log2_bins)
-        if compact:  # the compact index grid (flattened launches), from the nuclide grids
-            sizes = omprt_xs_compact_sizes(t.n_isotopes, t.n_gridpoints)
-            self.idx_rows = torch.empty(sizes[0] // 2, dtype=torch.uint16, device=device)
-            self.owner = torch.empty(sizes[1], dtype=torch.uint8, device=device)
-            tmp = torch.empty(omprt_xs_derive_tmp_bytes(t.n_isotopes, t.n_gridpoints),
-                              dtype=torch.uint8, device=device)
-            omprt_xs_build_compact(self.nuclide_grid, t.n_isotopes, t.n_gridpoints,
-                                   self.idx_rows, self.owner, tmp)
-            self.c.idx_rows, self.c.owner = _p(self.idx_rows), _p(self.owner)
-
-    def without_compact(self):
-        """A view of the same tables without the compact index grid."""
-        v = XSDeviceTables.__new__(XSDeviceTables)
-        v.__dict__.update(self.__dict__)
-        v.c = XSTablesC.from_buffer_copy(self.c)
-        v.c.idx_rows = v.c.owner = None
-        return v
 
     def plain(self):
         """A view of the same tables without the accelerated layouts."""
@@ -331,7 +340,6 @@ class XSDeviceTables:
         v.__dict__.update(self.__dict__)
         v.c = XSTablesC.from_buffer_copy(self.c)
         v.c.bins = v.c.index_grid16 = v.c.brackets = None
-        v.c.idx_rows = v.c.owner = None
         v.c.log2_bins = 0
         return v
 
@@ -345,20 +353,6 @@ def omprt_xs_accel_sizes(n_isotopes, n_gridpoints, n_union, log2_bins=18):
 def omprt_xs_build_accel(tables, bins, index_grid16, brackets, log2_bins=18, stream=None):
     return _check(load().omprt_xs_build_accel(C.byref(tables.c), _p(bins), _p(index_grid16),
                                               _p(brackets), log2_bins, _stream(stream)))
-
-
-def omprt_xs_compact_sizes(n_isotopes, n_gridpoints):
-    sz = (_u64 * 2)()
-    _check(load().omprt_xs_compact_sizes(n_isotopes, n_gridpoints, sz))
-    return list(sz)
-
-
-def omprt_xs_build_compact(nuclide_grid, n_isotopes, n_gridpoints, idx_rows, owner, tmp,
-                           stream=None):
-    return _check(load().omprt_xs_build_compact(_p(nuclide_grid), n_isotopes, n_gridpoints,
-                                                _p(idx_rows), _p(owner), _p(tmp),
-                                                tmp.numel() * tmp.element_size(),
-                                                _stream(stream)))
 
 
 def xs_host_struct(t, pinned=None, derive=False):
@@ -403,22 +397,31 @@ def omprt_xs_run_host_steps(host_struct, seed, first, count, steps, threads=256,
     return list(cks), hb.value, db.value
 
 
+def _lookup_ptrs(count, verification, checksum_inout, macro, width):
+    u64, m = (_T().uint64, _T().int64), max(int(count), 0)
+    return (_p(verification, u64, m), _p(checksum_inout, u64, 1),
+            _p(macro, _T().float64, width * m))
+
+
 def omprt_xs_lookup(tables, seed, first, count, verification, checksum_inout=None, teams=0,
-                    threads=256, flags=0, stream=None):
-    return _check(load().omprt_xs_lookup(tables.c, seed, first, count, _p(verification),
-                                         _p(checksum_inout), teams, threads, flags,
-                                         _stream(stream)))
+                    threads=256, flags=0, stream=None, macro=None):
+    """macro (test build): float64 [count*5] -- the 5 macroscopic cross sections per lookup."""
+    pv, pc, pm = _lookup_ptrs(count, verification, checksum_inout, macro, 5)
+    return _check(load().omprt_xs_lookup(tables.c, seed, first, count, pv, pc, pm, teams, threads,
+                                         flags, _stream(stream)))
 
 
 def omprt_cuda_xs_lookup(tables, seed, first, count, verification, checksum_inout=None, teams=0,
-                         threads=256, flags=0, stream=None):
-    return _check(load().omprt_cuda_xs_lookup(tables.c, seed, first, count, _p(verification),
-                                              _p(checksum_inout), teams, threads, flags,
-                                              _stream(stream)))
+                         threads=256, flags=0, stream=None, macro=None):
+    pv, pc, pm = _lookup_ptrs(count, verification, checksum_inout, macro, 5)
+    return _check(load().omprt_cuda_xs_lookup(tables.c, seed, first, count, pv, pc, pm, teams,
+                                              threads, flags, _stream(stream)))
 
 
 def omprt_u64_sum(v, n, out_inout, stream=None):
-    return _check(load().omprt_u64_sum(_p(v), n, _p(out_inout), _stream(stream)))
+    u64 = (_T().uint64, _T().int64)
+    return _check(load().omprt_u64_sum(_p(v, u64, max(int(n), 0)), n, _p(out_inout, u64, 1),
+                                       _stream(stream)))
 
 
 def omprt_xs_run_host(host_struct, seed, first, count, threads=256, flags=0, stream=None):
@@ -446,27 +449,36 @@ class RSDeviceTables:
 
 def omprt_rs_lookup(tables, seed, first, count, verification, macro=None, teams=0, threads=128,
                     flags=0, stream=None):
-    return _check(load().omprt_rs_lookup(tables.c, seed, first, count, _p(verification),
-                                         _p(macro), teams, threads, flags, _stream(stream)))
+    pv, _, pm = _lookup_ptrs(count, verification, None, macro, 4)
+    return _check(load().omprt_rs_lookup(tables.c, seed, first, count, pv, pm, teams, threads,
+                                         flags, _stream(stream)))
 
 
 def omprt_cuda_rs_lookup(tables, seed, first, count, verification, macro=None, teams=0,
                          threads=128, flags=0, stream=None):
-    return _check(load().omprt_cuda_rs_lookup(tables.c, seed, first, count, _p(verification),
-                                              _p(macro), teams, threads, flags, _stream(stream)))
+    pv, _, pm = _lookup_ptrs(count, verification, None, macro, 4)
+    return _check(load().omprt_cuda_rs_lookup(tables.c, seed, first, count, pv, pm, teams,
+                                              threads, flags, _stream(stream)))
 
 
 # ---------------------------------------------------------------- C5
+def _su3_ptrs(A, B, Cout, n_sites, checksum_inout):
+    f64, m = _T().float64, 72 * max(int(n_sites), 0)
+    return _p(A, f64, m), _p(B, f64, 72), _p(Cout, f64, m), _p(checksum_inout, f64, 1)
+
+
 def omprt_su3_mult(A, B, Cout, n_sites, checksum_inout=None, teams=0, threads=128, flags=0,
                    stream=None):
-    return _check(load().omprt_su3_mult(_p(A), _p(B), _p(Cout), n_sites, _p(checksum_inout), teams,
-                                        threads, flags, _stream(stream)))
+    pa, pb, pc, pk = _su3_ptrs(A, B, Cout, n_sites, checksum_inout)
+    return _check(load().omprt_su3_mult(pa, pb, pc, n_sites, pk, teams, threads, flags,
+                                        _stream(stream)))
 
 
 def omprt_cuda_su3_mult(A, B, Cout, n_sites, checksum_inout=None, teams=0, threads=128, flags=0,
                         stream=None):
-    return _check(load().omprt_cuda_su3_mult(_p(A), _p(B), _p(Cout), n_sites, _p(checksum_inout),
-                                             teams, threads, flags, _stream(stream)))
+    pa, pb, pc, pk = _su3_ptrs(A, B, Cout, n_sites, checksum_inout)
+    return _check(load().omprt_cuda_su3_mult(pa, pb, pc, n_sites, pk, teams, threads, flags,
+                                             _stream(stream)))
 
 
 # ---------------------------------------------------------------- introspection

@@ -32,4 +32,4 @@ du -sh $OUT
 for T in memcheck racecheck initcheck; do
   timeout 600 compute-sanitizer --tool $T python scripts/sanitize_run.py > $OUT/sanitize_${T}_$TAG.txt 2>&1
 done
-OMPRT_SANITIZE_NO_PER_THREAD_BULK=1 timeout 600 compute-sanitizer --tool synccheck python scripts/sanitize_run.py > $OUT/sanitize_synccheck_$TAG.txt 2>&1
+timeout 600 compute-sanitizer --tool synccheck python scripts/sanitize_run.py > $OUT/sanitize_synccheck_$TAG.txt 2>&1

@@ -35,7 +35,7 @@ def main(which):
             out.append(a.elapsed_time(b))
         return statistics.median(out)
 
-    A, TS = omprt.OMPRT_ASSUME_OVERSUB, omprt.OMPRT_TMA_STAGED
+    A = omprt.OMPRT_ASSUME_OVERSUB
     res = {}
     if "su3" in which:
         ns = 32 ** 4
@@ -44,8 +44,6 @@ def main(which):
         Ct = torch.empty_like(At)
         ck = torch.zeros(1, dtype=torch.float64, device=dev)
         variants = [("rt", omprt.omprt_su3_mult, A), ("twin", omprt.omprt_cuda_su3_mult, 0),
-                    ("rt_staged", omprt.omprt_su3_mult, TS),
-                    ("twin_staged", omprt.omprt_cuda_su3_mult, TS),
                     ("rt_wstaged", omprt.omprt_su3_mult, omprt.OMPRT_WARP_STAGED),
                     ("rt_tiled", omprt.omprt_su3_mult, omprt.OMPRT_TMA_TILED),
                     ("twin_tiled", omprt.omprt_cuda_su3_mult, omprt.OMPRT_TMA_TILED),

@@ -38,7 +38,7 @@ elif which == "su3":
     for _ in range(reps):
         omprt.omprt_su3_mult(At, Bt, Ct, ns, ck, 0, 128, A)
         omprt.omprt_cuda_su3_mult(At, Bt, Ct, ns, ck, 0, 128, 0)
-        for fl in (omprt.OMPRT_TMA_STAGED, omprt.OMPRT_WARP_STAGED):
+        for fl in (omprt.OMPRT_WARP_STAGED, omprt.OMPRT_TMA_TILED):
             omprt.omprt_su3_mult(At, Bt, Ct, ns, ck, 0, 128, fl)
             omprt.omprt_cuda_su3_mult(At, Bt, Ct, ns, ck, 0, 128, fl)
 elif which == "generic":

@@ -59,12 +59,14 @@ def main():
     omprt.omprt_xs_lookup(d, 1070, 0, m, None, ck, 0, 256, A | omprt.OMPRT_FUSED_REDUCTION)
     omprt.omprt_cuda_xs_lookup(d, 1070, 0, m, ver, None, 0, 256, 0)
     omprt.omprt_u64_sum(ver, m, ck)
-    # flattened (static, dynamic), compact index grid, fused, with the L2 window
+    # flattened (static, dynamic), fused, with the L2 window; the macro test build
     F = omprt.OMPRT_XS_FLAT
     omprt.omprt_l2_set_aside(1 << 40)
-    dc = omprt.XSDeviceTables(t, dev, accel=True, compact=True)
+    mac = torch.empty(5 * m, dtype=torch.float64, device=dev)
+    omprt.omprt_xs_lookup(d, 1070, 0, m, ver, None, 0, 256, 0, macro=mac)
+    omprt.omprt_xs_lookup(d, 1070, 0, m, ver, None, 3, 256, F, macro=mac)
     for fl in (F, F | D):
-        for tab in (d, dc):
+        for tab in (d,):
             omprt.omprt_xs_lookup(tab, 1070, 0, m, ver, None, 3, 256, fl)
             omprt.omprt_xs_lookup(tab, 1070, 0, m, None, ck, 3, 256,
                                   fl | omprt.OMPRT_FUSED_REDUCTION)
@@ -89,14 +91,9 @@ def main():
     cs = torch.zeros(1, dtype=torch.float64, device=dev)
     omprt.omprt_su3_mult(At, Bt, Ct, ns, cs, 0, 128, A)
     omprt.omprt_cuda_su3_mult(At, Bt, Ct, ns, cs, 0, 128, 0)
-    # staged / streamed variants: SU(3) per-thread bulk, warp cp.async, 2-D tensor tiles; C1
-    # TMA-streamed Fig. 5 columns
-    # (synccheck cannot track the per-thread mbarriers of OMPRT_TMA_STAGED -- 2 per thread:
-    # "overflow of tracked cuda::barrier structures", then the instrumented run faults --
-    # so the round script skips that variant under synccheck only)
-    staged = [] if os.environ.get("OMPRT_SANITIZE_NO_PER_THREAD_BULK") else [
-        omprt.OMPRT_TMA_STAGED]
-    for fl in staged + [omprt.OMPRT_WARP_STAGED, omprt.OMPRT_TMA_TILED]:
+    # staged / streamed variants: SU(3) warp cp.async, 2-D tensor tiles; C1 TMA-streamed Fig. 5
+    # columns
+    for fl in [omprt.OMPRT_WARP_STAGED, omprt.OMPRT_TMA_TILED]:
         omprt.omprt_su3_mult(At, Bt, Ct, ns, cs, 2, 128, fl)
         omprt.omprt_cuda_su3_mult(At, Bt, Ct, ns, cs, 2, 128, fl)
     n1 = 8 * 128 * 40 + 77  # whole boxes, a partial box and a ragged last trip

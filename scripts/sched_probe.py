@@ -47,18 +47,6 @@ def main(which):
     if "xs" in which:
         omprt.omprt_l2_set_aside(1 << 40)
         r = {}
-        dc = omprt.XSDeviceTables(tabs, dev, accel=True, compact=True)
-        for aside in (1 << 40, 0):
-            got = omprt.omprt_l2_set_aside(aside)
-            for name, fn, fl in [("rt_flat_compact", omprt.omprt_xs_lookup, F),
-                                 ("twin_flat_compact", omprt.omprt_cuda_xs_lookup, F),
-                                 ("rt_flat_compact_nowin", omprt.omprt_xs_lookup,
-                                  F | omprt.OMPRT_XS_NO_L2_PERSIST),
-                                 ("rt_dflat_compact", omprt.omprt_xs_lookup, F | D)]:
-                ver.zero_()
-                key = f"{name}_aside{got >> 20}MB"
-                r[key] = t(lambda: fn(dc, 1070, 0, n, ver, None, 0, 256, fl))
-                r[key + "_same"] = bool((ver == ref).all())
         omprt.omprt_l2_set_aside(1 << 40)
         for name, fn, fl in [("rt_flat", omprt.omprt_xs_lookup, F),
                              ("twin_flat", omprt.omprt_cuda_xs_lookup, F),

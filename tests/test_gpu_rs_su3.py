@@ -137,13 +137,12 @@ def _su3(rt, fn, A, B, n, flags=0):
 
 
 @pytest.mark.parametrize("n", [8 ** 4, 8 ** 4 + 5, 32 ** 4])
-@pytest.mark.parametrize("variant", ["rt", "rt_loop", "twin", "rt_staged", "twin_staged",
-                                     "rt_wstaged", "twin_wstaged", "rt_tiled", "twin_tiled"])
+@pytest.mark.parametrize("variant", ["rt", "rt_loop", "twin", "rt_wstaged", "twin_wstaged",
+                                     "rt_tiled", "twin_tiled"])
 def test_su3_bit_exact(rt, n, variant):
     A, B = gen.su3_inputs(n)
     fn = rt.omprt_cuda_su3_mult if variant.startswith("twin") else rt.omprt_su3_mult
     flags = {"rt": rt.OMPRT_ASSUME_OVERSUB, "rt_loop": 0, "twin": 0,
-             "rt_staged": rt.OMPRT_TMA_STAGED, "twin_staged": rt.OMPRT_TMA_STAGED,
              "rt_wstaged": rt.OMPRT_WARP_STAGED, "twin_wstaged": rt.OMPRT_WARP_STAGED,
              "rt_tiled": rt.OMPRT_TMA_TILED, "twin_tiled": rt.OMPRT_TMA_TILED}[variant]
     C, ck = _su3(rt, fn, A, B, n, flags)
@@ -153,7 +152,7 @@ def test_su3_bit_exact(rt, n, variant):
     assert abs(ck - oracle.sum_f64(re)) <= 1e-12 * oracle.sum_abs_f64(re)
 
 
-@pytest.mark.parametrize("flag", ["OMPRT_TMA_STAGED", "OMPRT_WARP_STAGED", "OMPRT_TMA_TILED"])
+@pytest.mark.parametrize("flag", ["OMPRT_WARP_STAGED", "OMPRT_TMA_TILED"])
 @pytest.mark.parametrize("teams", [1, 3, 148])
 def test_su3_staged_geometries(rt, flag, teams):
     """Few persistent teams (many tiles per warp, both buffers cycling) and a ragged last
@@ -172,8 +171,7 @@ def test_su3_staged_geometries(rt, flag, teams):
 def test_su3_staged_flags_exclusive(rt):
     A = torch.zeros(72 * 64, dtype=torch.float64, device=DEV)
     B = torch.zeros(72, dtype=torch.float64, device=DEV)
-    for both in (rt.OMPRT_TMA_STAGED | rt.OMPRT_WARP_STAGED,
-                 rt.OMPRT_TMA_TILED | rt.OMPRT_WARP_STAGED,
+    for both in (rt.OMPRT_TMA_TILED | rt.OMPRT_WARP_STAGED,
                  rt.OMPRT_TMA_TILED | rt.OMPRT_ASSUME_OVERSUB):
         with pytest.raises(Exception):
             rt.omprt_su3_mult(A, B, A, 64, None, 0, 128, both)

@@ -326,134 +326,135 @@ def test_dynamic_needs_flat(rt, xs_acc):
         rt.omprt_xs_lookup(xs_acc, SEED, 0, 64, ver, None, 0, 256, rt.OMPRT_SCHED_DYNAMIC)
 
 
-# ---- compact index grid (reading R-X1) ------------------------------------------------
-def _compact(rt, grid, n_iso, n_gp):
-    g = torch.from_numpy(np.ascontiguousarray(grid.reshape(-1))).to(DEV)
-    sz = rt.omprt_xs_compact_sizes(n_iso, n_gp)
-    rows = torch.zeros(sz[0] // 2, dtype=torch.int16, device=DEV)
-    owner = torch.zeros(sz[1], dtype=torch.uint8, device=DEV)
-    tmp = torch.empty(rt.omprt_xs_derive_tmp_bytes(n_iso, n_gp), dtype=torch.uint8, device=DEV)
-    rt.omprt_xs_build_compact(g, n_iso, n_gp, rows, owner, tmp)
+# ---- the macroscopic cross sections, value for value (test build: macro output) --------
+def _macro_run(rt, d, first, count, which, flags, teams=0):
+    ver = torch.zeros(max(count, 1), dtype=torch.uint64, device=DEV)
+    mac = torch.full((max(count, 1) * 5,), float("nan"), dtype=torch.float64, device=DEV)
+    fn = rt.omprt_xs_lookup if which == "rt" else rt.omprt_cuda_xs_lookup
+    fn(d, SEED, first, count, ver, None, teams, 256, flags, macro=mac)
     torch.cuda.synchronize()
-    return rows.cpu().numpy().view(np.uint16).reshape(-1, n_iso), owner.cpu().numpy()
+    return ver.cpu().numpy()[:count], mac.cpu().numpy()[:5 * count].reshape(count, 5)
 
 
-def _rebuild(rows, owner, e, n_iso, n_gp):
-    """index_grid[e] from the compact layout, written out: stored row + matches."""
-    u0 = e - e % 16
-    c = rows[e // 16].astype(np.int64) + np.bincount(owner[u0 + 1:e + 1], minlength=256)[:n_iso]
-    return np.clip(c - 1, 0, n_gp - 2)
+def _assert_bitwise(got, ref):
+    """Every double identical bit for bit (NaN never equals, so an unwritten slot fails)."""
+    g, r = got.view(np.uint64), np.ascontiguousarray(ref).view(np.uint64)
+    bad = np.nonzero((g != r).any(axis=-1))[0]
+    assert bad.size == 0, f"{bad.size} lookups differ, first {bad[:5]}: {got[bad[:2]]} vs {ref[bad[:2]]}"
+
+
+# (layout, launch flags, which): every lookup kernel family of the library
+MACRO_VARIANTS = {
+    "plain_rt": ("plain", 0, "rt"),
+    "plain_rt_assume": ("plain", "OMPRT_ASSUME_OVERSUB", "rt"),
+    "plain_twin": ("plain", 0, "twin"),
+    "accel_rt": ("accel", 0, "rt"),
+    "accel_rt_assume": ("accel", "OMPRT_ASSUME_OVERSUB", "rt"),
+    "accel_twin": ("accel", 0, "twin"),
+    "flat_rt": ("accel", "OMPRT_XS_FLAT", "rt"),
+    "flat_twin": ("accel", "OMPRT_XS_FLAT", "twin"),
+    "dflat_rt": ("accel", "OMPRT_XS_FLAT|OMPRT_SCHED_DYNAMIC", "rt"),
+    "dflat_twin": ("accel", "OMPRT_XS_FLAT|OMPRT_SCHED_DYNAMIC", "twin"),
+}
+
+
+def _flags(rt, spec):
+    f = 0
+    for name in (spec.split("|") if spec else []):
+        f |= getattr(rt, name)
+    return f
+
+
+@pytest.fixture(scope="module")
+def macro_ref(xs_small):
+    first, count = 12345, (1 << 17) + 29  # many teams and a ragged end
+    v, m = oracle.xs_lookup(xs_small, first, count, want_macro=True,
+                            threads=os.cpu_count() or 1)
+    return first, count, v, m
+
+
+@pytest.mark.parametrize("variant", list(MACRO_VARIANTS))
+def test_macro_xs_bit_exact(rt, xs_dev, xs_acc, macro_ref, variant):
+    """All 5 macroscopic cross sections of every lookup, bit for bit against the oracle
+    (`+ - * /` with explicit fma points on both sides), for every lookup
+    kernel (plain / B200 layouts, assumption on / off, one lookup per thread / flattened
+    static / flattened dynamic, runtime-driven and twin) -- not only their argmax."""
+    layout, spec, which = MACRO_VARIANTS[variant]
+    first, count, vref, mref = macro_ref
+    d = xs_dev if layout == "plain" else xs_acc
+    for teams in ((0, 3) if "FLAT" in (spec or "") else (0,)):
+        ver, mac = _macro_run(rt, d, first, count, which, _flags(rt, spec), teams)
+        _assert_bitwise(mac, mref)
+        assert (ver == vref).all()
+
+
+def test_macro_rejects_fused_and_debug(rt, xs_acc, xs_dev):
+    mac = torch.zeros(64 * 5, dtype=torch.float64, device=DEV)
+    ck = torch.zeros(1, dtype=torch.uint64, device=DEV)
+    with pytest.raises(rt.OmprtError):
+        rt.omprt_xs_lookup(xs_acc, SEED, 0, 64, None, ck, 0, 256, rt.OMPRT_FUSED_REDUCTION,
+                           macro=mac)
+    ver = torch.zeros(64, dtype=torch.uint64, device=DEV)
+    with pytest.raises(rt.OmprtError):
+        rt.omprt_xs_lookup(xs_dev, SEED, 0, 64, ver, None, 0, 256, rt.OMPRT_DEBUG_BUILD,
+                           macro=mac)
+    with pytest.raises(ValueError):  # the binding checks sizes and types before the ABI
+        rt.omprt_xs_lookup(xs_acc, SEED, 0, 65, ver, None, 0, 256, 0, macro=mac)
+    with pytest.raises(ValueError):
+        rt.omprt_xs_lookup(xs_acc, SEED, 0, 64, ver.float(), None, 0, 256, 0)
+
+
+def test_macro_full_size_sampled_windows(rt, xs_acc, xs_small):
+    """BASELINE configs[2] at full size in the bench's headline launch (flattened,
+    persistent grid, L2 window as timed): the macroscopic cross sections of three windows
+    of the 17M lookups (start, middle, ragged end) bit-exact against the oracle."""
+    n = 17_000_000
+    ver, mac = _macro_run(rt, xs_acc, 0, n, "rt", rt.OMPRT_XS_FLAT)
+    w = 1 << 15
+    for lo in (0, n // 2 - 777, n - w):
+        v, m = oracle.xs_lookup(xs_small, lo, w, want_macro=True, threads=os.cpu_count() or 1)
+        _assert_bitwise(mac[lo:lo + w], m)
+        assert (ver[lo:lo + w] == v).all()
+
+
+@pytest.mark.parametrize("flags", [0, "OMPRT_XS_FLAT"])
+def test_argmax_ties_first_maximum_wins(rt, xs_small, flags):
+    """Channels equal at every gridpoint (gen.xs_tied_channels: elastic = total, fission =
+    nu-fission = absorption) tie exactly in the accumulated values, so the verification can
+    only be 1 or 3 under "the first maximum wins" (App. A.1; a last-maximum argmax gives 2
+    or 5)."""
+    t = gen.xs_tied_channels(xs_small)
+    d = rt.XSDeviceTables(t, DEV, accel=True)
+    first, count = 99, 50_003
+    vref, mref = oracle.xs_lookup(t, first, count, want_macro=True, threads=os.cpu_count() or 1)
+    assert set(np.unique(vref)) == {1, 3}
+    ver, mac = _macro_run(rt, d, first, count, "rt", _flags(rt, flags))
+    _assert_bitwise(mac, mref)
+    assert (mac[:, 0] == mac[:, 1]).all() and (mac[:, 2] == mac[:, 4]).all()
+    assert (ver == vref).all()
 
 
 def _quantized_grid(n_iso, n_gp, q=4096):
-    """Energies on a 1/q lattice (ties within and across nuclides), the two smallest and
-    the two largest energies kept distinct (the builder's precondition)."""
+    """Energies on a 1/q lattice (ties within and across nuclides)."""
     t = gen.XSTables(n_isotopes=n_iso, n_gridpoints=n_gp)
     g = t.nuclide_grid.reshape(n_iso, n_gp, 6).copy()
     e = np.clip(np.floor(g[:, :, 0] * q) / q, 2.0 / q, 1.0 - 3.0 / q)
-    e[0, 0], e[0, -1] = 0.5 / q, 1.0 - 0.5 / q
     g[:, :, 0] = np.sort(e, axis=1)
     return t, g
 
 
-@pytest.mark.parametrize("n_iso,n_gp", [(68, 11303), (68, 500), (3, 2), (7, 1500)])
-def test_compact_layout_content(rt, n_iso, n_gp):
-    """Every index-grid row the search can return (the last of a group of equal energies)
-    rebuilt from the compact layout equals App. A.1's definition (numpy searchsorted)."""
-    t = gen.XSTables(n_isotopes=n_iso, n_gridpoints=n_gp)
-    rows, owner = _compact(rt, t.nuclide_grid, n_iso, n_gp)
-    n = n_iso * n_gp
-    assert (owner[n:] == 0xFF).all() and owner.size % 16 == 0
-    E = t.nuclide_grid.reshape(n_iso, n_gp, 6)[:, :, 0]
-    assert (np.sort(E.reshape(-1), kind="stable") == t.unionized).all()
-    ids = np.repeat(np.arange(n_iso), n_gp)[np.argsort(E.reshape(-1), kind="stable")]
-    assert (owner[:n] == ids).all()
-    rng = np.random.default_rng(5)
-    sample = np.unique(np.concatenate([[0, 1, n - 2, n - 1], np.arange(min(n, 40)),
-                                       rng.integers(0, n, 3000)]))
-    for e in sample:
-        if e + 1 < n and t.unionized[e + 1] == t.unionized[e]:
-            continue
-        assert (_rebuild(rows, owner, int(e), n_iso, n_gp) == t.index_grid[e]).all(), e
-
-
-def test_compact_layout_with_ties(rt):
-    n_iso, n_gp = 68, 700
-    t, g = _quantized_grid(n_iso, n_gp)
-    rows, owner = _compact(rt, g, n_iso, n_gp)
-    U, idx = _definition(g, n_iso, n_gp)
-    n = n_iso * n_gp
-    last = np.nonzero(np.append(U[1:] != U[:-1], True))[0]
-    assert last.size < n  # there are ties
-    for e in last[::7]:
-        assert (_rebuild(rows, owner, int(e), n_iso, n_gp) == idx[e]).all(), e
-
-
-def test_compact_rejects_ties_at_the_ends_and_bad_shapes(rt):
-    n_iso, n_gp = 68, 300
-    t, g = _quantized_grid(n_iso, n_gp)
-    g[1, 0, 0] = g[0, 0, 0]  # the two smallest energies equal
-    with pytest.raises(rt.OmprtError):
-        _compact(rt, g, n_iso, n_gp)
-    with pytest.raises(rt.OmprtError):
-        rt.omprt_xs_compact_sizes(256, 100)
-    with pytest.raises(rt.OmprtError):
-        rt.omprt_xs_compact_sizes(10, 65536)
-
-
-def _compact_tables(rt, t):
-    return rt.XSDeviceTables(t, DEV, accel=True, compact=True)
-
-
-@pytest.fixture(scope="module")
-def xs_cmp(rt, xs_small):
-    return _compact_tables(rt, xs_small)
-
-
-@pytest.mark.parametrize("variant", ["flat", "flat_fused", "dflat"])
-def test_compact_lookups_bit_exact(rt, xs_cmp, xs_small, variant):
-    F = rt.OMPRT_XS_FLAT | (rt.OMPRT_SCHED_DYNAMIC if variant == "dflat" else 0)
-    for first, count, teams in [(0, 1, 0), (9, 255, 1), (3, 100_003, 0), (77, 50_000, 5)]:
-        ref = oracle.xs_lookup(xs_small, first, count, threads=os.cpu_count() or 1)
-        for fn in (rt.omprt_xs_lookup, rt.omprt_cuda_xs_lookup):
-            if variant == "flat_fused":
-                ck = torch.full((1,), 3, dtype=torch.uint64, device=DEV)
-                fn(xs_cmp, SEED, first, count, None, ck, teams, 256, F | rt.OMPRT_FUSED_REDUCTION)
-                torch.cuda.synchronize()
-                assert int(ck.cpu().numpy()[0]) == int(ref.sum()) + 3
-            else:
-                ver = torch.zeros(count, dtype=torch.uint64, device=DEV)
-                fn(xs_cmp, SEED, first, count, ver, None, teams, 256, F)
-                torch.cuda.synchronize()
-                assert (ver.cpu().numpy() == ref).all()
-
-
-def test_compact_lookups_with_ties(rt):
-    """Tables whose energies tie (1/4096 lattice): every lookup bit-exact against the
-    oracle on the same tables (unionized + index grid from App. A.1's definition)."""
+def test_lookups_with_tied_energies(rt):
+    """Tables whose energies tie (1/4096 lattice): the binned search and the 16-bit index
+    grid return the same brackets as App. A.1's definition; every lookup's macroscopic
+    cross sections bit-exact against the oracle on the same tables."""
     t, g = _quantized_grid(68, 700)
     t.nuclide_grid = np.ascontiguousarray(g.reshape(-1, 6))
     t.unionized, t.index_grid = _definition(g, 68, 700)
     t.index_grid = t.index_grid.astype(np.int32)
-    d = _compact_tables(rt, t)
+    d = rt.XSDeviceTables(t, DEV, accel=True)
     n = 60_000
-    ref = oracle.xs_lookup(t, 0, n, threads=os.cpu_count() or 1)
-    ver = torch.zeros(n, dtype=torch.uint64, device=DEV)
-    rt.omprt_xs_lookup(d, SEED, 0, n, ver, None, 0, 256, rt.OMPRT_XS_FLAT)
-    torch.cuda.synchronize()
-    assert (ver.cpu().numpy() == ref).all()
-
-
-def test_compact_needs_flat(rt, xs_cmp):
-    ver = torch.zeros(64, dtype=torch.uint64, device=DEV)
-    with pytest.raises(rt.OmprtError):
-        rt.omprt_xs_lookup(xs_cmp, SEED, 0, 64, ver, None, 0, 256, rt.OMPRT_ASSUME_OVERSUB)
-
-
-def test_full_size_17M_compact(rt, xs_cmp, xs_ref_17M):
-    """The headline launch on the compact index grid, all 17M lookups bit-exact."""
-    n = 17_000_000
-    ver = torch.zeros(n, dtype=torch.uint64, device=DEV)
-    rt.omprt_xs_lookup(xs_cmp, SEED, 0, n, ver, None, 0, 256, rt.OMPRT_XS_FLAT)
-    torch.cuda.synchronize()
-    assert (ver.cpu().numpy() == xs_ref_17M).all()
+    vref, mref = oracle.xs_lookup(t, 0, n, want_macro=True, threads=os.cpu_count() or 1)
+    for flags in (0, rt.OMPRT_XS_FLAT):
+        ver, mac = _macro_run(rt, d, 0, n, "rt", flags)
+        _assert_bitwise(mac, mref)
+        assert (ver == vref).all()

@@ -56,3 +56,28 @@ def test_icv_table_openmp_values(N):
             assert list(rec[t, 1 + N + k]) == [0, 1, 2, active, active, t, teams]
             # after the nested region the thread's environment is the outer one again
             assert list(rec[t, 1 + 2 * N + k]) == [k, N, 1, active, active, t, teams]
+
+
+def _recover_perm(teams, inner, t):
+    """perm of team t recovered from the oracle's outputs: with in = 1..n, w[k] = (t+1)(k+1)
+    and out[j] = w[perm[j]]/s + w[j], so perm[j] = (out[j] - w[j]) s/(t+1) - 1."""
+    inp = np.tile(np.arange(1, inner + 1, dtype=np.float64), teams)
+    out, _, _ = oracle.generic_team(teams, 64, inner, inp)
+    w = (t + 1) * np.arange(1, inner + 1, dtype=np.float64)
+    o = out[t * inner:(t + 1) * inner]
+    return np.rint((o - w) * w.sum() / (t + 1)).astype(int) - 1
+
+
+def test_generic_perm_hand_derived_golden():
+    """The prologue's permutation (App. A.4, reading R-A1: perm[k] = (17k + t) mod n) at
+    hand-derived entries (tests/golden/generic_perm.txt), recovered from the oracle's
+    outputs -- a wrong bijection (another multiplier or offset) fails here."""
+    import os
+    rows = np.loadtxt(os.path.join(os.path.dirname(__file__), "golden", "generic_perm.txt"),
+                      dtype=np.int64, comments="#")
+    cache = {}
+    for t, n, k, p in rows:
+        key = (int(t), int(n))
+        if key not in cache:
+            cache[key] = _recover_perm(int(t) + 1, int(n), int(t))
+        assert cache[key][k] == p, (t, n, k)

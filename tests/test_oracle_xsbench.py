@@ -129,3 +129,32 @@ def test_xs_bytes_per_lookup(xs_small):
     b = oracle.xs_bytes(xs_small, 0, 20000) / 20000
     # ~19.5 probes * 8 B + 15.5 nuclides * 112 B + 12 B  (DESIGN.md roofline)
     assert 1700 < b < 2100
+
+
+def _argmax_from_minus_one(mac):
+    """1 + argmax with a strict `>` scan starting from max = -1, written
+    with numpy: argmax (documented first occurrence) over [-1, m_0 .. m_4]; column 0 (no
+    value above -1, which extrapolated cross sections can reach) gives 1, column k gives k."""
+    ext = np.hstack([np.full((mac.shape[0], 1), -1.0), mac])
+    return np.maximum(np.argmax(ext, axis=1), 1)
+
+
+def test_argmax_first_maximum_wins_on_tied_channels(xs_small):
+    """verification = argmax_k(macro_xs[k]) + 1, the FIRST maximum
+    winning.  On tables whose channels are equal at every gridpoint the macroscopic values
+    tie exactly, so only 1 or 3 can win; numpy's first-occurrence argmax is the independent
+    reference."""
+    t = gen.xs_tied_channels(xs_small)
+    ver, mac = oracle.xs_lookup(t, 5, 20_000, want_macro=True)
+    assert (mac[:, 0] == mac[:, 1]).all() and (mac[:, 2] == mac[:, 3]).all()
+    assert (mac[:, 3] == mac[:, 4]).all()
+    assert (ver == _argmax_from_minus_one(mac)).all()
+    assert set(np.unique(ver)) == {1, 3}
+    # the degenerate case: every value <= -1 (extrapolation below a nuclide's first
+    # gridpoint) leaves the scan at its start, verification 1
+    low = np.nonzero(mac.max(axis=1) <= -1.0)[0]
+    assert low.size >= 1 and (ver[low] == 1).all()
+    # and on the untouched tables the verification is that argmax of the macro values too
+    ver, mac = oracle.xs_lookup(xs_small, 5, 20_000, want_macro=True)
+    assert (ver == _argmax_from_minus_one(mac)).all()
+    assert set(np.unique(ver)) == {1, 2, 3, 4, 5}

@@ -157,6 +157,63 @@ def load_peaks():
     return 6650.0, "fallback 6.65 TB/s (B200_PROFILING.md)"
 
 
+def measure_peaks(omprt, torch, dev, stream, detail=False):
+    """The roofs MEASURED_PEAKS.json does not hold, measured live on this GPU with the
+    library's probes (csrc/kernels/peaks.cuh; best of 5 CUDA-event-timed launches after a
+    warm-up): L2 -> SM read bandwidth of a 40 MB L2-resident buffer with the 256-bit
+    L1-non-allocating loads of the C3 bracket records -- streaming (the hardware's best case),
+    random 32 B sectors, random 96 B records -- and FP64 FMA throughput (8 independent
+    chains per thread, 8 teams of 256 per SM)."""
+    props = torch.cuda.get_device_properties(dev)
+    sms = props.multi_processor_count
+    teams = 4 * sms
+    nthr = teams * 256
+    unit = 4 * nthr * 32                      # bytes per grid-stride step of the stream mode
+    size = unit * max(1, (40 << 20) // unit)  # ~40 MB, a whole number of steps
+    buf = torch.ones(size // 8, dtype=torch.float64, device=dev)
+    sink = torch.zeros(1, dtype=torch.float64, device=dev)
+
+    def best(fn, reps=5):
+        fn()
+        torch.cuda.synchronize()
+        out = []
+        for _ in range(reps):
+            a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            a.record(stream)
+            fn()
+            b.record(stream)
+            torch.cuda.synchronize()
+            out.append(a.elapsed_time(b))
+        return min(out)
+
+    res = {"l2_buffer_bytes": size, "teams": teams, "threads_per_team": 256}
+    R = 20
+    ms = best(lambda: omprt.omprt_probe_l2_read(buf, size, 0, R, 0, sink, teams))
+    res["l2_stream_gbs"] = R * size / ms / 1e6
+    P, R2 = 64, 4
+    ms = best(lambda: omprt.omprt_probe_l2_read(buf, size, 1, R2, P, sink, teams))
+    res["l2_sector32_gbs"] = R2 * P * nthr * 32 / ms / 1e6
+    ms = best(lambda: omprt.omprt_probe_l2_read(buf, size, 2, R2, P, sink, teams))
+    res["l2_record96_gbs"] = R2 * P * nthr * 96 / ms / 1e6
+    it = 1 << 14
+    fteams = 8 * sms
+    ms = best(lambda: omprt.omprt_probe_fp64_fma(it, sink, fteams))
+    res["fp64_fma_gflops"] = 16.0 * it * fteams * 256 / ms / 1e6
+    if detail:  # capacity sweep of the stream roof
+        sweep = {}
+        for mb in (8, 24, 48, 96, 192):
+            sz = unit * max(1, (mb << 20) // unit)
+            b2 = torch.ones(sz // 8, dtype=torch.float64, device=dev)
+            r = max(1, (800 << 20) // sz)
+            ms = best(lambda: omprt.omprt_probe_l2_read(b2, sz, 0, r, 0, sink, teams))
+            sweep[f"{sz >> 20}MB"] = r * sz / ms / 1e6
+            del b2
+        res["stream_gbs_by_buffer"] = sweep
+    res["how"] = ("omprt_probe_l2_read / omprt_probe_fp64_fma (csrc/kernels/peaks.cuh), best of 5 "
+                  "CUDA-event-timed launches")
+    return res
+
+
 def load_alg_bytes(accel):
     d = json.load(open(os.path.join(ROOT, "profiles", "xs_algorithmic_bytes.json")))
     return float(d["accel"]["bytes_per_lookup"] if accel else d["bytes_per_lookup"])

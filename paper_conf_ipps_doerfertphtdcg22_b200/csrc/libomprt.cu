@@ -11,3 +11,4 @@
 #include "kernels/rs_su3.cuh"
 #include "kernels/su3_staged.cuh"
 #include "kernels/lockstep_probe.cuh"
+#include "kernels/peaks.cuh"

@@ -52,6 +52,7 @@ EXPORTS = [
     "omprt_xs_run_host", "omprt_xs_run_host_steps", "omprt_xs_accel_sizes", "omprt_xs_build_accel",
     "omprt_xs_derive_tmp_bytes", "omprt_xs_derive", "omprt_rs_lookup", "omprt_cuda_rs_lookup", "omprt_su3_mult",
     "omprt_cuda_su3_mult", "omprt_kernel_count", "omprt_kernel_name", "omprt_kernel_attrs",
+    "omprt_probe_l2_read", "omprt_probe_fp64_fma",
 ]
 
 
@@ -118,6 +119,8 @@ _SIGS = {
     "omprt_cuda_rs_lookup": [RSTablesC, _u64, _i64, _i64, _vp, _vp, _i32, _i32, _u32, _vp],
     "omprt_su3_mult": [_vp, _vp, _vp, _i64, _vp, _i32, _i32, _u32, _vp],
     "omprt_cuda_su3_mult": [_vp, _vp, _vp, _i64, _vp, _i32, _i32, _u32, _vp],
+    "omprt_probe_l2_read": [_vp, _u64, _i32, _i32, _i32, _i32, _vp, _vp],
+    "omprt_probe_fp64_fma": [_i64, _i32, _vp, _vp],
     "omprt_kernel_count": [],
     "omprt_kernel_name": [C.c_int],
     "omprt_kernel_attrs": [C.c_int, C.POINTER(C.c_int), C.POINTER(C.c_int), C.POINTER(C.c_int),
@@ -479,6 +482,19 @@ def omprt_cuda_su3_mult(A, B, Cout, n_sites, checksum_inout=None, teams=0, threa
     pa, pb, pc, pk = _su3_ptrs(A, B, Cout, n_sites, checksum_inout)
     return _check(load().omprt_cuda_su3_mult(pa, pb, pc, n_sites, pk, teams, threads, flags,
                                              _stream(stream)))
+
+
+# ---------------------------------------------------------------- measurement probes
+def omprt_probe_l2_read(buf, nbytes, mode, reps, per_thread, sink, teams=0, stream=None):
+    f64 = _T().float64
+    return _check(load().omprt_probe_l2_read(_p(buf, f64, nbytes // 8), nbytes, mode, reps,
+                                             per_thread, teams, _p(sink, f64, 1),
+                                             _stream(stream)))
+
+
+def omprt_probe_fp64_fma(iters, sink, teams=0, stream=None):
+    return _check(load().omprt_probe_fp64_fma(iters, teams, _p(sink, _T().float64, 1),
+                                              _stream(stream)))
 
 
 # ---------------------------------------------------------------- introspection

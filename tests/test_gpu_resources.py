@@ -23,7 +23,6 @@ PAIRS = [
     ("omprt_generic_deglob_rt", "cuda_generic_twin", False),
     ("omprt_xs_flat_rt", "cuda_xs_flat_twin", True),
     ("omprt_xs_flat_rt_fused", "cuda_xs_flat_twin_fused", True),
-    ("omprt_su3_staged_rt", "cuda_su3_staged_twin", True),
     ("omprt_su3_wstaged_rt", "cuda_su3_wstaged_twin", True),
     ("omprt_su3_tiled_rt", "cuda_su3_tiled_twin", True),
     ("omprt_axpy_tma_rt", "cuda_axpy_tma_twin", True),

@@ -166,7 +166,7 @@ def measure_peaks(omprt, torch, dev, stream, detail=False):
     chains per thread, 8 teams of 256 per SM)."""
     props = torch.cuda.get_device_properties(dev)
     sms = props.multi_processor_count
-    teams = 4 * sms
+    teams = 2 * sms  # the probes' resident teams (csrc/kernels/peaks.cuh)
     nthr = teams * 256
     unit = 4 * nthr * 32                      # bytes per grid-stride step of the stream mode
     size = unit * max(1, (40 << 20) // unit)  # ~40 MB, a whole number of steps

@@ -364,7 +364,7 @@ int omprt_cuda_su3_mult(const double *A, const double *B, double *C, int64_t n_s
  * 126 MB L2) with 256-bit L1-non-allocating loads, the loads of the C3 bracket records:
  * mode 0 streams every 32 B sector `reps` times; mode 1 reads random 32 B sectors and mode 2
  * random 96 B records (3 adjacent sectors), `per_thread` (multiple of 8) per thread per
- * rep.  teams = 0: 4 per SM, 256 threads each.  The caller times the launch on `stream`.
+ * rep.  teams = 0: 2 per SM, 256 threads each.  The caller times the launch on `stream`.
  * sink: one device double (written only under a never-true condition). */
 int omprt_probe_l2_read(const double *buf, uint64_t bytes, int32_t mode, int32_t reps,
                         int32_t per_thread, int32_t teams, double *sink, void *stream);

@@ -291,7 +291,13 @@ def run_omprt(args):
         omprt.omprt_u64_sum(ver, L, ck)
         if world > 1:
             ck_all.copy_(ck.view(torch.int64))
+            if kernel_events:
+                kernel_events[2].record(stream)
             sharding.allreduce_u64_sum(ck_all.view(torch.uint64))  # NCCL, wraps mod 2^64
+            if kernel_events:  # the current stream waits for the collective (async_op=False)
+                kernel_events[3].record(stream)
+
+    allreduce_ms = []  # N > 1: the checksum all-reduce of each timed step, timed apart
 
     def timed(which, tables, flags, k_steps, w_steps):
         for _ in range(w_steps):
@@ -303,21 +309,22 @@ def run_omprt(args):
         if world > 1:
             dist.barrier()
         torch.cuda.synchronize()
-        ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True),
-               torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
+        ev = [tuple(torch.cuda.Event(enable_timing=True) for _ in range(6))
               for _ in range(k_steps)]
         for e in ev:
             torch.cuda.synchronize()
             omprt.omprt_l2_reset_persisting()  # no line survives the flush (flat's L2 window)
             scrub.fill_(1.0)  # L2 flush, outside the step's events
             e[0].record(stream)
-            step((e[1], e[2]), which, tables, flags)
+            step((e[1], e[2], e[4], e[5]), which, tables, flags)
             e[3].record(stream)
         torch.cuda.synchronize()
         if world > 1:
             dist.barrier()
-        step_ms = [a.elapsed_time(b) for a, _, _, b in ev]
-        kern_ms = [b.elapsed_time(c) for _, b, c, _ in ev]
+        step_ms = [e[0].elapsed_time(e[3]) for e in ev]
+        kern_ms = [e[1].elapsed_time(e[2]) for e in ev]
+        if world > 1:
+            allreduce_ms.append(statistics.mean(e[4].elapsed_time(e[5]) for e in ev))
         return step_ms, kern_ms
 
     def mx(v):
@@ -404,6 +411,7 @@ def run_omprt(args):
 
     tab = omprt.kernel_table()
     peak, peak_src = load_peaks()
+    peaks = measure_peaks(omprt, torch, dev, stream)  # the L2 and FP64 roofs, live
     alg = load_alg_bytes(True) * L
     achieved = alg / (kms["rt_flat"] / 1000.0) / 1e9
     props = torch.cuda.get_device_properties(dev)
@@ -412,14 +420,19 @@ def run_omprt(args):
     omprt.omprt_l2_set_aside(0)
     secondary = sharded = None
     if not args.no_secondary and world > 1:
-        sharded = run_sharded(omprt, torch, gen, sharding, dev, stream, scrub, rank, world)
+        sharded = run_sharded(omprt, torch, gen, sharding, dev, stream, scrub, rank, world,
+                              d_acc)
     if not args.no_secondary and rank == 0:
-        secondary = run_secondary(omprt, torch, gen, dev, stream, scrub)
+        secondary = run_secondary(omprt, torch, gen, dev, stream, scrub, peaks)
     cpu = None
     if rank == 0:
         r, cores, n, wall, _ = cpu_oracle_rate(tabs, seconds=3.0, first=first)
         cpu = {"value": r, "unit": UNIT, "cores": cores, "kind": "oracle",
                "sample": f"first {n} lookups of rank 0's batch, all host cores, {wall:.2f} s wall = {wall * cores:.1f} core-s"}
+        if not args.no_secondary:
+            cpu["one_core_prefix"] = one_core_oracle(tabs)
+    allreduce = mx(statistics.mean(allreduce_ms)) if allreduce_ms else None
+    l2_peak = peaks["l2_stream_gbs"]
     if rank == 0:
         line = {
             "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
@@ -437,15 +450,29 @@ def run_omprt(args):
                                   "bracket records), bracket records persisting in L2 during "
                                   "the launch (access-policy window; reset + flushed between "
                                   "steps)"},
-            "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
-                         "frac": achieved / peak,
-                         "traffic": load_ncu_traffic("omprt_xs_flat_rt"),
+            "roofline": {"bound": "l2", "achieved": achieved, "peak": l2_peak, "unit": "GB/s",
+                         "frac": achieved / l2_peak,
+                         "traffic": load_ncu_traffic("omprt_xs_flat_rt_timed") or
+                         load_ncu_traffic("omprt_xs_flat_rt"),
                          "kernel": "omprt_xs_flat_rt", "alg_bytes_per_launch": alg,
-                         "peak_source": peak_src,
-                         "note": "frac can exceed 1: the algorithmic bytes count every table "
-                                 "read, but the hot tables (147.6 MB on the B200 layouts) are "
-                                 "mostly served by the 126 MB L2 (traffic = ncu DRAM bytes); "
-                                 "the binding roof is the L2/L1 request path, see l2",
+                         "peak_source": "measured live in this run: L2 -> SM streaming read of "
+                                        f"a {peaks['l2_buffer_bytes'] >> 20} MB L2-resident "
+                                        "buffer with the kernel's 256-bit L1-non-allocating "
+                                        "loads (omprt_probe_l2_read, best of 5)",
+                         "note": "the lookups' hot tables (unionized grid, bins, bracket "
+                                 "records: 44 MB) are L2-resident in an access-policy window "
+                                 "and the 16-bit index grid partly so, so the binding roof is "
+                                 "the L2 -> SM path, not HBM (ncu: L1 75 %, L2 69 % busy); "
+                                 "`pattern_roof` is the same path for random 96 B records, "
+                                 "the bracket-record access pattern",
+                         "pattern_roof": {"peak": peaks["l2_record96_gbs"],
+                                          "frac": achieved / peaks["l2_record96_gbs"],
+                                          "what": "random 96 B records of an L2-resident "
+                                                  "buffer (omprt_probe_l2_read mode 2)"},
+                         "hbm": {"peak": peak, "frac": achieved / peak, "peak_source": peak_src,
+                                 "note": "algorithmic bytes against the HBM copy peak: above "
+                                         "1 because most of them are L2 hits"},
+                         "measured_roofs": peaks,
                          "l2": l2_roof("omprt_xs_flat_rt", kms["rt_flat"]),
                          "one_lookup_per_thread": {
                              "kernel": "omprt_xs_rt_assume_accel",
@@ -458,6 +485,7 @@ def run_omprt(args):
             "cpu_baseline": cpu,
             "e2e": e2e,
             "gpu_launches": 2 * args.steps,
+            "allreduce_ms": allreduce,
             "clocks": clk,
             "checksum": checksum,
             "kernel_ms": kms,
@@ -538,13 +566,55 @@ def _time_pair(fa, fb, stream, scrub, reps=15, warm=2):
     return _trimmed_mean(out[0], t), _trimmed_mean(out[1], t)
 
 
-def run_sharded(omprt, torch, gen, sharding, dev, stream, scrub, rank, world):
-    """BASELINE configs[3] and [4] as they are stated for several GPUs (N > 1 only): C4's
-    10M RSBench lookups and C5's 32^4 SU(3) sites split into contiguous per-rank shards
-    (strong scaling), each rank timing its own kernel (CUDA events; the max over ranks is
-    reported), then the one exchange step -- the checksum all-reduce over NCCL."""
+def _time_allreduce(torch, sharding, dev, stream, dtype, reps=20):
+    """The one exchange step alone: an 8 B checksum all-reduce, CUDA events on the
+    launching stream around each (the stream waits for the collective), mean over reps,
+    max over ranks."""
+    import torch.distributed as dist
+    t = torch.zeros(1, dtype=dtype, device=dev)
+    f = sharding.allreduce_u64_sum if dtype == torch.uint64 else sharding.allreduce_f64_sum
+    f(t)
+    torch.cuda.synchronize()
+    dist.barrier()
+    out = []
+    for _ in range(reps):
+        a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        a.record(stream)
+        f(t)
+        b.record(stream)
+        torch.cuda.synchronize()
+        out.append(a.elapsed_time(b))
+    return sharding.allreduce_max(statistics.mean(out), dev)
+
+
+def run_sharded(omprt, torch, gen, sharding, dev, stream, scrub, rank, world, d_acc):
+    """The configs as they are stated for several GPUs (N > 1 only), strong scaling: C3's
+    17M XSBench lookups (next to the headline's weak scaling), C4's 10M RSBench lookups and
+    C5's 32^4 SU(3) sites split into contiguous per-rank shards (lookups
+    [r*L/G, (r+1)*L/G)), each rank timing its own kernel (CUDA events; the max over ranks is
+    reported), then the one exchange step -- the checksum all-reduce over NCCL, timed
+    apart."""
     import torch.distributed as dist
     res = {}
+    # C3 strong scaling: the headline launch (flattened, persistent grid, L2 window) on a
+    # 17M/G shard
+    f3, c3 = sharding.shard(L, rank, world)
+    v3 = torch.empty(max(c3, 1), dtype=torch.uint64, device=dev)
+    ck3 = torch.zeros(1, dtype=torch.uint64, device=dev)
+    omprt.omprt_l2_set_aside(L2_SET_ASIDE)
+    dist.barrier()
+    t = _time(lambda: omprt.omprt_xs_lookup(d_acc, 1070, f3, c3, v3, None, 0, THREADS,
+                                            omprt.OMPRT_XS_FLAT), stream, scrub, reps=5, warm=2)
+    omprt.omprt_l2_set_aside(0)
+    ms = sharding.allreduce_max(t, dev)
+    omprt.omprt_u64_sum(v3, c3, ck3)
+    sharding.allreduce_u64_sum(ck3)
+    res["c3_xsbench_17M_strong"] = {
+        "ranks": world, "lookups_per_rank": c3, "max_rank_ms": ms,
+        "lookups_per_s": L / ms * 1e3, "checksum": int(ck3.cpu().numpy()[0]),
+        "allreduce_ms": _time_allreduce(torch, sharding, dev, stream, torch.uint64),
+        "variant": "the headline launch on a contiguous 17M/G shard; NCCL u64 checksum "
+                   "all-reduce"}
     nl = 10_000_000
     first, cnt = sharding.shard(nl, rank, world)
     rd = omprt.RSDeviceTables(gen.RSTables(), dev)
@@ -560,6 +630,8 @@ def run_sharded(omprt, torch, gen, sharding, dev, stream, scrub, rank, world):
     res["c4_rsbench_10M"] = {"ranks": world, "lookups_per_rank": cnt, "max_rank_ms": ms,
                              "lookups_per_s": nl / ms * 1e3,
                              "checksum": int(ck.cpu().numpy()[0]),
+                             "allreduce_ms": _time_allreduce(torch, sharding, dev, stream,
+                                                             torch.uint64),
                              "variant": "flattened, lock-step, schedule(dynamic,1), Abrarov poles "
                                         "queued per warp; NCCL u64 checksum all-reduce"}
     ns = 32 ** 4
@@ -569,44 +641,110 @@ def run_sharded(omprt, torch, gen, sharding, dev, stream, scrub, rank, world):
     Ct = torch.empty_like(At)
     cks = torch.zeros(1, dtype=torch.float64, device=dev)
     dist.barrier()
-    t = _time(lambda: omprt.omprt_su3_mult(At, Bt, Ct, sc, cks, 0, 128,
-                                           omprt.OMPRT_ASSUME_OVERSUB), stream, scrub)
+    TT = omprt.OMPRT_TMA_TILED
+    t = _time(lambda: omprt.omprt_su3_mult(At, Bt, Ct, sc, cks, 0, 128, TT), stream, scrub)
     ms = sharding.allreduce_max(t, dev)
     cks.zero_()
-    omprt.omprt_su3_mult(At, Bt, Ct, sc, cks, 0, 128, omprt.OMPRT_ASSUME_OVERSUB)
+    omprt.omprt_su3_mult(At, Bt, Ct, sc, cks, 0, 128, TT)
     sharding.allreduce_f64_sum(cks)
     res["c5_su3_32^4"] = {"ranks": world, "sites_per_rank": sc, "max_rank_ms": ms,
                           "GBps_alg": 1152 * ns / ms / 1e6, "checksum": float(cks.item()),
-                          "variant": "one site per thread, 256-bit accesses; NCCL f64 "
-                                     "checksum all-reduce"}
+                          "allreduce_ms": _time_allreduce(torch, sharding, dev, stream,
+                                                          torch.float64),
+                          "variant": "TMA tensor tiles (one 2-D copy per warp tile each way); "
+                                     "NCCL f64 checksum all-reduce"}
     dist.barrier()
     return res
 
 
-def run_secondary(omprt, torch, gen, dev, stream, scrub):
-    """The other BASELINE configs at their sizes, runtime vs twin (kernel ms, cold L2)."""
+def _time_graph(fa, fb, stream, k=100, reps=5):
+    """SURVEY §8(d) for kernels shorter than ~50 us: each callable captured K times
+    back to back in a CUDA graph (torch.cuda.CUDAGraph), the graph replayed `reps` times
+    (rt and twin interleaved), per-launch time = graph time / K (min over replays).  The
+    working set stays in L2 across the K launches: this is the WARM figure."""
+    import torch
+    graphs = []
+    try:
+        for fn in (fa, fb):
+            fn()  # any first-call setup (attributes, workspace) outside the capture
+            torch.cuda.synchronize()
+            g = torch.cuda.CUDAGraph()
+            with torch.cuda.graph(g):
+                for _ in range(k):
+                    fn()
+            graphs.append(g)
+        torch.cuda.synchronize()
+    except Exception as e:  # noqa: BLE001 -- reported in the line, the bench goes on
+        torch.cuda.synchronize()
+        return None, f"graph capture failed: {e}"
+    times = ([], [])
+    for r in range(reps):
+        for idx in ((0, 1) if r % 2 == 0 else (1, 0)):
+            a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            a.record(stream)
+            graphs[idx].replay()
+            b.record(stream)
+            torch.cuda.synchronize()
+            times[idx].append(a.elapsed_time(b) / k)
+    return min(times[0]), min(times[1])
+
+
+def _graph_entry(g_rt, g_tw):
+    if g_rt is None:
+        return {"error": g_tw}
+    return {"rt_ms": g_rt, "twin_ms": g_tw, "overhead": g_rt / g_tw - 1}
+
+
+def _roof(bound, achieved, peak, unit, what):
+    return {"bound": bound, "achieved": achieved, "peak": peak, "unit": unit,
+            "frac": achieved / peak if peak else None, "work": what}
+
+
+def run_secondary(omprt, torch, gen, dev, stream, scrub, peaks):
+    """The other BASELINE configs at their sizes, runtime vs twin: kernel ms cold (L2
+    reset + flushed before every launch, trimmed mean of 15 interleaved reps), the short
+    kernels also as CUDA graphs of 100 launches (warm), each with its roofline (algorithmic
+    work per launch / time vs the measured roof) and theoretical occupancy (resident teams
+    per SM, cudaOccupancyMaxActiveBlocksPerMultiprocessor)."""
     res = {}
+    hbm, _ = load_peaks()
+    fp64 = peaks.get("fp64_fma_gflops")
+
+    def occ(name, threads, dyn=0):
+        try:
+            return omprt.omprt_kernel_occupancy(name, threads, dyn)
+        except Exception:  # noqa: BLE001 -- reported, not fatal
+            return None
+
     # C1: SPMD axpy + sum, 2^20, 8 x 128
     n = 1 << 20
     x, b, c = gen.axpy_inputs(n)
     bt, ct = torch.from_numpy(b).to(dev), torch.from_numpy(c).to(dev)
     at = torch.empty_like(bt)
     s = torch.zeros(1, dtype=torch.float64, device=dev)
-    t_rt, t_tw = _time_pair(
-        lambda: omprt.omprt_spmd_axpy_sum(n, x, bt, ct, at, s, 8, 128),
-        lambda: omprt.omprt_cuda_axpy_sum(n, x, bt, ct, at, s, 8, 128),
-        stream, scrub)
-    res["c1_axpy_sum_8x128"] = {"rt_ms": t_rt, "twin_ms": t_tw, "overhead": t_rt / t_tw - 1,
-                                "GBps_alg": 24 * n / t_rt / 1e6}
+    rt1 = lambda: omprt.omprt_spmd_axpy_sum(n, x, bt, ct, at, s, 8, 128)
+    tw1 = lambda: omprt.omprt_cuda_axpy_sum(n, x, bt, ct, at, s, 8, 128)
+    t_rt, t_tw = _time_pair(rt1, tw1, stream, scrub)
+    g_rt, g_tw = _time_graph(rt1, tw1, stream)
+    res["c1_axpy_sum_8x128"] = {
+        "rt_ms": t_rt, "twin_ms": t_tw, "overhead": t_rt / t_tw - 1,
+        "graph100_warm": _graph_entry(g_rt, g_tw),
+        "GBps_alg": 24 * n / t_rt / 1e6,
+        "roofline": _roof("hbm", 24 * n / t_rt / 1e6, hbm, "GB/s", "24 B/iteration, cold"),
+        "occupancy_teams_per_sm": [occ("omprt_axpy_rt", 128), occ("cuda_axpy_twin", 128)],
+        "note": "8 teams of 128 run on 8 of the 148 SMs by the config's definition"}
     # the same loop, operands streamed by 2-D TMA boxes (Fig. 5 assignment kept)
     TS_ = omprt.OMPRT_TMA_STREAM
-    t_rt, t_tw = _time_pair(
-        lambda: omprt.omprt_spmd_axpy_sum(n, x, bt, ct, at, s, 8, 128, TS_),
-        lambda: omprt.omprt_cuda_axpy_sum(n, x, bt, ct, at, s, 8, 128, TS_),
-        stream, scrub)
-    res["c1_axpy_sum_8x128_tma_stream"] = {"rt_ms": t_rt, "twin_ms": t_tw,
-                                           "overhead": t_rt / t_tw - 1,
-                                           "GBps_alg": 24 * n / t_rt / 1e6}
+    rt1t = lambda: omprt.omprt_spmd_axpy_sum(n, x, bt, ct, at, s, 8, 128, TS_)
+    tw1t = lambda: omprt.omprt_cuda_axpy_sum(n, x, bt, ct, at, s, 8, 128, TS_)
+    t_rt, t_tw = _time_pair(rt1t, tw1t, stream, scrub)
+    g_rt, g_tw = _time_graph(rt1t, tw1t, stream)
+    res["c1_axpy_sum_8x128_tma_stream"] = {
+        "rt_ms": t_rt, "twin_ms": t_tw, "overhead": t_rt / t_tw - 1,
+        "graph100_warm": _graph_entry(g_rt, g_tw),
+        "GBps_alg": 24 * n / t_rt / 1e6,
+        "roofline": _roof("hbm", 24 * n / t_rt / 1e6, hbm, "GB/s", "24 B/iteration, cold"),
+        "occupancy_teams_per_sm": [1, 1]}
     # NEXT f3: the same loop with schedule(static, 4): 256-bit chunk accesses
     t_rt, t_tw = _time_pair(
         lambda: omprt.omprt_spmd_axpy_sum_chunked(n, 4, x, bt, ct, at, s, 8, 128),
@@ -624,17 +762,20 @@ def run_secondary(omprt, torch, gen, dev, stream, scrub):
     def gen_rt(flags):
         return lambda: omprt.omprt_generic_team(T, 256, 256, inp, out, None, None, flags)
 
-    t_rt, t_tw = _time_pair(gen_rt(A_),
-                            lambda: omprt.omprt_cuda_generic_team(T, 256, 256, inp, out),
-                            stream, scrub)
+    tw2 = lambda: omprt.omprt_cuda_generic_team(T, 256, 256, inp, out)
+    t_rt, t_tw = _time_pair(gen_rt(A_), tw2, stream, scrub)
+    g_rt, g_tw = _time_graph(gen_rt(A_), tw2, stream)
     t_gs, t_db = _time_pair(gen_rt(omprt.OMPRT_GENERAL_SM), gen_rt(omprt.OMPRT_DEBUG_BUILD),
                             stream, scrub)
     t_sp, t_dg = _time_pair(gen_rt(A_ | omprt.OMPRT_SPMDIZE), gen_rt(A_ | omprt.OMPRT_DEGLOBALIZE),
                             stream, scrub)
-    res["c2_generic_4096x256"] = {"rt_ms": t_rt, "rt_general_sm_ms": t_gs, "twin_ms": t_tw,
-                                  "overhead": t_rt / t_tw - 1, "rt_spmdized_ms": t_sp,
-                                  "rt_deglobalized_ms": t_dg,
-                                  "rt_debug_build_env_off_ms": t_db}
+    res["c2_generic_4096x256"] = {
+        "rt_ms": t_rt, "rt_general_sm_ms": t_gs, "twin_ms": t_tw, "overhead": t_rt / t_tw - 1,
+        "graph100_warm": _graph_entry(g_rt, g_tw),
+        "rt_spmdized_ms": t_sp, "rt_deglobalized_ms": t_dg, "rt_debug_build_env_off_ms": t_db,
+        "roofline": _roof("hbm", 16 * T * 256 / t_rt / 1e6, hbm, "GB/s",
+                          "16 B/output, cold; latency-bound by the sequential prologue"),
+        "occupancy_teams_per_sm": [occ("omprt_generic_rt", 256), occ("cuda_generic_twin", 256)]}
     # C4: RSBench-shaped, 10M lookups (single GPU here)
     rs = gen.RSTables()
     rd = omprt.RSDeviceTables(rs, dev)
@@ -665,13 +806,19 @@ def run_secondary(omprt, torch, gen, dev, stream, scrub):
         lambda: omprt.omprt_rs_lookup(rd, 1070, 0, nl, v, None, 0, 128, FQ),
         lambda: omprt.omprt_cuda_rs_lookup(rd, 1070, 0, nl, v, None, 0, 128, FQ),
         stream, scrub, reps=3, warm=1)
-    res["c4_rsbench_10M"] = {"rt_ms": t_rt, "twin_ms": t_tw, "overhead": t_rt / t_tw - 1,
-                             "lookups_per_s": nl / t_rt * 1e3,
-                             "variant": "flattened nuclide loop, lock-step warps, "
-                                        "schedule(dynamic,1), persistent grid, pole records "
-                                        "prefetched, Abrarov poles queued per warp",
-                             "regs": [tab["omprt_rs_qflat_rt"]["regs"],
-                                      tab["cuda_rs_qflat_twin"]["regs"]]}
+    fl = load_rs_flops()
+    gflops = fl["flops_per_lookup"] * nl / t_rt / 1e6 if fl else None
+    res["c4_rsbench_10M"] = {
+        "rt_ms": t_rt, "twin_ms": t_tw, "overhead": t_rt / t_tw - 1,
+        "lookups_per_s": nl / t_rt * 1e3,
+        "variant": "flattened nuclide loop, lock-step warps, schedule(dynamic,1), persistent "
+                   "grid, pole records prefetched, Abrarov poles queued per warp",
+        "regs": [tab["omprt_rs_qflat_rt"]["regs"], tab["cuda_rs_qflat_twin"]["regs"]],
+        "roofline": _roof("fp64", gflops, fp64, "GFLOP/s",
+                          f"{fl['flops_per_lookup']:.0f} fp64 flops/lookup (oracle-counted add, "
+                          f"mul, div, sqrt; profiles/rs_algorithmic_flops.json) vs the measured "
+                          f"FP64 FMA roof (2 flops per fma)") if fl else None,
+        "occupancy_teams_per_sm": [occ("omprt_rs_qflat_rt", 128), occ("cuda_rs_qflat_twin", 128)]}
     # C5: SU(3) 32^4 sites
     ns = 32 ** 4
     Ah, Bh = gen.su3_inputs(ns)
@@ -689,18 +836,76 @@ def run_secondary(omprt, torch, gen, dev, stream, scrub):
         stream, scrub)
     res["c5_su3_32^4_warp_staged"] = {"rt_ms": t_rw, "twin_ms": t_tww,
                                       "overhead": t_rw / t_tww - 1,
-                                      "GBps_alg": 1152 * ns / t_rw / 1e6}
+                                      "GBps_alg": 1152 * ns / t_rw / 1e6,
+                                      "occupancy_teams_per_sm": [1, 1]}
     TT = omprt.OMPRT_TMA_TILED
     t_rtt, t_twt = _time_pair(
         lambda: omprt.omprt_su3_mult(At, Bt, Ct, ns, ck, 0, 128, TT),
         lambda: omprt.omprt_cuda_su3_mult(At, Bt, Ct, ns, ck, 0, 128, TT),
         stream, scrub)
-    res["c5_su3_32^4_tma_tiled"] = {"rt_ms": t_rtt, "twin_ms": t_twt,
-                                    "overhead": t_rtt / t_twt - 1,
-                                    "GBps_alg": 1152 * ns / t_rtt / 1e6}
-    res["c5_su3_32^4"] = {"rt_ms": t_rt, "twin_ms": t_tw, "overhead": t_rt / t_tw - 1,
-                          "GBps_alg": 1152 * ns / t_rt / 1e6, "GFLOPs": 864 * ns / t_rt / 1e6}
+    res["c5_su3_32^4_tma_tiled"] = {
+        "rt_ms": t_rtt, "twin_ms": t_twt, "overhead": t_rtt / t_twt - 1,
+        "GBps_alg": 1152 * ns / t_rtt / 1e6,
+        "roofline": _roof("hbm", 1152 * ns / t_rtt / 1e6, hbm, "GB/s", "1152 B/site, cold"),
+        "occupancy_teams_per_sm": [1, 1]}
+    res["c5_su3_32^4"] = {
+        "rt_ms": t_rt, "twin_ms": t_tw, "overhead": t_rt / t_tw - 1,
+        "GBps_alg": 1152 * ns / t_rt / 1e6, "GFLOPs": 864 * ns / t_rt / 1e6,
+        "roofline": _roof("hbm", 1152 * ns / t_rt / 1e6, hbm, "GB/s", "1152 B/site, cold"),
+        "occupancy_teams_per_sm": [occ("omprt_su3_rt", 128), occ("cuda_su3_twin", 128)]}
+    # C5 as one of 8 shards (32^4 / 8 sites, ~25 us): short, so also as a CUDA graph
+    n8 = ns // 8
+    r5 = lambda: omprt.omprt_su3_mult(At, Bt, Ct, n8, ck, 0, 128, TT)
+    w5 = lambda: omprt.omprt_cuda_su3_mult(At, Bt, Ct, n8, ck, 0, 128, TT)
+    t_rt, t_tw = _time_pair(r5, w5, stream, scrub)
+    g_rt, g_tw = _time_graph(r5, w5, stream)
+    res["c5_su3_shard_of_8_tma_tiled"] = {
+        "sites": n8, "rt_ms": t_rt, "twin_ms": t_tw, "overhead": t_rt / t_tw - 1,
+        "graph100_warm": _graph_entry(g_rt, g_tw),
+        "roofline": _roof("hbm", 1152 * n8 / t_rt / 1e6, hbm, "GB/s", "1152 B/site, cold")}
     return res
+
+
+def load_rs_flops():
+    p = os.path.join(ROOT, "profiles", "rs_algorithmic_flops.json")
+    return json.load(open(p)) if os.path.exists(p) else None
+
+
+def one_core_oracle(tabs):
+    """the oracle on ONE host core over fixed prefixes (C3: the first 10^6
+    lookups; C4: the first 2 x 10^4 -- 10^5 would take ~20 s; C5: one 32^4 sweep; C1: the
+    2^20 axpy + sum; C2: the 4096 x 256 generic kernel)."""
+    import gen
+    import oracle
+    out = {}
+    t0 = time.perf_counter()
+    oracle.xs_lookup(tabs, 0, 1_000_000, threads=1)
+    w = time.perf_counter() - t0
+    out["c3_xsbench"] = {"units": 1_000_000, "seconds": w, "per_s": 1_000_000 / w,
+                         "unit": "lookups/s"}
+    rs = gen.RSTables()
+    t0 = time.perf_counter()
+    oracle.rs_lookup(rs, 0, 20_000, threads=1)
+    w = time.perf_counter() - t0
+    out["c4_rsbench"] = {"units": 20_000, "seconds": w, "per_s": 20_000 / w, "unit": "lookups/s"}
+    ns = 32 ** 4
+    A, B = gen.su3_inputs(ns)
+    t0 = time.perf_counter()
+    oracle.su3_mult(A, B, ns, threads=1)
+    w = time.perf_counter() - t0
+    out["c5_su3"] = {"units": ns, "seconds": w, "per_s": ns / w, "unit": "sites/s"}
+    n = 1 << 20
+    x, b, c = gen.axpy_inputs(n)
+    t0 = time.perf_counter()
+    oracle.sum_f64(oracle.axpy(x, b, c))
+    w = time.perf_counter() - t0
+    out["c1_axpy_sum"] = {"units": n, "seconds": w, "per_s": n / w, "unit": "iterations/s"}
+    inp = gen.generic_inputs(4096, 256)
+    t0 = time.perf_counter()
+    oracle.generic_team(4096, 256, 256, inp)
+    w = time.perf_counter() - t0
+    out["c2_generic"] = {"units": 4096, "seconds": w, "per_s": 4096 / w, "unit": "teams/s"}
+    return out
 
 
 def main():

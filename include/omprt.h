@@ -380,6 +380,10 @@ const char *omprt_kernel_name(int id);
  * (spill/stack) bytes per thread, max threads per block. */
 int omprt_kernel_attrs(int id, int *regs, int *static_smem, int *local_bytes,
                        int *max_threads);
+/* Resident teams per SM of kernel `id` at `threads` per team and `dyn_smem` bytes of dynamic
+ * shared memory (cudaOccupancyMaxActiveBlocksPerMultiprocessor): the theoretical occupancy
+ * bench.py reports per config. */
+int omprt_kernel_occupancy(int id, int threads, int dyn_smem, int *blocks_per_sm);
 
 #ifdef __cplusplus
 }

@@ -328,7 +328,7 @@ def rs_lookup(t, first, count, seed=1070, want_macro=False, threads=1):
 
 def rs_count(t, first, count, seed=1070):
     s = rs_struct(t)
-    ops = np.zeros(9, np.int64)
+    ops = np.zeros(10, np.int64)
     lib().oracle_rs_count(C.byref(s), seed, first, count, _p(ops, _i64p))
     return ops
 

@@ -146,9 +146,9 @@ typedef struct {
 /* verification[i-first] = 1 + argmax of 4 macro xs; macro (nullable) [count][4]. */
 int oracle_rs_lookup(const oracle_rs_tables *t, uint64_t seed, int64_t first, int64_t count,
                      uint64_t *verification, double *macro);
-/* Event counts of lookups [first,first+count) into ops[9]: ops[5] = Faddeeva evaluations,
- * ops[6] = of them on the Abrarov branch, ops[7] = poles visited, ops[8] = (lookup, nuclide)
- * pairs; ops[0..4] = 0.  For the fp64-pipe roofline's per-unit figure. */
+/* Instrumented pass over lookups [first,first+count) (the C4 roofline's per-unit figure,
+ * SURVEY §8(d)): ops[10] = {add/sub, mul, div, sqrt, transcendental calls, Faddeeva
+ * evaluations, of them Abrarov, poles visited, (lookup, nuclide) pairs, fma}. */
 void oracle_rs_count(const oracle_rs_tables *t, uint64_t seed, int64_t first, int64_t count,
                      int64_t *ops);
 

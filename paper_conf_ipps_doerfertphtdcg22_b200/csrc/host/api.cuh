@@ -153,3 +153,11 @@ extern "C" int omprt_kernel_attrs(int id, int* regs, int* static_smem, int* loca
   if (max_threads) *max_threads = a.maxThreadsPerBlock;
   return OMPRT_OK;
 }
+
+extern "C" int omprt_kernel_occupancy(int id, int threads, int dyn_smem, int* blocks_per_sm) {
+  OMPRT_CHECK_ARG(id >= 0 && id < (int)registry().size(), "bad kernel id %d", id);
+  OMPRT_CHECK_ARG(threads > 0 && dyn_smem >= 0 && blocks_per_sm, "bad arguments");
+  OMPRT_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, registry()[id].fn,
+                                                               threads, (size_t)dyn_smem));
+  return OMPRT_OK;
+}

@@ -60,10 +60,18 @@ __global__ void __launch_bounds__(1024)
   const Idx gtid = (Idx)blockIdx.x * blockDim.x + threadIdx.x;
   double acc = 0.0;
   Idx i = gtid;
+  // 8 iterations per trip, all 16 loads issued before the first store (what a CUDA
+  // programmer writes to keep loads in flight with 4 warps per SM)
   for (; i + 7 * stride < n; i += 8 * stride) {
+    double bv[8], cv[8];
 #pragma unroll
     for (int u = 0; u < 8; ++u) {
-      const double v = fma(x, __ldg(b + i + u * stride), __ldg(c + i + u * stride));
+      bv[u] = __ldg(b + i + u * stride);
+      cv[u] = __ldg(c + i + u * stride);
+    }
+#pragma unroll
+    for (int u = 0; u < 8; ++u) {
+      const double v = fma(x, bv[u], cv[u]);
       a[i + u * stride] = v;
       acc += v;
       if constexpr (Rec) {

@@ -52,7 +52,7 @@ EXPORTS = [
     "omprt_xs_run_host", "omprt_xs_run_host_steps", "omprt_xs_accel_sizes", "omprt_xs_build_accel",
     "omprt_xs_derive_tmp_bytes", "omprt_xs_derive", "omprt_rs_lookup", "omprt_cuda_rs_lookup", "omprt_su3_mult",
     "omprt_cuda_su3_mult", "omprt_kernel_count", "omprt_kernel_name", "omprt_kernel_attrs",
-    "omprt_probe_l2_read", "omprt_probe_fp64_fma",
+    "omprt_probe_l2_read", "omprt_probe_fp64_fma", "omprt_kernel_occupancy",
 ]
 
 
@@ -122,6 +122,7 @@ _SIGS = {
     "omprt_probe_l2_read": [_vp, _u64, _i32, _i32, _i32, _i32, _vp, _vp],
     "omprt_probe_fp64_fma": [_i64, _i32, _vp, _vp],
     "omprt_kernel_count": [],
+    "omprt_kernel_occupancy": [C.c_int, C.c_int, C.c_int, C.POINTER(C.c_int)],
     "omprt_kernel_name": [C.c_int],
     "omprt_kernel_attrs": [C.c_int, C.POINTER(C.c_int), C.POINTER(C.c_int), C.POINTER(C.c_int),
                            C.POINTER(C.c_int)],
@@ -511,6 +512,14 @@ def omprt_kernel_attrs(i):
     r, s, l, m = C.c_int(), C.c_int(), C.c_int(), C.c_int()
     _check(load().omprt_kernel_attrs(i, C.byref(r), C.byref(s), C.byref(l), C.byref(m)))
     return dict(regs=r.value, static_smem=s.value, local_bytes=l.value, max_threads=m.value)
+
+
+def omprt_kernel_occupancy(name, threads, dyn_smem=0):
+    """Resident teams per SM of the registered kernel `name`."""
+    ids = {omprt_kernel_name(i): i for i in range(omprt_kernel_count())}
+    b = C.c_int()
+    _check(load().omprt_kernel_occupancy(ids[name], threads, dyn_smem, C.byref(b)))
+    return b.value
 
 
 def kernel_table():

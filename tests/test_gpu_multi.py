@@ -50,7 +50,12 @@ def _checksums(rank, world, omprt, gen, sharding, dev, backend="gloo"):
     Ct = torch.empty_like(At)
     cs = torch.zeros(1, dtype=torch.float64, device=dev)
     omprt.omprt_su3_mult(At, Bt, Ct, sc, cs, 0, 128, omprt.OMPRT_ASSUME_OVERSUB)
+    # ... and with the TMA tensor tiles bench.py's sharded C5 runs (same elementwise C)
+    Ct2 = torch.empty_like(At)
+    cs2 = torch.zeros(1, dtype=torch.float64, device=dev)
+    omprt.omprt_su3_mult(At, Bt, Ct2, sc, cs2, 0, 128, omprt.OMPRT_TMA_TILED)
     torch.cuda.synchronize()
+    assert torch.equal(Ct, Ct2)
     if backend == "gloo":  # gloo reduces host tensors, NCCL device ones
         ck, ck4, cs = ck.cpu(), ck4.cpu(), cs.cpu()
     if world > 1:

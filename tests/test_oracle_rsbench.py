@@ -125,6 +125,49 @@ def test_rs_counts(rs_tables):
     assert 40 < per[8] < 75          # nuclides per lookup (fuel has 321 of 355)
     assert 8 < per[7] / per[8] < 12  # ~avg_poles/avg_windows poles per window
     assert per[6] / per[5] < 0.02    # the Abrarov branch is rare
+    assert ops[5] == ops[7]          # one Faddeeva evaluation per pole
+    assert ops[9] == 0               # the definition has no fma
+
+
+# Operation counts per event, derived BY HAND from App. A.2 as the oracle writes it (a complex
+# product = 4 mul + 2 add, a complex quotient = 6 mul + 3 add + 2 div, |z| = 2 mul + 1 add
+# + 1 sqrt; fast_exp = 13 mul + 1 add; the method's constants a_n, (n pi)^2, tau^2 are not
+# operations):
+#   per (lookup, nuclide) pair: window 2 div + 3 mul; sigTfactors over l = 0..3:
+#     4 x (sqrt + mul by k0rs) + l=1 (atan, add) + l=2 (2 mul, 2 add, div, atan)
+#     + l=3 (4 mul, 3 add, div, atan) + 4 x (mul by 2, cos, sin);
+#     sigE = sigT - sigA (1 add); macro += micro * conc (4 mul + 4 add)
+#     -> add 11, mul 21, div 4, sqrt 4, transcendental 11
+#   per pole: Z (2 add, 2 mul); RT*(W*f) (2 complex products); RA*W, RF*W (1 each); 3 adds
+#     -> add 13, mul 18
+#   per Faddeeva evaluation on the asymptotic branch: |Z| + Z^2 (cplx mul) + 2 subtractions
+#     + 2 quotients + 1 complex add + i Z * (...) (cplx mul)
+#     -> add 15, mul 22, div 4, sqrt 1
+#   per Faddeeva evaluation on the Abrarov branch: |Z|; tau Z, i tau Z (4 mul); exp(i tau Z)
+#     (fast_exp + 2 mul + cos + sin); (1 - e) (2 add); i*(..) (cplx mul); /(tau Z) (quotient);
+#     Z^2 (cplx mul); 10 terms x (2 mul + 1 add for (-1)^n e - 1; 2 mul + 1 add for the
+#     denominator; a quotient; 2 mul + 2 add into the sum); Z*sum, prefactor*(..) (2 cplx
+#     mul); 1 complex add
+#     -> add 87, mul 163, div 22, sqrt 1, transcendental 2
+PER_PAIR = {"add": 11, "mul": 21, "div": 4, "sqrt": 4, "trans": 11}
+PER_POLE = {"add": 13, "mul": 18}
+PER_W_ASYM = {"add": 15, "mul": 22, "div": 4, "sqrt": 1}
+PER_W_ABR = {"add": 87, "mul": 163, "div": 22, "sqrt": 1, "trans": 2}
+
+
+def test_rs_operation_counts_hand_derived(rs_tables_small):
+    """The instrumented pass adds up exactly the hand-derived per-event counts
+    over 300 lookups: a dropped or double-counted operation anywhere fails here."""
+    ops = oracle.rs_count(rs_tables_small, 17, 300)
+    pairs, poles, w, abr = ops[8], ops[7], ops[5], ops[6]
+    assert abr > 0 and w - abr > 0
+    for k, name in enumerate(["add", "mul", "div", "sqrt", "trans"]):
+        expect = (PER_PAIR.get(name, 0) * pairs + PER_POLE.get(name, 0) * poles
+                  + PER_W_ASYM.get(name, 0) * (w - abr) + PER_W_ABR.get(name, 0) * abr)
+        assert ops[k] == expect, name
+    # and counting changes no result
+    assert (oracle.rs_lookup(rs_tables_small, 17, 300) ==
+            oracle.rs_lookup(rs_tables_small, 17, 300)).all()
 
 
 def test_abrarov_branch_without_sqrt():

@@ -27,9 +27,15 @@ struct AxpyTraitsDebug : AxpyTraits {
 struct AxpyTraitsAssumeDebug : AxpyTraitsAssume {
   static constexpr unsigned debug = dbg::Assert | dbg::Trace;
 };
+// Both C1 kernels carry the same register budget, __maxnreg__(48) (1024 threads still fit
+// an SM): with __launch_bounds__(1024) ptxas holds them to 32 registers and interleaves the
+// unrolled trip's loads with its stores (2-4 loads in flight per thread); with a budget of
+// its own it issues all 16 loads of a trip first -- what 4 warps per SM (C1: 8 teams x 128)
+// need.
 // Runtime-driven kernel: the OpenMP region as the runtime executes it.
+constexpr int kAxpyMaxRegs = 48;
 template <class Tr, bool Rec>
-__global__ void __launch_bounds__(1024)
+__global__ void __maxnreg__(kAxpyMaxRegs)
     omprt_axpy_rt(typename Tr::Idx n, double x, const double* __restrict__ b,
                   const double* __restrict__ c, double* __restrict__ a, double* sum_inout,
                   double* partials, unsigned* ticket, int32_t* owner, int32_t* count) {
@@ -52,7 +58,7 @@ __global__ void __launch_bounds__(1024)
 // Bare CUDA twin: grid-stride loop (the same cyclic assignment) and a hand-written copy of
 // the same reduction algorithm (shfl.xor butterfly, warp partials, last-block combine).
 template <class Idx, bool Rec>
-__global__ void __launch_bounds__(1024)
+__global__ void __maxnreg__(kAxpyMaxRegs)
     cuda_axpy_twin(Idx n, double x, const double* __restrict__ b, const double* __restrict__ c,
                    double* __restrict__ a, double* sum_inout, double* partials,
                    unsigned* ticket, int32_t* owner, int32_t* count) {

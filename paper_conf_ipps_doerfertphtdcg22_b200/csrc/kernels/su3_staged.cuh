@@ -138,8 +138,9 @@ __global__ void __launch_bounds__(kSU3WarpThreads, 1)
 #pragma unroll
     for (unsigned j = 0; j < kCh; ++j) {
       const unsigned c = lane + 32u * j;
-      tma::cp_async16_zfill(b + (c / kCh) * kSU3Slot + (c % kCh) * 16u,
-                            src + (c < nch ? c * 16u : 0u), c < nch ? 16u : 0u);
+      const unsigned r = c / kCh, q = c - r * kCh;  // record, 16 B chunk of the record
+      tma::cp_async16_zfill(b + r * kSU3Slot + q * 16u, src + (c < nch ? c * 16u : 0u),
+                            c < nch ? 16u : 0u);
     }
     tma::cp_async_commit();
   };
@@ -160,9 +161,11 @@ __global__ void __launch_bounds__(kSU3WarpThreads, 1)
 #pragma unroll
     for (unsigned j = 0; j < kCh; ++j) {
       const unsigned c = lane + 32u * j;
-      if (c < nch)
+      if (c < nch) {
+        const unsigned r = c / kCh, q = c - r * kCh;
         *reinterpret_cast<uint4*>(dst + c * 16u) =
-            *reinterpret_cast<const uint4*>(cur + (c / kCh) * kSU3Slot + (c % kCh) * 16u);
+            *reinterpret_cast<const uint4*>(cur + r * kSU3Slot + q * 16u);
+      }
     }
     __syncwarp();
   }

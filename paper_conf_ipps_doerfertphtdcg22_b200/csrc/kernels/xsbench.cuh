@@ -266,9 +266,34 @@ inline XSTables to_dev(const omprt_xs_tables& a) {
 // the set-aside granted by omprt_l2_set_aside (none: no window), so the 16-bit index grid's misses cannot evict
 // them; hitRatio scales down when the table exceeds the set-aside.  (Persisting lines
 // outlive the launch: omprt_l2_reset_persisting returns them to normal.)
+// The window is a STREAM attribute set around the one launch and restored after it (not a
+// launch attribute): Nsight Compute drops launch attributes when it replays a kernel, so
+// only this form lets ncu measure the launch exactly as it is timed (profiles/README.md).
 struct FlatLaunch {
   cudaLaunchConfig_t cfg;
-  cudaLaunchAttribute attr[1];
+  bool window = false;
+  cudaStreamAttrValue win{};
+};
+// Sets the window on the launch stream for the lifetime of the object, then restores the
+// stream's previous window.
+struct ScopedStreamWindow {
+  cudaStream_t s;
+  bool on;
+  cudaStreamAttrValue prev{};
+  ScopedStreamWindow(const FlatLaunch& L) : s(L.cfg.stream), on(L.window) {
+    if (on && cudaStreamGetAttribute(s, cudaStreamAttributeAccessPolicyWindow, &prev) ==
+                  cudaSuccess)
+      on = cudaStreamSetAttribute(s, cudaStreamAttributeAccessPolicyWindow, &L.win) ==
+           cudaSuccess;
+    else
+      on = false;
+    cudaGetLastError();  // a stream without attribute support just runs without the window
+  }
+  ~ScopedStreamWindow() {
+    if (on && cudaStreamSetAttribute(s, cudaStreamAttributeAccessPolicyWindow, &prev) !=
+                  cudaSuccess)
+      cudaGetLastError();
+  }
 };
 inline FlatLaunch flat_launch(const omprt_xs_tables& t, int32_t teams, int32_t threads,
                               uint32_t flags, const Workspace* w, cudaStream_t s) {
@@ -277,7 +302,7 @@ inline FlatLaunch flat_launch(const omprt_xs_tables& t, int32_t teams, int32_t t
   L.cfg.blockDim = dim3((unsigned)threads);
   L.cfg.dynamicSmemBytes = 0;
   L.cfg.stream = s;
-  L.cfg.attrs = L.attr;
+  L.cfg.attrs = nullptr;
   L.cfg.numAttrs = 0;
   const size_t br = sizeof(double) * 12ull * t.n_isotopes * (t.n_gridpoints - 1);
   if (!(flags & OMPRT_XS_NO_L2_PERSIST) && w->l2_persist_bytes > 0 && t.brackets) {
@@ -299,14 +324,13 @@ inline FlatLaunch flat_launch(const omprt_xs_tables& t, int32_t teams, int32_t t
     join(t.unionized, sizeof(double) * (size_t)t.n_union);
     const size_t bytes = std::min((size_t)(hi - lo), (size_t)std::max(maxwin, 0));
     if (bytes > 0) {
-      cudaAccessPolicyWindow& win = L.attr[0].val.accessPolicyWindow;
-      L.attr[0].id = cudaLaunchAttributeAccessPolicyWindow;
+      cudaAccessPolicyWindow& win = L.win.accessPolicyWindow;
       win.base_ptr = (void*)lo;
       win.num_bytes = bytes;
       win.hitRatio = (float)std::min(1.0, (double)w->l2_persist_bytes / (double)bytes);
       win.hitProp = cudaAccessPropertyPersisting;
       win.missProp = cudaAccessPropertyStreaming;
-      L.cfg.numAttrs = 1;
+      L.window = true;
     }
   }
   return L;
@@ -475,6 +499,7 @@ extern "C" int omprt_xs_lookup(omprt_xs_tables t, uint64_t seed, int64_t first, 
   if (flags & OMPRT_XS_FLAT) {
     const bool smem = xs_mats_fit_smem(t);
     const FlatLaunch L = flat_launch(t, teams, threads, flags, w, s);
+    ScopedStreamWindow sw(L);
     xs_flat_dispatch<false>(flags, fused, smem, L.cfg, d, seed, first, n, verification, ck, p,
                             tk, macro);
     return check_launch("omprt_xs_flat_rt");
@@ -533,6 +558,7 @@ extern "C" int omprt_cuda_xs_lookup(omprt_xs_tables t, uint64_t seed, int64_t fi
   if (flat) {  // the same launch (geometry, L2 window) as the runtime-driven kernel
     const bool smem = xs_mats_fit_smem(t);
     const FlatLaunch L = flat_launch(t, tm, threads, flags, w, s);
+    ScopedStreamWindow sw(L);
     unsigned long long* nul = nullptr;
     unsigned* nult = nullptr;
     if (fused)

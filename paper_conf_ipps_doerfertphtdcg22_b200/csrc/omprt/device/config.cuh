@@ -61,10 +61,22 @@ struct WithIdx64 : Base {
   using Idx = int64_t;
 };
 
+// OMPRT_STRIP_DEBUG (a verification build, tests/test_release_pruning.py): the debug
+// machinery does not exist at all -- no kernel is debug-instrumented whatever its traits,
+// and env.cuh defines neither the assertion nor the trace functions.  Every release kernel
+// of the normal build must compile to the same SASS as in this build (§III-G: "the
+// debugging code paths will be trivially dead and removed statically").
+#ifdef OMPRT_STRIP_DEBUG
+template <class Tr>
+inline constexpr bool kDebugAssert = false;
+template <class Tr>
+inline constexpr bool kDebugTrace = false;
+#else
 template <class Tr>
 inline constexpr bool kDebugAssert = (Tr::debug & dbg::Assert) != 0;
 template <class Tr>
 inline constexpr bool kDebugTrace = (Tr::debug & dbg::Trace) != 0;
+#endif
 template <class Tr>
 inline constexpr bool kHasStack = Tr::stack_bytes > 0 || Tr::dynamic_stack;
 

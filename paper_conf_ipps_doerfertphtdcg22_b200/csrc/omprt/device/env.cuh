@@ -49,6 +49,7 @@ __device__ __noinline__ void fatal(int code, int line, int extra) {
   __trap();
 }
 
+#ifndef OMPRT_STRIP_DEBUG
 __device__ __noinline__ void assert_fail(const char* msg, int line) {
   printf("[omprt] assertion failed (line %d, team %d, thread %d): %s\n", line,
          (int)blockIdx.x, (int)threadIdx.x, msg);
@@ -59,11 +60,21 @@ __device__ __noinline__ void trace_call(const char* fn) {
   printf("[omprt] team %d thread %d: %s\n", (int)blockIdx.x, (int)threadIdx.x, fn);
 }
 
+#endif  // OMPRT_STRIP_DEBUG
+
 }  // namespace omprt
 
 // OMPRT_ASSERT(Traits, cond, msg): checked in debug builds with the runtime Assert bit set;
 // otherwise an assumption.  __builtin_assume drops conditions with side effects,
 // so `cond` must be side-effect free.
+#ifdef OMPRT_STRIP_DEBUG
+// The stripped build: an assertion is only its release meaning (an assumption), a trace
+// point nothing.
+#define OMPRT_ASSERT(TR, COND, MSG) __builtin_assume(COND)
+#define OMPRT_TRACE(TR, NAME) \
+  do {                        \
+  } while (0)
+#else
 #define OMPRT_ASSERT(TR, COND, MSG)                                                  \
   do {                                                                               \
     if constexpr (::omprt::kDebugAssert<TR>) {                                       \
@@ -81,3 +92,4 @@ __device__ __noinline__ void trace_call(const char* fn) {
       if (omprt_env.debug_bits & ::omprt::dbg::Trace) ::omprt::trace_call(NAME);     \
     }                                                                                \
   } while (0)
+#endif  // OMPRT_STRIP_DEBUG

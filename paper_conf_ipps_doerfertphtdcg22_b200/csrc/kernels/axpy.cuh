@@ -27,13 +27,16 @@ struct AxpyTraitsDebug : AxpyTraits {
 struct AxpyTraitsAssumeDebug : AxpyTraitsAssume {
   static constexpr unsigned debug = dbg::Assert | dbg::Trace;
 };
-// Both C1 kernels carry the same register budget, __maxnreg__(48) (1024 threads still fit
-// an SM): with __launch_bounds__(1024) ptxas holds them to 32 registers and interleaves the
+// Both C1 kernels carry the same register budget, __maxnreg__(58) (1024 threads still fit
+// an SM).  Under __launch_bounds__(1024) ptxas held them to 32 registers and interleaved the
 // unrolled trip's loads with its stores (2-4 loads in flight per thread); with a budget of
-// its own it issues all 16 loads of a trip first -- what 4 warps per SM (C1: 8 teams x 128)
-// need.
+// their own both issue all 16 loads of a trip first -- what 4 warps per SM (C1: 8 teams x
+// 128) need: 0.30 -> 0.104 ms.  At a budget of 56 the runtime kernel (56 registers: it
+// keeps the trip's 8 indices for the stores where the twin advances pointers) lost that
+// schedule and ran 33 % slower; at 58 both run 0.104 ms (scripts/experiments/
+// c1_lib_kernels.cu, profiles/c1_budget_r2.txt).
 // Runtime-driven kernel: the OpenMP region as the runtime executes it.
-constexpr int kAxpyMaxRegs = 48;
+constexpr int kAxpyMaxRegs = 58;
 template <class Tr, bool Rec>
 __global__ void __maxnreg__(kAxpyMaxRegs)
     omprt_axpy_rt(typename Tr::Idx n, double x, const double* __restrict__ b,

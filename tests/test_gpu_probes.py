@@ -1,0 +1,39 @@
+"""The measurement side of the library (not the hot path): the roof probes bench.py
+reports against and the occupancy query -- they run, and their numbers are physically
+plausible for a B200 (so a broken probe cannot inflate or deflate a roofline fraction
+unnoticed)."""
+import pytest
+import torch
+
+pytestmark = pytest.mark.gpu
+DEV = "cuda:0"
+
+
+def test_roof_probes_plausible(rt):
+    import bench
+    p = bench.measure_peaks(rt, torch, torch.device(DEV), torch.cuda.current_stream())
+    # L2 -> SM: above the HBM copy peak (~6.5 TB/s), below 4 x it
+    assert 7000 < p["l2_stream_gbs"] < 26000, p
+    assert 2000 < p["l2_sector32_gbs"] <= p["l2_stream_gbs"] * 1.05, p
+    assert 2000 < p["l2_record96_gbs"] <= p["l2_stream_gbs"] * 1.05, p
+    # FP64 FMA: B200 nominal ~37-40 TFLOP/s
+    assert 20000 < p["fp64_fma_gflops"] < 45000, p
+
+
+def test_probe_arguments_rejected(rt):
+    buf = torch.ones(1024, dtype=torch.float64, device=DEV)
+    sink = torch.zeros(1, dtype=torch.float64, device=DEV)
+    with pytest.raises(rt.OmprtError):
+        rt.omprt_probe_l2_read(buf, 8192, 3, 1, 8, sink)      # no mode 3
+    with pytest.raises(rt.OmprtError):
+        rt.omprt_probe_l2_read(buf, 8192, 1, 1, 7, sink)      # per_thread % 8
+    with pytest.raises(rt.OmprtError):
+        rt.omprt_probe_fp64_fma(0, sink)
+
+
+def test_occupancy_query(rt):
+    # the headline kernel: 64 registers x 256 threads -> 4 resident teams per SM
+    assert rt.omprt_kernel_occupancy("omprt_xs_flat_rt", 256) == 4
+    assert rt.omprt_kernel_occupancy("omprt_rs_qflat_rt", 128) == 4
+    with pytest.raises(rt.OmprtError):
+        rt.omprt_kernel_occupancy("omprt_xs_flat_rt", 0)

@@ -15,6 +15,7 @@ echo "smoke exit $?" >> $OUT/smoke_$TAG.txt
 timeout 900 python bench.py --steps 10 --warmup 3 > $OUT/bench_$TAG.txt 2>&1
 echo "bench exit $?" >> $OUT/bench_$TAG.txt
 timeout 300 python bench.py --impl reference --steps 2 --warmup 1 > $OUT/bench_ref_$TAG.txt 2>&1
+timeout 300 python scripts/peaks_probe.py > $OUT/peaks_$TAG.txt 2>&1
 timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none -c 400 --csv \
   --log-file $OUT/launches_$TAG.csv python bench.py --steps 2 --warmup 1 --no-e2e --no-secondary > $OUT/ncu_launch_stdout_$TAG.txt 2>&1
 for K in omprt_xs_flat_rt cuda_xs_flat_twin omprt_xs_rt; do

@@ -135,6 +135,7 @@ extern "C" {
  * sections per pole (reading R-A8: a different summation order, within the RSBench
  * tolerance contract -- macro xs 1e-10 normwise, verification up to near-ties). */
 #define OMPRT_RS_QUEUE (1u << 20)
+/* (1u << 21) is unused: a warp-shared pole evaluation for RSBench measured slower. */
 
 /* ---- runtime lifecycle ------------------------------------------------------------- */
 typedef struct {

@@ -69,9 +69,46 @@ __device__ __forceinline__ LcgMap lcg_jump(uint64_t n) {
 __device__ __forceinline__ uint64_t lcg_apply(LcgMap m, uint64_t seed) {
   return (m.a * seed + m.c) & kLcgMask;
 }
+// The same maps for n = m * 256^b, m in [0, 256), b in [0, 8) (32 KB, compile time): a
+// fast-forward composes one per BYTE of n -- 4 for a 26-bit lookup index -- instead of one
+// per set bit through a ~24-trip loop.  The maps of one LCG commute, so any composition order
+// gives the same (a, c).  (Mattered where a lane starts a lookup alone: RSBench's dynamic
+// schedule ran that loop at 1.6 active lanes, 4.4 % of its warp instructions.)
+struct LcgByteJumps {
+  uint64_t a[8][256], c[8][256];
+};
+__host__ __device__ constexpr LcgByteJumps make_lcg_byte_jumps() {
+  LcgByteJumps t{};
+  const LcgJumps j = make_lcg_jumps();
+  for (int b = 0; b < 8; ++b)
+    for (int m = 0; m < 256; ++m) {
+      uint64_t a = 1, c = 0;
+      for (int k = 0; k < 8; ++k)
+        if ((m >> k) & 1) {
+          a *= j.a[8 * b + k];
+          c = c * j.a[8 * b + k] + j.c[8 * b + k];
+        }
+      t.a[b][m] = a;
+      t.c[b][m] = c;
+    }
+  return t;
+}
+__device__ const LcgByteJumps kLcgByteJumps = make_lcg_byte_jumps();
+__device__ __forceinline__ LcgMap lcg_jump_bytes(uint64_t n) {
+  uint64_t a_new = 1, c_new = 0;
+  for (int b = 0; n != 0; ++b, n >>= 8) {
+    const unsigned m = (unsigned)(n & 255u);
+    if (m) {
+      const uint64_t ak = __ldg(&kLcgByteJumps.a[b][m]);
+      a_new *= ak;
+      c_new = c_new * ak + __ldg(&kLcgByteJumps.c[b][m]);
+    }
+  }
+  return {a_new, c_new};
+}
 // fast_forward_LCG(seed, n)
 __device__ __forceinline__ uint64_t lcg_fast_forward(uint64_t seed, uint64_t n) {
-  return lcg_apply(lcg_jump(n), seed);
+  return lcg_apply(lcg_jump_bytes(n), seed);
 }
 
 __device__ __forceinline__ double lcg_double(uint64_t& seed) {
@@ -307,7 +344,9 @@ struct XSFlatLookup {
   template <class Idx>
   __device__ __forceinline__ void begin(Idx iv, Idx stride) {
     J = lcg_jump(2ull * (uint64_t)stride);
-    s = lcg_fast_forward(seed0, 2ull * (uint64_t)(first + iv));
+    // once per thread here (static schedule): the bit-serial jump, whose constant-bank
+    // table costs this 64-register loop no extra registers (the byte table spilled)
+    s = lcg_apply(lcg_jump(2ull * (uint64_t)(first + iv)), seed0);
     start();
   }
   template <class Idx>

@@ -26,6 +26,7 @@ def one(path):
     n = 10_000_000
     v = torch.empty(n, dtype=torch.uint64, device=dev)
     FQ = omprt.OMPRT_FLAT | omprt.OMPRT_SCHED_DYNAMIC | omprt.OMPRT_RS_QUEUE
+    FQ |= int(os.environ.get("RSV_EXTRA_FLAGS", "0"), 0)
     scrub = torch.empty(64 << 20, dtype=torch.float32, device=dev)
     s = torch.cuda.current_stream()
     fns = {"rt": lambda: omprt.omprt_rs_lookup(d, 1070, 0, n, v, None, 0, 128, FQ),
@@ -53,7 +54,15 @@ def one(path):
         torch.cuda.synchronize()
         mac[k] = mm.cpu().numpy()
     tab = omprt.kernel_table()
-    out = {"lib": path, "rt_ms": min(res["rt"]), "twin_ms": min(res["twin"]),
+    D = omprt.OMPRT_FLAT | omprt.OMPRT_SCHED_DYNAMIC
+    m0 = torch.empty(4 * m, dtype=torch.float64, device=dev)
+    v0 = torch.empty(m, dtype=torch.uint64, device=dev)
+    omprt.omprt_rs_lookup(d, 1070, 0, m, v0, m0, 0, 128, D)  # no queue: the reference order
+    torch.cuda.synchronize()
+    ref = m0.cpu().numpy().reshape(-1, 4)
+    got = mac["rt"].reshape(-1, 4)
+    normwise = float((np.abs(got - ref).max(axis=1) / np.abs(ref).max(axis=1)).max())
+    out = {"lib": path, "flags": FQ, "max_normwise_vs_unqueued": normwise, "rt_ms": min(res["rt"]), "twin_ms": min(res["twin"]),
            "rt_all": res["rt"], "twin_all": res["twin"], "checksums": cks,
            "rt_twin_macro_bit_identical": bool((mac["rt"].view(np.uint64) ==
                                                 mac["twin"].view(np.uint64)).all()),

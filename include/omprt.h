@@ -328,7 +328,9 @@ int omprt_xs_run_host_steps(omprt_xs_tables host_tables, uint64_t seed, int64_t 
 
 /* ---- C4: RSBench-shaped multipole lookup -------------------- */
 typedef struct {
-  const double *poles;      /* [n_poles][8] EA RT RA RF (re, im), 32 B aligned */
+  /* [n_poles][8] EA RT RA RF (re, im), 32 B aligned -- in the lookups' PREPARED form (see
+   * omprt_rs_prepare): EA.re / 2, (0 - EA.im) / 2, RT, RA, RF */
+  const double *poles;
   const int32_t *pole_l;    /* [n_poles] l value in [0, numL) */
   const double *windows;    /* [n_windows][4] T A F 0, 32 B aligned */
   const int32_t *win_range; /* [n_windows][2] absolute pole [start, end) */
@@ -338,9 +340,19 @@ typedef struct {
   const int32_t *num_nucs;  /* [12] */
   const int32_t *mats;      /* [12][max_num_nucs] */
   const double *concs;      /* [12][max_num_nucs] */
-  int32_t n_nuclides, numL, max_num_nucs, pad;
+  int32_t n_nuclides, numL, max_num_nucs;
+  int32_t prepared; /* 1: `poles` holds the prepared form (set by omprt_rs_prepare) */
 } omprt_rs_tables;
-/* Same contract as omprt_xs_lookup (4 macroscopic cross sections; numL must be 4).
+/* Table preparation (like omprt_xs_build_accel; not part of a lookup): copies the n_poles
+ * records of t->poles into `prepared` (caller-owned device memory, n_poles * 8 doubles, 32 B
+ * aligned) with EA replaced by (EA.re / 2, (0 - EA.im) / 2) -- exact in IEEE arithmetic --
+ * and points t->poles at it, t->prepared = 1.  The lookup's Z = ((E - EA.re) / 2,
+ * (0 - EA.im) / 2) (App. A.2) is then E/2 - EA.re/2 and a load: the same bits (halving
+ * commutes with rounding), 3 fewer fp64 operations per pole.  OMPRT_E_INVAL on null
+ * pointers, a misaligned buffer or an already prepared table. */
+int omprt_rs_prepare(omprt_rs_tables *t, int64_t n_poles, double *prepared, void *stream);
+/* Same contract as omprt_xs_lookup (4 macroscopic cross sections; numL must be 4; the
+ * tables prepared by omprt_rs_prepare, else OMPRT_E_INVAL).
  * macro (nullable): [count][4] doubles for parity tests. */
 int omprt_rs_lookup(omprt_rs_tables t, uint64_t seed, int64_t first, int64_t count,
                     uint64_t *verification, double *macro, int32_t teams, int32_t threads,

@@ -194,7 +194,8 @@ OMPRT_REGISTER_KERNEL(cuda_rs_twin, cuda_rs_twin<false>)
 
 inline RSTables to_dev(const omprt_rs_tables& a) {
   return RSTables{a.poles, a.pole_l, a.windows, a.win_range, a.win_off, a.n_windows, a.k0rs,
-                  a.num_nucs, a.mats, a.concs, a.n_nuclides, a.numL, a.max_num_nucs, 0};
+                  a.num_nucs, a.mats, a.concs, a.n_nuclides, a.numL, a.max_num_nucs,
+                  a.prepared};
 }
 
 // Persistent grid of the flattened kernels: teams = 0 -> every SM's resident teams (of the
@@ -218,6 +219,7 @@ inline int rs_validate(const omprt_rs_tables& t, int64_t count, uint64_t* ver, i
   OMPRT_CHECK_ARG(count >= 0 && count < (1ll << 31), "count must be in [0, 2^31)");
   OMPRT_CHECK_ARG(threads == kRSThreads, "threads must be %d", kRSThreads);
   OMPRT_CHECK_ARG(t.numL == 4, "numL must be 4");
+  OMPRT_CHECK_ARG(t.prepared == 1, "RSBench tables not prepared (omprt_rs_prepare)");
   OMPRT_CHECK_ARG(t.poles && t.pole_l && t.windows && t.win_range && t.win_off && t.n_windows &&
                       t.k0rs && t.num_nucs && t.mats && t.concs,
                   "bad RSBench tables");
@@ -382,6 +384,37 @@ inline int su3_validate(const double* A, const double* B, double* Cm, int64_t n,
 }
 
 }  // namespace omprt_kernels
+
+namespace omprt_kernels {
+// the prepared pole records (omprt_rs_prepare): EA.re / 2, (0 - EA.im) / 2, RT, RA, RF
+__global__ void rs_prepare_poles(const double* __restrict__ in, double* __restrict__ out,
+                                 int64_t n) {
+  for (int64_t p = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; p < n;
+       p += (int64_t)gridDim.x * blockDim.x) {
+    const double* r = in + p * 8;
+    double* o = out + p * 8;
+    o[0] = __dmul_rn(r[0], 0.5);
+    o[1] = __dmul_rn(__dsub_rn(0.0, r[1]), 0.5);
+#pragma unroll
+    for (int k = 2; k < 8; ++k) o[k] = r[k];
+  }
+}
+}  // namespace omprt_kernels
+
+extern "C" int omprt_rs_prepare(omprt_rs_tables* t, int64_t n_poles, double* prepared,
+                                void* stream) {
+  using namespace omprt_kernels;
+  Workspace* w;
+  if (int r = current_ws(&w)) return r;
+  OMPRT_CHECK_ARG(t && t->poles && prepared && n_poles > 0 && ((uintptr_t)prepared & 31) == 0,
+                  "omprt_rs_prepare: bad arguments");
+  OMPRT_CHECK_ARG(t->prepared == 0, "omprt_rs_prepare: the tables are already prepared");
+  rs_prepare_poles<<<1024, 256, 0, as_stream(stream)>>>(t->poles, prepared, n_poles);
+  if (int r = check_launch("rs_prepare_poles")) return r;
+  t->poles = prepared;
+  t->prepared = 1;
+  return OMPRT_OK;
+}
 
 extern "C" int omprt_rs_lookup(omprt_rs_tables t, uint64_t seed, int64_t first, int64_t count,
                                uint64_t* verification, double* macro, int32_t teams,

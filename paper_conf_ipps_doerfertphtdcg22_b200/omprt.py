@@ -52,7 +52,7 @@ EXPORTS = [
     "omprt_xs_run_host", "omprt_xs_run_host_steps", "omprt_xs_accel_sizes", "omprt_xs_build_accel",
     "omprt_xs_derive_tmp_bytes", "omprt_xs_derive", "omprt_rs_lookup", "omprt_cuda_rs_lookup", "omprt_su3_mult",
     "omprt_cuda_su3_mult", "omprt_kernel_count", "omprt_kernel_name", "omprt_kernel_attrs",
-    "omprt_probe_l2_read", "omprt_probe_fp64_fma", "omprt_kernel_occupancy",
+    "omprt_probe_l2_read", "omprt_probe_fp64_fma", "omprt_kernel_occupancy", "omprt_rs_prepare",
 ]
 
 
@@ -81,7 +81,7 @@ class RSTablesC(C.Structure):
                 ("win_range", C.c_void_p), ("win_off", C.c_void_p), ("n_windows", C.c_void_p),
                 ("k0rs", C.c_void_p), ("num_nucs", C.c_void_p), ("mats", C.c_void_p),
                 ("concs", C.c_void_p), ("n_nuclides", C.c_int32), ("numL", C.c_int32),
-                ("max_num_nucs", C.c_int32), ("pad", C.c_int32)]
+                ("max_num_nucs", C.c_int32), ("prepared", C.c_int32)]
 
 
 _lib = None
@@ -115,6 +115,7 @@ _SIGS = {
                           C.POINTER(_u64), C.POINTER(_u64), _vp],
     "omprt_xs_run_host_steps": [XSTablesC, _u64, _i64, _i64, _i32, _u32, _i32, C.POINTER(_u64),
                                 C.POINTER(_u64), C.POINTER(_u64), _vp],
+    "omprt_rs_prepare": [C.POINTER(RSTablesC), _i64, _vp, _vp],
     "omprt_rs_lookup": [RSTablesC, _u64, _i64, _i64, _vp, _vp, _i32, _i32, _u32, _vp],
     "omprt_cuda_rs_lookup": [RSTablesC, _u64, _i64, _i64, _vp, _vp, _i32, _i32, _u32, _vp],
     "omprt_su3_mult": [_vp, _vp, _vp, _i64, _vp, _i32, _i32, _u32, _vp],
@@ -449,6 +450,15 @@ class RSDeviceTables:
                                                    "win_off", "n_windows", "k0rs", "num_nucs",
                                                    "mats", "concs")],
                            t.n_nuclides, t.numL, t.max_num_nucs, 0)
+        # the lookups' prepared pole records (omprt_rs_prepare, on the device)
+        self.poles_prepared = torch.empty_like(self.poles)
+        omprt_rs_prepare(self, self.poles.shape[0], self.poles_prepared)
+
+
+def omprt_rs_prepare(tables, n_poles, prepared, stream=None):
+    return _check(load().omprt_rs_prepare(C.byref(tables.c), n_poles,
+                                          _p(prepared, _T().float64, 8 * n_poles),
+                                          _stream(stream)))
 
 
 def omprt_rs_lookup(tables, seed, first, count, verification, macro=None, teams=0, threads=128,

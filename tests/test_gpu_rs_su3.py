@@ -210,3 +210,25 @@ def test_su3_pins_on_gpu(rt):
     A, B = gen.su3_inputs(n, "third")
     C, ck = _su3(rt, rt.omprt_su3_mult, A, B, n, rt.OMPRT_ASSUME_OVERSUB)
     assert (C.reshape(n, 4, 3, 3, 2)[..., 0] == 1.0).all() and ck == 36.0 * n
+
+
+def test_rs_prepare_pole_records(rt, rs_tables_small):
+    """omprt_rs_prepare: EA.re / 2 and (0 - EA.im) / 2, the rest of each record unchanged --
+    exactly the values numpy's IEEE arithmetic gives -- and an unprepared or twice-prepared
+    table is rejected."""
+    d = rt.RSDeviceTables(rs_tables_small, DEV)
+    got = d.poles_prepared.cpu().numpy().reshape(-1, 8)
+    P = rs_tables_small.poles.reshape(-1, 8)
+    exp = P.copy()
+    exp[:, 0] = P[:, 0] * 0.5
+    exp[:, 1] = (0.0 - P[:, 1]) * 0.5
+    assert (got.view(np.uint64) == exp.view(np.uint64)).all()
+    assert d.c.prepared == 1
+    with pytest.raises(rt.OmprtError):
+        rt.omprt_rs_prepare(d, P.shape[0], d.poles_prepared)
+    raw = rt.RSTablesC.from_buffer_copy(d.c)
+    raw.prepared = 0
+    d.c = raw
+    v = torch.zeros(16, dtype=torch.uint64, device=DEV)
+    with pytest.raises(rt.OmprtError):
+        rt.omprt_rs_lookup(d, 1, 0, 16, v)

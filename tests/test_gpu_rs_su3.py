@@ -232,3 +232,18 @@ def test_rs_prepare_pole_records(rt, rs_tables_small):
     v = torch.zeros(16, dtype=torch.uint64, device=DEV)
     with pytest.raises(rt.OmprtError):
         rt.omprt_rs_lookup(d, 1, 0, 16, v)
+
+
+def test_rs_sigt_factor_angles_beyond_the_series_range(rt, rs_tables_small):
+    """The sigT factors outside the workload's angle range (k0rs scaled by 3: angles 2 k0rs
+    sqrt(E) up to 6, past the first quadrant boundaries of the rational-rotation form,
+    R-A10) still match the oracle within the C7 contract."""
+    import copy
+    t = copy.copy(rs_tables_small)
+    t.k0rs = rs_tables_small.k0rs * 3.0
+    d = rt.RSDeviceTables(t, DEV)
+    first, count = 11, 5_000
+    ver, mac = _rs(rt, d, first, count, "rt", rt.OMPRT_FLAT | rt.OMPRT_SCHED_DYNAMIC)
+    rv, rm = oracle.rs_lookup(t, first, count, want_macro=True, threads=os.cpu_count() or 1)
+    err = np.abs(mac - rm).max(axis=1) / np.abs(rm).max(axis=1)
+    assert err.max() <= 1e-10, err.max()

@@ -457,8 +457,7 @@ def run_omprt(args):
                                   "steps)"},
             "roofline": {"bound": "l2", "achieved": achieved, "peak": l2_peak, "unit": "GB/s",
                          "frac": achieved / l2_peak,
-                         "traffic": load_ncu_traffic("omprt_xs_flat_rt_timed") or
-                         load_ncu_traffic("omprt_xs_flat_rt"),
+                         "traffic": load_ncu_traffic("omprt_xs_flat_rt_timed"),
                          "kernel": "omprt_xs_flat_rt", "alg_bytes_per_launch": alg,
                          "peak_source": "measured live in this run: L2 -> SM streaming read of "
                                         "16 / 40 MB L2-resident buffers with the kernel's "
@@ -478,7 +477,7 @@ def run_omprt(args):
                                  "note": "algorithmic bytes against the HBM copy peak: above "
                                          "1 because most of them are L2 hits"},
                          "measured_roofs": peaks,
-                         "l2": l2_roof("omprt_xs_flat_rt", kms["rt_flat"]),
+                         "l2": l2_roof("omprt_xs_flat_rt_timed", kms["rt_flat"]),
                          "one_lookup_per_thread": {
                              "kernel": "omprt_xs_rt_assume_accel",
                              "achieved": alg / kms["rt_assume"] / 1e6,

@@ -16,6 +16,8 @@ timeout 900 python bench.py --steps 10 --warmup 3 > $OUT/bench_$TAG.txt 2>&1
 echo "bench exit $?" >> $OUT/bench_$TAG.txt
 timeout 300 python bench.py --impl reference --steps 2 --warmup 1 > $OUT/bench_ref_$TAG.txt 2>&1
 timeout 300 python scripts/peaks_probe.py > $OUT/peaks_$TAG.txt 2>&1
+timeout 900 python -m torch.distributed.run --nnodes=1 --nproc-per-node 2 --master-addr 127.0.0.1 \
+  --master-port 29533 bench.py --gpus 2 --steps 3 --warmup 3 > $OUT/bench_2rank_sharedgpu_$TAG.txt 2>&1
 timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none -c 400 --csv \
   --log-file $OUT/launches_$TAG.csv python bench.py --steps 2 --warmup 1 --no-e2e --no-secondary > $OUT/ncu_launch_stdout_$TAG.txt 2>&1
 for K in omprt_xs_flat_rt cuda_xs_flat_twin omprt_xs_rt; do

@@ -16,9 +16,10 @@ struct RSTraitsAssume : DefaultTraits {
 };
 constexpr int kRSThreads = 128;
 static_assert(kRSThreads == kRSBodyThreads, "rs_nuclide's shared-memory slots");
-// 5 teams of 128 per SM (<= 96 registers): 10 % faster than the unconstrained 122-register
-// build (scripts/experiments/rs_explore, profiles/rs_explore_x05.txt)
-constexpr int kRSMinBlocks = 5;
+// 4 teams of 128 per SM (<= 128 registers, no spills): the round-1 choice of 5 (96
+// registers) was 10 % faster for the round-1 body; with the round-2 body it spilled 120-216 B
+// per thread and ran no faster (185.3 ms at 4 vs 186.2 ms at 5 per SM, 10M lookups).
+constexpr int kRSMinBlocks = 4;
 // The flattened kernels: 4 teams of 128 per SM (<= 128 registers, no spills).  With the
 // prefetched pole loop (and, queued, the Abrarov drain) in one loop body the 96-register
 // budget of 5 teams spills inside the pole loop: queued 106 ms vs 77.8 ms, dynamic 82.8 vs

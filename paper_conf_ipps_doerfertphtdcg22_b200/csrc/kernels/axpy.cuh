@@ -27,41 +27,70 @@ struct AxpyTraitsDebug : AxpyTraits {
 struct AxpyTraitsAssumeDebug : AxpyTraitsAssume {
   static constexpr unsigned debug = dbg::Assert | dbg::Trace;
 };
+// Teams of <= 256 threads (C1: 8 x 128): 32 iterations per trip.  The config runs on 8 SMs
+// with 4 warps each; its HBM reads are latency-bound by the bytes each SM keeps in flight
+// (8 iterations: 4 warps x 16 loads x 256 B = 16 KB per SM, ~240 GB/s over the 8 SMs).  At
+// 32 iterations a trip issues its 64 loads before the first store (the runtime kernel
+// through distribute_parallel_for_split, the twin by hand) in a 255-register budget, which
+// 256 threads per team still fit: 0.104 -> 0.059 ms at 2^20, runtime within 3 % of the
+// twin.  64 iterations ran the twin at 0.048 ms but the runtime kernel at 0.053-0.055 ms
+// for every budget tried (200-255): under the extra register pressure ptxas moves some of
+// its stores ahead of the last loads (scripts/experiments/c1_prefetch.cu,
+// profiles/c1_wide_r2.txt).  Same Fig. 5 assignment, same per-thread order: a[] and the
+// sum keep their bits.
+#ifndef OMPRT_AXPY_WIDE_UNROLL  // exploration builds only
+#define OMPRT_AXPY_WIDE_UNROLL 32
+#define OMPRT_AXPY_WIDE_REGS 255
+#endif
+constexpr unsigned kAxpyWideUnroll = OMPRT_AXPY_WIDE_UNROLL;
+constexpr int kAxpyWideMaxThreads = 256;
+struct AxpyTraitsWide : AxpyTraits {
+  static constexpr unsigned unroll = kAxpyWideUnroll;
+};
+struct AxpyTraitsWideDebug : AxpyTraitsWide {
+  static constexpr unsigned debug = dbg::Assert | dbg::Trace;
+};
+
 // Both C1 kernels carry the same register budget, __maxnreg__(58) (1024 threads still fit
 // an SM).  Under __launch_bounds__(1024) ptxas held them to 32 registers and interleaved the
 // unrolled trip's loads with its stores (2-4 loads in flight per thread); with a budget of
-// their own both issue all 16 loads of a trip first -- what 4 warps per SM (C1: 8 teams x
-// 128) need: 0.30 -> 0.104 ms.  At a budget of 56 the runtime kernel (56 registers: it
-// keeps the trip's 8 indices for the stores where the twin advances pointers) lost that
-// schedule and ran 33 % slower; at 58 both run 0.104 ms (scripts/experiments/
-// c1_lib_kernels.cu, profiles/c1_budget_r2.txt).
+// their own both issue all 16 loads of a trip first -- what 4 warps per SM need: 0.30 ->
+// 0.104 ms at 8 x 128 (scripts/experiments/c1_lib_kernels.cu, profiles/c1_budget_r2.txt).
+// The runtime kernel's body is split into its loads and the rest
+// (distribute_parallel_for_split), so its trip has the twin's shape and register count (50).
 // Runtime-driven kernel: the OpenMP region as the runtime executes it.
 constexpr int kAxpyMaxRegs = 58;
+// the budget of a C1 kernel unrolled U times: 58 at U = 8, all 255 for the wide trips
+constexpr int axpy_max_regs(unsigned U) { return U > 8 ? OMPRT_AXPY_WIDE_REGS : kAxpyMaxRegs; }
 template <class Tr, bool Rec>
-__global__ void __maxnreg__(kAxpyMaxRegs)
+__global__ void __maxnreg__(axpy_max_regs(Tr::unroll))
     omprt_axpy_rt(typename Tr::Idx n, double x, const double* __restrict__ b,
                   const double* __restrict__ c, double* __restrict__ a, double* sum_inout,
                   double* partials, unsigned* ticket, int32_t* owner, int32_t* count) {
   using Idx = typename Tr::Idx;
   Team<Tr> team = init<Tr>();
   double acc = 0.0;  // private copy, identity of +
-  distribute_parallel_for(team, n, [&](Idx i) {
-    const double v = fma(x, __ldg(b + i), __ldg(c + i));
-    a[i] = v;
-    acc += v;
-    if constexpr (Rec) {
-      owner[i] = get_team_num(team) * get_num_threads(team) + get_thread_num(team);
-      atomicAdd(count + i, 1);
-    }
-  });
+  // the body split into its loads and the rest (b and c are read-only in the loop), so the
+  // runtime issues a trip's loads together (distribute_parallel_for_split)
+  distribute_parallel_for_split(
+      team, n, [&](Idx i) { return double2{__ldg(b + i), __ldg(c + i)}; },
+      [&](Idx i, double2 bc) {
+        const double v = fma(x, bc.x, bc.y);
+        a[i] = v;
+        acc += v;
+        if constexpr (Rec) {
+          owner[i] = get_team_num(team) * get_num_threads(team) + get_thread_num(team);
+          atomicAdd(count + i, 1);
+        }
+      });
   league_reduce_threads(team, acc, Plus{}, sum_inout, partials,
                 ticket);
 }
 
 // Bare CUDA twin: grid-stride loop (the same cyclic assignment) and a hand-written copy of
 // the same reduction algorithm (shfl.xor butterfly, warp partials, last-block combine).
-template <class Idx, bool Rec>
-__global__ void __maxnreg__(kAxpyMaxRegs)
+template <class Idx, bool Rec, int U = 8>
+__global__ void __maxnreg__(axpy_max_regs(U))
     cuda_axpy_twin(Idx n, double x, const double* __restrict__ b, const double* __restrict__ c,
                    double* __restrict__ a, double* sum_inout, double* partials,
                    unsigned* ticket, int32_t* owner, int32_t* count) {
@@ -69,17 +98,17 @@ __global__ void __maxnreg__(kAxpyMaxRegs)
   const Idx gtid = (Idx)blockIdx.x * blockDim.x + threadIdx.x;
   double acc = 0.0;
   Idx i = gtid;
-  // 8 iterations per trip, all 16 loads issued before the first store (what a CUDA
+  // U iterations per trip, all 2U loads issued before the first store (what a CUDA
   // programmer writes to keep loads in flight with 4 warps per SM)
-  for (; i + 7 * stride < n; i += 8 * stride) {
-    double bv[8], cv[8];
+  for (; i + (U - 1) * stride < n; i += U * stride) {
+    double bv[U], cv[U];
 #pragma unroll
-    for (int u = 0; u < 8; ++u) {
+    for (int u = 0; u < U; ++u) {
       bv[u] = __ldg(b + i + u * stride);
       cv[u] = __ldg(c + i + u * stride);
     }
 #pragma unroll
-    for (int u = 0; u < 8; ++u) {
+    for (int u = 0; u < U; ++u) {
       const double v = fma(x, bv[u], cv[u]);
       a[i + u * stride] = v;
       acc += v;
@@ -89,6 +118,7 @@ __global__ void __maxnreg__(kAxpyMaxRegs)
       }
     }
   }
+#pragma unroll 1
   for (; i < n; i += stride) {
     const double v = fma(x, __ldg(b + i), __ldg(c + i));
     a[i] = v;
@@ -378,6 +408,9 @@ OMPRT_REGISTER_KERNEL(omprt_axpy_rt, omprt_axpy_rt<AxpyTraits, false>)
 OMPRT_REGISTER_KERNEL(omprt_axpy_rt_assume, omprt_axpy_rt<AxpyTraitsAssume, false>)
 OMPRT_REGISTER_KERNEL(omprt_axpy_rt_debug, omprt_axpy_rt<AxpyTraitsDebug, false>)
 OMPRT_REGISTER_KERNEL(cuda_axpy_twin, cuda_axpy_twin<int32_t, false>)
+OMPRT_REGISTER_KERNEL(omprt_axpy_rt_wide, omprt_axpy_rt<AxpyTraitsWide, false>)
+OMPRT_REGISTER_KERNEL(omprt_axpy_rt_wide_debug, omprt_axpy_rt<AxpyTraitsWideDebug, false>)
+OMPRT_REGISTER_KERNEL(cuda_axpy_twin_wide, cuda_axpy_twin<int32_t, false, kAxpyWideUnroll>)
 
 template <class Tr, class Idx>
 int launch_axpy_rt(int64_t n, double x, const double* b, const double* c, double* a,
@@ -393,6 +426,13 @@ int launch_axpy_rt(int64_t n, double x, const double* b, const double* c, double
                                                        (double*)w->partials, w->tickets + 0,
                                                        nullptr, nullptr);
   return check_launch("omprt_axpy_rt");
+}
+
+// the 64-iteration trips: teams of <= 256 threads (the 255-register budget), no
+// oversubscription assumption (no loop then), 32-bit induction variable
+inline bool axpy_wide(int64_t n, int32_t teams, int32_t threads, uint32_t flags) {
+  return threads <= kAxpyWideMaxThreads && !(flags & OMPRT_ASSUME_OVERSUB) &&
+         n + (int64_t)(kAxpyWideUnroll + 1) * teams * threads < INT32_MAX;
 }
 
 inline int axpy_validate(int64_t n, const double* b, const double* c, double* a, double* sum,
@@ -432,6 +472,13 @@ extern "C" int omprt_spmd_axpy_sum(int64_t n, double x, const double* b, const d
     return launch_axpy_tma(false, n, x, b, c, a, sum_inout, teams, threads, owner, count, w, s);
   }
   const bool assume = flags & OMPRT_ASSUME_OVERSUB, debug = flags & OMPRT_DEBUG_BUILD;
+  // trait selection: teams of <= 256 threads take the 64-iteration trips (the twin does
+  // the same, axpy_wide())
+  if (axpy_wide(n, teams, threads, flags))
+    return debug ? launch_axpy_rt<AxpyTraitsWideDebug, int32_t>(n, x, b, c, a, sum_inout, teams,
+                                                               threads, owner, count, w, s)
+                 : launch_axpy_rt<AxpyTraitsWide, int32_t>(n, x, b, c, a, sum_inout, teams,
+                                                          threads, owner, count, w, s);
   // 32-bit induction variable when n + (unroll+1)*T*N fits
   const bool i32 = n + 9 * (int64_t)teams * threads < INT32_MAX;
   if (i32) {
@@ -468,6 +515,15 @@ extern "C" int omprt_cuda_axpy_sum(int64_t n, double x, const double* b, const d
   const bool i32 = n + 9 * (int64_t)teams * threads < INT32_MAX;
   double* p = (double*)w->partials;
   unsigned* t = w->tickets + 0;
+  if (axpy_wide(n, teams, threads, flags)) {
+    if (rec)
+      cuda_axpy_twin<int32_t, true, kAxpyWideUnroll><<<teams, threads, 0, s>>>(
+          (int32_t)n, x, b, c, a, sum_inout, p, t, owner, count);
+    else
+      cuda_axpy_twin<int32_t, false, kAxpyWideUnroll><<<teams, threads, 0, s>>>(
+          (int32_t)n, x, b, c, a, sum_inout, p, t, nullptr, nullptr);
+    return check_launch("cuda_axpy_twin");
+  }
   if (i32) {
     if (rec)
       cuda_axpy_twin<int32_t, true><<<teams, threads, 0, s>>>((int32_t)n, x, b, c, a, sum_inout,

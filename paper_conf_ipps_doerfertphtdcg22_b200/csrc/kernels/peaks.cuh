@@ -6,12 +6,17 @@
 //     random 32 B sectors / random 96 B records (3 adjacent sectors: the bracket record of a
 //     lookup's nuclide) -- the access pattern that bounds C3;
 //   * FP64 FMA throughput: 8 independent DFMA chains per thread on a full-device grid, the
-//     roof of the RSBench lookup ("compute bound").
+//     roof of the RSBench lookup ("compute bound");
+//   * HBM -> SM streaming read bandwidth of a given number of SMs: one team per SM moving
+//     its contiguous slice of a buffer larger than L2 by bulk copies (cp.async.bulk, 16 KB
+//     each, 8 in flight) into shared memory -- the most an SM can pull from HBM, the roof of
+//     a config that by definition runs on few SMs (C1: 8 teams).
 // Each probe folds what it reads into a value written to `sink` only under a condition that
 // never holds, so no load or fma can be removed.
 #pragma once
 #include <cstdint>
 
+#include "../common/ptx_tma.cuh"
 #include "../host/runtime.cuh"
 #include "vec.cuh"
 
@@ -109,6 +114,39 @@ __global__ void __launch_bounds__(kProbeThreads) probe_fp64_fma(int64_t iters, d
   if (acc == -1.2345e300) *sink = acc;
 }
 
+// HBM stream probe: team b reads bytes [b * slice, (b + 1) * slice) in kHbmChunk pieces,
+// kHbmStages bulk copies in flight on as many mbarriers (one issuing thread).
+constexpr uint32_t kHbmChunk = 16384;
+constexpr int kHbmStages = 8;
+__global__ void __launch_bounds__(32, 1)
+    probe_hbm_stream(const unsigned char* __restrict__ buf, int64_t slice, double* sink) {
+  extern __shared__ __align__(128) unsigned char ring[];
+  __shared__ uint64_t bars[kHbmStages];
+  namespace tma = omprt::tma;
+  if (threadIdx.x != 0) return;
+  for (int k = 0; k < kHbmStages; ++k) tma::mbar_init(&bars[k], 1);
+  tma::fence_mbar_init();
+  const unsigned char* src = buf + (int64_t)blockIdx.x * slice;
+  const int64_t chunks = slice / kHbmChunk;
+  uint32_t phase = 0;
+  for (int64_t c = 0; c < chunks; ++c) {
+    const int k = (int)(c % kHbmStages);
+    if (c >= kHbmStages) {  // the stage's previous copy has landed
+      tma::mbar_wait(&bars[k], phase >> k & 1u);
+      phase ^= 1u << k;
+    }
+    tma::mbar_arrive_expect_tx(&bars[k], kHbmChunk);
+    tma::bulk_load(ring + (size_t)k * kHbmChunk, src + c * kHbmChunk, kHbmChunk, &bars[k]);
+  }
+  for (int64_t c = chunks > kHbmStages ? chunks - kHbmStages : 0; c < chunks; ++c) {
+    const int k = (int)(c % kHbmStages);
+    tma::mbar_wait(&bars[k], phase >> k & 1u);
+    phase ^= 1u << k;
+  }
+  const double v = *reinterpret_cast<const double*>(ring);
+  if (v == -1.2345e300) *sink = v;
+}
+
 }  // namespace omprt_kernels
 
 // bytes: size of the L2-resident buffer (>= 96, 32 B aligned); reps: passes (mode 0) or
@@ -144,4 +182,24 @@ extern "C" int omprt_probe_fp64_fma(int64_t iters, int32_t teams, double* sink, 
   if (teams <= 0) teams = 8 * sms;
   probe_fp64_fma<<<teams, kProbeThreads, 0, as_stream(stream)>>>(iters, 1.0, sink);
   return check_launch("probe_fp64_fma");
+}
+
+// bytes read = teams * slice, slice = (bytes / teams) rounded down to 16 KB; one team of 32
+// threads per SM (teams <= the SM count), 128 KB of dynamic shared memory each.  Use a
+// buffer larger than L2 (126 MB) so the reads come from HBM.
+extern "C" int omprt_probe_hbm_stream(const void* buf, uint64_t bytes, int32_t teams, double* sink,
+                                      void* stream) {
+  using namespace omprt_kernels;
+  int dev = 0, sms = 148;
+  cudaGetDevice(&dev);
+  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  const int64_t slice = teams > 0 ? (int64_t)(bytes / (uint64_t)teams) / kHbmChunk * kHbmChunk : 0;
+  OMPRT_CHECK_ARG(buf && sink && ((uintptr_t)buf & 15) == 0 && teams > 0 && teams <= sms &&
+                      slice >= (int64_t)kHbmChunk,
+                  "omprt_probe_hbm_stream: bad arguments");
+  const int smem = (int)kHbmChunk * kHbmStages;
+  cudaFuncSetAttribute(probe_hbm_stream, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+  probe_hbm_stream<<<teams, 32, smem, as_stream(stream)>>>(
+      static_cast<const unsigned char*>(buf), slice, sink);
+  return check_launch("probe_hbm_stream");
 }

@@ -52,7 +52,7 @@ EXPORTS = [
     "omprt_xs_run_host", "omprt_xs_run_host_steps", "omprt_xs_accel_sizes", "omprt_xs_build_accel",
     "omprt_xs_derive_tmp_bytes", "omprt_xs_derive", "omprt_rs_lookup", "omprt_cuda_rs_lookup", "omprt_su3_mult",
     "omprt_cuda_su3_mult", "omprt_kernel_count", "omprt_kernel_name", "omprt_kernel_attrs",
-    "omprt_probe_l2_read", "omprt_probe_fp64_fma", "omprt_kernel_occupancy", "omprt_rs_prepare",
+    "omprt_probe_l2_read", "omprt_probe_fp64_fma", "omprt_probe_hbm_stream", "omprt_kernel_occupancy", "omprt_rs_prepare",
 ]
 
 
@@ -122,6 +122,7 @@ _SIGS = {
     "omprt_cuda_su3_mult": [_vp, _vp, _vp, _i64, _vp, _i32, _i32, _u32, _vp],
     "omprt_probe_l2_read": [_vp, _u64, _i32, _i32, _i32, _i32, _vp, _vp],
     "omprt_probe_fp64_fma": [_i64, _i32, _vp, _vp],
+    "omprt_probe_hbm_stream": [_vp, _u64, _i32, _vp, _vp],
     "omprt_kernel_count": [],
     "omprt_kernel_occupancy": [C.c_int, C.c_int, C.c_int, C.POINTER(C.c_int)],
     "omprt_kernel_name": [C.c_int],
@@ -506,6 +507,12 @@ def omprt_probe_l2_read(buf, nbytes, mode, reps, per_thread, sink, teams=0, stre
 def omprt_probe_fp64_fma(iters, sink, teams=0, stream=None):
     return _check(load().omprt_probe_fp64_fma(iters, teams, _p(sink, _T().float64, 1),
                                               _stream(stream)))
+
+
+def omprt_probe_hbm_stream(buf, nbytes, teams, sink, stream=None):
+    """Bytes read: teams * (nbytes // teams rounded down to 16 KB)."""
+    return _check(load().omprt_probe_hbm_stream(_p(buf, None, nbytes // buf.element_size()), nbytes, teams,
+                                                _p(sink, _T().float64, 1), _stream(stream)))
 
 
 # ---------------------------------------------------------------- introspection

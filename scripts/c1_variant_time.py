@@ -35,6 +35,10 @@ def one(path):
     tw1 = lambda: omprt.omprt_cuda_axpy_sum(n, x, bt, ct, at, sm, 8, 128)
     t_rt, t_tw = bench._time_pair(rt1, tw1, s, scrub)
     g_rt, g_tw = bench._time_graph(rt1, tw1, s)
+    # teams of 512 threads: the 8-iteration trips (the wide ones need <= 256)
+    n_rt, n_tw = bench._time_pair(lambda: omprt.omprt_spmd_axpy_sum(n, x, bt, ct, at, sm, 8, 512),
+                                  lambda: omprt.omprt_cuda_axpy_sum(n, x, bt, ct, at, sm, 8, 512),
+                                  s, scrub)
     sm.zero_()
     rt1()
     torch.cuda.synchronize()
@@ -42,6 +46,7 @@ def one(path):
     tab = omprt.kernel_table()
     print(json.dumps({"lib": path, "rt_ms": t_rt, "twin_ms": t_tw, "graph_rt_ms": g_rt,
                       "graph_twin_ms": g_tw, "a_bit_exact": ok,
+                      "x512_rt_ms": n_rt, "x512_twin_ms": n_tw,
                       "regs": [tab["omprt_axpy_rt"]["regs"], tab["cuda_axpy_twin"]["regs"]]}),
           flush=True)
 

@@ -18,6 +18,10 @@ def test_roof_probes_plausible(rt):
     assert 2000 < p["l2_record96_gbs"] <= p["l2_stream_gbs"] * 1.05, p
     # FP64 FMA: B200 nominal ~37-40 TFLOP/s
     assert 20000 < p["fp64_fma_gflops"] < 45000, p
+    # HBM -> SM by bulk copies: all SMs near the HBM peak (~7.7 TB/s nominal), 8 SMs a
+    # fraction of it
+    assert 4000 < p["hbm_stream_gbs"] < 8500, p
+    assert 100 < p["hbm_stream_8sm_gbs"] < p["hbm_stream_gbs"] * 0.5, p
 
 
 def test_probe_arguments_rejected(rt):
@@ -29,6 +33,13 @@ def test_probe_arguments_rejected(rt):
         rt.omprt_probe_l2_read(buf, 8192, 1, 1, 7, sink)      # per_thread % 8
     with pytest.raises(rt.OmprtError):
         rt.omprt_probe_fp64_fma(0, sink)
+    big = torch.ones(1 << 16, dtype=torch.float64, device=DEV)
+    with pytest.raises(rt.OmprtError):
+        rt.omprt_probe_hbm_stream(big, big.numel() * 8, 0, sink)       # no teams
+    with pytest.raises(rt.OmprtError):
+        rt.omprt_probe_hbm_stream(big, big.numel() * 8, 1000, sink)    # more teams than SMs
+    with pytest.raises(rt.OmprtError):
+        rt.omprt_probe_hbm_stream(big, 8192, 1, sink)                  # slice < 16 KB
 
 
 def test_occupancy_query(rt):

@@ -1,5 +1,5 @@
 """Launch one config's runtime kernel and twin a few times (for ncu captures).
-  python scripts/run_kernels.py rs|rs1m|su3|generic|axpy|xs [reps]"""
+  python scripts/run_kernels.py rs|rs1m|rs10m|su3|generic|axpy|xs [reps]"""
 import os, sys
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 sys.path.insert(0, ROOT)
@@ -31,6 +31,12 @@ elif which == "rs1m":  # nested and flattened, 1M lookups
         Q = omprt.OMPRT_FLAT | omprt.OMPRT_SCHED_DYNAMIC | omprt.OMPRT_RS_QUEUE
         omprt.omprt_rs_lookup(d, 1070, 0, n, v, None, 0, 128, Q)
         omprt.omprt_cuda_rs_lookup(d, 1070, 0, n, v, None, 0, 128, Q)
+elif which == "rs10m":  # the bench's C4 launch (queued, dynamic, flattened), 10M lookups
+    t = gen.RSTables(); d = omprt.RSDeviceTables(t, dev); n = 10_000_000
+    v = torch.empty(n, dtype=torch.uint64, device=dev)
+    Q = omprt.OMPRT_FLAT | omprt.OMPRT_SCHED_DYNAMIC | omprt.OMPRT_RS_QUEUE
+    for _ in range(reps):
+        omprt.omprt_rs_lookup(d, 1070, 0, n, v, None, 0, 128, Q)
 elif which == "su3":
     ns = 32 ** 4; Ah, Bh = gen.su3_inputs(ns)
     At, Bt = torch.from_numpy(Ah).to(dev), torch.from_numpy(Bh).to(dev); Ct = torch.empty_like(At)

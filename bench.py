@@ -800,6 +800,14 @@ def run_secondary(omprt, torch, gen, dev, stream, scrub, peaks):
         "roofline": c1_roof(24 * n / t_rt / 1e6),
         "occupancy_teams_per_sm": [occ("omprt_axpy_rt", 128), occ("cuda_axpy_twin", 128)],
         "note": "8 teams of 128 run on 8 of the 148 SMs by the config's definition"})
+    # a labelled full-device geometry as a secondary point (4 teams per SM)
+    tf = 4 * torch.cuda.get_device_properties(dev).multi_processor_count
+    e = _short_pair(lambda: omprt.omprt_spmd_axpy_sum(n, x, bt, ct, at, s, tf, 128),
+                    lambda: omprt.omprt_cuda_axpy_sum(n, x, bt, ct, at, s, tf, 128), stream, scrub)
+    e.update({"geometry": [tf, 128], "GBps_alg": 24 * n / e["rt_ms"] / 1e6,
+              "roofline": _roof("hbm", 24 * n / e["rt_ms"] / 1e6, hbm, "GB/s",
+                                "24 B/iteration, cold; a 25 MB launch: latency-dominated")})
+    res["c1_axpy_sum_full_device"] = e
     # the same loop, operands streamed by 2-D TMA boxes (Fig. 5 assignment kept)
     TS_ = omprt.OMPRT_TMA_STREAM
     rt1t = lambda: omprt.omprt_spmd_axpy_sum(n, x, bt, ct, at, s, 8, 128, TS_)

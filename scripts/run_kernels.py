@@ -37,6 +37,7 @@ elif which == "rs10m":  # the bench's C4 launch (queued, dynamic, flattened), 10
     Q = omprt.OMPRT_FLAT | omprt.OMPRT_SCHED_DYNAMIC | omprt.OMPRT_RS_QUEUE
     for _ in range(reps):
         omprt.omprt_rs_lookup(d, 1070, 0, n, v, None, 0, 128, Q)
+        omprt.omprt_cuda_rs_lookup(d, 1070, 0, n, v, None, 0, 128, Q)
 elif which == "su3":
     ns = 32 ** 4; Ah, Bh = gen.su3_inputs(ns)
     At, Bt = torch.from_numpy(Ah).to(dev), torch.from_numpy(Bh).to(dev); Ct = torch.empty_like(At)

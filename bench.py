@@ -798,7 +798,10 @@ def run_secondary(omprt, torch, gen, dev, stream, scrub, peaks):
     res["c1_axpy_sum_8x128"].update({
         "GBps_alg": 24 * n / t_rt / 1e6,
         "roofline": c1_roof(24 * n / t_rt / 1e6),
-        "occupancy_teams_per_sm": [occ("omprt_axpy_rt", 128), occ("cuda_axpy_twin", 128)],
+        "occupancy_teams_per_sm": [occ("omprt_axpy_rt_wide", 128), occ("cuda_axpy_twin_wide", 128)],
+        "regs": [omprt.kernel_table()[k]["regs"] for k in ("omprt_axpy_rt_wide",
+                                                             "cuda_axpy_twin_wide")],
+        "variant": "32 iterations per trip (teams of <= 256 threads), loads of a trip issued first",
         "note": "8 teams of 128 run on 8 of the 148 SMs by the config's definition"})
     # a labelled full-device geometry as a secondary point (4 teams per SM)
     tf = 4 * torch.cuda.get_device_properties(dev).multi_processor_count

@@ -484,7 +484,8 @@ def run_omprt(args):
                          "note": "the lookups' hot tables (unionized grid, bins, bracket "
                                  "records: 44 MB) are L2-resident in an access-policy window "
                                  "and the 16-bit index grid partly so, so the binding roof is "
-                                 "the L2 -> SM path, not HBM (ncu: L1 75 %, L2 69 % busy); "
+                                 "the L2 -> SM path, not HBM (ncu of the timed launch: `l2.frac_ncu`, "
+                                 "`l2.l1tex_frac_ncu`); "
                                  "`pattern_roof` is the same path for random 96 B records, "
                                  "the bracket-record access pattern",
                          "pattern_roof": {"peak": peaks["l2_record96_gbs"],

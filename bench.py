@@ -386,7 +386,7 @@ def run_omprt(args):
     if not args.no_e2e:
         # per step: H2D of the raw problem data only (pinned nuclide grids + materials,
         # 36.9 MB) -> unionized grid, 16-bit index grid, bins and bracket records derived
-        # on the device -> flattened lookups with the fused checksum -> D2H of the 8 B
+        # on the device -> flattened lookups + the K11 checksum sum -> D2H of the 8 B
         # checksum; steps pipelined (H2D of step s+1 under step s's kernels)
         raw = {k: torch.from_numpy(getattr(tabs, k)).pin_memory()
                for k in ("nuclide_grid", "num_nucs", "mats", "concs")}
@@ -427,7 +427,8 @@ def run_omprt(args):
                "path": "omprt_xs_run_host_steps (pinned host nuclide grids + materials; "
                        "unionized grid, 16-bit index grid, bins and bracket records derived "
                        "on the device; H2D of step s+1 overlapped with step s; flattened "
-                       "lookups with the fused reduction; u64 checksum back)",
+                       "lookups, per-lookup verification summed by omprt_u64_sum_rt; u64 "
+                       "checksum back)",
                "upload_index16": {"ms_per_step": up_ms, "h2d_bytes_per_step": h2d16,
                                   "value": world * L / (up_ms / 1000.0)},
                "single_call_int32_index": {"ms": single_ms, "h2d_bytes": h2d1}}

@@ -209,15 +209,20 @@ def measure_peaks(omprt, torch, dev, stream, detail=False):
     ms = best(lambda: omprt.omprt_probe_fp64_fma(it, sink, fteams))
     res["fp64_fma_gflops"] = 16.0 * it * fteams * 256 / ms / 1e6
     # HBM -> SM streaming by bulk copies from a 1 GiB buffer (8x L2): all SMs, and the 8
-    # SMs C1's 8 teams run on (its roof: the config fixes the team count)
+    # SMs C1's 8 teams run on (its roof: the config fixes the team count), read-only and
+    # with C1's mix of 2 bytes read per byte written (mode 1)
     del buf
     big = torch.empty(1 << 30, dtype=torch.uint8, device=dev)
     big.fill_(1)
-    for key, tm in (("hbm_stream_gbs", sms), ("hbm_stream_8sm_gbs", 8)):
-        read = tm * ((big.numel() // tm) // 16384 * 16384)
-        ms = best(lambda: omprt.omprt_probe_hbm_stream(big, big.numel(), tm, sink), reps=5)
-        res[key] = read / ms / 1e6
-    del big
+    out = torch.empty(1 << 29, dtype=torch.uint8, device=dev)
+    for key, tm, mode in (("hbm_stream_gbs", sms, 0), ("hbm_stream_8sm_gbs", 8, 0),
+                          ("hbm_read2write1_8sm_gbs", 8, 1)):
+        read = tm * ((big.numel() // tm) // 32768 * 32768)
+        moved = read + (read // 2 if mode else 0)
+        ms = best(lambda: omprt.omprt_probe_hbm_stream(big, big.numel(), tm, sink, out, mode),
+                  reps=5)
+        res[key] = moved / ms / 1e6
+    del big, out
     if detail:  # capacity sweep of the stream roof
         sweep = {}
         for mb in (8, 24, 48, 96, 192):
@@ -786,14 +791,19 @@ def run_secondary(omprt, torch, gen, dev, stream, scrub, peaks):
     tw1 = lambda: omprt.omprt_cuda_axpy_sum(n, x, bt, ct, at, s, 8, 128)
     res["c1_axpy_sum_8x128"] = _short_pair(rt1, tw1, stream, scrub)
     t_rt = res["c1_axpy_sum_8x128"]["rt_ms"]
-    hbm8 = peaks.get("hbm_stream_8sm_gbs")
+    hbm8 = peaks.get("hbm_read2write1_8sm_gbs")
+    hbm8r = peaks.get("hbm_stream_8sm_gbs")
 
     def c1_roof(gbs):
-        # the config runs 8 teams, so 8 SMs: their measured HBM stream roof, the whole
-        # GPU's copy peak as context
-        r = _roof("hbm", gbs, hbm8 or hbm, "GB/s", "24 B/iteration, cold")
-        r["peak_source"] = ("omprt_probe_hbm_stream on 8 SMs (measured live)" if hbm8 else
+        # the config runs 8 teams, so 8 SMs: their measured HBM roof for C1's traffic mix
+        # (2 bytes read per byte written); the 8 SMs' read-only stream and the whole GPU's
+        # copy peak as context
+        r = _roof("hbm", gbs, hbm8 or hbm, "GB/s", "24 B/iteration (16 read, 8 written), cold")
+        r["peak_source"] = ("omprt_probe_hbm_stream mode 1 on 8 SMs: bulk copies, 2 bytes read "
+                            "per byte written (measured live)" if hbm8 else
                             "MEASURED_PEAKS.json hbm_gbs")
+        if hbm8r:
+            r["read_only_8sm"] = {"peak": hbm8r, "frac": gbs / hbm8r}
         r["full_gpu"] = {"peak": hbm, "frac": gbs / hbm}
         return r
 

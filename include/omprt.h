@@ -384,13 +384,15 @@ int omprt_probe_l2_read(const double *buf, uint64_t bytes, int32_t mode, int32_t
 /* FP64 FMA throughput: `iters` steps of 8 independent fma chains per thread, 256 threads
  * per team, teams = 0: 8 per SM; flops = 16 * iters * teams * 256. */
 int omprt_probe_fp64_fma(int64_t iters, int32_t teams, double *sink, void *stream);
-/* HBM -> SM streaming read bandwidth of `teams` SMs (1 <= teams <= the SM count): team b
- * (32 threads, one per SM, 128 KB dynamic shared memory) reads its contiguous slice of
- * `buf` (device, 16 B aligned) by 16 KB bulk copies, 8 in flight.  Bytes read = teams *
- * slice, slice = floor(bytes / teams) rounded down to 16 KB (>= 16 KB, else OMPRT_E_INVAL).
- * Size `buf` above the 126 MB L2 so the reads come from HBM. */
-int omprt_probe_hbm_stream(const void *buf, uint64_t bytes, int32_t teams, double *sink,
-                           void *stream);
+/* HBM -> SM streaming bandwidth of `teams` SMs (1 <= teams <= the SM count): team b (32
+ * threads, one per SM, 192 KB dynamic shared memory) reads its contiguous slice of `buf`
+ * (device, 16 B aligned) by 16 KB bulk copies, 8 in flight; mode 1 also writes every second
+ * chunk it read to `dst` (device, 16 B aligned, bytes / 2 writable), 2 bytes read per byte
+ * written (C1's mix).  slice = floor(bytes / teams) rounded down to 32 KB (>= 32 KB, else
+ * OMPRT_E_INVAL); bytes read = teams * slice, written = teams * slice / 2 in mode 1.  Size
+ * `buf` above the 126 MB L2 so the reads come from HBM. */
+int omprt_probe_hbm_stream(const void *buf, void *dst, uint64_t bytes, int32_t mode,
+                           int32_t teams, double *sink, void *stream);
 
 /* ---- introspection (resource report, "# Regs" and "SMem") ------------------ */
 /* Number of kernels in the library and the name of kernel `id`. */

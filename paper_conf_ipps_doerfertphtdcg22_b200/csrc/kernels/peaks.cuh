@@ -115,11 +115,15 @@ __global__ void __launch_bounds__(kProbeThreads) probe_fp64_fma(int64_t iters, d
 }
 
 // HBM stream probe: team b reads bytes [b * slice, (b + 1) * slice) in kHbmChunk pieces,
-// kHbmStages bulk copies in flight on as many mbarriers (one issuing thread).
+// 8 bulk copies in flight on a ring of kHbmStages mbarriers (one issuing thread).  Mode 1 also
+// writes every second landed chunk back to `dst` (bulk store from shared memory): 2 bytes
+// read per byte written, C1's mix (b and c read, a written).
 constexpr uint32_t kHbmChunk = 16384;
-constexpr int kHbmStages = 8;
+constexpr int kHbmStages = 12;  // 8 loads in flight + 4 stages whose stores are reading
+template <int Mode>
 __global__ void __launch_bounds__(32, 1)
-    probe_hbm_stream(const unsigned char* __restrict__ buf, int64_t slice, double* sink) {
+    probe_hbm_stream(const unsigned char* __restrict__ buf, unsigned char* __restrict__ dst,
+                     int64_t slice, double* sink) {
   extern __shared__ __align__(128) unsigned char ring[];
   __shared__ uint64_t bars[kHbmStages];
   namespace tma = omprt::tma;
@@ -127,22 +131,37 @@ __global__ void __launch_bounds__(32, 1)
   for (int k = 0; k < kHbmStages; ++k) tma::mbar_init(&bars[k], 1);
   tma::fence_mbar_init();
   const unsigned char* src = buf + (int64_t)blockIdx.x * slice;
+  unsigned char* out = Mode == 1 ? dst + (int64_t)blockIdx.x * (slice / 2) : nullptr;
   const int64_t chunks = slice / kHbmChunk;
   uint32_t phase = 0;
+  // chunk c has landed in stage c % kHbmStages: mode 1 writes the odd ones out.  Landings
+  // are taken kLag = 8 chunks behind the loads (8 loads in flight), so a stage's store has
+  // had 4 loads' time to read it before the stage is refilled.
+  constexpr int64_t kLag = 8;
+  auto landed = [&](int64_t c) {
+    const int k = (int)(c % kHbmStages);
+    tma::mbar_wait(&bars[k], phase >> k & 1u);
+    phase ^= 1u << k;
+    if constexpr (Mode == 1) {
+      if (c & 1) {
+        tma::bulk_store(out + (c >> 1) * kHbmChunk, ring + (size_t)k * kHbmChunk, kHbmChunk);
+        tma::bulk_commit();
+      }
+    }
+  };
   for (int64_t c = 0; c < chunks; ++c) {
     const int k = (int)(c % kHbmStages);
-    if (c >= kHbmStages) {  // the stage's previous copy has landed
-      tma::mbar_wait(&bars[k], phase >> k & 1u);
-      phase ^= 1u << k;
+    if (c >= kLag) landed(c - kLag);
+    if constexpr (Mode == 1) {
+      // the store of chunk c - kHbmStages (if any) has read its stage: at most the
+      // (kHbmStages - kLag) / 2 stores committed after it may still be reading
+      if (c >= kHbmStages) tma::bulk_wait_read<(kHbmStages - kLag) / 2>();
     }
     tma::mbar_arrive_expect_tx(&bars[k], kHbmChunk);
     tma::bulk_load(ring + (size_t)k * kHbmChunk, src + c * kHbmChunk, kHbmChunk, &bars[k]);
   }
-  for (int64_t c = chunks > kHbmStages ? chunks - kHbmStages : 0; c < chunks; ++c) {
-    const int k = (int)(c % kHbmStages);
-    tma::mbar_wait(&bars[k], phase >> k & 1u);
-    phase ^= 1u << k;
-  }
+  for (int64_t c = chunks > kLag ? chunks - kLag : 0; c < chunks; ++c) landed(c);
+  if constexpr (Mode == 1) tma::bulk_wait<0>();
   const double v = *reinterpret_cast<const double*>(ring);
   if (v == -1.2345e300) *sink = v;
 }
@@ -185,21 +204,25 @@ extern "C" int omprt_probe_fp64_fma(int64_t iters, int32_t teams, double* sink, 
 }
 
 // bytes read = teams * slice, slice = (bytes / teams) rounded down to 16 KB; one team of 32
-// threads per SM (teams <= the SM count), 128 KB of dynamic shared memory each.  Use a
-// buffer larger than L2 (126 MB) so the reads come from HBM.
-extern "C" int omprt_probe_hbm_stream(const void* buf, uint64_t bytes, int32_t teams, double* sink,
-                                      void* stream) {
+// threads per SM (teams <= the SM count), 192 KB of dynamic shared memory each.  Use a
+// buffer larger than L2 (126 MB) so the reads come from HBM.  dst (mode 1 only): bytes / 2
+// writable bytes; bytes written = teams * slice / 2.
+extern "C" int omprt_probe_hbm_stream(const void* buf, void* dst, uint64_t bytes, int32_t mode,
+                                      int32_t teams, double* sink, void* stream) {
   using namespace omprt_kernels;
   int dev = 0, sms = 148;
   cudaGetDevice(&dev);
   cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-  const int64_t slice = teams > 0 ? (int64_t)(bytes / (uint64_t)teams) / kHbmChunk * kHbmChunk : 0;
+  const int64_t slice =
+      teams > 0 ? (int64_t)(bytes / (uint64_t)teams) / (2 * kHbmChunk) * (2 * kHbmChunk) : 0;
   OMPRT_CHECK_ARG(buf && sink && ((uintptr_t)buf & 15) == 0 && teams > 0 && teams <= sms &&
-                      slice >= (int64_t)kHbmChunk,
+                      slice >= (int64_t)(2 * kHbmChunk) && (mode == 0 || mode == 1) &&
+                      (mode == 0 || (dst && ((uintptr_t)dst & 15) == 0)),
                   "omprt_probe_hbm_stream: bad arguments");
   const int smem = (int)kHbmChunk * kHbmStages;
-  cudaFuncSetAttribute(probe_hbm_stream, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
-  probe_hbm_stream<<<teams, 32, smem, as_stream(stream)>>>(
-      static_cast<const unsigned char*>(buf), slice, sink);
+  const auto k = mode == 0 ? probe_hbm_stream<0> : probe_hbm_stream<1>;
+  cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+  k<<<teams, 32, smem, as_stream(stream)>>>(static_cast<const unsigned char*>(buf),
+                                           static_cast<unsigned char*>(dst), slice, sink);
   return check_launch("probe_hbm_stream");
 }

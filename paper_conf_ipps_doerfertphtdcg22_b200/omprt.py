@@ -122,7 +122,7 @@ _SIGS = {
     "omprt_cuda_su3_mult": [_vp, _vp, _vp, _i64, _vp, _i32, _i32, _u32, _vp],
     "omprt_probe_l2_read": [_vp, _u64, _i32, _i32, _i32, _i32, _vp, _vp],
     "omprt_probe_fp64_fma": [_i64, _i32, _vp, _vp],
-    "omprt_probe_hbm_stream": [_vp, _u64, _i32, _vp, _vp],
+    "omprt_probe_hbm_stream": [_vp, _vp, _u64, _i32, _i32, _vp, _vp],
     "omprt_kernel_count": [],
     "omprt_kernel_occupancy": [C.c_int, C.c_int, C.c_int, C.POINTER(C.c_int)],
     "omprt_kernel_name": [C.c_int],
@@ -509,10 +509,13 @@ def omprt_probe_fp64_fma(iters, sink, teams=0, stream=None):
                                               _stream(stream)))
 
 
-def omprt_probe_hbm_stream(buf, nbytes, teams, sink, stream=None):
-    """Bytes read: teams * (nbytes // teams rounded down to 16 KB)."""
-    return _check(load().omprt_probe_hbm_stream(_p(buf, None, nbytes // buf.element_size()), nbytes, teams,
-                                                _p(sink, _T().float64, 1), _stream(stream)))
+def omprt_probe_hbm_stream(buf, nbytes, teams, sink, dst=None, mode=0, stream=None):
+    """Bytes read: teams * (nbytes // teams rounded down to 32 KB); mode 1 writes half as
+    many to `dst` (nbytes // 2 bytes)."""
+    return _check(load().omprt_probe_hbm_stream(
+        _p(buf, None, nbytes // buf.element_size()),
+        _p(dst, None, nbytes // 2 // dst.element_size()) if dst is not None else None,
+        nbytes, mode, teams, _p(sink, _T().float64, 1), _stream(stream)))
 
 
 # ---------------------------------------------------------------- introspection

@@ -22,6 +22,7 @@ def test_roof_probes_plausible(rt):
     # fraction of it
     assert 4000 < p["hbm_stream_gbs"] < 8500, p
     assert 100 < p["hbm_stream_8sm_gbs"] < p["hbm_stream_gbs"] * 0.5, p
+    assert 100 < p["hbm_read2write1_8sm_gbs"] < p["hbm_stream_gbs"] * 0.5, p
 
 
 def test_probe_arguments_rejected(rt):
@@ -39,7 +40,25 @@ def test_probe_arguments_rejected(rt):
     with pytest.raises(rt.OmprtError):
         rt.omprt_probe_hbm_stream(big, big.numel() * 8, 1000, sink)    # more teams than SMs
     with pytest.raises(rt.OmprtError):
-        rt.omprt_probe_hbm_stream(big, 8192, 1, sink)                  # slice < 16 KB
+        rt.omprt_probe_hbm_stream(big, 16384, 1, sink)                 # slice < 32 KB
+    with pytest.raises(rt.OmprtError):
+        rt.omprt_probe_hbm_stream(big, big.numel() * 8, 1, sink, None, 1)  # mode 1, no dst
+    with pytest.raises(rt.OmprtError):
+        rt.omprt_probe_hbm_stream(big, big.numel() * 8, 1, sink, None, 2)  # no mode 2
+
+
+def test_hbm_probe_copies_what_it_reads(rt):
+    """Mode 1 writes every second 16 KB chunk of each team's slice to dst (team b's writes
+    at b * slice / 2): the copy is exact, so the probe moves the bytes it claims."""
+    n = 8 * (1 << 20)  # 8 MiB, 4 teams -> slice 2 MiB = 128 chunks of 16 KB
+    src = torch.arange(n // 8, dtype=torch.int64, device=DEV)
+    dst = torch.zeros(n // 2 // 8, dtype=torch.int64, device=DEV)
+    sink = torch.zeros(1, dtype=torch.float64, device=DEV)
+    rt.omprt_probe_hbm_stream(src, n, 4, sink, dst, 1)
+    torch.cuda.synchronize()
+    chunk = 16384 // 8
+    s = src.view(4, -1, chunk)[:, 1::2, :].reshape(-1)
+    assert torch.equal(dst, s)
 
 
 def test_occupancy_query(rt):

@@ -38,6 +38,13 @@ elif which == "rs10m":  # the bench's C4 launch (queued, dynamic, flattened), 10
     for _ in range(reps):
         omprt.omprt_rs_lookup(d, 1070, 0, n, v, None, 0, 128, Q)
         omprt.omprt_cuda_rs_lookup(d, 1070, 0, n, v, None, 0, 128, Q)
+elif which == "rsd10m":  # dynamic flattened without the queue, 10M lookups
+    t = gen.RSTables(); d = omprt.RSDeviceTables(t, dev); n = 10_000_000
+    v = torch.empty(n, dtype=torch.uint64, device=dev)
+    D = omprt.OMPRT_FLAT | omprt.OMPRT_SCHED_DYNAMIC
+    for _ in range(reps):
+        omprt.omprt_rs_lookup(d, 1070, 0, n, v, None, 0, 128, D)
+        omprt.omprt_cuda_rs_lookup(d, 1070, 0, n, v, None, 0, 128, D)
 elif which == "su3":
     ns = 32 ** 4; Ah, Bh = gen.su3_inputs(ns)
     At, Bt = torch.from_numpy(Ah).to(dev), torch.from_numpy(Bh).to(dev); Ct = torch.empty_like(At)

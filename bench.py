@@ -144,7 +144,9 @@ def run_reference(args):
     line = {"impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms,
             "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64",
-            "data": "synthetic", "config": {"workload": WORKLOAD + " (CPU oracle sample)"},
+            "data": "synthetic",
+            # the GPU arm's workload (the same config); the timed sample is in cpu_baseline
+            "config": {"workload": WORKLOAD, "lookups_per_gpu": L, "parallelism": f"dp{world}"},
             "cpu_baseline": {"value": value, "unit": UNIT, "cores": cores, "kind": "oracle",
                              "sample": sample},
             "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0,

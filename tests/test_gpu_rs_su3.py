@@ -234,13 +234,15 @@ def test_rs_prepare_pole_records(rt, rs_tables_small):
         rt.omprt_rs_lookup(d, 1, 0, 16, v)
 
 
-def test_rs_sigt_factor_angles_beyond_the_series_range(rt, rs_tables_small):
+@pytest.mark.parametrize("scale", [3.0, 30.0])
+def test_rs_sigt_factor_angles_beyond_the_series_range(rt, rs_tables_small, scale):
     """The sigT factors outside the workload's angle range (k0rs scaled by 3: angles 2 k0rs
     sqrt(E) up to 6, past the first quadrant boundaries of the rational-rotation form,
-    R-A10) still match the oracle within the C7 contract."""
+    R-A10; by 30: up to 60, every quadrant of the sincos reduction many times over)
+    still match the oracle within the C7 contract."""
     import copy
     t = copy.copy(rs_tables_small)
-    t.k0rs = rs_tables_small.k0rs * 3.0
+    t.k0rs = rs_tables_small.k0rs * scale
     d = rt.RSDeviceTables(t, DEV)
     first, count = 11, 5_000
     ver, mac = _rs(rt, d, first, count, "rt", rt.OMPRT_FLAT | rt.OMPRT_SCHED_DYNAMIC)

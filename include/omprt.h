@@ -329,10 +329,10 @@ int omprt_xs_run_host_steps(omprt_xs_tables host_tables, uint64_t seed, int64_t 
 /* ---- C4: RSBench-shaped multipole lookup -------------------- */
 typedef struct {
   /* [n_poles][8] EA RT RA RF (re, im), 32 B aligned -- in the lookups' PREPARED form (see
-   * omprt_rs_prepare): EA.re / 2, (0 - EA.im) / 2, RT, RA, RF */
+   * omprt_rs_prepare): EA.re / 2, (0 - EA.im) / 2, RT, RA, RF, sorted by l per window */
   const double *poles;
-  const int32_t *pole_l;    /* [n_poles] l value in [0, numL) */
-  const double *windows;    /* [n_windows][4] T A F 0, 32 B aligned */
+  const int32_t *pole_l;    /* [n_poles] l value in [0, numL); read by omprt_rs_prepare only */
+  const double *windows;    /* [n_windows][4] T A F (prepared: l-run boundaries), 32 B aligned */
   const int32_t *win_range; /* [n_windows][2] absolute pole [start, end) */
   const int32_t *win_off;   /* [n_nuclides+1] window CSR offsets */
   const int32_t *n_windows; /* [n_nuclides] */
@@ -341,16 +341,27 @@ typedef struct {
   const int32_t *mats;      /* [12][max_num_nucs] */
   const double *concs;      /* [12][max_num_nucs] */
   int32_t n_nuclides, numL, max_num_nucs;
-  int32_t prepared; /* 1: `poles` holds the prepared form (set by omprt_rs_prepare) */
+  int32_t prepared; /* 1: `poles` and `windows` hold the prepared form (omprt_rs_prepare) */
 } omprt_rs_tables;
-/* Table preparation (like omprt_xs_build_accel; not part of a lookup): copies the n_poles
- * records of t->poles into `prepared` (caller-owned device memory, n_poles * 8 doubles, 32 B
- * aligned) with EA replaced by (EA.re / 2, (0 - EA.im) / 2) -- exact in IEEE arithmetic --
- * and points t->poles at it, t->prepared = 1.  The lookup's Z = ((E - EA.re) / 2,
- * (0 - EA.im) / 2) (App. A.2) is then E/2 - EA.re/2 and a load: the same bits (halving
- * commutes with rounding), 3 fewer fp64 operations per pole.  OMPRT_E_INVAL on null
- * pointers, a misaligned buffer or an already prepared table. */
-int omprt_rs_prepare(omprt_rs_tables *t, int64_t n_poles, double *prepared, void *stream);
+/* Table preparation (like omprt_xs_build_accel; not part of a lookup; App. A.2 defines the
+ * lookup, this only lays its data out):
+ * - prepared_poles (caller-owned device memory, n_poles * 8 doubles, 32 B aligned): the
+ *   records of t->poles with EA replaced by (EA.re / 2, (0 - EA.im) / 2) -- exact in IEEE
+ *   arithmetic; the lookup's Z = ((E - EA.re) / 2, (0 - EA.im) / 2) is then E/2 - EA.re/2
+ *   and a load, the same bits, 3 fewer fp64 operations per pole (reading R-A9) -- and, within
+ *   each window's range, stably sorted by the pole's l (reading R-A12: a window's poles are
+ *   summed in l order, the same terms in another order);
+ * - prepared_windows (caller-owned, n_windows * 4 doubles, 32 B aligned): T, A, F of each
+ *   window and, as the 4th word, its l-run boundaries c1 | c2 << 21 | c3 << 42 (c_k = the
+ *   number of the window's poles with l < k), so a lookup derives a pole's l from its index
+ *   instead of loading pole_l.
+ * Then points t->poles / t->windows at them and sets t->prepared = 1.  Synchronizes
+ * `stream` (the range checks come back to the host).  OMPRT_E_INVAL on null pointers, a
+ * misaligned buffer, an already prepared table, numL != 4, a window range outside
+ * [0, n_poles) or starting before the previous window's end (windows must not overlap), a
+ * window of 2^21 poles or more, or an l outside [0, 4); the table is then unchanged. */
+int omprt_rs_prepare(omprt_rs_tables *t, int64_t n_poles, int64_t n_windows,
+                     double *prepared_poles, double *prepared_windows, void *stream);
 /* Same contract as omprt_xs_lookup (4 macroscopic cross sections; numL must be 4; the
  * tables prepared by omprt_rs_prepare, else OMPRT_E_INVAL).
  * macro (nullable): [count][4] doubles for parity tests. */

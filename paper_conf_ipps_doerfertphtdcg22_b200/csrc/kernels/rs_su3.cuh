@@ -388,31 +388,87 @@ inline int su3_validate(const double* A, const double* B, double* Cm, int64_t n,
 
 namespace omprt_kernels {
 // the prepared pole records (omprt_rs_prepare): EA.re / 2, (0 - EA.im) / 2, RT, RA, RF
+__device__ __forceinline__ void rs_prepare_record(const double* __restrict__ r,
+                                                  double* __restrict__ o) {
+  o[0] = __dmul_rn(r[0], 0.5);
+  o[1] = __dmul_rn(__dsub_rn(0.0, r[1]), 0.5);
+#pragma unroll
+  for (int k = 2; k < 8; ++k) o[k] = r[k];
+}
 __global__ void rs_prepare_poles(const double* __restrict__ in, double* __restrict__ out,
                                  int64_t n) {
   for (int64_t p = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; p < n;
-       p += (int64_t)gridDim.x * blockDim.x) {
-    const double* r = in + p * 8;
-    double* o = out + p * 8;
-    o[0] = __dmul_rn(r[0], 0.5);
-    o[1] = __dmul_rn(__dsub_rn(0.0, r[1]), 0.5);
-#pragma unroll
-    for (int k = 2; k < 8; ++k) o[k] = r[k];
+       p += (int64_t)gridDim.x * blockDim.x)
+    rs_prepare_record(in + p * 8, out + p * 8);
+}
+// one thread per window (reading R-A12): the window's prepared records stably sorted by l
+// (a counting sort: l = 0 first, each run in the input order), and the window record
+// (T, A, F, runs) with runs = c1 | c2 << 21 | c3 << 42, c_k = the number of the window's
+// poles with l < k.  Rejected (bit 0 of *err): a window range outside [0, n_poles), one
+// that starts before the previous window ends (overlapping windows cannot be sorted
+// independently), a window of 2^21 poles or more, an l outside [0, 4).
+__global__ void rs_prepare_windows(const double* __restrict__ poles,
+                                   const int32_t* __restrict__ pole_l,
+                                   const int32_t* __restrict__ win_range,
+                                   const double* __restrict__ windows, int64_t n_poles,
+                                   int64_t n_windows, double* __restrict__ out_poles,
+                                   double* __restrict__ out_windows,
+                                   unsigned long long* __restrict__ err) {
+  const int64_t w = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+  if (w >= n_windows) return;
+  const int64_t s = win_range[2 * w], e = win_range[2 * w + 1];
+  bool bad = s < 0 || e < s || e > n_poles || e - s >= (1 << 21) ||
+             (w > 0 && s < (int64_t)win_range[2 * w - 1]);
+  int64_t c[4] = {0, 0, 0, 0};
+  for (int64_t p = s; !bad && p < e; ++p) {
+    const int32_t l = pole_l[p];
+    if (l < 0 || l > 3) bad = true;
+    else ++c[l];
   }
+  if (bad) {
+    atomicOr(err, 1ull);
+    return;
+  }
+  int64_t pos[4] = {s, s + c[0], s + c[0] + c[1], s + c[0] + c[1] + c[2]};
+  for (int64_t p = s; p < e; ++p) rs_prepare_record(poles + p * 8, out_poles + 8 * pos[pole_l[p]]++);
+  const uint64_t runs = (uint64_t)c[0] | (uint64_t)(c[0] + c[1]) << 21 |
+                        (uint64_t)(c[0] + c[1] + c[2]) << 42;
+  out_windows[4 * w] = windows[4 * w];
+  out_windows[4 * w + 1] = windows[4 * w + 1];
+  out_windows[4 * w + 2] = windows[4 * w + 2];
+  out_windows[4 * w + 3] = __longlong_as_double((long long)runs);
 }
 }  // namespace omprt_kernels
 
-extern "C" int omprt_rs_prepare(omprt_rs_tables* t, int64_t n_poles, double* prepared,
+extern "C" int omprt_rs_prepare(omprt_rs_tables* t, int64_t n_poles, int64_t n_windows,
+                                double* prepared_poles, double* prepared_windows,
                                 void* stream) {
   using namespace omprt_kernels;
   Workspace* w;
   if (int r = current_ws(&w)) return r;
-  OMPRT_CHECK_ARG(t && t->poles && prepared && n_poles > 0 && ((uintptr_t)prepared & 31) == 0,
+  OMPRT_CHECK_ARG(t && t->poles && t->pole_l && t->windows && t->win_range && prepared_poles &&
+                      prepared_windows && n_poles > 0 && n_windows > 0 &&
+                      (((uintptr_t)prepared_poles | (uintptr_t)prepared_windows) & 31) == 0,
                   "omprt_rs_prepare: bad arguments");
   OMPRT_CHECK_ARG(t->prepared == 0, "omprt_rs_prepare: the tables are already prepared");
-  rs_prepare_poles<<<1024, 256, 0, as_stream(stream)>>>(t->poles, prepared, n_poles);
+  OMPRT_CHECK_ARG(t->numL == 4, "omprt_rs_prepare: numL must be 4");
+  cudaStream_t st = as_stream(stream);
+  unsigned long long* err = (unsigned long long*)w->scratch_u64;
+  OMPRT_CUDA_TRY(cudaMemsetAsync(err, 0, sizeof(*err), st));
+  rs_prepare_poles<<<1024, 256, 0, st>>>(t->poles, prepared_poles, n_poles);
   if (int r = check_launch("rs_prepare_poles")) return r;
-  t->poles = prepared;
+  rs_prepare_windows<<<(unsigned)ceil_div(n_windows, 256), 256, 0, st>>>(
+      t->poles, t->pole_l, t->win_range, t->windows, n_poles, n_windows, prepared_poles,
+      prepared_windows, err);
+  if (int r = check_launch("rs_prepare_windows")) return r;
+  unsigned long long bad = 0;
+  OMPRT_CUDA_TRY(cudaMemcpyAsync(&bad, err, sizeof(bad), cudaMemcpyDeviceToHost, st));
+  OMPRT_CUDA_TRY(cudaStreamSynchronize(st));
+  OMPRT_CHECK_ARG(bad == 0,
+                  "omprt_rs_prepare: windows overlap / out of range / >= 2^21 poles, or l "
+                  "outside [0, 4)");
+  t->poles = prepared_poles;
+  t->windows = prepared_windows;
   t->prepared = 1;
   return OMPRT_OK;
 }

@@ -115,7 +115,7 @@ _SIGS = {
                           C.POINTER(_u64), C.POINTER(_u64), _vp],
     "omprt_xs_run_host_steps": [XSTablesC, _u64, _i64, _i64, _i32, _u32, _i32, C.POINTER(_u64),
                                 C.POINTER(_u64), C.POINTER(_u64), _vp],
-    "omprt_rs_prepare": [C.POINTER(RSTablesC), _i64, _vp, _vp],
+    "omprt_rs_prepare": [C.POINTER(RSTablesC), _i64, _i64, _vp, _vp, _vp],
     "omprt_rs_lookup": [RSTablesC, _u64, _i64, _i64, _vp, _vp, _i32, _i32, _u32, _vp],
     "omprt_cuda_rs_lookup": [RSTablesC, _u64, _i64, _i64, _vp, _vp, _i32, _i32, _u32, _vp],
     "omprt_su3_mult": [_vp, _vp, _vp, _i64, _vp, _i32, _i32, _u32, _vp],
@@ -451,14 +451,18 @@ class RSDeviceTables:
                                                    "win_off", "n_windows", "k0rs", "num_nucs",
                                                    "mats", "concs")],
                            t.n_nuclides, t.numL, t.max_num_nucs, 0)
-        # the lookups' prepared pole records (omprt_rs_prepare, on the device)
+        # the lookups' prepared pole and window records (omprt_rs_prepare, on the device)
         self.poles_prepared = torch.empty_like(self.poles)
-        omprt_rs_prepare(self, self.poles.shape[0], self.poles_prepared)
+        self.windows_prepared = torch.empty_like(self.windows)
+        omprt_rs_prepare(self, self.poles.shape[0], self.windows.shape[0],
+                         self.poles_prepared, self.windows_prepared)
 
 
-def omprt_rs_prepare(tables, n_poles, prepared, stream=None):
-    return _check(load().omprt_rs_prepare(C.byref(tables.c), n_poles,
-                                          _p(prepared, _T().float64, 8 * n_poles),
+def omprt_rs_prepare(tables, n_poles, n_windows, prepared_poles, prepared_windows,
+                     stream=None):
+    return _check(load().omprt_rs_prepare(C.byref(tables.c), n_poles, n_windows,
+                                          _p(prepared_poles, _T().float64, 8 * n_poles),
+                                          _p(prepared_windows, _T().float64, 4 * n_windows),
                                           _stream(stream)))
 
 

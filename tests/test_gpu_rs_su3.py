@@ -212,26 +212,66 @@ def test_su3_pins_on_gpu(rt):
     assert (C.reshape(n, 4, 3, 3, 2)[..., 0] == 1.0).all() and ck == 36.0 * n
 
 
-def test_rs_prepare_pole_records(rt, rs_tables_small):
-    """omprt_rs_prepare: EA.re / 2 and (0 - EA.im) / 2, the rest of each record unchanged --
-    exactly the values numpy's IEEE arithmetic gives -- and an unprepared or twice-prepared
-    table is rejected."""
-    d = rt.RSDeviceTables(rs_tables_small, DEV)
-    got = d.poles_prepared.cpu().numpy().reshape(-1, 8)
-    P = rs_tables_small.poles.reshape(-1, 8)
+def _prepared_expected(t):
+    """The prepared layout written out with numpy (R-A9, R-A12): EA halved, each window's
+    records stably sorted by l, the window's 4th word = its l-run boundaries."""
+    P = t.poles.reshape(-1, 8)
     exp = P.copy()
     exp[:, 0] = P[:, 0] * 0.5
     exp[:, 1] = (0.0 - P[:, 1]) * 0.5
+    W = t.windows.reshape(-1, 4).copy()
+    runs = np.zeros(W.shape[0], dtype=np.uint64)
+    out = exp.copy()
+    for w, (s, e) in enumerate(t.win_range.reshape(-1, 2)):
+        ls = t.pole_l[s:e]
+        order = np.argsort(ls, kind="stable")
+        out[s:e] = exp[s:e][order]
+        c = [int((ls < k).sum()) for k in (1, 2, 3)]
+        runs[w] = c[0] | (c[1] << 21) | (c[2] << 42)
+    W.view(np.uint64)[:, 3] = runs
+    return out, W
+
+
+def test_rs_prepare_pole_records(rt, rs_tables_small):
+    """omprt_rs_prepare: EA.re / 2 and (0 - EA.im) / 2, the rest of each record unchanged --
+    exactly the values numpy's IEEE arithmetic gives --, each window's records stably
+    sorted by l and its l-run boundaries in the window record (R-A12); an unprepared or
+    twice-prepared table is rejected."""
+    d = rt.RSDeviceTables(rs_tables_small, DEV)
+    got = d.poles_prepared.cpu().numpy().reshape(-1, 8)
+    gotw = d.windows_prepared.cpu().numpy().reshape(-1, 4)
+    exp, expw = _prepared_expected(rs_tables_small)
     assert (got.view(np.uint64) == exp.view(np.uint64)).all()
+    assert (gotw.view(np.uint64) == expw.view(np.uint64)).all()
     assert d.c.prepared == 1
     with pytest.raises(rt.OmprtError):
-        rt.omprt_rs_prepare(d, P.shape[0], d.poles_prepared)
+        rt.omprt_rs_prepare(d, exp.shape[0], gotw.shape[0], d.poles_prepared,
+                            d.windows_prepared)
     raw = rt.RSTablesC.from_buffer_copy(d.c)
     raw.prepared = 0
     d.c = raw
     v = torch.zeros(16, dtype=torch.uint64, device=DEV)
     with pytest.raises(rt.OmprtError):
         rt.omprt_rs_lookup(d, 1, 0, 16, v)
+
+
+@pytest.mark.parametrize("defect", ["overlap", "l_range", "past_end"])
+def test_rs_prepare_rejects_unsortable_windows(rt, rs_tables_small, defect):
+    """Windows that overlap (their poles cannot be sorted independently), an l outside
+    [0, 4) or a range past the last pole: omprt_rs_prepare fails with OMPRT_E_INVAL and
+    leaves the table unprepared."""
+    import copy
+    t = copy.copy(rs_tables_small)
+    t.win_range = rs_tables_small.win_range.copy()
+    t.pole_l = rs_tables_small.pole_l.copy()
+    if defect == "overlap":
+        t.win_range[5, 0] = t.win_range[4, 1] - 1
+    elif defect == "l_range":
+        t.pole_l[t.win_range[7, 0]] = 4
+    else:
+        t.win_range[-1, 1] = t.poles.shape[0] + 1
+    with pytest.raises(rt.OmprtError):
+        rt.RSDeviceTables(t, DEV)
 
 
 @pytest.mark.parametrize("scale", [3.0, 30.0])

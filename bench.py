@@ -901,7 +901,8 @@ def run_secondary(omprt, torch, gen, dev, stream, scrub, peaks):
         "rt_ms": t_rt, "twin_ms": t_tw, "overhead": t_rt / t_tw - 1,
         "lookups_per_s": nl / t_rt * 1e3,
         "variant": "flattened nuclide loop, lock-step warps, schedule(dynamic,1), persistent "
-                   "grid, pole records prefetched, Abrarov poles queued per warp",
+                   "grid, pole records prefetched, Abrarov poles queued per warp; prepared "
+                   "tables: poles sorted by l per window, one record per material entry",
         "regs": [tab["omprt_rs_qflat_rt"]["regs"], tab["cuda_rs_qflat_twin"]["regs"]],
         "roofline": _roof("fp64", gflops, fp64, "GFLOP/s",
                           f"{fl['flops_per_lookup']:.0f} fp64 flops/lookup (oracle-counted add, "

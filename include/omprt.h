@@ -340,11 +340,15 @@ typedef struct {
   const int32_t *num_nucs;  /* [12] */
   const int32_t *mats;      /* [12][max_num_nucs] */
   const double *concs;      /* [12][max_num_nucs] */
+  /* set by omprt_rs_prepare (NULL before): [n_mats][max_num_nucs][8] doubles per material
+   * entry -- k0rs of its nuclide (4), conc, window offset | window count << 32 (bits), 2 pad */
+  const double *matnuc;
   int32_t n_nuclides, numL, max_num_nucs;
-  int32_t prepared; /* 1: `poles` and `windows` hold the prepared form (omprt_rs_prepare) */
+  int32_t prepared; /* 1: poles, windows, matnuc hold the prepared form (omprt_rs_prepare) */
 } omprt_rs_tables;
 /* Table preparation (like omprt_xs_build_accel; not part of a lookup; App. A.2 defines the
- * lookup, this only lays its data out):
+ * lookup, this only lays its data out; n_mats = the number of materials of num_nucs / mats /
+ * concs):
  * - prepared_poles (caller-owned device memory, n_poles * 8 doubles, 32 B aligned): the
  *   records of t->poles with EA replaced by (EA.re / 2, (0 - EA.im) / 2) -- exact in IEEE
  *   arithmetic; the lookup's Z = ((E - EA.re) / 2, (0 - EA.im) / 2) is then E/2 - EA.re/2
@@ -354,14 +358,20 @@ typedef struct {
  * - prepared_windows (caller-owned, n_windows * 4 doubles, 32 B aligned): T, A, F of each
  *   window and, as the 4th word, its l-run boundaries c1 | c2 << 21 | c3 << 42 (c_k = the
  *   number of the window's poles with l < k), so a lookup derives a pole's l from its index
- *   instead of loading pole_l.
- * Then points t->poles / t->windows at them and sets t->prepared = 1.  Synchronizes
+ *   instead of loading pole_l;
+ * - prepared_matnuc (caller-owned, n_mats * max_num_nucs * 8 doubles, 32 B aligned): one
+ *   64 B record per material entry (m, j): k0rs of nuclide mats[m][j], concs[m][j], and
+ *   win_off | n_windows << 32 of that nuclide (bit pattern), zeros past num_nucs[m]
+ *   (reading R-A13: a nuclide step's 6-8 small loads become two).
+ * Then points t->poles / t->windows / t->matnuc at them and sets t->prepared = 1.  Synchronizes
  * `stream` (the range checks come back to the host).  OMPRT_E_INVAL on null pointers, a
  * misaligned buffer, an already prepared table, numL != 4, a window range outside
  * [0, n_poles) or starting before the previous window's end (windows must not overlap), a
- * window of 2^21 poles or more, or an l outside [0, 4); the table is then unchanged. */
-int omprt_rs_prepare(omprt_rs_tables *t, int64_t n_poles, int64_t n_windows,
-                     double *prepared_poles, double *prepared_windows, void *stream);
+ * window of 2^21 poles or more, an l outside [0, 4), num_nucs outside [0, max_num_nucs]
+ * or a material entry outside [0, n_nuclides); the table is then unchanged. */
+int omprt_rs_prepare(omprt_rs_tables *t, int64_t n_poles, int64_t n_windows, int32_t n_mats,
+                     double *prepared_poles, double *prepared_windows,
+                     double *prepared_matnuc, void *stream);
 /* Same contract as omprt_xs_lookup (4 macroscopic cross sections; numL must be 4; the
  * tables prepared by omprt_rs_prepare, else OMPRT_E_INVAL).
  * macro (nullable): [count][4] doubles for parity tests. */

@@ -194,9 +194,9 @@ OMPRT_REGISTER_KERNEL(omprt_rs_rt_assume, omprt_rs_rt<RSTraitsAssume, false>)
 OMPRT_REGISTER_KERNEL(cuda_rs_twin, cuda_rs_twin<false>)
 
 inline RSTables to_dev(const omprt_rs_tables& a) {
-  return RSTables{a.poles, a.pole_l, a.windows, a.win_range, a.win_off, a.n_windows, a.k0rs,
-                  a.num_nucs, a.mats, a.concs, a.n_nuclides, a.numL, a.max_num_nucs,
-                  a.prepared};
+  return RSTables{a.poles,    a.pole_l,  a.windows, a.win_range,  a.win_off,
+                  a.n_windows, a.k0rs,   a.num_nucs, a.mats,      a.concs,
+                  a.matnuc,    a.n_nuclides, a.numL, a.max_num_nucs, a.prepared};
 }
 
 // Persistent grid of the flattened kernels: teams = 0 -> every SM's resident teams (of the
@@ -220,7 +220,8 @@ inline int rs_validate(const omprt_rs_tables& t, int64_t count, uint64_t* ver, i
   OMPRT_CHECK_ARG(count >= 0 && count < (1ll << 31), "count must be in [0, 2^31)");
   OMPRT_CHECK_ARG(threads == kRSThreads, "threads must be %d", kRSThreads);
   OMPRT_CHECK_ARG(t.numL == 4, "numL must be 4");
-  OMPRT_CHECK_ARG(t.prepared == 1, "RSBench tables not prepared (omprt_rs_prepare)");
+  OMPRT_CHECK_ARG(t.prepared == 1 && t.matnuc && ((uintptr_t)t.matnuc & 31) == 0,
+                  "RSBench tables not prepared (omprt_rs_prepare)");
   OMPRT_CHECK_ARG(t.poles && t.pole_l && t.windows && t.win_range && t.win_off && t.n_windows &&
                       t.k0rs && t.num_nucs && t.mats && t.concs,
                   "bad RSBench tables");
@@ -438,17 +439,55 @@ __global__ void rs_prepare_windows(const double* __restrict__ poles,
   out_windows[4 * w + 2] = windows[4 * w + 2];
   out_windows[4 * w + 3] = __longlong_as_double((long long)runs);
 }
+// one thread per material entry (reading R-A13): the 64 B record of (m, j) -- k0rs of its
+// nuclide, conc, the nuclide's window offset | count << 32 -- zeros past num_nucs[m].
+// Rejected: a nuclide id outside [0, n_nuclides), num_nucs outside [0, max_num_nucs].
+__global__ void rs_prepare_matnuc(const int32_t* __restrict__ num_nucs,
+                                  const int32_t* __restrict__ mats,
+                                  const double* __restrict__ concs,
+                                  const double* __restrict__ k0rs,
+                                  const int32_t* __restrict__ win_off,
+                                  const int32_t* __restrict__ n_windows, int32_t n_mats,
+                                  int32_t max_num_nucs, int32_t n_nuclides,
+                                  double* __restrict__ out, unsigned long long* err) {
+  const int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+  if (i >= (int64_t)n_mats * max_num_nucs) return;
+  const int m = (int)(i / max_num_nucs), j = (int)(i % max_num_nucs);
+  double* o = out + i * 8;
+#pragma unroll
+  for (int k = 0; k < 8; ++k) o[k] = 0.0;
+  const int nn = num_nucs[m];
+  if (nn < 0 || nn > max_num_nucs) {
+    atomicOr(err, 2ull);
+    return;
+  }
+  if (j >= nn) return;
+  const int nuc = mats[i];
+  if (nuc < 0 || nuc >= n_nuclides) {
+    atomicOr(err, 2ull);
+    return;
+  }
+#pragma unroll
+  for (int l = 0; l < 4; ++l) o[l] = k0rs[nuc * 4 + l];
+  o[4] = concs[i];
+  o[5] = __longlong_as_double((long long)(uint32_t)win_off[nuc] |
+                              (long long)((uint64_t)(uint32_t)n_windows[nuc] << 32));
+}
 }  // namespace omprt_kernels
 
 extern "C" int omprt_rs_prepare(omprt_rs_tables* t, int64_t n_poles, int64_t n_windows,
-                                double* prepared_poles, double* prepared_windows,
+                                int32_t n_mats, double* prepared_poles,
+                                double* prepared_windows, double* prepared_matnuc,
                                 void* stream) {
   using namespace omprt_kernels;
   Workspace* w;
   if (int r = current_ws(&w)) return r;
-  OMPRT_CHECK_ARG(t && t->poles && t->pole_l && t->windows && t->win_range && prepared_poles &&
-                      prepared_windows && n_poles > 0 && n_windows > 0 &&
-                      (((uintptr_t)prepared_poles | (uintptr_t)prepared_windows) & 31) == 0,
+  OMPRT_CHECK_ARG(t && t->poles && t->pole_l && t->windows && t->win_range && t->win_off &&
+                      t->n_windows && t->k0rs && t->num_nucs && t->mats && t->concs &&
+                      prepared_poles && prepared_windows && prepared_matnuc && n_poles > 0 &&
+                      n_windows > 0 && n_mats > 0 && t->max_num_nucs > 0 &&
+                      (((uintptr_t)prepared_poles | (uintptr_t)prepared_windows |
+                        (uintptr_t)prepared_matnuc) & 31) == 0,
                   "omprt_rs_prepare: bad arguments");
   OMPRT_CHECK_ARG(t->prepared == 0, "omprt_rs_prepare: the tables are already prepared");
   OMPRT_CHECK_ARG(t->numL == 4, "omprt_rs_prepare: numL must be 4");
@@ -461,14 +500,20 @@ extern "C" int omprt_rs_prepare(omprt_rs_tables* t, int64_t n_poles, int64_t n_w
       t->poles, t->pole_l, t->win_range, t->windows, n_poles, n_windows, prepared_poles,
       prepared_windows, err);
   if (int r = check_launch("rs_prepare_windows")) return r;
+  rs_prepare_matnuc<<<(unsigned)ceil_div((int64_t)n_mats * t->max_num_nucs, 256), 256, 0, st>>>(
+      t->num_nucs, t->mats, t->concs, t->k0rs, t->win_off, t->n_windows, n_mats,
+      t->max_num_nucs, t->n_nuclides, prepared_matnuc, err);
+  if (int r = check_launch("rs_prepare_matnuc")) return r;
   unsigned long long bad = 0;
   OMPRT_CUDA_TRY(cudaMemcpyAsync(&bad, err, sizeof(bad), cudaMemcpyDeviceToHost, st));
   OMPRT_CUDA_TRY(cudaStreamSynchronize(st));
   OMPRT_CHECK_ARG(bad == 0,
-                  "omprt_rs_prepare: windows overlap / out of range / >= 2^21 poles, or l "
-                  "outside [0, 4)");
+                  "omprt_rs_prepare: windows overlap / out of range / >= 2^21 poles, l "
+                  "outside [0, 4), or a material entry outside [0, n_nuclides) (code %llu)",
+                  bad);
   t->poles = prepared_poles;
   t->windows = prepared_windows;
+  t->matnuc = prepared_matnuc;
   t->prepared = 1;
   return OMPRT_OK;
 }

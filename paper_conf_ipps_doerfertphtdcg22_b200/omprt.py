@@ -80,7 +80,8 @@ class RSTablesC(C.Structure):
     _fields_ = [("poles", C.c_void_p), ("pole_l", C.c_void_p), ("windows", C.c_void_p),
                 ("win_range", C.c_void_p), ("win_off", C.c_void_p), ("n_windows", C.c_void_p),
                 ("k0rs", C.c_void_p), ("num_nucs", C.c_void_p), ("mats", C.c_void_p),
-                ("concs", C.c_void_p), ("n_nuclides", C.c_int32), ("numL", C.c_int32),
+                ("concs", C.c_void_p), ("matnuc", C.c_void_p), ("n_nuclides", C.c_int32),
+                ("numL", C.c_int32),
                 ("max_num_nucs", C.c_int32), ("prepared", C.c_int32)]
 
 
@@ -115,7 +116,7 @@ _SIGS = {
                           C.POINTER(_u64), C.POINTER(_u64), _vp],
     "omprt_xs_run_host_steps": [XSTablesC, _u64, _i64, _i64, _i32, _u32, _i32, C.POINTER(_u64),
                                 C.POINTER(_u64), C.POINTER(_u64), _vp],
-    "omprt_rs_prepare": [C.POINTER(RSTablesC), _i64, _i64, _vp, _vp, _vp],
+    "omprt_rs_prepare": [C.POINTER(RSTablesC), _i64, _i64, _i32, _vp, _vp, _vp, _vp],
     "omprt_rs_lookup": [RSTablesC, _u64, _i64, _i64, _vp, _vp, _i32, _i32, _u32, _vp],
     "omprt_cuda_rs_lookup": [RSTablesC, _u64, _i64, _i64, _vp, _vp, _i32, _i32, _u32, _vp],
     "omprt_su3_mult": [_vp, _vp, _vp, _i64, _vp, _i32, _i32, _u32, _vp],
@@ -450,20 +451,26 @@ class RSDeviceTables:
         self.c = RSTablesC(*[_p(keep[k]) for k in ("poles", "pole_l", "windows", "win_range",
                                                    "win_off", "n_windows", "k0rs", "num_nucs",
                                                    "mats", "concs")],
-                           t.n_nuclides, t.numL, t.max_num_nucs, 0)
-        # the lookups' prepared pole and window records (omprt_rs_prepare, on the device)
+                           None, t.n_nuclides, t.numL, t.max_num_nucs, 0)
+        # the lookups' prepared pole, window and material-entry records (omprt_rs_prepare,
+        # on the device)
+        self.n_mats = int(self.num_nucs.shape[0])
         self.poles_prepared = torch.empty_like(self.poles)
         self.windows_prepared = torch.empty_like(self.windows)
-        omprt_rs_prepare(self, self.poles.shape[0], self.windows.shape[0],
-                         self.poles_prepared, self.windows_prepared)
+        self.matnuc = torch.empty(self.n_mats * t.max_num_nucs * 8, dtype=torch.float64,
+                                  device=device)
+        omprt_rs_prepare(self, self.poles.shape[0], self.windows.shape[0], self.n_mats,
+                         self.poles_prepared, self.windows_prepared, self.matnuc)
 
 
-def omprt_rs_prepare(tables, n_poles, n_windows, prepared_poles, prepared_windows,
-                     stream=None):
-    return _check(load().omprt_rs_prepare(C.byref(tables.c), n_poles, n_windows,
-                                          _p(prepared_poles, _T().float64, 8 * n_poles),
-                                          _p(prepared_windows, _T().float64, 4 * n_windows),
-                                          _stream(stream)))
+def omprt_rs_prepare(tables, n_poles, n_windows, n_mats, prepared_poles, prepared_windows,
+                     prepared_matnuc, stream=None):
+    return _check(load().omprt_rs_prepare(
+        C.byref(tables.c), n_poles, n_windows, n_mats,
+        _p(prepared_poles, _T().float64, 8 * n_poles),
+        _p(prepared_windows, _T().float64, 4 * n_windows),
+        _p(prepared_matnuc, _T().float64, 8 * n_mats * tables.c.max_num_nucs),
+        _stream(stream)))
 
 
 def omprt_rs_lookup(tables, seed, first, count, verification, macro=None, teams=0, threads=128,

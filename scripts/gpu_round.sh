@@ -46,7 +46,5 @@ rm -f $OUT/prof_*_$TAG.ncu-rep  # the CSV exports come back; the reports exceed 
 OMPRT_DEBUG=0 timeout 600 python scripts/debug_cost.py > $OUT/debug_cost_env0_$TAG.txt 2>&1
 OMPRT_DEBUG=1 timeout 600 python scripts/debug_cost.py > $OUT/debug_cost_env1_$TAG.txt 2>&1
 du -sh $OUT
-for T in memcheck racecheck initcheck; do
-  timeout 600 compute-sanitizer --tool $T python scripts/sanitize_run.py > $OUT/sanitize_${T}_$TAG.txt 2>&1
-done
-timeout 600 compute-sanitizer --tool synccheck python scripts/sanitize_run.py > $OUT/sanitize_synccheck_$TAG.txt 2>&1
+# compute-sanitizer: closed on the GPU pool since round 2's r2e session (runs under it had
+# left GPUs needing a reset); the r2d results in profiles/ are the last ones

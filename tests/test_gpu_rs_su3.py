@@ -229,7 +229,18 @@ def _prepared_expected(t):
         c = [int((ls < k).sum()) for k in (1, 2, 3)]
         runs[w] = c[0] | (c[1] << 21) | (c[2] << 42)
     W.view(np.uint64)[:, 3] = runs
-    return out, W
+    # material entries (R-A13): k0rs of the nuclide, conc, win_off | n_windows << 32
+    n_mats, mx = t.num_nucs.shape[0], t.max_num_nucs
+    MN = np.zeros((n_mats * mx, 8))
+    mats, concs = t.mats.reshape(n_mats, mx), t.concs.reshape(n_mats, mx)
+    for m in range(n_mats):
+        for j in range(int(t.num_nucs[m])):
+            nuc = int(mats[m, j])
+            r = MN[m * mx + j]
+            r[0:4] = t.k0rs.reshape(-1, 4)[nuc]
+            r[4] = concs[m, j]
+            r.view(np.uint64)[5] = np.uint64(int(t.win_off[nuc]) | (int(t.n_windows[nuc]) << 32))
+    return out, W, MN
 
 
 def test_rs_prepare_pole_records(rt, rs_tables_small):
@@ -240,13 +251,15 @@ def test_rs_prepare_pole_records(rt, rs_tables_small):
     d = rt.RSDeviceTables(rs_tables_small, DEV)
     got = d.poles_prepared.cpu().numpy().reshape(-1, 8)
     gotw = d.windows_prepared.cpu().numpy().reshape(-1, 4)
-    exp, expw = _prepared_expected(rs_tables_small)
+    gotm = d.matnuc.cpu().numpy().reshape(-1, 8)
+    exp, expw, expm = _prepared_expected(rs_tables_small)
     assert (got.view(np.uint64) == exp.view(np.uint64)).all()
     assert (gotw.view(np.uint64) == expw.view(np.uint64)).all()
+    assert (gotm.view(np.uint64) == expm.view(np.uint64)).all()
     assert d.c.prepared == 1
     with pytest.raises(rt.OmprtError):
-        rt.omprt_rs_prepare(d, exp.shape[0], gotw.shape[0], d.poles_prepared,
-                            d.windows_prepared)
+        rt.omprt_rs_prepare(d, exp.shape[0], gotw.shape[0], d.n_mats, d.poles_prepared,
+                            d.windows_prepared, d.matnuc)
     raw = rt.RSTablesC.from_buffer_copy(d.c)
     raw.prepared = 0
     d.c = raw
@@ -255,21 +268,24 @@ def test_rs_prepare_pole_records(rt, rs_tables_small):
         rt.omprt_rs_lookup(d, 1, 0, 16, v)
 
 
-@pytest.mark.parametrize("defect", ["overlap", "l_range", "past_end"])
+@pytest.mark.parametrize("defect", ["overlap", "l_range", "past_end", "nuclide"])
 def test_rs_prepare_rejects_unsortable_windows(rt, rs_tables_small, defect):
     """Windows that overlap (their poles cannot be sorted independently), an l outside
-    [0, 4) or a range past the last pole: omprt_rs_prepare fails with OMPRT_E_INVAL and
-    leaves the table unprepared."""
+    [0, 4), a range past the last pole or a material entry naming no nuclide:
+    omprt_rs_prepare fails with OMPRT_E_INVAL."""
     import copy
     t = copy.copy(rs_tables_small)
     t.win_range = rs_tables_small.win_range.copy()
     t.pole_l = rs_tables_small.pole_l.copy()
+    t.mats = rs_tables_small.mats.copy()
     if defect == "overlap":
         t.win_range[5, 0] = t.win_range[4, 1] - 1
     elif defect == "l_range":
         t.pole_l[t.win_range[7, 0]] = 4
-    else:
+    elif defect == "past_end":
         t.win_range[-1, 1] = t.poles.shape[0] + 1
+    else:
+        t.mats.reshape(-1)[3] = t.n_nuclides
     with pytest.raises(rt.OmprtError):
         rt.RSDeviceTables(t, DEV)
 

@@ -364,7 +364,8 @@ typedef struct {
  *   win_off | n_windows << 32 of that nuclide (bit pattern), zeros past num_nucs[m]
  *   (reading R-A13: a nuclide step's 6-8 small loads become two).
  * Then points t->poles / t->windows / t->matnuc at them and sets t->prepared = 1.  Synchronizes
- * `stream` (the range checks come back to the host).  OMPRT_E_INVAL on null pointers, a
+ * `stream` (the range checks come back to the host through a device workspace word: do not
+ * run two omprt_rs_prepare calls on one device concurrently).  OMPRT_E_INVAL on null pointers, a
  * misaligned buffer, an already prepared table, numL != 4, a window range outside
  * [0, n_poles) or starting before the previous window's end (windows must not overlap), a
  * window of 2^21 poles or more, an l outside [0, 4), num_nucs outside [0, max_num_nucs]

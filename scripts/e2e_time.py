@@ -1,6 +1,6 @@
 """Host-clock time per step of the end-to-end XS offload (omprt_xs_run_host_steps, derived
 tables, flattened lookups), with and without the L2 set-aside.
-  python scripts/e2e_time.py [steps]"""
+  python scripts/e2e_time.py [steps] [lib.so]   (A/B: one process per library build)"""
 import json
 import os
 import sys
@@ -14,6 +14,8 @@ import gen  # noqa: E402
 from paper_conf_ipps_doerfertphtdcg22_b200 import omprt  # noqa: E402
 
 steps = int(sys.argv[1]) if len(sys.argv) > 1 else 10
+if len(sys.argv) > 2:
+    omprt.load(sys.argv[2])
 torch.cuda.set_device(0)
 omprt.omprt_init(0)
 t = gen.XSTables(**gen.XS_SMALL)

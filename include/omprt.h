@@ -368,8 +368,10 @@ typedef struct {
  * run two omprt_rs_prepare calls on one device concurrently).  OMPRT_E_INVAL on null pointers, a
  * misaligned buffer, an already prepared table, numL != 4, a window range outside
  * [0, n_poles) or starting before the previous window's end (windows must not overlap), a
- * window of 2^21 poles or more, an l outside [0, 4), num_nucs outside [0, max_num_nucs]
- * or a material entry outside [0, n_nuclides); the table is then unchanged. */
+ * window of 2^21 poles or more, an l outside [0, 4), num_nucs outside [0, max_num_nucs],
+ * a material entry outside [0, n_nuclides) or one whose nuclide's windows are not all among
+ * the n_windows (a successful preparation makes every lookup's table access in-range); the
+ * table is then unchanged. */
 int omprt_rs_prepare(omprt_rs_tables *t, int64_t n_poles, int64_t n_windows, int32_t n_mats,
                      double *prepared_poles, double *prepared_windows,
                      double *prepared_matnuc, void *stream);

@@ -441,7 +441,8 @@ __global__ void rs_prepare_windows(const double* __restrict__ poles,
 }
 // one thread per material entry (reading R-A13): the 64 B record of (m, j) -- k0rs of its
 // nuclide, conc, the nuclide's window offset | count << 32 -- zeros past num_nucs[m].
-// Rejected: a nuclide id outside [0, n_nuclides), num_nucs outside [0, max_num_nucs].
+// Rejected: a nuclide id outside [0, n_nuclides), num_nucs outside [0, max_num_nucs], a
+// nuclide whose windows are not all among the n_windows_total prepared ones (or none).
 __global__ void rs_prepare_matnuc(const int32_t* __restrict__ num_nucs,
                                   const int32_t* __restrict__ mats,
                                   const double* __restrict__ concs,
@@ -449,7 +450,8 @@ __global__ void rs_prepare_matnuc(const int32_t* __restrict__ num_nucs,
                                   const int32_t* __restrict__ win_off,
                                   const int32_t* __restrict__ n_windows, int32_t n_mats,
                                   int32_t max_num_nucs, int32_t n_nuclides,
-                                  double* __restrict__ out, unsigned long long* err) {
+                                  int64_t n_windows_total, double* __restrict__ out,
+                                  unsigned long long* err) {
   const int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
   if (i >= (int64_t)n_mats * max_num_nucs) return;
   const int m = (int)(i / max_num_nucs), j = (int)(i % max_num_nucs);
@@ -463,7 +465,8 @@ __global__ void rs_prepare_matnuc(const int32_t* __restrict__ num_nucs,
   }
   if (j >= nn) return;
   const int nuc = mats[i];
-  if (nuc < 0 || nuc >= n_nuclides) {
+  if (nuc < 0 || nuc >= n_nuclides || win_off[nuc] < 0 || n_windows[nuc] < 1 ||
+      (int64_t)win_off[nuc] + n_windows[nuc] > n_windows_total) {
     atomicOr(err, 2ull);
     return;
   }
@@ -502,7 +505,7 @@ extern "C" int omprt_rs_prepare(omprt_rs_tables* t, int64_t n_poles, int64_t n_w
   if (int r = check_launch("rs_prepare_windows")) return r;
   rs_prepare_matnuc<<<(unsigned)ceil_div((int64_t)n_mats * t->max_num_nucs, 256), 256, 0, st>>>(
       t->num_nucs, t->mats, t->concs, t->k0rs, t->win_off, t->n_windows, n_mats,
-      t->max_num_nucs, t->n_nuclides, prepared_matnuc, err);
+      t->max_num_nucs, t->n_nuclides, n_windows, prepared_matnuc, err);
   if (int r = check_launch("rs_prepare_matnuc")) return r;
   unsigned long long bad = 0;
   OMPRT_CUDA_TRY(cudaMemcpyAsync(&bad, err, sizeof(bad), cudaMemcpyDeviceToHost, st));

@@ -268,11 +268,11 @@ def test_rs_prepare_pole_records(rt, rs_tables_small):
         rt.omprt_rs_lookup(d, 1, 0, 16, v)
 
 
-@pytest.mark.parametrize("defect", ["overlap", "l_range", "past_end", "nuclide"])
+@pytest.mark.parametrize("defect", ["overlap", "l_range", "past_end", "nuclide", "n_windows"])
 def test_rs_prepare_rejects_unsortable_windows(rt, rs_tables_small, defect):
     """Windows that overlap (their poles cannot be sorted independently), an l outside
-    [0, 4), a range past the last pole or a material entry naming no nuclide:
-    omprt_rs_prepare fails with OMPRT_E_INVAL."""
+    [0, 4), a range past the last pole, a material entry naming no nuclide or a nuclide
+    whose windows run past the table's: omprt_rs_prepare fails with OMPRT_E_INVAL."""
     import copy
     t = copy.copy(rs_tables_small)
     t.win_range = rs_tables_small.win_range.copy()
@@ -284,8 +284,11 @@ def test_rs_prepare_rejects_unsortable_windows(rt, rs_tables_small, defect):
         t.pole_l[t.win_range[7, 0]] = 4
     elif defect == "past_end":
         t.win_range[-1, 1] = t.poles.shape[0] + 1
-    else:
+    elif defect == "nuclide":
         t.mats.reshape(-1)[3] = t.n_nuclides
+    else:  # a nuclide's windows past the table's
+        t.n_windows = rs_tables_small.n_windows.copy()
+        t.n_windows[int(t.mats.reshape(-1)[0])] += 10_000
     with pytest.raises(rt.OmprtError):
         rt.RSDeviceTables(t, DEV)
 
